@@ -1,0 +1,183 @@
+/* ggrid.h — C ABI of the B200-native lazy-update grid index ("G-Grid") for snapshot
+ * kNN queries over moving objects in road networks.
+ *
+ * Paper: C. Li, Y. Gu, J. Qi, J. He, Q. Deng, G. Yu, "A GPU Accelerated Update Efficient
+ * Index for kNN Queries in Road Networks", ICDE 2018.  Citations "P@N" are 0-based
+ * character offsets into /root/reference/PAPER.md (one line), see SURVEY.md §0.1.
+ *
+ * Conventions (all calls):
+ *  - Plain pointers and sizes; no torch / C++ types.  Every pointer argument named
+ *    "host or device" may be either; the library detects which (cudaPointerGetAttributes)
+ *    and never retains it after the call returns.
+ *  - Return value 0 = GGRID_OK, negative = error (see GGRID_E*); ggrid_strerror() names it.
+ *    On an error no observable state changes (ingest rejects the whole batch).
+ *  - All integers are unsigned 32-bit unless noted ("4-byte integers", P@59405).
+ *    Distances are u32; a location at network distance >= 2^32-1 is unreachable
+ *    (reading R18).  GGRID_PAD = 0xFFFFFFFF pads missing answers.
+ *  - The handle is bound to one CUDA device; calls are synchronous on return
+ *    (the library's stream is drained) and not thread-safe on the same handle.
+ */
+#ifndef GGRID_H
+#define GGRID_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GGRID_OK 0
+#define GGRID_EINVAL (-1)    /* bad argument (range, null pointer, k, offsets, ...) */
+#define GGRID_ENOMEM (-2)    /* device or host allocation failed / log arena exhausted */
+#define GGRID_ECUDA (-3)     /* a CUDA runtime error (sticky errors included) */
+#define GGRID_ENCCL (-4)     /* reserved for the multi-GPU exchange */
+#define GGRID_EOVERFLOW (-5) /* the global arrival index seq would exceed 2^32-1 */
+#define GGRID_PAD 0xFFFFFFFFu
+
+/* Road network G = <V, E> (P@7808-8419): a directed graph, arc a = src[a] -> dst[a] with
+ * weight w[a] >= 1; an undirected road is two arcs of equal weight (P@8380).
+ * The ARC INDEX a (0..n_arcs-1) is the edge id used by updates and queries.
+ * x, y (optional, may be NULL) are vertex coordinates used only to lay out the grid
+ * cells (P@11972-13692); answers never depend on them. All arrays are host pointers. */
+typedef struct ggrid_graph {
+  uint32_t n_vertices;
+  uint32_t n_arcs;
+  const uint32_t* src;
+  const uint32_t* dst;
+  const uint32_t* w;
+  const int32_t* x;
+  const int32_t* y;
+} ggrid_graph;
+
+/* Build options; pass NULL for defaults (each 0 field also means "default"). */
+typedef struct ggrid_opts {
+  int device;              /* CUDA device ordinal; -1 or 0 = current device       */
+  uint32_t max_k;          /* largest k accepted by ggrid_knn (default 256)       */
+  uint32_t max_objects;    /* object ids must be < max_objects (default 2^24)     */
+  uint64_t log_capacity;   /* record arena capacity in records (default 2^26)     */
+  uint32_t delta;          /* expansion bucket width; 0 = mean arc weight          */
+  uint32_t seed_neighbors; /* 0 = default on: flush c_q and its neighbour cells up
+                              front (Alg. 4 line 1); 2 = off (c_q only)            */
+  uint32_t profile;        /* 1 = time every kernel launch with CUDA events        */
+  uint32_t reserved;
+  void* stream;            /* cudaStream_t to run on, or NULL (library stream)    */
+} ggrid_opts;
+
+typedef struct ggrid_s* ggrid_t;
+
+/* Location update message m = <o, e, d, t> (P@10382-10606): object o is on arc e at
+ * distance d from the arc's source (0 <= d < w[e]) at time t.  16 bytes. */
+typedef struct ggrid_update {
+  uint32_t obj;
+  uint32_t edge;
+  uint32_t offset;
+  uint32_t t;
+} ggrid_update;
+
+/* Query q = <k, e, d> (P@45698): a location (edge, offset), 0 <= offset < w[edge]. */
+typedef struct ggrid_query {
+  uint32_t edge;
+  uint32_t offset;
+} ggrid_query;
+
+/* Kernel kinds reported by ggrid_stats. */
+enum {
+  GGRID_K_INGEST_CLASSIFY = 0,
+  GGRID_K_INGEST_ALLOC = 1,
+  GGRID_K_INGEST_SCATTER = 2,
+  GGRID_K_SEED = 3,
+  GGRID_K_FLUSH = 4,
+  GGRID_K_EXPAND = 5,
+  GGRID_K_EXPAND_BIG = 6,
+  GGRID_K_OTHER = 7,
+  GGRID_NK = 8
+};
+
+typedef struct ggrid_stats_t {
+  uint64_t n_updates;        /* updates ingested (= next seq)                        */
+  uint64_t n_queries;        /* queries answered                                     */
+  uint64_t knn_calls;
+  uint64_t knn_rounds;       /* flush+expand rounds over all knn calls               */
+  uint64_t cells_flushed;
+  uint64_t records_flushed;  /* cached records read by flushes                       */
+  uint64_t objects_written;  /* compacted entries written by flushes                 */
+  uint64_t arena_used;       /* records (incl. garbage) in the log arena             */
+  uint64_t arena_capacity;
+  uint64_t gc_runs;
+  uint64_t launches;         /* kernel launches issued by the library, all kinds     */
+  uint64_t kernel_launches[GGRID_NK];
+  double kernel_ms[GGRID_NK];/* summed CUDA-event device time (opts.profile = 1)     */
+  uint32_t n_cells;
+  uint32_t cell_size;
+  uint32_t delta;
+  uint32_t n_vertices;
+  uint32_t n_arcs;
+  uint32_t max_objects;
+} ggrid_stats_t;
+
+/* Build the index (graph grid, P@11423-15818; object table P@15869; message lists
+ * P@16303-17438).  cell_size = the cell capacity delta^c (P@11972): cells are runs of at
+ * most cell_size vertices in Z-order (P@13067-13692) of the quantised coordinates.
+ * Errors: EINVAL (n_vertices = 0 or >= 2^32-1, arc endpoint out of range, w = 0,
+ * cell_size = 0, null pointers, max_k = 0 > 65536), ENOMEM, ECUDA.
+ * Ownership: inputs are copied; *out is owned by the caller until ggrid_free. */
+int ggrid_build(const ggrid_graph* g, uint32_t cell_size, const ggrid_opts* opts, ggrid_t* out);
+
+/* Append n updates (Alg. 1, P@18177-19248, lazy: P@17773-17981).  The global arrival
+ * index seq of u[i] is (updates ingested before this call) + i.  An object's location is
+ * its update with the largest (t, seq) (readings R7/R8); t needs no order.
+ * u: host or device pointer to n records.  Errors: EINVAL (obj >= max_objects,
+ * edge >= n_arcs, offset >= w[edge]: the whole batch is rejected), EOVERFLOW, ENOMEM
+ * (log arena full even after garbage collection), ECUDA. */
+int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n);
+
+/* Answer n_q kNN queries (Def. 1, P@9206-9761; Alg. 4-6, P@44429-52751) on the snapshot
+ * of all updates ingested before the call.  Row i of out_obj / out_dist (n_q*k each,
+ * host or device pointers) holds the k nearest objects in ascending (dist, obj) order,
+ * padded with GGRID_PAD when fewer than k objects are reachable.  Flushes the cells the
+ * queries touch (lazy message cleaning, Alg. 2) as a side effect; answers never depend
+ * on what was flushed before.  q: host or device pointer to n_q queries.
+ * Errors: EINVAL (k = 0 or k > max_k, bad edge/offset, null pointers), ENOMEM, ECUDA. */
+int ggrid_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
+              uint32_t* out_dist);
+
+/* Release every resource of h (NULL is accepted). */
+int ggrid_free(ggrid_t h);
+
+/* Static string naming rc. */
+const char* ggrid_strerror(int rc);
+
+/* ---- test / bench hooks -------------------------------------------------------- */
+
+/* Eager message cleaning of every cell with cached updates (lazy == eager invariant). */
+int ggrid_flush_all(ggrid_t h);
+
+/* Dump the objects located in `cell` (flushing it first if it has cached updates):
+ * up to cap entries of (obj, edge, offset) into host or device arrays; *n receives the
+ * number of objects in the cell (may exceed cap).  Order unspecified.
+ * Errors: EINVAL (cell >= n_cells, null n). */
+int ggrid_cell_objects(ggrid_t h, uint32_t cell, uint32_t* obj, uint32_t* edge, uint32_t* off,
+                       uint32_t cap, uint32_t* n);
+
+/* Counters and per-kernel timings (host pointer). */
+int ggrid_stats(ggrid_t h, ggrid_stats_t* s);
+
+/* Reset the per-kernel launch counters and timings in ggrid_stats. */
+int ggrid_stats_reset(ggrid_t h);
+
+/* The grid partition: cell_of_vertex[v] for every user vertex id (host pointer,
+ * n_vertices entries). */
+int ggrid_vertex_cell(ggrid_t h, uint32_t* cell_of_vertex);
+
+/* Z-value of grid position (x, y): bits of y and x interleaved, y above x at every
+ * level (P@13347-13521: (3,4) -> 37).  Pure host function. */
+uint64_t ggrid_zvalue(uint32_t x, uint32_t y);
+
+/* Library version string. */
+const char* ggrid_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* GGRID_H */

@@ -1,0 +1,250 @@
+"""B200-native lazy-update grid index (G-Grid) for snapshot kNN over moving objects.
+
+Thin Python binding over the C ABI in include/ggrid.h (libggrid.so, built in-tree by
+`paper_conf_icde_li0qhdy18_b200.build`).  Argument marshalling only: every step of
+ingest / flush / expansion / top-k runs in the CUDA kernels of csrc/.  There is no CPU
+fallback: if libggrid.so is missing or no CUDA device is present the calls raise.
+
+The same names as the C ABI are exported (ggrid_build, ggrid_ingest, ggrid_knn, ...), plus
+a small `GGrid` convenience class.  Arrays may be numpy arrays (host) or torch tensors
+(host or CUDA); the library detects host vs device pointers itself.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libggrid.so")
+
+GGRID_OK, GGRID_EINVAL, GGRID_ENOMEM, GGRID_ECUDA, GGRID_ENCCL, GGRID_EOVERFLOW = 0, -1, -2, -3, -4, -5
+PAD = 0xFFFFFFFF
+KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "flush", "expand",
+                "expand_big", "other"]
+EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_flush_all",
+           "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
+           "ggrid_version"]
+
+
+class GGridError(RuntimeError):
+    def __init__(self, rc: int, what: str):
+        self.rc = rc
+        super().__init__(f"{what}: {strerror(rc)} ({rc})")
+
+
+class ggrid_graph(ctypes.Structure):
+    _fields_ = [("n_vertices", ctypes.c_uint32), ("n_arcs", ctypes.c_uint32),
+                ("src", ctypes.c_void_p), ("dst", ctypes.c_void_p), ("w", ctypes.c_void_p),
+                ("x", ctypes.c_void_p), ("y", ctypes.c_void_p)]
+
+
+class ggrid_opts(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("max_k", ctypes.c_uint32), ("max_objects", ctypes.c_uint32),
+                ("log_capacity", ctypes.c_uint64), ("delta", ctypes.c_uint32),
+                ("seed_neighbors", ctypes.c_uint32), ("profile", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32), ("stream", ctypes.c_void_p)]
+
+
+NK = 8
+
+
+class ggrid_stats_t(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_uint64) for n in
+                ["n_updates", "n_queries", "knn_calls", "knn_rounds", "cells_flushed", "records_flushed",
+                 "objects_written", "arena_used", "arena_capacity", "gc_runs", "launches"]] + [
+        ("kernel_launches", ctypes.c_uint64 * NK), ("kernel_ms", ctypes.c_double * NK)] + [
+        (n, ctypes.c_uint32) for n in ["n_cells", "cell_size", "delta", "n_vertices", "n_arcs", "max_objects"]]
+
+
+_lib = None
+
+
+def lib():
+    """Load libggrid.so (raises if it has not been built — no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: run `python -m paper_conf_icde_li0qhdy18_b200.build`")
+        L = ctypes.CDLL(LIB_PATH)
+        P, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+        sig = {
+            "ggrid_build": ([ctypes.POINTER(ggrid_graph), u32, ctypes.POINTER(ggrid_opts), ctypes.POINTER(P)], i32),
+            "ggrid_ingest": ([P, P, u64], i32),
+            "ggrid_knn": ([P, P, u32, u32, P, P], i32),
+            "ggrid_free": ([P], i32),
+            "ggrid_strerror": ([i32], ctypes.c_char_p),
+            "ggrid_flush_all": ([P], i32),
+            "ggrid_cell_objects": ([P, u32, P, P, P, u32, ctypes.POINTER(u32)], i32),
+            "ggrid_stats": ([P, ctypes.POINTER(ggrid_stats_t)], i32),
+            "ggrid_stats_reset": ([P], i32),
+            "ggrid_vertex_cell": ([P, P], i32),
+            "ggrid_zvalue": ([u32, u32], u64),
+            "ggrid_version": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = L
+    return _lib
+
+
+def strerror(rc: int) -> str:
+    return lib().ggrid_strerror(int(rc)).decode()
+
+
+def _check(rc: int, what: str):
+    if rc != GGRID_OK:
+        raise GGridError(rc, what)
+
+
+def _ptr(a):
+    """Raw pointer of a contiguous numpy array or torch tensor (host or device)."""
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        assert a.flags["C_CONTIGUOUS"]
+        return a.ctypes.data
+    assert a.is_contiguous()
+    return a.data_ptr()
+
+
+def _u32(a):
+    if isinstance(a, np.ndarray):
+        return np.ascontiguousarray(a, dtype=np.uint32)
+    import torch
+    assert a.dtype in (torch.int32, torch.uint32), a.dtype
+    return a.contiguous()
+
+
+# ------------------------------------------------------------------------ the C ABI names
+def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 256,
+                max_objects: int = 1 << 24, log_capacity: int = 0, delta: int = 0,
+                seed_neighbors: bool = True, profile: bool = False, stream=None):
+    """ggrid_build(graph, cell_size) -> handle (c_void_p).  graph: dict(n_vertices, src, dst, w[, x, y])."""
+    src, dst, w = (np.ascontiguousarray(graph[k], np.uint32) for k in ("src", "dst", "w"))
+    x = graph.get("x")
+    y = graph.get("y")
+    x = None if x is None else np.ascontiguousarray(x, np.int32)
+    y = None if y is None else np.ascontiguousarray(y, np.int32)
+    g = ggrid_graph(int(graph["n_vertices"]), len(src), src.ctypes.data, dst.ctypes.data, w.ctypes.data,
+                    None if x is None else x.ctypes.data, None if y is None else y.ctypes.data)
+    o = ggrid_opts(int(device), int(max_k), int(max_objects), int(log_capacity), int(delta),
+                   0 if seed_neighbors else 2, 1 if profile else 0, 0, stream)
+    h = ctypes.c_void_p()
+    _check(lib().ggrid_build(ctypes.byref(g), int(cell_size), ctypes.byref(o), ctypes.byref(h)), "ggrid_build")
+    return h
+
+
+def ggrid_ingest(h, updates, n: int | None = None):
+    """Append updates: (n, 4) u32 (obj, edge, offset, t) numpy array or torch tensor."""
+    u = _u32(updates)
+    cnt = int(u.shape[0]) if n is None else int(n)
+    _check(lib().ggrid_ingest(h, _ptr(u), cnt), "ggrid_ingest")
+
+
+def ggrid_knn(h, queries, k: int, out_obj=None, out_dist=None):
+    """Answer queries ((n, 2) u32 (edge, offset)); returns (out_obj, out_dist) of shape (n, k).
+
+    Outputs default to numpy arrays; pass preallocated torch tensors (int32/uint32, host or
+    CUDA) to receive them in place."""
+    q = _u32(queries)
+    nq = int(q.shape[0])
+    if out_obj is None:
+        out_obj = np.empty((nq, k), np.uint32)
+    if out_dist is None:
+        out_dist = np.empty((nq, k), np.uint32)
+    _check(lib().ggrid_knn(h, _ptr(q), nq, int(k), _ptr(out_obj), _ptr(out_dist)), "ggrid_knn")
+    return out_obj, out_dist
+
+
+def ggrid_free(h):
+    if h:
+        lib().ggrid_free(h)
+
+
+def ggrid_flush_all(h):
+    _check(lib().ggrid_flush_all(h), "ggrid_flush_all")
+
+
+def ggrid_cell_objects(h, cell: int, cap: int = 1 << 16):
+    obj = np.empty(cap, np.uint32)
+    edge = np.empty(cap, np.uint32)
+    off = np.empty(cap, np.uint32)
+    n = ctypes.c_uint32()
+    _check(lib().ggrid_cell_objects(h, int(cell), obj.ctypes.data, edge.ctypes.data, off.ctypes.data, cap,
+                                    ctypes.byref(n)), "ggrid_cell_objects")
+    if n.value > cap:
+        return ggrid_cell_objects(h, cell, int(n.value))
+    m = n.value
+    return obj[:m].copy(), edge[:m].copy(), off[:m].copy()
+
+
+def ggrid_stats(h) -> dict:
+    s = ggrid_stats_t()
+    _check(lib().ggrid_stats(h, ctypes.byref(s)), "ggrid_stats")
+    d = {f: getattr(s, f) for f, _ in ggrid_stats_t._fields_ if f not in ("kernel_launches", "kernel_ms")}
+    d["kernel_launches"] = dict(zip(KERNEL_KINDS, list(s.kernel_launches)))
+    d["kernel_ms"] = dict(zip(KERNEL_KINDS, list(s.kernel_ms)))
+    return d
+
+
+def ggrid_stats_reset(h):
+    _check(lib().ggrid_stats_reset(h), "ggrid_stats_reset")
+
+
+def ggrid_vertex_cell(h, n_vertices: int):
+    out = np.empty(n_vertices, np.uint32)
+    _check(lib().ggrid_vertex_cell(h, out.ctypes.data), "ggrid_vertex_cell")
+    return out
+
+
+def ggrid_zvalue(x: int, y: int) -> int:
+    return int(lib().ggrid_zvalue(int(x), int(y)))
+
+
+def ggrid_version() -> str:
+    return lib().ggrid_version().decode()
+
+
+class GGrid:
+    """Owning wrapper: GGrid(graph, cell_size, **opts).ingest(u).knn(q, k)."""
+
+    def __init__(self, graph: dict, cell_size: int, **opts):
+        self.n_vertices = int(graph["n_vertices"])
+        self.h = ggrid_build(graph, cell_size, **opts)
+
+    def ingest(self, updates):
+        ggrid_ingest(self.h, updates)
+        return self
+
+    def knn(self, queries, k: int, out_obj=None, out_dist=None):
+        return ggrid_knn(self.h, queries, k, out_obj, out_dist)
+
+    def flush_all(self):
+        ggrid_flush_all(self.h)
+
+    def cell_objects(self, cell: int):
+        return ggrid_cell_objects(self.h, cell)
+
+    def vertex_cell(self):
+        return ggrid_vertex_cell(self.h, self.n_vertices)
+
+    def stats(self):
+        return ggrid_stats(self.h)
+
+    def stats_reset(self):
+        ggrid_stats_reset(self.h)
+
+    def close(self):
+        if self.h:
+            ggrid_free(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,643 @@
+// api.cu — the C ABI (include/ggrid.h): host-side graph-grid build, device memory
+// management, ingest / knn orchestration, garbage collection of the record arena.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <utility>
+#include <vector>
+
+#include "ggrid.h"
+#include "internal.cuh"
+
+using namespace gg;
+
+namespace {
+
+bool debug_on() {
+  static int v = -1;
+  if (v < 0) v = getenv("GGRID_DEBUG") ? 1 : 0;
+  return v == 1;
+}
+
+#define CK(x)                                                                             \
+  do {                                                                                    \
+    cudaError_t e_ = (x);                                                                 \
+    if (e_ != cudaSuccess) {                                                              \
+      if (debug_on()) fprintf(stderr, "ggrid: %s:%d %s: %s\n", __FILE__, __LINE__, #x,    \
+                              cudaGetErrorString(e_));                                    \
+      return e_ == cudaErrorMemoryAllocation ? GGRID_ENOMEM : GGRID_ECUDA;                \
+    }                                                                                     \
+  } while (0)
+
+#define RC(x)                  \
+  do {                         \
+    int r_ = (x);              \
+    if (r_ != GGRID_OK) return r_; \
+  } while (0)
+
+// grow-only device buffer
+struct DBuf {
+  void* p = nullptr;
+  size_t n = 0;
+  int ensure(size_t bytes) {
+    if (bytes <= n) return GGRID_OK;
+    if (p) cudaFree(p);
+    p = nullptr;
+    n = 0;
+    size_t want = std::max<size_t>(bytes, 4096);
+    if (cudaMalloc(&p, want) != cudaSuccess) {
+      cudaGetLastError();
+      return GGRID_ENOMEM;
+    }
+    n = want;
+    return GGRID_OK;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    n = 0;
+  }
+  template <class T>
+  T* as() const {
+    return static_cast<T*>(p);
+  }
+};
+
+bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+}  // namespace
+
+struct ggrid_s {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int sm_count = 148;
+  uint32_t V = 0, A = 0, cs = 1, n_cells = 0, delta = 1, max_k = 256, max_objects = 0;
+  int seed_neighbors = 1;
+  int profile = 0;
+  std::vector<uint32_t> user_cell;
+  DevGraph g{};
+  DevState s{};
+  std::vector<void*> allocs;
+  DevStatus* d_status = nullptr;
+  DevStatus* h_status = nullptr;  // pinned
+  uint64_t seq_next = 0;
+  uint32_t epoch = 0;
+  DBuf upd_stage, tmp, q_stage, out_stage, lists, l2_scratch, dump_stage, gc_buf, misc;
+  ggrid_stats_t stats{};
+  std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending_ev;
+  std::vector<cudaEvent_t> ev_pool;
+
+  template <class T>
+  int alloc(T** p, size_t count, bool zero = true) {
+    *p = nullptr;
+    size_t bytes = std::max<size_t>(count * sizeof(T), 16);
+    if (cudaMalloc((void**)p, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      return GGRID_ENOMEM;
+    }
+    allocs.push_back(*p);
+    if (zero && cudaMemset(*p, 0, bytes) != cudaSuccess) return GGRID_ECUDA;
+    return GGRID_OK;
+  }
+
+  cudaEvent_t get_event() {
+    if (!ev_pool.empty()) {
+      cudaEvent_t e = ev_pool.back();
+      ev_pool.pop_back();
+      return e;
+    }
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    return e;
+  }
+
+  // every kernel launch goes through here: counted, and timed in profile mode
+  template <class F>
+  void launch(int kind, F&& f) {
+    stats.launches++;
+    stats.kernel_launches[kind]++;
+    if (profile) {
+      cudaEvent_t a = get_event(), b = get_event();
+      cudaEventRecord(a, stream);
+      f();
+      cudaEventRecord(b, stream);
+      pending_ev.push_back({kind, {a, b}});
+    } else {
+      f();
+    }
+  }
+
+  // drain the stream, collect event timings, refresh the status mirror
+  int sync() {
+    CK(cudaMemcpyAsync(h_status, d_status, sizeof(DevStatus), cudaMemcpyDeviceToHost, stream));
+    CK(cudaStreamSynchronize(stream));
+    for (auto& pe : pending_ev) {
+      float ms = 0.f;
+      if (cudaEventElapsedTime(&ms, pe.second.first, pe.second.second) == cudaSuccess)
+        stats.kernel_ms[pe.first] += ms;
+      ev_pool.push_back(pe.second.first);
+      ev_pool.push_back(pe.second.second);
+    }
+    pending_ev.clear();
+    CK(cudaGetLastError());
+    return GGRID_OK;
+  }
+
+  int set_status_u32(unsigned int* field, unsigned int v) {
+    CK(cudaMemsetAsync(field, 0, sizeof(unsigned int), stream));
+    if (v) CK(cudaMemcpyAsync(field, &v, sizeof v, cudaMemcpyHostToDevice, stream));
+    return GGRID_OK;
+  }
+
+  int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin) {
+    CK(cudaMemsetAsync(&d_status->flush_work, 0, sizeof(unsigned int), stream));
+    launch(GGRID_K_FLUSH, [&] { launch_flush(g, s, out, out_top, begin, sm_count, stream); });
+    return GGRID_OK;
+  }
+
+  int gc();
+  int ensure_arena(uint64_t need_records, uint32_t need_ext);
+  // upper bound of the records a flush of every dirty cell can write: each live object is
+  // valid in exactly one cell, plus <= 3 padding records per cell (dirty cells <= extents)
+  uint64_t flush_need() const {
+    return (uint64_t)h_status->n_live + 4ull * std::min<uint64_t>(n_cells, h_status->ext_top) + 16;
+  }
+};
+
+// ------------------------------------------------------------------------------------------
+// Garbage collection of the log arena: every cell (clean or not) is cleaned into a fresh
+// arena, which is copied back to the start of the main one; the extent pool is emptied.
+int ggrid_s::gc() {
+  RC(sync());
+  const uint64_t live = (uint64_t)h_status->n_live + 4ull * n_cells + 16;
+  const size_t per = 4 + 8 + 4 + 4 + 4;
+  RC(gc_buf.ensure(live * per + 64));
+  Arena t;
+  unsigned char* b = gc_buf.as<unsigned char>();
+  t.key = reinterpret_cast<unsigned long long*>(b);
+  t.obj = reinterpret_cast<uint32_t*>(t.key + live);
+  t.vsrc = t.obj + live;
+  t.off = t.vsrc + live;
+  t.edge = t.off + live;
+  t.cap = live;
+  unsigned long long* d_top = nullptr;
+  RC(misc.ensure(64));
+  d_top = misc.as<unsigned long long>();
+  CK(cudaMemsetAsync(d_top, 0, 8, stream));
+  epoch++;
+  RC(set_status_u32(&d_status->n_flush, 0));
+  launch(GGRID_K_OTHER, [&] { launch_mark_dirty(g, s, epoch, 1, stream); });
+  RC(flush_list_run(t, d_top, 0));
+  unsigned long long top = 0;
+  CK(cudaMemcpyAsync(&top, d_top, 8, cudaMemcpyDeviceToHost, stream));
+  RC(sync());
+  if (h_status->err & ERR_ARENA) return GGRID_ENOMEM;
+  CK(cudaMemcpyAsync(s.ar.obj, t.obj, top * 4, cudaMemcpyDeviceToDevice, stream));
+  CK(cudaMemcpyAsync(s.ar.key, t.key, top * 8, cudaMemcpyDeviceToDevice, stream));
+  CK(cudaMemcpyAsync(s.ar.vsrc, t.vsrc, top * 4, cudaMemcpyDeviceToDevice, stream));
+  CK(cudaMemcpyAsync(s.ar.off, t.off, top * 4, cudaMemcpyDeviceToDevice, stream));
+  CK(cudaMemcpyAsync(s.ar.edge, t.edge, top * 4, cudaMemcpyDeviceToDevice, stream));
+  CK(cudaMemcpyAsync(&d_status->arena_top, &top, 8, cudaMemcpyHostToDevice, stream));
+  RC(set_status_u32(&d_status->ext_top, 0));
+  RC(sync());
+  gc_buf.release();
+  stats.gc_runs++;
+  return GGRID_OK;
+}
+
+int ggrid_s::ensure_arena(uint64_t need_records, uint32_t need_ext) {
+  const bool fits_a = h_status->arena_top + need_records <= s.ar.cap;
+  const bool fits_e = (uint64_t)h_status->ext_top + need_ext <= s.ext_cap;
+  if (fits_a && fits_e) return GGRID_OK;
+  RC(gc());
+  if (h_status->arena_top + need_records > s.ar.cap) return GGRID_ENOMEM;
+  if ((uint64_t)h_status->ext_top + need_ext > s.ext_cap) return GGRID_ENOMEM;
+  return GGRID_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+extern "C" {
+
+const char* ggrid_version(void) { return "ggrid-b200 0.1 (sm_100a)"; }
+
+const char* ggrid_strerror(int rc) {
+  switch (rc) {
+    case GGRID_OK: return "ok";
+    case GGRID_EINVAL: return "invalid argument";
+    case GGRID_ENOMEM: return "out of memory";
+    case GGRID_ECUDA: return "CUDA error";
+    case GGRID_ENCCL: return "NCCL error";
+    case GGRID_EOVERFLOW: return "arrival index overflow (more than 2^32 updates)";
+    default: return "unknown error";
+  }
+}
+
+uint64_t ggrid_zvalue(uint32_t x, uint32_t y) {
+  uint64_t z = 0;
+  for (int b = 0; b < 32; ++b) {
+    z |= (uint64_t)((x >> b) & 1u) << (2 * b);
+    z |= (uint64_t)((y >> b) & 1u) << (2 * b + 1);
+  }
+  return z;
+}
+
+int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opts, ggrid_t* out) {
+  if (!gr || !out) return GGRID_EINVAL;
+  *out = nullptr;
+  const uint32_t V = gr->n_vertices, A = gr->n_arcs;
+  if (V == 0 || V >= 0xFFFFFFFEu || A >= 0xFFFFFFFEu || cell_size == 0) return GGRID_EINVAL;
+  if (A > 0 && (!gr->src || !gr->dst || !gr->w)) return GGRID_EINVAL;
+  if ((gr->x == nullptr) != (gr->y == nullptr)) return GGRID_EINVAL;
+  for (uint32_t a = 0; a < A; ++a)
+    if (gr->src[a] >= V || gr->dst[a] >= V || gr->w[a] == 0) return GGRID_EINVAL;
+  ggrid_opts o{};
+  if (opts) o = *opts;
+  if (o.max_k == 0) o.max_k = 256;
+  if (o.max_k > expand_max_k(expand_levels() - 1)) return GGRID_EINVAL;
+  if (o.max_objects == 0) o.max_objects = 1u << 24;
+  if (o.max_objects == 0xFFFFFFFFu) return GGRID_EINVAL;
+  if (o.log_capacity == 0) o.log_capacity = 1ull << 26;
+  if (o.log_capacity > 0xFFFFFFF0ull) return GGRID_EINVAL;
+
+  ggrid_s* h = new (std::nothrow) ggrid_s();
+  if (!h) return GGRID_ENOMEM;
+  auto fail = [&](int rc) {
+    ggrid_free(h);
+    return rc;
+  };
+  if (o.device > 0) {
+    if (cudaSetDevice(o.device) != cudaSuccess) return fail(GGRID_ECUDA);
+  }
+  if (cudaGetDevice(&h->device) != cudaSuccess) return fail(GGRID_ECUDA);
+  cudaDeviceGetAttribute(&h->sm_count, cudaDevAttrMultiProcessorCount, h->device);
+  if (o.stream) {
+    h->stream = (cudaStream_t)o.stream;
+  } else {
+    if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess)
+      return fail(GGRID_ECUDA);
+    h->own_stream = true;
+  }
+  h->V = V;
+  h->A = A;
+  h->cs = cell_size;
+  h->n_cells = (uint32_t)((V + (uint64_t)cell_size - 1) / cell_size);
+  h->max_k = o.max_k;
+  h->max_objects = o.max_objects;
+  h->seed_neighbors = o.seed_neighbors == 2 ? 0 : 1;
+  h->profile = o.profile ? 1 : 0;
+
+  // ---- graph grid: Z-order of quantised coordinates, cells = runs of cell_size vertices
+  std::vector<uint32_t> order(V);
+  for (uint32_t v = 0; v < V; ++v) order[v] = v;
+  if (gr->x) {
+    int64_t mnx = INT64_MAX, mxx = INT64_MIN, mny = INT64_MAX, mxy = INT64_MIN;
+    for (uint32_t v = 0; v < V; ++v) {
+      mnx = std::min<int64_t>(mnx, gr->x[v]);
+      mxx = std::max<int64_t>(mxx, gr->x[v]);
+      mny = std::min<int64_t>(mny, gr->y[v]);
+      mxy = std::max<int64_t>(mxy, gr->y[v]);
+    }
+    const int64_t sx = std::max<int64_t>(1, mxx - mnx), sy = std::max<int64_t>(1, mxy - mny);
+    std::vector<uint64_t> key(V);
+    for (uint32_t v = 0; v < V; ++v) {
+      uint32_t qx = (uint32_t)(((int64_t)gr->x[v] - mnx) * 65535 / sx);
+      uint32_t qy = (uint32_t)(((int64_t)gr->y[v] - mny) * 65535 / sy);
+      key[v] = (ggrid_zvalue(qx, qy) << 32) | v;
+    }
+    std::sort(key.begin(), key.end());
+    for (uint32_t i = 0; i < V; ++i) order[i] = (uint32_t)key[i];
+  }
+  std::vector<uint32_t> newid(V);
+  for (uint32_t i = 0; i < V; ++i) newid[order[i]] = i;
+  h->user_cell.resize(V);
+  for (uint32_t v = 0; v < V; ++v) h->user_cell[v] = newid[v] / cell_size;
+
+  // ---- CSR over internal ids, inverted index (user edge -> src, w, dst)
+  std::vector<uint32_t> rowptr((size_t)V + 1, 0);
+  for (uint32_t a = 0; a < A; ++a) rowptr[newid[gr->src[a]] + 1]++;
+  for (uint32_t v = 0; v < V; ++v) rowptr[v + 1] += rowptr[v];
+  std::vector<uint2> adj(A), einfo(A);
+  std::vector<uint32_t> edst(A);
+  {
+    std::vector<uint32_t> fill(rowptr.begin(), rowptr.end() - 1);
+    uint64_t wsum = 0;
+    for (uint32_t a = 0; a < A; ++a) {
+      const uint32_t u = newid[gr->src[a]], v = newid[gr->dst[a]];
+      adj[fill[u]++] = make_uint2(v, gr->w[a]);
+      einfo[a] = make_uint2(u, gr->w[a]);
+      edst[a] = v;
+      wsum += gr->w[a];
+    }
+    h->delta = o.delta ? o.delta : (uint32_t)std::max<uint64_t>(1, A ? wsum / A : 1);
+  }
+  // ---- cell adjacency (P@47172: c_i neighbours c_j if an arc goes from c_i to c_j)
+  std::vector<uint64_t> cpairs;
+  for (uint32_t a = 0; a < A; ++a) {
+    const uint32_t cu = einfo[a].x / cell_size, cv = edst[a] / cell_size;
+    if (cu != cv) cpairs.push_back(((uint64_t)cu << 32) | cv);
+  }
+  std::sort(cpairs.begin(), cpairs.end());
+  cpairs.erase(std::unique(cpairs.begin(), cpairs.end()), cpairs.end());
+  std::vector<uint32_t> cptr((size_t)h->n_cells + 1, 0), cadj(cpairs.size());
+  for (size_t i = 0; i < cpairs.size(); ++i) {
+    cptr[(cpairs[i] >> 32) + 1]++;
+    cadj[i] = (uint32_t)cpairs[i];
+  }
+  for (uint32_t c = 0; c < h->n_cells; ++c) cptr[c + 1] += cptr[c];
+
+  // ---- device graph
+  uint32_t *d_rowptr, *d_edst, *d_cptr, *d_cadj;
+  uint2 *d_adj, *d_einfo;
+  int rc;
+  if ((rc = h->alloc(&d_rowptr, (size_t)V + 1, false))) return fail(rc);
+  if ((rc = h->alloc(&d_adj, A, false))) return fail(rc);
+  if ((rc = h->alloc(&d_einfo, A, false))) return fail(rc);
+  if ((rc = h->alloc(&d_edst, A, false))) return fail(rc);
+  if ((rc = h->alloc(&d_cptr, (size_t)h->n_cells + 1, false))) return fail(rc);
+  if ((rc = h->alloc(&d_cadj, cadj.size(), false))) return fail(rc);
+  if (cudaMemcpy(d_rowptr, rowptr.data(), rowptr.size() * 4, cudaMemcpyHostToDevice) ||
+      cudaMemcpy(d_adj, adj.data(), (size_t)A * 8, cudaMemcpyHostToDevice) ||
+      cudaMemcpy(d_einfo, einfo.data(), (size_t)A * 8, cudaMemcpyHostToDevice) ||
+      cudaMemcpy(d_edst, edst.data(), (size_t)A * 4, cudaMemcpyHostToDevice) ||
+      cudaMemcpy(d_cptr, cptr.data(), cptr.size() * 4, cudaMemcpyHostToDevice) ||
+      (cadj.size() && cudaMemcpy(d_cadj, cadj.data(), cadj.size() * 4, cudaMemcpyHostToDevice)))
+    return fail(GGRID_ECUDA);
+  h->g = DevGraph{V, A, cell_size, h->n_cells, h->delta, d_rowptr, d_adj, d_einfo, d_edst, d_cptr, d_cadj};
+
+  // ---- dynamic state
+  DevState& s = h->s;
+  s.max_objects = o.max_objects;
+  if ((rc = h->alloc(&s.ot_key, o.max_objects))) return fail(rc);
+  const uint64_t cap = (o.log_capacity + 3) & ~3ull;
+  s.ar.cap = cap;
+  if ((rc = h->alloc(&s.ar.obj, cap + 4, false))) return fail(rc);
+  if ((rc = h->alloc(&s.ar.key, cap + 4, false))) return fail(rc);
+  if ((rc = h->alloc(&s.ar.vsrc, cap + 4, false))) return fail(rc);
+  if ((rc = h->alloc(&s.ar.off, cap + 4, false))) return fail(rc);
+  if ((rc = h->alloc(&s.ar.edge, cap + 4, false))) return fail(rc);
+  s.ext_cap = (uint32_t)std::min<uint64_t>(std::max<uint64_t>(1u << 20, 16ull * h->n_cells), 1u << 27);
+  if ((rc = h->alloc(&s.x_start, s.ext_cap, false))) return fail(rc);
+  if ((rc = h->alloc(&s.x_len, s.ext_cap, false))) return fail(rc);
+  if ((rc = h->alloc(&s.x_next, s.ext_cap, false))) return fail(rc);
+  if ((rc = h->alloc(&s.cell_head, h->n_cells, false))) return fail(rc);
+  if (cudaMemset(s.cell_head, 0xFF, (size_t)h->n_cells * 4)) return fail(GGRID_ECUDA);
+  if ((rc = h->alloc(&s.cell_pending, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&s.cell_req, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&s.v_obj, V))) return fail(rc);
+  if ((rc = h->alloc(&s.cell_comp, h->n_cells))) return fail(rc);
+  s.vcnt = nullptr;
+  if (cell_size > 4096 && (rc = h->alloc(&s.vcnt, V))) return fail(rc);
+  if ((rc = h->alloc(&s.bcount, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&s.bbase, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&s.flush_list, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&h->d_status, 1))) return fail(rc);
+  s.st = h->d_status;
+  if (cudaMallocHost((void**)&h->h_status, sizeof(DevStatus)) != cudaSuccess) return fail(GGRID_ENOMEM);
+  memset(h->h_status, 0, sizeof(DevStatus));
+  h->stats.arena_capacity = cap;
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(GGRID_ECUDA);
+  *out = h;
+  return GGRID_OK;
+}
+
+int ggrid_free(ggrid_t h) {
+  if (!h) return GGRID_OK;
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  for (void* p : h->allocs) cudaFree(p);
+  for (DBuf* b : {&h->upd_stage, &h->tmp, &h->q_stage, &h->out_stage, &h->lists, &h->l2_scratch,
+                  &h->dump_stage, &h->gc_buf, &h->misc})
+    b->release();
+  for (auto& pe : h->pending_ev) {
+    cudaEventDestroy(pe.second.first);
+    cudaEventDestroy(pe.second.second);
+  }
+  for (cudaEvent_t e : h->ev_pool) cudaEventDestroy(e);
+  if (h->h_status) cudaFreeHost(h->h_status);
+  if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+  delete h;
+  return GGRID_OK;
+}
+
+int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
+  if (!h) return GGRID_EINVAL;
+  if (n == 0) return GGRID_OK;
+  if (!u) return GGRID_EINVAL;
+  if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
+  CK(cudaSetDevice(h->device));
+  const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
+  RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
+  const uint4* d_u = reinterpret_cast<const uint4*>(u);
+  if (!is_device_ptr(u)) {
+    RC(h->upd_stage.ensure(n * sizeof(uint4)));
+    CK(cudaMemcpyAsync(h->upd_stage.p, u, n * sizeof(uint4), cudaMemcpyHostToDevice, h->stream));
+    d_u = h->upd_stage.as<uint4>();
+  }
+  RC(h->tmp.ensure(n * sizeof(uint2)));
+  unsigned int zero_bad[2] = {0u, 0xFFFFFFFFu};
+  CK(cudaMemcpyAsync(&h->d_status->err, zero_bad, 8, cudaMemcpyHostToDevice, h->stream));
+  const uint32_t seq0 = (uint32_t)h->seq_next;
+  const DevGraph& g = h->g;
+  const DevState& s = h->s;
+  uint2* tmp = h->tmp.as<uint2>();
+  cudaStream_t st = h->stream;
+  h->launch(GGRID_K_INGEST_CLASSIFY, [&] { launch_ingest_classify(d_u, n, g, s, tmp, st); });
+  h->launch(GGRID_K_INGEST_ALLOC, [&] { launch_ingest_alloc(g, s, st); });
+  h->launch(GGRID_K_INGEST_SCATTER, [&] { launch_ingest_scatter(d_u, n, seq0, g, s, tmp, st); });
+  RC(h->sync());
+  const unsigned err = h->h_status->err;
+  if (err & (ERR_OBJ | ERR_EDGE | ERR_OFF)) return GGRID_EINVAL;
+  if (err & ERR_ARENA) return GGRID_ENOMEM;
+  h->seq_next += n;
+  h->stats.n_updates = h->seq_next;
+  return GGRID_OK;
+}
+
+static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
+                    uint32_t* out_dist) {
+  CK(cudaSetDevice(h->device));
+  cudaStream_t st = h->stream;
+  // every flushed cell writes at most its live objects (+ alignment padding)
+  RC(h->ensure_arena(h->flush_need(), 0));
+  const uint2* d_q = reinterpret_cast<const uint2*>(q);
+  if (!is_device_ptr(q)) {
+    RC(h->q_stage.ensure((size_t)n_q * 8));
+    CK(cudaMemcpyAsync(h->q_stage.p, q, (size_t)n_q * 8, cudaMemcpyHostToDevice, st));
+    d_q = h->q_stage.as<uint2>();
+  }
+  const bool dev_o = is_device_ptr(out_obj), dev_d = is_device_ptr(out_dist);
+  uint32_t* d_oo = out_obj;
+  uint32_t* d_od = out_dist;
+  const size_t outn = (size_t)n_q * k;
+  if (!dev_o || !dev_d) {
+    RC(h->out_stage.ensure(outn * 8));
+    if (!dev_o) d_oo = h->out_stage.as<uint32_t>();
+    if (!dev_d) d_od = h->out_stage.as<uint32_t>() + outn;
+  }
+  const int L = expand_levels();
+  RC(h->lists.ensure((size_t)2 * L * n_q * 4));
+  uint32_t* lists = h->lists.as<uint32_t>();
+  auto list = [&](int buf, int lvl) { return lists + ((size_t)buf * L + lvl) * n_q; };
+
+  h->epoch++;
+  const uint32_t epoch = h->epoch;
+  // reset err, n_flush, flush_work, n_next[*], flush_end
+  CK(cudaMemsetAsync(&h->d_status->err, 0, sizeof(unsigned), st));
+  CK(cudaMemsetAsync(&h->d_status->n_flush, 0, offsetof(DevStatus, pad) - offsetof(DevStatus, n_flush), st));
+  const DevGraph& g = h->g;
+  const DevState& s = h->s;
+  h->launch(GGRID_K_SEED, [&] { launch_seed(d_q, n_q, g, s, epoch, h->seed_neighbors, st); });
+
+  int lvl0 = 0;
+  while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
+  std::vector<uint32_t> n_in(L, 0);
+  n_in[lvl0] = n_q;
+  std::vector<const uint32_t*> in_list(L, nullptr);
+  int cur = 0;
+  uint32_t flush_begin = 0;
+  for (int round = 0;; ++round) {
+    if (round > 100000) return GGRID_ECUDA;
+    RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin));
+    CK(cudaMemsetAsync(h->d_status->n_next, 0, sizeof(h->d_status->n_next), st));
+    for (int lvl = 0; lvl < L; ++lvl) {
+      if (!n_in[lvl]) continue;
+      void* scratch = nullptr;
+      uint32_t sw = 0;
+      if (lvl == L - 1) {
+        const size_t wb = expand_warp_bytes(lvl, h->V);
+        sw = (uint32_t)std::max<size_t>(1, std::min<size_t>(64, (size_t(2) << 30) / wb));
+        sw = std::min<uint32_t>(sw, n_in[lvl]);
+        RC(h->l2_scratch.ensure(wb * sw));
+        scratch = h->l2_scratch.p;
+      }
+      uint32_t* retry = list(cur ^ 1, lvl);
+      uint32_t* promote = lvl + 1 < L ? list(cur ^ 1, lvl + 1) : nullptr;
+      const uint32_t* qlist = in_list[lvl];
+      const uint32_t nn = n_in[lvl];
+      const int kind = lvl == 0 ? GGRID_K_EXPAND : GGRID_K_EXPAND_BIG;
+      h->launch(kind, [&] {
+        launch_expand(lvl, d_q, qlist, nn, k, g, s, epoch, retry, promote, d_oo, d_od, scratch, sw, st);
+      });
+    }
+    RC(h->sync());
+    h->stats.knn_rounds++;
+    const unsigned err = h->h_status->err;
+    if (err & ERR_QUERY) return GGRID_EINVAL;
+    if (err & (ERR_ARENA | ERR_FAIL)) return GGRID_ENOMEM;
+    flush_begin = h->h_status->flush_end;
+    bool any = false;
+    for (int lvl = 0; lvl < L; ++lvl) {
+      n_in[lvl] = h->h_status->n_next[lvl];
+      in_list[lvl] = list(cur ^ 1, lvl);
+      any |= n_in[lvl] != 0;
+    }
+    cur ^= 1;
+    if (!any) break;
+  }
+  if (!dev_o) CK(cudaMemcpyAsync(out_obj, d_oo, outn * 4, cudaMemcpyDeviceToHost, st));
+  if (!dev_d) CK(cudaMemcpyAsync(out_dist, d_od, outn * 4, cudaMemcpyDeviceToHost, st));
+  RC(h->sync());
+  h->stats.n_queries += n_q;
+  h->stats.knn_calls++;
+  return GGRID_OK;
+}
+
+int ggrid_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
+              uint32_t* out_dist) {
+  if (!h || k == 0 || k > h->max_k) return GGRID_EINVAL;
+  if (n_q == 0) return GGRID_OK;
+  if (!q || !out_obj || !out_dist) return GGRID_EINVAL;
+  return knn_impl(h, q, n_q, k, out_obj, out_dist);
+}
+
+int ggrid_flush_all(ggrid_t h) {
+  if (!h) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  RC(h->ensure_arena(h->flush_need(), 0));
+  h->epoch++;
+  RC(h->set_status_u32(&h->d_status->n_flush, 0));
+  h->launch(GGRID_K_OTHER, [&] { launch_mark_dirty(h->g, h->s, h->epoch, 0, h->stream); });
+  RC(h->flush_list_run(h->s.ar, &h->d_status->arena_top, 0));
+  RC(h->sync());
+  if (h->h_status->err & ERR_ARENA) return GGRID_ENOMEM;
+  return GGRID_OK;
+}
+
+int ggrid_cell_objects(ggrid_t h, uint32_t cell, uint32_t* obj, uint32_t* edge, uint32_t* off,
+                       uint32_t cap, uint32_t* n) {
+  if (!h || !n || cell >= h->n_cells) return GGRID_EINVAL;
+  if (cap && (!obj || !edge || !off)) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  RC(h->ensure_arena(h->flush_need(), 0));
+  h->epoch++;
+  RC(h->set_status_u32(&h->d_status->n_flush, 1));
+  CK(cudaMemcpyAsync(h->s.flush_list, &cell, 4, cudaMemcpyHostToDevice, h->stream));
+  RC(h->flush_list_run(h->s.ar, &h->d_status->arena_top, 0));
+  RC(h->dump_stage.ensure(16 + (size_t)cap * 12));
+  uint32_t* d_n = h->dump_stage.as<uint32_t>();
+  uint32_t* d_o = d_n + 4;
+  uint32_t* d_e = d_o + cap;
+  uint32_t* d_f = d_e + cap;
+  CK(cudaMemsetAsync(d_n, 0, 4, h->stream));
+  h->launch(GGRID_K_OTHER, [&] { launch_dump_cell(h->g, h->s, cell, d_o, d_e, d_f, cap, d_n, h->stream); });
+  uint32_t cnt = 0;
+  CK(cudaMemcpyAsync(&cnt, d_n, 4, cudaMemcpyDeviceToHost, h->stream));
+  RC(h->sync());
+  const uint32_t m = std::min(cnt, cap);
+  if (m) {
+    CK(cudaMemcpy(obj, d_o, (size_t)m * 4, cudaMemcpyDefault));
+    CK(cudaMemcpy(edge, d_e, (size_t)m * 4, cudaMemcpyDefault));
+    CK(cudaMemcpy(off, d_f, (size_t)m * 4, cudaMemcpyDefault));
+  }
+  *n = cnt;
+  return GGRID_OK;
+}
+
+int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
+  if (!h || !out) return GGRID_EINVAL;
+  RC(h->sync());
+  ggrid_stats_t s = h->stats;
+  s.cells_flushed = h->h_status->cells_flushed;
+  s.records_flushed = h->h_status->records_flushed;
+  s.objects_written = h->h_status->objects_written;
+  s.arena_used = h->h_status->arena_top;
+  s.arena_capacity = h->s.ar.cap;
+  s.n_cells = h->n_cells;
+  s.cell_size = h->cs;
+  s.delta = h->delta;
+  s.n_vertices = h->V;
+  s.n_arcs = h->A;
+  s.max_objects = h->max_objects;
+  *out = s;
+  return GGRID_OK;
+}
+
+int ggrid_stats_reset(ggrid_t h) {
+  if (!h) return GGRID_EINVAL;
+  RC(h->sync());
+  h->stats.launches = 0;
+  for (int i = 0; i < GGRID_NK; ++i) {
+    h->stats.kernel_launches[i] = 0;
+    h->stats.kernel_ms[i] = 0.0;
+  }
+  return GGRID_OK;
+}
+
+int ggrid_vertex_cell(ggrid_t h, uint32_t* cell_of_vertex) {
+  if (!h || !cell_of_vertex) return GGRID_EINVAL;
+  memcpy(cell_of_vertex, h->user_cell.data(), (size_t)h->V * 4);
+  return GGRID_OK;
+}
+
+}  // extern "C"

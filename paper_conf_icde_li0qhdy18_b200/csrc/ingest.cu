@@ -1,0 +1,202 @@
+// ingest.cu — caching location-update messages (Alg. 1, P@18177-19248) on the device.
+//
+// The paper appends each message to the bucket list of cell getCell(m.e) on the CPU,
+// appends a tombstone to the old cell and overwrites the object table (Alg. 1).  Here a
+// batch of n updates becomes, in three launches:
+//   classify : validate, find cell(src(e)) via the inverted index (P@15006), warp-
+//              aggregated rank within the cell (one atomic per distinct cell per warp);
+//   alloc    : one thread per cell carves this batch's extent for the cell out of the
+//              bump arena (warp-aggregated) and links it at the head of the cell's chain;
+//   scatter  : writes the SoA record and RED.MAX-es (t<<32|seq) into ot_key[o].
+// No tombstones: a record is valid iff its key equals ot_key[obj] (reading R8/R9), which
+// also makes out-of-order arrivals harmless.
+#include "internal.cuh"
+
+namespace gg {
+
+__global__ void __launch_bounds__(256) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
+                                                         DevGraph g, DevState s,
+                                                         uint2* __restrict__ tmp) {
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint4 m = upd[i];
+  unsigned bad = 0;
+  uint2 e = make_uint2(0, 1);
+  if (m.x >= s.max_objects) bad |= ERR_OBJ;
+  if (m.y >= g.A) {
+    bad |= ERR_EDGE;
+  } else {
+    e = g.einfo[m.y];
+    if (m.z >= e.y) bad |= ERR_OFF;
+  }
+  if (bad) {
+    atomicOr(&s.st->err, bad);
+    atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
+    return;
+  }
+  uint32_t c = cell_of(e.x, g.cs);
+  unsigned act = __activemask();
+  unsigned grp = __match_any_sync(act, c);
+  int leader = __ffs(grp) - 1;
+  unsigned base = 0;
+  if ((int)(threadIdx.x & 31) == leader) base = atomicAdd(&s.bcount[c], (unsigned)__popc(grp));
+  base = __shfl_sync(grp, base, leader);
+  tmp[i] = make_uint2(e.x, base + __popc(grp & lanemask_lt()));
+}
+
+__global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
+  uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
+  const bool err = s.st->err != 0;
+  uint32_t cnt = (c < g.n_cells) ? s.bcount[c] : 0;
+  if (err) {
+    if (c < g.n_cells && cnt) s.bcount[c] = 0;
+    return;
+  }
+  unsigned lane = threadIdx.x & 31;
+  // extents start on 4-record boundaries so the flush can use 128-bit loads
+  uint32_t alloc = (cnt + 3u) & ~3u;
+  uint32_t incl = alloc;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= (unsigned)o) incl += y;
+  }
+  uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  unsigned nonempty = __ballot_sync(0xffffffffu, cnt > 0);
+  if (nonempty == 0) return;
+  unsigned long long base = 0;
+  unsigned ebase = 0;
+  if (lane == 0) {
+    base = atomicAdd(&s.st->arena_top, (unsigned long long)total);
+    ebase = atomicAdd(&s.st->ext_top, (unsigned)__popc(nonempty));
+  }
+  base = __shfl_sync(0xffffffffu, base, 0);
+  ebase = __shfl_sync(0xffffffffu, ebase, 0);
+  if (cnt == 0) return;
+  unsigned long long start = base + (incl - alloc);
+  unsigned e = ebase + __popc(nonempty & lanemask_lt());
+  if (start + alloc > s.ar.cap || e >= s.ext_cap) {  // host pre-checks make this unreachable
+    atomicOr(&s.st->err, (unsigned)ERR_ARENA);
+    return;
+  }
+  s.x_start[e] = (uint32_t)start;
+  s.x_len[e] = cnt;
+  s.x_next[e] = s.cell_head[c];
+  s.cell_head[c] = e;
+  s.cell_pending[c] += cnt;
+  s.bbase[c] = (uint32_t)start;
+  s.bcount[c] = 0;
+}
+
+__global__ void __launch_bounds__(256) k_ingest_scatter(const uint4* __restrict__ upd, uint64_t n,
+                                                        uint32_t seq0, DevGraph g, DevState s,
+                                                        const uint2* __restrict__ tmp) {
+  if (s.st->err) return;
+  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint4 m = upd[i];
+  uint2 vr = tmp[i];
+  uint32_t pos = s.bbase[cell_of(vr.x, g.cs)] + vr.y;
+  unsigned long long key = ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
+  s.ar.obj[pos] = m.x;
+  s.ar.key[pos] = key;
+  s.ar.vsrc[pos] = vr.x;
+  s.ar.off[pos] = m.z;
+  s.ar.edge[pos] = m.y;
+  unsigned long long old = atomicMax(&s.ot_key[m.x], key);
+  if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+}
+
+void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
+                            uint2* tmp, cudaStream_t st) {
+  unsigned blocks = (unsigned)((n + 255) / 256);
+  k_ingest_classify<<<blocks, 256, 0, st>>>(upd, n, g, s, tmp);
+}
+void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st) {
+  k_ingest_alloc<<<(g.n_cells + 255) / 256, 256, 0, st>>>(g, s);
+}
+void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
+                           const DevState& s, const uint2* tmp, cudaStream_t st) {
+  unsigned blocks = (unsigned)((n + 255) / 256);
+  k_ingest_scatter<<<blocks, 256, 0, st>>>(upd, n, seq0, g, s, tmp);
+}
+
+// ---------------------------------------------------------------------------------------
+// Alg. 4 line 1 (P@45660): c_q = getCell(q.e) and getNeighbors({c_q}) are cleaned first.
+__global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint32_t nq, DevGraph g,
+                                              DevState s, uint32_t epoch, int neighbors) {
+  uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nq) return;
+  uint2 qq = q[i];
+  if (qq.x >= g.A) {
+    atomicOr(&s.st->err, (unsigned)ERR_QUERY);
+    return;
+  }
+  uint2 e = g.einfo[qq.x];
+  if (qq.y >= e.y) {
+    atomicOr(&s.st->err, (unsigned)ERR_QUERY);
+    return;
+  }
+  uint32_t c = cell_of(e.x, g.cs);
+  request_flush(s, c, epoch);
+  if (neighbors) {
+    for (uint32_t j = g.cadj_ptr[c]; j < g.cadj_ptr[c + 1]; ++j) request_flush(s, g.cadj[j], epoch);
+  } else {
+    request_flush(s, cell_of(g.edst[qq.x], g.cs), epoch);
+  }
+}
+
+void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s, uint32_t epoch,
+                 int neighbors, cudaStream_t st) {
+  if (nq == 0) return;
+  k_seed<<<(nq + 255) / 256, 256, 0, st>>>(q, nq, g, s, epoch, neighbors);
+}
+
+// Every dirty cell (eager cleaning; all_cells additionally queues clean cells for GC).
+__global__ void __launch_bounds__(256) k_mark_dirty(DevGraph g, DevState s, uint32_t epoch,
+                                                    int all_cells) {
+  uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= g.n_cells) return;
+  bool want = all_cells ? true : (s.cell_head[c] != NONE);
+  if (!want) return;
+  unsigned act = __activemask();
+  int leader = __ffs(act) - 1;
+  unsigned base = 0;
+  if ((int)(threadIdx.x & 31) == leader) base = atomicAdd(&s.st->n_flush, (unsigned)__popc(act));
+  base = __shfl_sync(act, base, leader);
+  s.flush_list[base + __popc(act & lanemask_lt())] = c;
+  s.cell_req[c] = epoch;
+}
+
+void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int all_cells,
+                       cudaStream_t st) {
+  k_mark_dirty<<<(g.n_cells + 255) / 256, 256, 0, st>>>(g, s, epoch, all_cells);
+}
+
+// Valid objects of one clean cell (test hook ggrid_cell_objects).
+__global__ void k_dump_cell(DevGraph g, DevState s, uint32_t c, uint32_t* obj, uint32_t* edge,
+                            uint32_t* off, uint32_t cap, uint32_t* n_out) {
+  uint32_t vb = c * g.cs;
+  uint32_t ve = min(g.V, vb + g.cs);
+  for (uint32_t v = vb + threadIdx.x; v < ve; v += blockDim.x) {
+    uint2 vo = s.v_obj[v];
+    for (uint32_t j = 0; j < vo.y; ++j) {
+      uint32_t p = vo.x + j;
+      uint32_t o = s.ar.obj[p];
+      if (s.ar.key[p] != s.ot_key[o]) continue;  // moved away since the cell was cleaned
+      uint32_t i = atomicAdd(n_out, 1u);
+      if (i < cap) {
+        obj[i] = o;
+        edge[i] = s.ar.edge[p];
+        off[i] = s.ar.off[p];
+      }
+    }
+  }
+}
+
+void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t* obj,
+                      uint32_t* edge, uint32_t* off, uint32_t cap, uint32_t* n_out, cudaStream_t st) {
+  k_dump_cell<<<1, 256, 0, st>>>(g, s, c, obj, edge, off, cap, n_out);
+}
+
+}  // namespace gg

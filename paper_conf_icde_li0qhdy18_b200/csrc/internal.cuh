@@ -1,0 +1,136 @@
+// internal.cuh — device-side data layout of the B200 G-Grid.
+//
+// Everything the hot path touches lives in HBM in flat arrays:
+//   graph grid  : CSR over internal (Z-ordered) vertex ids; cells are runs of cell_size
+//                 consecutive internal ids (P@11972-13692, reading R16), so cell(v) = v/cs.
+//   object table: ot_key[o] = max (t<<32 | seq) over o's updates (P@15869, reading R7/R8).
+//   message log : a bump-allocated record arena (SoA: obj, key, vsrc, off, edge) holding
+//                 per-cell append-only extents (one per ingest batch per cell, a chain
+//                 newest-first) = the paper's message lists of buckets (P@16303-17318),
+//                 plus each cell's compacted object list (the cleaned result R[c],
+//                 P@22008-22213) sorted by source vertex, indexed per vertex by v_obj.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "ggrid.h"
+
+namespace gg {
+
+constexpr uint32_t NONE = 0xFFFFFFFFu;
+constexpr uint32_t INF = 0xFFFFFFFFu;  // u32 distance "unreachable" (reading R18)
+constexpr unsigned long long EMPTY64 = ~0ull;
+
+enum ErrBits : unsigned {
+  ERR_OBJ = 1u,      // update obj >= max_objects
+  ERR_EDGE = 2u,     // update/query edge >= n_arcs
+  ERR_OFF = 4u,      // offset >= w[edge]
+  ERR_ARENA = 8u,    // arena / extent pool exhausted on device (should not happen)
+  ERR_QUERY = 16u,   // query edge/offset invalid
+  ERR_FAIL = 32u,    // a query overflowed the largest expansion variant
+};
+
+// Device-resident counters (one struct, read back with one D2H copy at sync points).
+struct DevStatus {
+  unsigned long long arena_top;  // next free record in the arena
+  unsigned long long records_flushed;
+  unsigned long long objects_written;
+  unsigned long long cells_flushed;
+  unsigned int ext_top;     // next free extent
+  unsigned int err;         // ErrBits
+  unsigned int bad_index;   // smallest offending index (ingest)
+  unsigned int n_live;      // objects with at least one update
+  unsigned int n_flush;     // entries in flush_list
+  unsigned int flush_work;  // persistent flush work counter
+  unsigned int n_next[4];   // per expansion level: queries queued for the next round
+  unsigned int flush_end;   // n_flush as seen by the last flush launch
+  unsigned int pad;
+};
+
+struct DevGraph {
+  uint32_t V, A, cs, n_cells, delta;
+  const uint32_t* rowptr;    // [V+1] out-arc CSR by internal source
+  const uint2* adj;          // [A]  (internal dst, w) in CSR order
+  const uint2* einfo;        // [A]  user edge -> (internal src, w)
+  const uint32_t* edst;      // [A]  user edge -> internal dst
+  const uint32_t* cadj_ptr;  // [n_cells+1] cell adjacency (P@47172)
+  const uint32_t* cadj;
+};
+
+struct Arena {  // SoA record arena
+  uint32_t* obj;
+  unsigned long long* key;
+  uint32_t* vsrc;
+  uint32_t* off;
+  uint32_t* edge;
+  unsigned long long cap;
+};
+
+struct DevState {
+  unsigned long long* ot_key;  // [max_objects]
+  uint32_t max_objects;
+  Arena ar;
+  uint32_t* x_start;  // extents
+  uint32_t* x_len;
+  uint32_t* x_next;
+  uint32_t ext_cap;
+  uint32_t* cell_head;     // newest pending extent or NONE (NONE = clean)
+  uint32_t* cell_pending;  // cached records not yet cleaned
+  uint32_t* cell_req;      // request epoch stamp (dedup of flush requests)
+  uint2* v_obj;            // [V] (arena start, count) of the objects at each vertex
+  uint2* cell_comp;        // [n_cells] (arena start, count) of the cell's compacted list
+  uint32_t* vcnt;          // [V] flush scratch, only when cell_size > 4096 (else null)
+  uint32_t* bcount;        // [n_cells] per-batch counts
+  uint32_t* bbase;         // [n_cells] per-batch arena base
+  uint32_t* flush_list;    // [n_cells]
+  DevStatus* st;
+};
+
+__host__ __device__ inline uint32_t cell_of(uint32_t v, uint32_t cs) { return v / cs; }
+
+__device__ inline unsigned lanemask_lt() {
+  unsigned m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// Request a flush of cell c in this knn epoch (deduplicated by the epoch stamp).
+__device__ inline void request_flush(const DevState& s, uint32_t c, uint32_t epoch) {
+  if (s.cell_head[c] == NONE) return;
+  if (atomicExch(&s.cell_req[c], epoch) != epoch) {
+    unsigned i = atomicAdd(&s.st->n_flush, 1u);
+    s.flush_list[i] = c;
+  }
+}
+
+}  // namespace gg
+
+// Launchers (defined in the .cu files; called by api.cu).
+namespace gg {
+void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
+                            uint2* tmp, cudaStream_t st);
+void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);
+void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
+                           const DevState& s, const uint2* tmp, cudaStream_t st);
+void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s, uint32_t epoch,
+                 int neighbors, cudaStream_t st);
+void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int all_cells,
+                       cudaStream_t st);
+// Flush the cells flush_list[begin .. st->n_flush) writing compacted lists into `out`
+// (out == s.ar for a regular flush; a fresh arena for garbage collection).
+void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
+                  unsigned long long* out_top, uint32_t begin, int sm_count, cudaStream_t st);
+int flush_smem_bytes();
+// Expansion (Alg. 5/6 semantics) for the queries qlist[0..n) at variant `level`.
+// Outcomes: answered (rows written), retried at the same level (retry_list, a needed cell
+// had cached updates) or promoted to the next level (promote_list, capacity overflow).
+void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
+                   const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
+                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist, void* scratch,
+                   uint32_t scratch_warps, cudaStream_t st);
+int expand_levels();
+uint32_t expand_max_k(int level);
+size_t expand_warp_bytes(int level, uint32_t V);
+void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t* obj,
+                      uint32_t* edge, uint32_t* off, uint32_t cap, uint32_t* n_out, cudaStream_t st);
+}  // namespace gg

@@ -1,0 +1,501 @@
+// knn.cu — candidate construction and refinement of a kNN query (Alg. 4 lines 5-10,
+// Alg. 5 GPU_SDist, GPU_First_k, Def. 3 GPU_Unresolved, Alg. 6 Refine_kNN;
+// P@47779-52751), one warp per query.
+//
+// The paper runs |V| rounds of Bellman-Ford over the candidate cells with one thread per
+// vertex (Alg. 5, P@48476-50421), picks the k nearest candidates, then refines them on CPU
+// threads with one Dijkstra per unresolved boundary vertex (Alg. 6).  Both are prior art
+// here.  This kernel computes the same exact answer with one bounded, label-correcting
+// delta-stepping expansion per query that never leaves the GPU:
+//
+//   * D lives in a per-warp shared-memory open-addressing table keyed by vertex; one
+//     64-bit word (v<<32 | dist) so relaxation is a single atomicMin (same key => min on
+//     the distance).  Seeds follow reading R1 (d=0 -> D[src]=0, else D[dst]=w-d).
+//   * Each round takes the frontier bucket [m, m+delta) (m = frontier minimum) and relaxes
+//     its out-arcs lane-per-arc (warp-cooperative adjacency scan: a warp scan of the degrees
+//     of 32 active vertices, then each lane binary-searches its arc).
+//   * Every vertex with D < m is final; its objects are harvested from the cell's cleaned
+//     list (v_obj index) as exact candidates dist = D[src(e_o)] + d_o (P@49436), objects on
+//     q's own arc ahead of q at d_o - d_q (reading R2), stale entries dropped by
+//     key == ot_key.  Harvesting a vertex of a cell with cached updates requests that cell's
+//     flush and the query is retried next round (lazy cleaning, Alg. 4 lines 2-4).
+//   * Stop once k candidates have dist < m (every unharvested object is >= m): this is
+//     Def. 3's unresolved-vertex rule taken inclusively (reading R13) and Alg. 6's refinement
+//     fused into the same expansion.  Output: k smallest (dist<<32 | obj) (readings R5, R6).
+// Capacities are per variant ("level"); a query that overflows one is retried on the next.
+#include <algorithm>
+
+#include "internal.cuh"
+
+namespace gg {
+
+namespace {
+
+enum { DONE = 0, RETRY = 1, OVERFLOW = 2 };
+constexpr int MAXP = 128;  // probe limit of the vertex table
+
+struct Caps {
+  uint32_t H, F, X, C;  // table slots (pow2), frontier, expanded list, candidates
+};
+
+// byte layout of one warp's working memory
+struct WarpMem {
+  unsigned long long* dtab;  // H
+  unsigned long long* cand;  // C
+  uint32_t* front0;          // F
+  uint32_t* front1;          // F
+  uint32_t* act;             // F
+  uint32_t* exl;             // X
+  uint32_t* fin;             // H/32
+  uint32_t* listed;          // H/32
+  uint32_t* scan;            // 32
+  uint32_t* rp;              // 32
+  uint32_t* du;              // 32
+};
+
+__host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
+  return 8ull * c.H + 8ull * c.C + 4ull * (3ull * c.F + c.X + 2ull * (c.H / 32) + 96);
+}
+
+__device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
+  WarpMem m;
+  m.dtab = reinterpret_cast<unsigned long long*>(base);
+  m.cand = m.dtab + c.H;
+  uint32_t* p = reinterpret_cast<uint32_t*>(m.cand + c.C);
+  m.front0 = p; p += c.F;
+  m.front1 = p; p += c.F;
+  m.act = p; p += c.F;
+  m.exl = p; p += c.X;
+  m.fin = p; p += c.H / 32;
+  m.listed = p; p += c.H / 32;
+  m.scan = p; p += 32;
+  m.rp = p; p += 32;
+  m.du = p;
+  return m;
+}
+
+__device__ __forceinline__ uint32_t vhash(uint32_t v) {
+  uint32_t h = v * 2654435761u;
+  return h ^ (h >> 15);
+}
+
+// insert-or-min of (v, d); returns the slot (or -1 if the table is full)
+__device__ __forceinline__ int tab_relax(unsigned long long* dtab, uint32_t hmask, uint32_t v,
+                                         uint32_t d, bool& improved) {
+  const unsigned long long nv = ((unsigned long long)v << 32) | d;
+  const uint32_t h = vhash(v);
+  volatile unsigned long long* vt = dtab;
+#pragma unroll 1
+  for (int p = 0; p < MAXP; ++p) {
+    const uint32_t sl = (h + p) & hmask;
+    unsigned long long cur = vt[sl];
+    if (cur == EMPTY64) {
+      const unsigned long long old = atomicCAS(&dtab[sl], EMPTY64, nv);
+      if (old == EMPTY64) {
+        improved = true;
+        return (int)sl;
+      }
+      cur = old;
+    }
+    if ((uint32_t)(cur >> 32) == v) {
+      const unsigned long long old = atomicMin(&dtab[sl], nv);
+      improved = (uint32_t)old > d;
+      return (int)sl;
+    }
+  }
+  improved = false;
+  return -1;
+}
+
+// warp bitonic sort of cand[0..n) ascending (n padded to a power of two <= cap)
+__device__ void warp_sort(unsigned long long* a, uint32_t n, uint32_t cap, int lane) {
+  uint32_t n2 = 1;
+  while (n2 < n) n2 <<= 1;
+  if (n2 > cap) n2 = cap;  // n <= cap always
+  for (uint32_t i = n + lane; i < n2; i += 32) a[i] = EMPTY64;
+  __syncwarp();
+  for (uint32_t size = 2; size <= n2; size <<= 1) {
+    for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+      for (uint32_t i = lane; i < n2 / 2; i += 32) {
+        const uint32_t lo = 2 * i - (i & (stride - 1));
+        const uint32_t hi = lo + stride;
+        const bool asc = (lo & size) == 0;
+        const unsigned long long x = a[lo], y = a[hi];
+        if ((x > y) == asc) {
+          a[lo] = y;
+          a[hi] = x;
+        }
+      }
+      __syncwarp();
+    }
+  }
+}
+
+struct QParams {
+  DevGraph g;
+  DevState s;
+  const uint2* q;
+  const uint32_t* qlist;
+  uint32_t n;
+  uint32_t k;
+  uint32_t epoch;
+  int level;
+  int last_level;
+  uint32_t* retry_list;     // same level, next round
+  uint32_t* promote_list;   // next level, next round
+  uint32_t* out_obj;
+  uint32_t* out_dist;
+  Caps caps;
+  unsigned char* scratch;   // global working memory (level 2) or null (shared)
+  uint32_t warps_per_cta;
+};
+
+// Ask for the flush of every dirty cell the frontier / pending harvest will need, so a
+// retried query is unlikely to stop again for the same reason.
+__device__ void request_lookahead(const QParams& P, const WarpMem& m, const uint32_t* front,
+                                  uint32_t nf, uint32_t nx, int lane) {
+  for (uint32_t i = lane; i < nf; i += 32) {
+    const uint32_t v = (uint32_t)(m.dtab[front[i]] >> 32);
+    request_flush(P.s, cell_of(v, P.g.cs), P.epoch);
+  }
+  for (uint32_t i = lane; i < nx; i += 32) {
+    const uint32_t v = (uint32_t)(m.dtab[m.exl[i]] >> 32);
+    request_flush(P.s, cell_of(v, P.g.cs), P.epoch);
+  }
+}
+
+__device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int lane) {
+  const unsigned FULL = 0xffffffffu;
+  const DevGraph& g = P.g;
+  const DevState& s = P.s;
+  const Caps& cp = P.caps;
+  const uint32_t hmask = cp.H - 1;
+  const uint32_t k = P.k;
+  const unsigned lt = lanemask_lt();
+
+  for (uint32_t i = lane; i < cp.H; i += 32) m.dtab[i] = EMPTY64;
+  for (uint32_t i = lane; i < cp.H / 32; i += 32) {
+    m.fin[i] = 0;
+    m.listed[i] = 0;
+  }
+  __syncwarp();
+
+  const uint2 q = P.q[qi];
+  if (q.x >= g.A) return DONE;   // invalid query: reported by the seed kernel (EINVAL)
+  const uint2 ei = g.einfo[q.x];  // (internal src, w)
+  if (q.y >= ei.y) return DONE;
+  uint32_t seed_v, seed_d;
+  if (q.y == 0) {
+    seed_v = ei.x;
+    seed_d = 0;
+  } else {
+    seed_v = g.edst[q.x];
+    seed_d = ei.y - q.y;
+  }
+  uint32_t* front = m.front0;
+  uint32_t* nfront = m.front1;
+  uint32_t nf = 1, nx = 0, nc = 0;
+  if (lane == 0) {
+    bool imp;
+    const int sl = tab_relax(m.dtab, hmask, seed_v, seed_d, imp);
+    front[0] = (uint32_t)sl;
+    m.fin[sl >> 5] |= 1u << (sl & 31);
+  }
+  __syncwarp();
+
+  // objects on q's own arc ahead of q (reading R2); they are stored at vertex src(q.e)
+  if (q.y > 0) {
+    const uint32_t c = cell_of(ei.x, g.cs);
+    if (s.cell_head[c] != NONE) {
+      if (lane == 0) request_flush(s, c, P.epoch);
+      return RETRY;
+    }
+    const uint2 vo = s.v_obj[ei.x];
+    for (uint32_t j0 = 0; j0 < vo.y; j0 += 32) {
+      const uint32_t j = j0 + lane;
+      bool has = false;
+      unsigned long long dk = 0;
+      if (j < vo.y) {
+        const uint32_t p = vo.x + j;
+        const uint32_t ob = s.ar.obj[p];
+        const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
+        if (oe == q.x && oo >= q.y && s.ar.key[p] == s.ot_key[ob]) {
+          has = true;
+          dk = ((unsigned long long)(oo - q.y) << 32) | ob;
+        }
+      }
+      const unsigned hm = __ballot_sync(FULL, has);
+      if (nc + __popc(hm) > cp.C) return OVERFLOW;
+      if (has) m.cand[nc + __popc(hm & lt)] = dk;
+      nc += __popc(hm);
+    }
+    __syncwarp();
+  }
+
+  for (;;) {
+    // ---- 1. frontier minimum: every vertex with D < m is final -------------------------
+    uint32_t ml = INF;
+    for (uint32_t i = lane; i < nf; i += 32) ml = min(ml, (uint32_t)m.dtab[front[i]]);
+    const uint32_t mn = __reduce_min_sync(FULL, ml);
+    const uint32_t blo = nf ? mn : INF;
+
+    // ---- 2. harvest the objects of the newly final vertices -----------------------------
+    uint32_t keep = 0;
+    for (uint32_t b0 = 0; b0 < nx; b0 += 32) {
+      const uint32_t i = b0 + lane;
+      const uint32_t sl = i < nx ? m.exl[i] : NONE;
+      const unsigned long long ent = sl != NONE ? m.dtab[sl] : EMPTY64;
+      const uint32_t d = (uint32_t)ent, u = (uint32_t)(ent >> 32);
+      const bool take = sl != NONE && (nf == 0 || d < blo);
+      const bool stay = sl != NONE && !take;
+      const unsigned smk = __ballot_sync(FULL, stay);
+      __syncwarp();
+      if (stay) m.exl[keep + __popc(smk & lt)] = sl;
+      keep += __popc(smk);
+      uint2 vo = make_uint2(0, 0);
+      bool dirty = false;
+      if (take) {
+        const uint32_t c = cell_of(u, g.cs);
+        if (s.cell_head[c] != NONE) {
+          dirty = true;
+          request_flush(s, c, P.epoch);
+        } else {
+          vo = s.v_obj[u];
+        }
+      }
+      if (__any_sync(FULL, dirty)) {
+        request_lookahead(P, m, front, nf, 0, lane);
+        return RETRY;
+      }
+      for (uint32_t j = 0; __any_sync(FULL, j < vo.y); ++j) {
+        bool has = false;
+        unsigned long long dk = 0;
+        if (j < vo.y) {
+          const uint32_t p = vo.x + j;
+          const uint32_t ob = s.ar.obj[p];
+          const unsigned long long kk = s.ar.key[p];
+          const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
+          const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
+          if (!same_ahead && kk == s.ot_key[ob]) {
+            const unsigned long long dd = (unsigned long long)d + oo;
+            if (dd < INF) {
+              has = true;
+              dk = (dd << 32) | ob;
+            }
+          }
+        }
+        const unsigned hm = __ballot_sync(FULL, has);
+        if (nc + __popc(hm) > cp.C) {
+          // keep only the k best so far: a dropped candidate has >= k better ones
+          warp_sort(m.cand, nc, cp.C, lane);
+          nc = min(nc, k);
+          if (nc + __popc(hm) > cp.C) return OVERFLOW;
+        }
+        if (has) m.cand[nc + __popc(hm & lt)] = dk;
+        nc += __popc(hm);
+      }
+    }
+    nx = keep;
+    __syncwarp();
+
+    // ---- 3. termination: k candidates strictly closer than any unharvested object -------
+    if (nf == 0) break;
+    uint32_t cl = 0;
+    for (uint32_t i = lane; i < nc; i += 32) cl += (uint32_t)(m.cand[i] >> 32) < blo;
+    if (__reduce_add_sync(FULL, cl) >= k) break;
+
+    // ---- 4. activate the bucket [m, m + delta) -------------------------------------------
+    const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
+    uint32_t na = 0, nn = 0;
+    for (uint32_t b0 = 0; b0 < nf; b0 += 32) {
+      const uint32_t i = b0 + lane;
+      const uint32_t sl = i < nf ? front[i] : NONE;
+      const bool a = sl != NONE && (uint32_t)m.dtab[sl] < bhi;
+      const bool r = sl != NONE && !a;
+      const unsigned am = __ballot_sync(FULL, a), rm = __ballot_sync(FULL, r);
+      bool newl = false;
+      if (a) {
+        m.act[na + __popc(am & lt)] = sl;
+        atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
+        const uint32_t bit = 1u << (sl & 31);
+        newl = !(atomicOr(&m.listed[sl >> 5], bit) & bit);
+      }
+      if (r) nfront[nn + __popc(rm & lt)] = sl;
+      na += __popc(am);
+      nn += __popc(rm);
+      const unsigned lm = __ballot_sync(FULL, newl);
+      if (nx + __popc(lm) > cp.X) return OVERFLOW;
+      if (newl) m.exl[nx + __popc(lm & lt)] = sl;
+      nx += __popc(lm);
+    }
+    __syncwarp();
+
+    // ---- 5. relax the active vertices' out-arcs, lane per arc ----------------------------
+    for (uint32_t b0 = 0; b0 < na; b0 += 32) {
+      const uint32_t i = b0 + lane;
+      uint32_t rp0 = 0, deg = 0, du = INF;
+      if (i < na) {
+        const unsigned long long ent = m.dtab[m.act[i]];
+        const uint32_t u = (uint32_t)(ent >> 32);
+        du = (uint32_t)ent;
+        rp0 = g.rowptr[u];
+        deg = g.rowptr[u + 1] - rp0;
+      }
+      uint32_t x = deg;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += y;
+      }
+      const uint32_t total = __shfl_sync(FULL, x, 31);
+      m.scan[lane] = x;
+      m.rp[lane] = rp0;
+      m.du[lane] = du;
+      __syncwarp();
+      for (uint32_t t0 = 0; t0 < total; t0 += 32) {
+        const uint32_t t = t0 + lane;
+        bool has = false, ovf = false;
+        uint32_t slot = 0;
+        if (t < total) {
+          int lo = 0, hi = 31;
+          while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (m.scan[mid] > t) hi = mid; else lo = mid + 1;
+          }
+          const uint32_t excl = lo ? m.scan[lo - 1] : 0;
+          const uint2 a = g.adj[m.rp[lo] + (t - excl)];
+          const unsigned long long nd = (unsigned long long)m.du[lo] + a.y;
+          if (nd < INF) {
+            bool imp;
+            const int r = tab_relax(m.dtab, hmask, a.x, (uint32_t)nd, imp);
+            if (r < 0) {
+              ovf = true;
+            } else if (imp) {
+              const uint32_t bit = 1u << (r & 31);
+              if (!(atomicOr(&m.fin[r >> 5], bit) & bit)) {
+                has = true;
+                slot = (uint32_t)r;
+              }
+            }
+          }
+        }
+        if (__any_sync(FULL, ovf)) return OVERFLOW;
+        const unsigned hm = __ballot_sync(FULL, has);
+        if (nn + __popc(hm) > cp.F) return OVERFLOW;
+        if (has) nfront[nn + __popc(hm & lt)] = slot;
+        nn += __popc(hm);
+      }
+      __syncwarp();
+    }
+    uint32_t* tmp = front;
+    front = nfront;
+    nfront = tmp;
+    nf = nn;
+    __syncwarp();
+  }
+
+  // ---- 6. the k smallest (dist, obj) ------------------------------------------------------
+  warp_sort(m.cand, nc, cp.C, lane);
+  for (uint32_t r = lane; r < k; r += 32) {
+    const bool ok = r < nc;
+    const unsigned long long dk = ok ? m.cand[r] : EMPTY64;
+    P.out_obj[(size_t)qi * k + r] = ok ? (uint32_t)dk : GGRID_PAD;
+    P.out_dist[(size_t)qi * k + r] = ok ? (uint32_t)(dk >> 32) : GGRID_PAD;
+  }
+  return DONE;
+}
+
+__global__ void k_expand(QParams P) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const int lane = threadIdx.x & 31;
+  const uint32_t warp = threadIdx.x >> 5;
+  const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
+  const uint32_t gw = blockIdx.x * P.warps_per_cta + warp;
+  const uint32_t nwarps = gridDim.x * P.warps_per_cta;
+  unsigned char* base = P.scratch ? P.scratch + (size_t)gw * wbytes : smem_raw + (size_t)warp * wbytes;
+  const WarpMem m = carve(base, P.caps);
+  for (uint32_t li = gw; li < P.n; li += nwarps) {
+    const uint32_t qi = P.qlist ? P.qlist[li] : li;
+    const int r = run_query(P, m, qi, lane);
+    if (lane == 0 && r != DONE) {
+      if (r == RETRY) {
+        P.retry_list[atomicAdd(&P.s.st->n_next[P.level], 1u)] = qi;
+      } else if (P.level < P.last_level) {
+        P.promote_list[atomicAdd(&P.s.st->n_next[P.level + 1], 1u)] = qi;
+      } else {
+        atomicOr(&P.s.st->err, (unsigned)ERR_FAIL);
+      }
+    }
+    __syncwarp();
+  }
+}
+
+// level 0: small balls (k <= 128), 4 warps per CTA in shared memory
+// level 1: large balls, 1 warp per CTA in shared memory
+// level 2: global-memory working set sized from |V| (fewer than k reachable objects, ...)
+constexpr int NLEVELS = 3;
+const Caps kCaps0 = {1024, 256, 256, 256};
+const Caps kCaps1 = {8192, 2048, 2048, 1024};
+constexpr uint32_t kWarps0 = 4, kWarps1 = 1, kWarps2 = 1;
+
+Caps caps_for(int level, uint32_t V) {
+  if (level == 0) return kCaps0;
+  if (level == 1) return kCaps1;
+  uint32_t H = 1u << 14;
+  while (H < 2ull * V && H < (1u << 27)) H <<= 1;
+  const uint32_t F = std::min<uint32_t>(H / 2, 1u << 22);
+  return Caps{H, F, F, 8192};
+}
+
+bool g_attr_set[NLEVELS] = {false, false, false};
+}  // namespace
+
+int expand_levels() { return NLEVELS; }
+
+uint32_t expand_max_k(int level) { return level == 0 ? 128 : (level == 1 ? 512 : 4096); }
+
+size_t expand_warp_bytes(int level, uint32_t V) {
+  const Caps c = caps_for(level, V);
+  return (warpmem_bytes(c) + 15) & ~size_t(15);
+}
+
+void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
+                   const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
+                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist, void* scratch,
+                   uint32_t scratch_warps, cudaStream_t st) {
+  if (n == 0) return;
+  QParams P;
+  P.g = g;
+  P.s = s;
+  P.q = q;
+  P.qlist = qlist;
+  P.n = n;
+  P.k = k;
+  P.epoch = epoch;
+  P.level = level;
+  P.last_level = NLEVELS - 1;
+  P.retry_list = retry_list;
+  P.promote_list = promote_list;
+  P.out_obj = out_obj;
+  P.out_dist = out_dist;
+  P.caps = caps_for(level, g.V);
+  const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
+  if (level < 2) {
+    P.scratch = nullptr;
+    P.warps_per_cta = level == 0 ? kWarps0 : kWarps1;
+    const int smem = (int)(wbytes * P.warps_per_cta);
+    if (!g_attr_set[level]) {
+      cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+      g_attr_set[level] = true;
+    }
+    const uint32_t blocks = (n + P.warps_per_cta - 1) / P.warps_per_cta;
+    k_expand<<<blocks, 32 * P.warps_per_cta, smem, st>>>(P);
+  } else {
+    P.scratch = static_cast<unsigned char*>(scratch);
+    P.warps_per_cta = kWarps2;
+    const uint32_t blocks = std::min<uint32_t>((n + kWarps2 - 1) / kWarps2, std::max<uint32_t>(1, scratch_warps / kWarps2));
+    k_expand<<<blocks, 32 * kWarps2, 0, st>>>(P);
+  }
+}
+
+}  // namespace gg

@@ -1,0 +1,282 @@
+"""Parity of the CUDA path (through the C ABI) against the CPU oracle (-m gpu).
+
+The bar (north_star): integer work, so bit-exact — identical object ids AND
+distances per query, ties broken by id, padding identical.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def gg():
+    import torch
+
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icde_li0qhdy18_b200 import build
+
+    build.build()
+    import paper_conf_icde_li0qhdy18_b200 as m
+
+    return m
+
+
+def _oracle(g, upd, q, k, mode=oracle.FULL):
+    return oracle.knn_from_updates(g, upd, q, k, mode=mode)
+
+
+def _assert_same(got, ref, msg=""):
+    go, gd = got
+    ro, rd = ref
+    if not (np.array_equal(go, ro) and np.array_equal(gd, rd)):
+        bad = np.flatnonzero(~((go == ro).all(1) & (gd == rd).all(1)))
+        i = int(bad[0])
+        raise AssertionError(f"{msg}: {len(bad)} rows differ; first row {i}: got {list(zip(gd[i], go[i]))} "
+                             f"ref {list(zip(rd[i], ro[i]))}")
+
+
+# ---------------------------------------------------------------------------------- C0
+@pytest.mark.parametrize("cell_size", [1, 16, 64, 1024])
+def test_c0_knn_bit_exact(gg, cell_size):
+    """BASELINE configs[0]: 32x32 lattice, w in {1..4} (ties), 100 objects, 1k cached updates
+    with late / duplicate timestamps, 100 queries; every cell_size gives the oracle's answer
+    (partition independence)."""
+    g = synth.lattice_graph(32, 32, 1, 4)
+    upd = synth.RandomWalk(g, 100, inject=True).ticks(10)
+    q = synth.queries(g, 100)
+    grid = gg.GGrid(g, cell_size, max_objects=128)
+    grid.ingest(upd)
+    for k in (1, 3, 10, 100, 130):
+        _assert_same(grid.knn(q, k), _oracle(g, upd, q, k), f"cs={cell_size} k={k}")
+    grid.close()
+
+
+def test_c0_interleaved_rounds_lazy_equals_eager(gg):
+    """Interleaved ingest / query rounds; a lazy handle and an eager one (flush_all after
+    every ingest) agree with the oracle's snapshot at every round."""
+    g = synth.lattice_graph(32, 32, 1, 4)
+    walk = synth.RandomWalk(g, 100, inject=True)
+    lazy = gg.GGrid(g, 16, max_objects=128)
+    eager = gg.GGrid(g, 16, max_objects=128)
+    hist = []
+    for r in range(8):
+        u = walk.ticks(3)
+        hist.append(u)
+        lazy.ingest(u)
+        eager.ingest(u)
+        eager.flush_all()
+        allu = np.concatenate(hist)
+        q = synth.queries(g, 64, seed=100 + r)
+        ref = _oracle(g, allu, q, 5)
+        _assert_same(lazy.knn(q, 5), ref, f"lazy round {r}")
+        _assert_same(eager.knn(q, 5), ref, f"eager round {r}")
+    lazy.close()
+    eager.close()
+
+
+def test_flush_parity_and_cells(gg):
+    """After ggrid_flush_all the cells' object lists are exactly the oracle's latest-per-object
+    snapshot, each object once, in the cell of its arc's source vertex; flushing twice is a
+    no-op (idempotent)."""
+    g = synth.table_ii_graph("NY", scale=0.05)
+    upd = synth.RandomWalk(g, 2000, inject=True).ticks(12)
+    grid = gg.GGrid(g, 256, max_objects=4096)
+    for part in np.array_split(upd, 5):
+        grid.ingest(part)
+    grid.flush_all()
+    vcell = grid.vertex_cell()
+    n_cells = grid.stats()["n_cells"]
+
+    def dump():
+        rows = []
+        for c in range(n_cells):
+            o, e, d = grid.cell_objects(c)
+            assert np.all(vcell[g["src"][e]] == c)
+            rows += list(zip(o.tolist(), e.tolist(), d.tolist()))
+        return sorted(rows)
+
+    got = dump()
+    ids, e, d = oracle.snapshot_objects(upd)
+    assert got == sorted(zip(ids.tolist(), e.tolist(), d.tolist()))
+    grid.flush_all()
+    assert dump() == got
+    grid.close()
+
+
+def test_batch_independence_and_pointer_kinds(gg):
+    import torch
+
+    g = synth.table_ii_graph("NY", scale=0.05)
+    upd = synth.RandomWalk(g, 1000).ticks(5)
+    q = synth.queries(g, 200)
+    k = 7
+    ref = _oracle(g, upd, q, k)
+    grid = gg.GGrid(g, 256, max_objects=1024)
+    grid.ingest(torch.from_numpy(upd.view(np.int32)).cuda())  # device input
+    one = [grid.knn(q[i:i + 1], k) for i in range(0, 40)]
+    _assert_same((np.concatenate([a for a, _ in one]), np.concatenate([b for _, b in one])),
+                 (ref[0][:40], ref[1][:40]), "Q=1 calls")
+    qo = torch.empty((len(q), k), dtype=torch.int32, device="cuda")
+    qd = torch.empty((len(q), k), dtype=torch.int32, device="cuda")
+    grid.knn(torch.from_numpy(q.view(np.int32)).cuda(), k, qo, qd)  # device in / out
+    _assert_same((qo.cpu().numpy().view(np.uint32), qd.cpu().numpy().view(np.uint32)), ref, "device io")
+    po = torch.empty((len(q), k), dtype=torch.int32).pin_memory()
+    pd = torch.empty((len(q), k), dtype=torch.int32).pin_memory()
+    grid.knn(torch.from_numpy(q.view(np.int32)).pin_memory(), k, po, pd)  # pinned host
+    _assert_same((po.numpy().view(np.uint32), pd.numpy().view(np.uint32)), ref, "pinned io")
+    grid.close()
+
+
+# ----------------------------------------------------------------- tiny graphs / edge cases
+@pytest.mark.parametrize("seed", range(40))
+def test_random_digraphs(gg, seed):
+    """Random directed multigraphs with self-loops, unreachable parts and ties."""
+    rng = np.random.default_rng(500 + seed)
+    V = int(rng.integers(2, 40))
+    A = int(rng.integers(1, 4 * V))
+    g = dict(n_vertices=V, src=rng.integers(0, V, A).astype(np.uint32),
+             dst=rng.integers(0, V, A).astype(np.uint32), w=rng.integers(1, 6, A).astype(np.uint32))
+    n_obj = int(rng.integers(1, 30))
+    n_upd = int(rng.integers(1, 200))
+    upd = np.zeros((n_upd, 4), np.uint32)
+    upd[:, 0] = rng.integers(0, n_obj, n_upd)
+    upd[:, 1] = rng.integers(0, A, n_upd)
+    upd[:, 2] = (rng.random(n_upd) * g["w"][upd[:, 1]]).astype(np.uint32)
+    upd[:, 3] = rng.integers(0, 20, n_upd)
+    q = np.zeros((30, 2), np.uint32)
+    q[:, 0] = rng.integers(0, A, 30)
+    q[:, 1] = (rng.random(30) * g["w"][q[:, 0]]).astype(np.uint32)
+    for cs in (1, 3, V):
+        grid = gg.GGrid(g, cs, max_objects=64, delta=int(rng.integers(1, 8)))
+        for part in np.array_split(upd, 3):
+            if len(part):
+                grid.ingest(part)
+        for k in (1, 4, 40):
+            _assert_same(grid.knn(q, k), _oracle(g, upd, q, k), f"seed={seed} cs={cs} k={k}")
+        grid.close()
+
+
+def test_fig1_fixture_through_library(gg):
+    d, g = synth.fig1_fixture()
+    W = d["lattice"]["width"]
+
+    def arc(a, b):
+        return int(np.flatnonzero((g["src"] == a[1] * W + a[0]) & (g["dst"] == b[1] * W + b[0]))[0])
+
+    upd = np.array([[o["id"], arc(o["from"], o["to"]), o["offset"], 0] for o in d["objects"]], np.uint32)
+    q = np.array([[arc(d["query"]["from"], d["query"]["to"]), d["query"]["offset"]]], np.uint32)
+    grid = gg.GGrid(g, 8, max_objects=16)
+    grid.ingest(upd)
+    o, _ = grid.knn(q, 3)
+    assert o[0].tolist() == d["paper_answer"]  # <o5, o2, o4>
+    o, dist = grid.knn(q, 9)
+    assert [[int(a), int(b)] for a, b in zip(o[0], dist[0])] == d["hand_order"]
+    grid.close()
+
+
+def test_u32_distance_range(gg):
+    big = 1 << 31
+    g = dict(n_vertices=3, src=np.array([0, 1], np.uint32), dst=np.array([1, 2], np.uint32),
+             w=np.array([big, big], np.uint32))
+    upd = np.array([[1, 1, big - 2, 0], [2, 1, big - 1, 0], [3, 0, 5, 0]], np.uint32)
+    grid = gg.GGrid(g, 2, max_objects=8)
+    grid.ingest(upd)
+    o, d = grid.knn(np.array([[0, 0]], np.uint32), 3)
+    assert o.tolist() == [[3, 1, gg.PAD]] and d.tolist() == [[5, (1 << 32) - 2, gg.PAD]]
+    grid.close()
+
+
+def test_delta_independence(gg):
+    g = synth.table_ii_graph("NY", scale=0.03)
+    upd = synth.RandomWalk(g, 500, inject=True).ticks(4)
+    q = synth.queries(g, 100)
+    ref = _oracle(g, upd, q, 10)
+    for delta in (1, 97, 1000, 1 << 30):
+        grid = gg.GGrid(g, 128, max_objects=512, delta=delta)
+        grid.ingest(upd)
+        _assert_same(grid.knn(q, 10), ref, f"delta={delta}")
+        grid.close()
+
+
+def test_large_k_and_sparse_objects_use_every_level(gg):
+    """k above the level-0 limit and fewer reachable objects than k: levels 1 and 2."""
+    g = synth.table_ii_graph("NY", scale=0.05)
+    upd = synth.RandomWalk(g, 40).ticks(2)
+    q = synth.queries(g, 20)
+    grid = gg.GGrid(g, 512, max_objects=64, max_k=1024)
+    grid.ingest(upd)
+    for k in (129, 600):
+        _assert_same(grid.knn(q, k), _oracle(g, upd, q, k), f"k={k}")
+    st = grid.stats()
+    assert st["kernel_launches"]["expand_big"] > 0
+    grid.close()
+
+
+def test_einval_rejects_batch_atomically(gg):
+    g = synth.lattice_graph(8, 8, 1, 4)
+    grid = gg.GGrid(g, 16, max_objects=32, max_k=8)
+    good = synth.RandomWalk(g, 20).ticks(2)
+    grid.ingest(good)
+    for bad_row in ([40, 0, 0, 0], [1, len(g["src"]), 0, 0], [1, 3, int(g["w"][3]), 0]):
+        bad = np.concatenate([good[:5], np.array([bad_row], np.uint32), good[5:9]])
+        with pytest.raises(gg.GGridError) as e:
+            grid.ingest(bad)
+        assert e.value.rc == gg.GGRID_EINVAL
+    q = synth.queries(g, 10)
+    _assert_same(grid.knn(q, 4), _oracle(g, good, q, 4), "after rejected batches")
+    for k in (0, 9):
+        with pytest.raises(gg.GGridError):
+            grid.knn(q, k)
+    with pytest.raises(gg.GGridError):
+        grid.knn(np.array([[len(g["src"]), 0]], np.uint32), 2)
+    with pytest.raises(gg.GGridError):
+        grid.knn(np.array([[3, int(g["w"][3])]], np.uint32), 2)
+    assert grid.stats()["n_updates"] == len(good)
+    grid.close()
+
+
+def test_garbage_collection_keeps_answers(gg):
+    g = synth.table_ii_graph("NY", scale=0.03)
+    walk = synth.RandomWalk(g, 800, inject=True)
+    grid = gg.GGrid(g, 128, max_objects=1024, log_capacity=12_000)
+    hist = []
+    for r in range(12):
+        u = walk.ticks(3)
+        hist.append(u)
+        grid.ingest(u)
+        q = synth.queries(g, 50, seed=7 + r)
+        _assert_same(grid.knn(q, 6), _oracle(g, np.concatenate(hist), q, 6), f"round {r}")
+    assert grid.stats()["gc_runs"] > 0
+    grid.close()
+
+
+# ----------------------------------------------------------------- BASELINE-scale configs
+def test_c1_ny_bit_exact(gg):
+    """configs[1] at full size: NY-shaped graph, 10k objects, 1M cached updates, k=10;
+    every one of 2,000 queries checked against the full-Dijkstra oracle."""
+    g = synth.config_graph("C1")
+    upd = synth.RandomWalk(g, 10_000, inject=True).ticks(100)
+    q = synth.queries(g, 2000)
+    grid = gg.GGrid(g, 1024, max_objects=10_000)
+    grid.ingest(upd)
+    got = grid.knn(q, 10)
+    _assert_same(got, _oracle(g, upd, q, 10), "C1")
+    grid.close()
+
+
+def test_c2_fla_k_sweep(gg):
+    """configs[2]: FLA-shaped, 100k objects, k = 10..50 (sampled 300 queries, EARLY oracle
+    cross-checked against FULL on a subset in test_oracle)."""
+    g = synth.config_graph("C2")
+    upd = synth.RandomWalk(g, 100_000).ticks(10)
+    q = synth.queries(g, 300)
+    grid = gg.GGrid(g, 1024, max_objects=100_000)
+    grid.ingest(upd)
+    for k in (10, 20, 30, 40, 50):
+        _assert_same(grid.knn(q, k), _oracle(g, upd, q, k, mode=oracle.EARLY), f"C2 k={k}")
+    grid.close()
