@@ -1,0 +1,348 @@
+"""Benchmark: kNN queries/s including the lazy flush at a fixed update rate (BASELINE.json).
+
+One step = one pass of the whole hot path over one batch of synthetic input:
+  ggrid_ingest(r*Q cached location updates)   (Alg. 1: a0)
+  ggrid_knn(Q queries, k)                      (cell selection, lazy flush, expansion,
+                                                 candidate top-k, unresolved, refinement:
+                                                 a1-a6 of SURVEY §8(a))
+value = queries answered / device time of the steps (CUDA events on the library's stream,
+max over ranks).  Default workload: BASELINE configs[1] (NY-shaped graph, 10k objects,
+1M cached updates per step = 100 ticks of the random walk, Q = 10^4 queries, k = 10).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C1|C0|C2|C3]
+    python bench.py --impl reference ...    # the CPU oracle as the reference arm
+Multi-GPU (torchrun): each rank owns a replica of the index, ingests the same update
+stream and answers its own Q queries (weak scaling of the query work).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+CONFIG_TEXT = {
+    "C0": "Fig.1-scale toy: ~1k-vertex synthetic grid road graph, 100 moving objects, 1k cached updates, k=3, 100 queries",
+    "C1": "NY-shaped synthetic road graph (~264k vertices, ~734k edges), 10k objects, k=10, 1M cached updates",
+    "C2": "FLA-shaped synthetic road graph (~1.07M vertices), 100k objects, k=10-50 sweep",
+    "C3": "USA-shaped synthetic road graph (~24M vertices, ~58M edges), 1M objects, k=10, batched queries",
+}
+METRIC = "kNN queries/sec incl. lazy flush at fixed update rate"
+
+# Algorithmic bytes per unit (restated in DESIGN.md §5)
+INGEST_BYTES_PER_UPDATE = 48          # 16 record + 4 arc->cell + 8 RED.MAX + 20 SoA write
+FLUSH_BYTES_PER_RECORD = 12           # obj + key
+FLUSH_BYTES_PER_WINNER = 12 + 8 + 24  # payload read + ot_key + compacted write
+FLUSH_BYTES_PER_VERTEX = 8            # v_obj index entry per vertex of a flushed cell
+# expansion: counted work (ggrid_stats expand_*), bytes each unit must move
+EXPAND_BYTES_PER_VERTEX = 8    # rowptr[u], rowptr[u+1]
+EXPAND_BYTES_PER_ARC = 8       # adj (dst, w)
+EXPAND_BYTES_PER_HARVEST = 12  # cell_head (dirty check) + v_obj (start, count)
+EXPAND_BYTES_PER_OBJECT = 28   # obj, key, edge, off + ot_key (validity)
+EXPAND_BYTES_PER_QUERY = 16    # query (edge, off) + inverted index (src, w)
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def workload(cfg: str, queries: int | None):
+    c = dict(synth.CONFIGS[cfg])
+    if queries:
+        c["n_queries"] = queries
+    return c
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(gpu), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = [r.split(",") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            r = [x.strip() for x in r]
+            try:
+                sm.append(float(r[1]))
+                mx.append(float(r[2]))
+            except (ValueError, IndexError):
+                continue
+            for n, v in zip(names, r[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# -------------------------------------------------------------------------- oracle arm
+def time_oracle(g, cfg, upd_step, queries, n_sample, threads=0):
+    """The CPU oracle as it stands on a bounded sample: snapshot of one step's updates +
+    n_sample full-Dijkstra queries; returns (queries/s scaled to the step, sample text, cores)."""
+    import oracle
+
+    cores = threads if threads > 0 else oracle.hardware_threads()
+    snap = oracle.Snapshot(cfg["n_objects"])
+    t0 = time.perf_counter()
+    snap.apply(upd_step)
+    t_snap = time.perf_counter() - t0
+    ids, e, d = snap.objects()
+    qs = queries[:n_sample]
+    t0 = time.perf_counter()
+    oracle.knn(g, ids, e, d, qs, cfg["k"], mode=oracle.FULL, threads=cores)
+    t_q = time.perf_counter() - t0
+    Q = len(queries)
+    per_step = t_snap + t_q * Q / len(qs)
+    sample = (f"snapshot of one step's {len(upd_step)} updates ({t_snap:.3f}s) + {len(qs)} of the step's {Q} "
+              f"queries, full-graph Dijkstra ({t_q:.2f}s), scaled to the step")
+    return Q / per_step, sample, cores
+
+
+def run_reference(args, cfg_name):
+    world, rank, _ = dist_setup()
+    if world > 1 and rank != 0:
+        return
+    cfg = workload(cfg_name, args.queries)
+    g = synth.config_graph(cfg_name)
+    walk = synth.RandomWalk(g, cfg["n_objects"])
+    n_sample = args.ref_sample
+    times = []
+    sample_txt, cores = "", 0
+    for s in range(args.warmup + args.steps):
+        upd = walk.ticks(cfg["updates_per_object"])
+        q = synth.queries(g, cfg["n_queries"], seed=synth.SEED_QUERIES + s)
+        qps, sample_txt, cores = time_oracle(g, cfg, upd, q, n_sample)
+        if s >= args.warmup:
+            times.append(cfg["n_queries"] / qps)
+    value = cfg["n_queries"] * len(times) / sum(times)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic", "config": {"workload": CONFIG_TEXT[cfg_name], "config_id": cfg_name,
+                                            "queries_per_step": cfg["n_queries"], "k": cfg["k"]},
+            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
+                             "sample": sample_txt},
+            "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- our arm
+def run_ours(args, cfg_name):
+    import torch
+
+    import paper_conf_icde_li0qhdy18_b200 as gg
+
+    world, rank, local = dist_setup()
+    if world > 1:
+        import torch.distributed as dist
+
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.cuda.current_device()
+    cfg = workload(cfg_name, args.queries)
+    Q, k = cfg["n_queries"], cfg["k"]
+    g = synth.config_graph(cfg_name)
+    walk = synth.RandomWalk(g, cfg["n_objects"])
+    stream = torch.cuda.Stream()
+    grid = gg.GGrid(g, args.cell_size or cfg["cell_size"], max_objects=cfg["n_objects"], profile=True,
+                    log_capacity=args.log_capacity, delta=args.delta, stream=stream.cuda_stream)
+    out_o = torch.empty((Q, k), dtype=torch.int32, device="cuda")
+    out_d = torch.empty((Q, k), dtype=torch.int32, device="cuda")
+    l2 = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
+
+    def step_inputs(s):
+        u = walk.ticks(cfg["updates_per_object"])
+        q = synth.queries(g, Q, seed=synth.SEED_QUERIES + 1000 * rank + s)
+        return u, q
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            torch.distributed.barrier()
+
+    # ---- device-resident timed region -------------------------------------------------
+    times = []
+    st0 = None
+    for s in range(args.warmup + args.steps):
+        u, q = step_inputs(s)
+        du = torch.from_numpy(u.view(np.int32)).to("cuda")
+        dq = torch.from_numpy(q.view(np.int32)).to("cuda")
+        with torch.cuda.stream(stream):
+            l2.zero_()  # flush L2 between timed iterations (outside the events)
+        barrier()
+        if s == args.warmup:
+            grid.stats_reset()
+            st0 = grid.stats()
+            clocks = ClockSampler(dev)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        grid.ingest(du)
+        grid.knn(dq, k, out_o, out_d)
+        e1.record(stream)
+        e1.synchronize()
+        if s >= args.warmup:
+            times.append(e0.elapsed_time(e1))
+    barrier()
+    clk = clocks.stop()
+    st1 = grid.stats()
+    total_ms = sum(times)
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        total_ms = float(t.item())
+    K = args.steps
+    value = world * Q * K / (total_ms / 1e3)
+    n_upd = cfg["n_objects"] * cfg["updates_per_object"]
+
+    # ---- per-kernel roofline from the profile-mode events of the timed region -----------
+    peak, peak_kind = load_peaks()
+    kms = st1["kernel_ms"]
+    kl = st1["kernel_launches"]
+    ingest_ms = kms["ingest_classify"] + kms["ingest_alloc"] + kms["ingest_scatter"]
+    rec = st1["records_flushed"] - st0["records_flushed"]
+    win = st1["objects_written"] - st0["objects_written"]
+    cells = st1["cells_flushed"] - st0["cells_flushed"]
+    cs = st1["cell_size"]
+    dx = {n: st1["expand_" + n] - st0["expand_" + n] for n in ("iterations", "vertices", "arcs", "harvested", "objects")}
+    expand_bytes = (dx["vertices"] * EXPAND_BYTES_PER_VERTEX + dx["arcs"] * EXPAND_BYTES_PER_ARC
+                    + dx["harvested"] * EXPAND_BYTES_PER_HARVEST + dx["objects"] * EXPAND_BYTES_PER_OBJECT
+                    + Q * K * (EXPAND_BYTES_PER_QUERY + 8 * k))
+    flush_bytes = rec * FLUSH_BYTES_PER_RECORD + win * FLUSH_BYTES_PER_WINNER + cells * cs * FLUSH_BYTES_PER_VERTEX
+    kern = {
+        "ingest": (ingest_ms, n_upd * K * INGEST_BYTES_PER_UPDATE,
+                   kl["ingest_classify"] + kl["ingest_alloc"] + kl["ingest_scatter"]),
+        "flush": (kms["flush"], flush_bytes, kl["flush"]),
+        "expand": (kms["expand"] + kms["expand_big"], expand_bytes, kl["expand"] + kl["expand_big"]),
+    }
+    dom = max(kern, key=lambda n: kern[n][0])
+    dms, dbytes, dl = kern[dom]
+    achieved = dbytes / (dms / 1e3) / 1e9 if dms > 0 else 0.0
+    per_kernel = {n: {"ms_total": v[0], "launches": v[2], "alg_bytes": v[1],
+                      "gbs": (v[1] / (v[0] / 1e3) / 1e9) if v[0] > 0 else 0.0} for n, v in kern.items()}
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", f"traffic_{cfg_name}.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(dom)
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": traffic, "kernel": dom, "peak_source": peak_kind}
+    updates_per_s = n_upd * K / (ingest_ms / 1e3) if ingest_ms > 0 else None
+
+    # ---- e2e through the public API with pinned host buffers -------------------------------
+    e2e_times = []
+    h_o = torch.empty((Q, k), dtype=torch.int32).pin_memory()
+    h_d = torch.empty((Q, k), dtype=torch.int32).pin_memory()
+    n_e2e = max(1, min(K, args.e2e_steps))
+    for s in range(n_e2e + 1):
+        u, q = step_inputs(10_000 + s)
+        hu = torch.from_numpy(u.view(np.int32)).pin_memory()
+        hq = torch.from_numpy(q.view(np.int32)).pin_memory()
+        barrier()
+        t0 = time.perf_counter()
+        grid.ingest(hu)
+        grid.knn(hq, k, h_o, h_d)
+        t1 = time.perf_counter()
+        if s > 0:
+            e2e_times.append(t1 - t0)
+    e2e_total = sum(e2e_times)
+    if world > 1:
+        t = torch.tensor([e2e_total], dtype=torch.float64, device="cuda")
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        e2e_total = float(t.item())
+    e2e = {"value": world * Q * len(e2e_times) / e2e_total, "unit": "queries/s",
+           "h2d_bytes_per_step": n_upd * 16 + Q * 8, "d2h_bytes_per_step": Q * k * 8}
+
+    # ---- CPU oracle beside it (rank 0, N=1 only) -------------------------------------------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        u, q = step_inputs(20_000)
+        qps, sample, cores = time_oracle(g, cfg, u, q, args.ref_sample)
+        cpu = {"value": qps, "unit": "queries/s", "cores": cores, "kind": "oracle", "sample": sample}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": K,
+                "warmup": args.warmup, "ms_per_step": total_ms / K, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": {"workload": CONFIG_TEXT[cfg_name], "config_id": cfg_name, "graph": synth.CONFIGS[cfg_name]["graph"],
+                           "n_vertices": int(g["n_vertices"]), "n_arcs": int(len(g["src"])),
+                           "objects": cfg["n_objects"], "updates_per_step": n_upd, "queries_per_step_per_gpu": Q,
+                           "k": k, "cell_size": cs, "l2": "flushed between timed steps (256 MB write)",
+                           "parallelism": f"replicas x{world}, queries sharded"},
+                "updates_per_s": updates_per_s, "per_kernel": per_kernel, "roofline": roofline,
+                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(st1["launches"]), "clocks": clk,
+                "knn_rounds_per_step": (st1["knn_rounds"] - st0["knn_rounds"]) / K,
+                "expand_work_per_query": {n: v / (Q * K) for n, v in dx.items()}, "delta": st1["delta"]}
+        print(json.dumps(line), flush=True)
+    grid.close()
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C1", choices=["C0", "C1", "C2", "C3"])
+    ap.add_argument("--queries", type=int, default=0)
+    ap.add_argument("--cell-size", type=int, default=0)
+    ap.add_argument("--delta", type=int, default=0)
+    ap.add_argument("--log-capacity", type=int, default=0)
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--ref-sample", type=int, default=400)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    assert args.warmup >= 3 or args.impl == "reference" or os.environ.get("BENCH_ALLOW_SHORT"), "W >= 3"
+    if args.impl == "reference":
+        run_reference(args, args.config)
+    else:
+        run_ours(args, args.config)
+
+
+if __name__ == "__main__":
+    main()

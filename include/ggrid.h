@@ -105,6 +105,11 @@ typedef struct ggrid_stats_t {
   uint64_t arena_capacity;
   uint64_t gc_runs;
   uint64_t launches;         /* kernel launches issued by the library, all kinds     */
+  uint64_t expand_iterations;/* delta-stepping rounds over all answered queries      */
+  uint64_t expand_vertices;  /* vertex expansions (out-arc scans)                    */
+  uint64_t expand_arcs;      /* arc relaxations                                      */
+  uint64_t expand_harvested; /* settled vertices whose object lists were read        */
+  uint64_t expand_objects;   /* object entries read while harvesting                 */
   uint64_t kernel_launches[GGRID_NK];
   double kernel_ms[GGRID_NK];/* summed CUDA-event device time (opts.profile = 1)     */
   uint32_t n_cells;

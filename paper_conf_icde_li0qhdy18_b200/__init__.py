@@ -53,7 +53,8 @@ NK = 8
 class ggrid_stats_t(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in
                 ["n_updates", "n_queries", "knn_calls", "knn_rounds", "cells_flushed", "records_flushed",
-                 "objects_written", "arena_used", "arena_capacity", "gc_runs", "launches"]] + [
+                 "objects_written", "arena_used", "arena_capacity", "gc_runs", "launches", "expand_iterations",
+                 "expand_vertices", "expand_arcs", "expand_harvested", "expand_objects"]] + [
         ("kernel_launches", ctypes.c_uint64 * NK), ("kernel_ms", ctypes.c_double * NK)] + [
         (n, ctypes.c_uint32) for n in ["n_cells", "cell_size", "delta", "n_vertices", "n_arcs", "max_objects"]]
 

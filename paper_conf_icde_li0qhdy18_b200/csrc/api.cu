@@ -492,9 +492,9 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
 
   h->epoch++;
   const uint32_t epoch = h->epoch;
-  // reset err, n_flush, flush_work, n_next[*], flush_end
+  // reset err, n_flush, flush_work, n_next[*], flush_end, expand_work[*]
   CK(cudaMemsetAsync(&h->d_status->err, 0, sizeof(unsigned), st));
-  CK(cudaMemsetAsync(&h->d_status->n_flush, 0, offsetof(DevStatus, pad) - offsetof(DevStatus, n_flush), st));
+  CK(cudaMemsetAsync(&h->d_status->n_flush, 0, offsetof(DevStatus, round_end) - offsetof(DevStatus, n_flush), st));
   const DevGraph& g = h->g;
   const DevState& s = h->s;
   h->launch(GGRID_K_SEED, [&] { launch_seed(d_q, n_q, g, s, epoch, h->seed_neighbors, st); });
@@ -510,6 +510,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
     if (round > 100000) return GGRID_ECUDA;
     RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin));
     CK(cudaMemsetAsync(h->d_status->n_next, 0, sizeof(h->d_status->n_next), st));
+    CK(cudaMemsetAsync(h->d_status->expand_work, 0, sizeof(h->d_status->expand_work), st));
     for (int lvl = 0; lvl < L; ++lvl) {
       if (!n_in[lvl]) continue;
       void* scratch = nullptr;
@@ -527,7 +528,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
       const uint32_t nn = n_in[lvl];
       const int kind = lvl == 0 ? GGRID_K_EXPAND : GGRID_K_EXPAND_BIG;
       h->launch(kind, [&] {
-        launch_expand(lvl, d_q, qlist, nn, k, g, s, epoch, retry, promote, d_oo, d_od, scratch, sw, st);
+        launch_expand(lvl, d_q, qlist, nn, k, g, s, epoch, retry, promote, d_oo, d_od, scratch, sw, h->sm_count, st);
       });
     }
     RC(h->sync());
@@ -611,6 +612,11 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
   s.cells_flushed = h->h_status->cells_flushed;
   s.records_flushed = h->h_status->records_flushed;
   s.objects_written = h->h_status->objects_written;
+  s.expand_iterations = h->h_status->ex_iters;
+  s.expand_vertices = h->h_status->ex_vertices;
+  s.expand_arcs = h->h_status->ex_arcs;
+  s.expand_harvested = h->h_status->ex_harvested;
+  s.expand_objects = h->h_status->ex_objects;
   s.arena_used = h->h_status->arena_top;
   s.arena_capacity = h->s.ar.cap;
   s.n_cells = h->n_cells;

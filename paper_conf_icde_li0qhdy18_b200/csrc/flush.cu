@@ -22,7 +22,7 @@
 namespace gg {
 
 namespace {
-constexpr int FT = 256;               // threads per CTA
+constexpr int FT = 512;               // threads per CTA
 constexpr int TCAP = 2048;            // table slots (power of two)
 constexpr int HCAP = 4096;            // per-vertex counters kept in smem
 constexpr int RPT = 4;                // records per thread per tile

@@ -14,34 +14,76 @@
 
 namespace gg {
 
-__global__ void __launch_bounds__(256) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
-                                                         DevGraph g, DevState s,
-                                                         uint2* __restrict__ tmp) {
-  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  uint4 m = upd[i];
-  unsigned bad = 0;
-  uint2 e = make_uint2(0, 1);
-  if (m.x >= s.max_objects) bad |= ERR_OBJ;
-  if (m.y >= g.A) {
-    bad |= ERR_EDGE;
-  } else {
-    e = g.einfo[m.y];
-    if (m.z >= e.y) bad |= ERR_OFF;
+// CTA-level aggregation: each CTA takes CU consecutive updates, counts them per cell in a
+// shared-memory hash (rank within the CTA), then claims one global range per distinct
+// cell with a single atomicAdd on bcount[cell] (few cells => no hot-spot serialisation).
+constexpr int CT = 256;            // threads
+constexpr int CPT = 8;             // updates per thread
+constexpr int CU = CT * CPT;       // updates per CTA
+constexpr int CH = 4096;           // hash slots (>= 2*CU)
+
+__global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
+                                                        DevGraph g, DevState s,
+                                                        uint2* __restrict__ tmp) {
+  __shared__ uint32_t h_cell[CH];
+  __shared__ uint32_t h_cnt[CH];
+  const int tid = threadIdx.x;
+  for (int i = tid; i < CH; i += CT) {
+    h_cell[i] = NONE;
+    h_cnt[i] = 0;
   }
-  if (bad) {
-    atomicOr(&s.st->err, bad);
-    atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
-    return;
+  __syncthreads();
+  const uint64_t base = (uint64_t)blockIdx.x * CU;
+  int slot[CPT];
+  uint32_t vs[CPT], lr[CPT];
+#pragma unroll
+  for (int j = 0; j < CPT; ++j) {
+    const uint64_t i = base + (uint64_t)j * CT + tid;
+    slot[j] = -1;
+    if (i >= n) continue;
+    const uint4 m = upd[i];
+    unsigned bad = 0;
+    uint2 e = make_uint2(0, 1);
+    if (m.x >= s.max_objects) bad |= ERR_OBJ;
+    if (m.y >= g.A) {
+      bad |= ERR_EDGE;
+    } else {
+      e = g.einfo[m.y];
+      if (m.z >= e.y) bad |= ERR_OFF;
+    }
+    if (bad) {
+      atomicOr(&s.st->err, bad);
+      atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
+      continue;
+    }
+    const uint32_t c = cell_of(e.x, g.cs);
+    uint32_t h = (c * 2654435761u) >> 20;  // 12 bits
+    volatile uint32_t* vc = h_cell;
+    for (;;) {
+      const uint32_t cur = vc[h];
+      if (cur == c) break;
+      if (cur == NONE) {
+        const uint32_t old = atomicCAS(&h_cell[h], NONE, c);
+        if (old == NONE || old == c) break;
+      }
+      h = (h + 1) & (CH - 1);
+    }
+    slot[j] = (int)h;
+    vs[j] = e.x;
+    lr[j] = atomicAdd(&h_cnt[h], 1u);
   }
-  uint32_t c = cell_of(e.x, g.cs);
-  unsigned act = __activemask();
-  unsigned grp = __match_any_sync(act, c);
-  int leader = __ffs(grp) - 1;
-  unsigned base = 0;
-  if ((int)(threadIdx.x & 31) == leader) base = atomicAdd(&s.bcount[c], (unsigned)__popc(grp));
-  base = __shfl_sync(grp, base, leader);
-  tmp[i] = make_uint2(e.x, base + __popc(grp & lanemask_lt()));
+  __syncthreads();
+  for (int i = tid; i < CH; i += CT) {
+    const uint32_t c = h_cell[i];
+    if (c != NONE) h_cnt[i] = atomicAdd(&s.bcount[c], h_cnt[i]);
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < CPT; ++j) {
+    if (slot[j] < 0) continue;
+    const uint64_t i = base + (uint64_t)j * CT + tid;
+    tmp[i] = make_uint2(vs[j], h_cnt[slot[j]] + lr[j]);
+  }
 }
 
 __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
@@ -109,8 +151,8 @@ __global__ void __launch_bounds__(256) k_ingest_scatter(const uint4* __restrict_
 
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
                             uint2* tmp, cudaStream_t st) {
-  unsigned blocks = (unsigned)((n + 255) / 256);
-  k_ingest_classify<<<blocks, 256, 0, st>>>(upd, n, g, s, tmp);
+  unsigned blocks = (unsigned)((n + CU - 1) / CU);
+  k_ingest_classify<<<blocks, CT, 0, st>>>(upd, n, g, s, tmp);
 }
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st) {
   k_ingest_alloc<<<(g.n_cells + 255) / 256, 256, 0, st>>>(g, s);

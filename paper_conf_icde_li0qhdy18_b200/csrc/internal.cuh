@@ -36,6 +36,7 @@ struct DevStatus {
   unsigned long long records_flushed;
   unsigned long long objects_written;
   unsigned long long cells_flushed;
+  unsigned long long ex_iters, ex_vertices, ex_arcs, ex_harvested, ex_objects;  // expansion work
   unsigned int ext_top;     // next free extent
   unsigned int err;         // ErrBits
   unsigned int bad_index;   // smallest offending index (ingest)
@@ -44,7 +45,8 @@ struct DevStatus {
   unsigned int flush_work;  // persistent flush work counter
   unsigned int n_next[4];   // per expansion level: queries queued for the next round
   unsigned int flush_end;   // n_flush as seen by the last flush launch
-  unsigned int pad;
+  unsigned int expand_work[4];  // per-level dynamic work counters of the expand launches
+  unsigned int round_end;   // (marks the end of the per-round reset region)
 };
 
 struct DevGraph {
@@ -127,7 +129,7 @@ int flush_smem_bytes();
 void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
                    const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
                    uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist, void* scratch,
-                   uint32_t scratch_warps, cudaStream_t st);
+                   uint32_t scratch_warps, int sm_count, cudaStream_t st);
 int expand_levels();
 uint32_t expand_max_k(int level);
 size_t expand_warp_bytes(int level, uint32_t V);

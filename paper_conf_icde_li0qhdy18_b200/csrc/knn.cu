@@ -11,9 +11,10 @@
 //   * D lives in a per-warp shared-memory open-addressing table keyed by vertex; one
 //     64-bit word (v<<32 | dist) so relaxation is a single atomicMin (same key => min on
 //     the distance).  Seeds follow reading R1 (d=0 -> D[src]=0, else D[dst]=w-d).
-//   * Each round takes the frontier bucket [m, m+delta) (m = frontier minimum) and relaxes
-//     its out-arcs lane-per-arc (warp-cooperative adjacency scan: a warp scan of the degrees
-//     of 32 active vertices, then each lane binary-searches its arc).
+//   * Each round walks the frontier in chunks of 32; the lanes whose D lies in the bucket
+//     [m, m+delta) (m = frontier minimum) relax their out-arcs lane-per-arc
+//     (warp-cooperative adjacency scan: a warp scan of the degrees, the chunk's arcs
+//     flattened into shared memory, one arc per lane).
 //   * Every vertex with D < m is final; its objects are harvested from the cell's cleaned
 //     list (v_obj index) as exact candidates dist = D[src(e_o)] + d_o (P@49436), objects on
 //     q's own arc ahead of q at d_o - d_q (reading R2), stale entries dropped by
@@ -32,7 +33,8 @@ namespace gg {
 namespace {
 
 enum { DONE = 0, RETRY = 1, OVERFLOW = 2 };
-constexpr int MAXP = 128;  // probe limit of the vertex table
+constexpr int MAXP = 128;       // probe limit of the vertex table
+constexpr uint32_t ARCMAX = 128;  // flattened arcs per 32-vertex chunk (else binary search)
 
 struct Caps {
   uint32_t H, F, X, C;  // table slots (pow2), frontier, expanded list, candidates
@@ -44,17 +46,18 @@ struct WarpMem {
   unsigned long long* cand;  // C
   uint32_t* front0;          // F
   uint32_t* front1;          // F
-  uint32_t* act;             // F
   uint32_t* exl;             // X
   uint32_t* fin;             // H/32
   uint32_t* listed;          // H/32
   uint32_t* scan;            // 32
   uint32_t* rp;              // 32
   uint32_t* du;              // 32
+  uint32_t* own_arc;         // ARCMAX: arcs of the current chunk's active vertices
+  uint32_t* own_du;          // ARCMAX: D of each staged arc's source
 };
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 8ull * c.C + 4ull * (3ull * c.F + c.X + 2ull * (c.H / 32) + 96);
+  return 8ull * c.H + 8ull * c.C + 4ull * (2ull * c.F + c.X + 2ull * (c.H / 32) + 96 + 2 * ARCMAX);
 }
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
@@ -64,13 +67,14 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   uint32_t* p = reinterpret_cast<uint32_t*>(m.cand + c.C);
   m.front0 = p; p += c.F;
   m.front1 = p; p += c.F;
-  m.act = p; p += c.F;
   m.exl = p; p += c.X;
   m.fin = p; p += c.H / 32;
   m.listed = p; p += c.H / 32;
   m.scan = p; p += 32;
   m.rp = p; p += 32;
-  m.du = p;
+  m.du = p; p += 32;
+  m.own_arc = p; p += ARCMAX;
+  m.own_du = p;
   return m;
 }
 
@@ -83,35 +87,39 @@ __device__ __forceinline__ uint32_t vhash(uint32_t v) {
 __device__ __forceinline__ int tab_relax(unsigned long long* dtab, uint32_t hmask, uint32_t v,
                                          uint32_t d, bool& improved) {
   const unsigned long long nv = ((unsigned long long)v << 32) | d;
-  const uint32_t h = vhash(v);
+  uint32_t sl = vhash(v) & hmask;
   volatile unsigned long long* vt = dtab;
 #pragma unroll 1
   for (int p = 0; p < MAXP; ++p) {
-    const uint32_t sl = (h + p) & hmask;
     unsigned long long cur = vt[sl];
+    if ((uint32_t)(cur >> 32) == v) {
+      if ((uint32_t)cur <= d) {  // not an improvement (e.g. the twin arc back): no atomic
+        improved = false;
+        return (int)sl;
+      }
+      const unsigned long long old = atomicMin(&dtab[sl], nv);
+      improved = (uint32_t)old > d;
+      return (int)sl;
+    }
     if (cur == EMPTY64) {
       const unsigned long long old = atomicCAS(&dtab[sl], EMPTY64, nv);
       if (old == EMPTY64) {
         improved = true;
         return (int)sl;
       }
-      cur = old;
+      if ((uint32_t)(old >> 32) == v) continue;  // same vertex inserted meanwhile: re-read
     }
-    if ((uint32_t)(cur >> 32) == v) {
-      const unsigned long long old = atomicMin(&dtab[sl], nv);
-      improved = (uint32_t)old > d;
-      return (int)sl;
-    }
+    sl = (sl + 1) & hmask;
   }
   improved = false;
   return -1;
 }
 
-// warp bitonic sort of cand[0..n) ascending (n padded to a power of two <= cap)
+// warp bitonic sort of a[0..n) ascending (n padded to a power of two <= cap)
 __device__ void warp_sort(unsigned long long* a, uint32_t n, uint32_t cap, int lane) {
   uint32_t n2 = 1;
   while (n2 < n) n2 <<= 1;
-  if (n2 > cap) n2 = cap;  // n <= cap always
+  if (n2 > cap) n2 = cap;
   for (uint32_t i = n + lane; i < n2; i += 32) a[i] = EMPTY64;
   __syncwarp();
   for (uint32_t size = 2; size <= n2; size <<= 1) {
@@ -146,20 +154,32 @@ struct QParams {
   uint32_t* out_obj;
   uint32_t* out_dist;
   Caps caps;
-  unsigned char* scratch;   // global working memory (level 2) or null (shared)
+  unsigned char* scratch;   // global working memory (last level) or null (shared)
   uint32_t warps_per_cta;
 };
 
-// Ask for the flush of every dirty cell the frontier / pending harvest will need, so a
-// retried query is unlikely to stop again for the same reason.
+// Append one ballot's worth of candidates; when full, keep only the k best so far (a
+// dropped candidate has >= k better ones, so it can never be in the answer).
+__device__ __forceinline__ bool cand_push(const WarpMem& m, uint32_t& nc, uint32_t C, uint32_t k,
+                                          bool has, unsigned long long dk, int lane, unsigned lt) {
+  const unsigned hm = __ballot_sync(0xffffffffu, has);
+  if (!hm) return true;
+  if (nc + __popc(hm) > C) {
+    warp_sort(m.cand, nc, C, lane);
+    nc = min(nc, k);
+    if (nc + __popc(hm) > C) return false;
+  }
+  if (has) m.cand[nc + __popc(hm & lt)] = dk;
+  nc += __popc(hm);
+  return true;
+}
+
+// Ask for the flush of every dirty cell the frontier will need, so a retried query is
+// unlikely to stop again for the same reason.
 __device__ void request_lookahead(const QParams& P, const WarpMem& m, const uint32_t* front,
-                                  uint32_t nf, uint32_t nx, int lane) {
+                                  uint32_t nf, int lane) {
   for (uint32_t i = lane; i < nf; i += 32) {
     const uint32_t v = (uint32_t)(m.dtab[front[i]] >> 32);
-    request_flush(P.s, cell_of(v, P.g.cs), P.epoch);
-  }
-  for (uint32_t i = lane; i < nx; i += 32) {
-    const uint32_t v = (uint32_t)(m.dtab[m.exl[i]] >> 32);
     request_flush(P.s, cell_of(v, P.g.cs), P.epoch);
   }
 }
@@ -224,15 +244,15 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
           dk = ((unsigned long long)(oo - q.y) << 32) | ob;
         }
       }
-      const unsigned hm = __ballot_sync(FULL, has);
-      if (nc + __popc(hm) > cp.C) return OVERFLOW;
-      if (has) m.cand[nc + __popc(hm & lt)] = dk;
-      nc += __popc(hm);
+      if (!cand_push(m, nc, cp.C, k, has, dk, lane, lt)) return OVERFLOW;
     }
     __syncwarp();
   }
 
+  // work counters (warp-uniform), published once per answered query
+  uint32_t c_iter = 0, c_vert = 0, c_arcs = 0, c_harv = 0, c_objs = 0;
   for (;;) {
+    ++c_iter;
     // ---- 1. frontier minimum: every vertex with D < m is final -------------------------
     uint32_t ml = INF;
     for (uint32_t i = lane; i < nf; i += 32) ml = min(ml, (uint32_t)m.dtab[front[i]]);
@@ -264,10 +284,14 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
         }
       }
       if (__any_sync(FULL, dirty)) {
-        request_lookahead(P, m, front, nf, 0, lane);
+        request_lookahead(P, m, front, nf, lane);
         return RETRY;
       }
-      for (uint32_t j = 0; __any_sync(FULL, j < vo.y); ++j) {
+      c_harv += __popc(__ballot_sync(FULL, take));
+      const uint32_t most = __reduce_max_sync(FULL, vo.y);
+      if (most == 0) continue;
+      c_objs += __reduce_add_sync(FULL, vo.y);
+      for (uint32_t j = 0; j < most; ++j) {
         bool has = false;
         unsigned long long dk = 0;
         if (j < vo.y) {
@@ -284,15 +308,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
             }
           }
         }
-        const unsigned hm = __ballot_sync(FULL, has);
-        if (nc + __popc(hm) > cp.C) {
-          // keep only the k best so far: a dropped candidate has >= k better ones
-          warp_sort(m.cand, nc, cp.C, lane);
-          nc = min(nc, k);
-          if (nc + __popc(hm) > cp.C) return OVERFLOW;
-        }
-        if (has) m.cand[nc + __popc(hm & lt)] = dk;
-        nc += __popc(hm);
+        if (!cand_push(m, nc, cp.C, k, has, dk, lane, lt)) return OVERFLOW;
       }
     }
     nx = keep;
@@ -300,47 +316,44 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
 
     // ---- 3. termination: k candidates strictly closer than any unharvested object -------
     if (nf == 0) break;
-    uint32_t cl = 0;
-    for (uint32_t i = lane; i < nc; i += 32) cl += (uint32_t)(m.cand[i] >> 32) < blo;
-    if (__reduce_add_sync(FULL, cl) >= k) break;
+    if (nc >= k) {
+      uint32_t cl = 0;
+      for (uint32_t i = lane; i < nc; i += 32) cl += (uint32_t)(m.cand[i] >> 32) < blo;
+      if (__reduce_add_sync(FULL, cl) >= k) break;
+    }
 
-    // ---- 4. activate the bucket [m, m + delta) -------------------------------------------
+    // ---- 4+5. walk the frontier; relax the out-arcs of the bucket [m, m + delta) ---------
     const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
-    uint32_t na = 0, nn = 0;
+    uint32_t nn = 0;
     for (uint32_t b0 = 0; b0 < nf; b0 += 32) {
       const uint32_t i = b0 + lane;
       const uint32_t sl = i < nf ? front[i] : NONE;
-      const bool a = sl != NONE && (uint32_t)m.dtab[sl] < bhi;
+      const unsigned long long ent = sl != NONE ? m.dtab[sl] : EMPTY64;
+      const bool a = sl != NONE && (uint32_t)ent < bhi;
       const bool r = sl != NONE && !a;
-      const unsigned am = __ballot_sync(FULL, a), rm = __ballot_sync(FULL, r);
-      bool newl = false;
-      if (a) {
-        m.act[na + __popc(am & lt)] = sl;
-        atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
-        const uint32_t bit = 1u << (sl & 31);
-        newl = !(atomicOr(&m.listed[sl >> 5], bit) & bit);
-      }
+      const unsigned rm = __ballot_sync(FULL, r);
       if (r) nfront[nn + __popc(rm & lt)] = sl;
-      na += __popc(am);
       nn += __popc(rm);
+      bool newl = false;
+      uint32_t rp0 = 0, deg = 0, du = INF;
+      if (a) {
+        const uint32_t bit = 1u << (sl & 31);
+        atomicAnd(&m.fin[sl >> 5], ~bit);  // re-queued if improved from here on
+        newl = !(atomicOr(&m.listed[sl >> 5], bit) & bit);
+        const uint32_t u = (uint32_t)(ent >> 32);
+        // re-read D after clearing the frontier bit (an improvement in between re-queues u)
+        du = (uint32_t)m.dtab[sl];
+        rp0 = g.rowptr[u];
+        deg = g.rowptr[u + 1] - rp0;
+      }
       const unsigned lm = __ballot_sync(FULL, newl);
       if (nx + __popc(lm) > cp.X) return OVERFLOW;
       if (newl) m.exl[nx + __popc(lm & lt)] = sl;
       nx += __popc(lm);
-    }
-    __syncwarp();
+      const unsigned am = __ballot_sync(FULL, a);
+      if (!am) continue;
+      c_vert += __popc(am);
 
-    // ---- 5. relax the active vertices' out-arcs, lane per arc ----------------------------
-    for (uint32_t b0 = 0; b0 < na; b0 += 32) {
-      const uint32_t i = b0 + lane;
-      uint32_t rp0 = 0, deg = 0, du = INF;
-      if (i < na) {
-        const unsigned long long ent = m.dtab[m.act[i]];
-        const uint32_t u = (uint32_t)(ent >> 32);
-        du = (uint32_t)ent;
-        rp0 = g.rowptr[u];
-        deg = g.rowptr[u + 1] - rp0;
-      }
       uint32_t x = deg;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
@@ -348,33 +361,51 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
         if (lane >= o) x += y;
       }
       const uint32_t total = __shfl_sync(FULL, x, 31);
-      m.scan[lane] = x;
-      m.rp[lane] = rp0;
-      m.du[lane] = du;
+      c_arcs += total;
+      const bool staged = total <= ARCMAX;
+      if (staged) {
+        // flatten the chunk's arcs: lane j writes its deg arcs at [x - deg, x)
+        for (uint32_t e = 0; e < deg; ++e) {
+          m.own_arc[x - deg + e] = rp0 + e;
+          m.own_du[x - deg + e] = du;
+        }
+      } else {
+        m.scan[lane] = x;
+        m.rp[lane] = rp0;
+        m.du[lane] = du;
+      }
       __syncwarp();
       for (uint32_t t0 = 0; t0 < total; t0 += 32) {
         const uint32_t t = t0 + lane;
         bool has = false, ovf = false;
         uint32_t slot = 0;
         if (t < total) {
-          int lo = 0, hi = 31;
-          while (lo < hi) {
-            const int mid = (lo + hi) >> 1;
-            if (m.scan[mid] > t) hi = mid; else lo = mid + 1;
+          uint32_t arc, dsrc;
+          if (staged) {
+            arc = m.own_arc[t];
+            dsrc = m.own_du[t];
+          } else {  // high-degree chunk: binary-search the owner of arc t
+            int lo = 0, hi = 31;
+            while (lo < hi) {
+              const int mid = (lo + hi) >> 1;
+              if (m.scan[mid] > t) hi = mid; else lo = mid + 1;
+            }
+            const uint32_t excl = lo ? m.scan[lo - 1] : 0;
+            arc = m.rp[lo] + (t - excl);
+            dsrc = m.du[lo];
           }
-          const uint32_t excl = lo ? m.scan[lo - 1] : 0;
-          const uint2 a = g.adj[m.rp[lo] + (t - excl)];
-          const unsigned long long nd = (unsigned long long)m.du[lo] + a.y;
+          const uint2 av = g.adj[arc];
+          const unsigned long long nd = (unsigned long long)dsrc + av.y;
           if (nd < INF) {
             bool imp;
-            const int r = tab_relax(m.dtab, hmask, a.x, (uint32_t)nd, imp);
-            if (r < 0) {
+            const int rr = tab_relax(m.dtab, hmask, av.x, (uint32_t)nd, imp);
+            if (rr < 0) {
               ovf = true;
             } else if (imp) {
-              const uint32_t bit = 1u << (r & 31);
-              if (!(atomicOr(&m.fin[r >> 5], bit) & bit)) {
+              const uint32_t bit = 1u << (rr & 31);
+              if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
                 has = true;
-                slot = (uint32_t)r;
+                slot = (uint32_t)rr;
               }
             }
           }
@@ -402,6 +433,13 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
     P.out_obj[(size_t)qi * k + r] = ok ? (uint32_t)dk : GGRID_PAD;
     P.out_dist[(size_t)qi * k + r] = ok ? (uint32_t)(dk >> 32) : GGRID_PAD;
   }
+  if (lane == 0) {
+    atomicAdd(&s.st->ex_iters, (unsigned long long)c_iter);
+    atomicAdd(&s.st->ex_vertices, (unsigned long long)c_vert);
+    atomicAdd(&s.st->ex_arcs, (unsigned long long)c_arcs);
+    atomicAdd(&s.st->ex_harvested, (unsigned long long)c_harv);
+    atomicAdd(&s.st->ex_objects, (unsigned long long)c_objs);
+  }
   return DONE;
 }
 
@@ -411,10 +449,13 @@ __global__ void k_expand(QParams P) {
   const uint32_t warp = threadIdx.x >> 5;
   const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
   const uint32_t gw = blockIdx.x * P.warps_per_cta + warp;
-  const uint32_t nwarps = gridDim.x * P.warps_per_cta;
   unsigned char* base = P.scratch ? P.scratch + (size_t)gw * wbytes : smem_raw + (size_t)warp * wbytes;
   const WarpMem m = carve(base, P.caps);
-  for (uint32_t li = gw; li < P.n; li += nwarps) {
+  for (;;) {  // persistent: queries fetched dynamically
+    uint32_t li = 0;
+    if (lane == 0) li = atomicAdd(&P.s.st->expand_work[P.level], 1u);
+    li = __shfl_sync(0xffffffffu, li, 0);
+    if (li >= P.n) break;
     const uint32_t qi = P.qlist ? P.qlist[li] : li;
     const int r = run_query(P, m, qi, lane);
     if (lane == 0 && r != DONE) {
@@ -430,29 +471,27 @@ __global__ void k_expand(QParams P) {
   }
 }
 
-// level 0: small balls (k <= 128), 4 warps per CTA in shared memory
-// level 1: large balls, 1 warp per CTA in shared memory
-// level 2: global-memory working set sized from |V| (fewer than k reachable objects, ...)
-constexpr int NLEVELS = 3;
-const Caps kCaps0 = {1024, 256, 256, 256};
-const Caps kCaps1 = {8192, 2048, 2048, 1024};
-constexpr uint32_t kWarps0 = 4, kWarps1 = 1, kWarps2 = 1;
+// Capacity ladder.  Levels 0-2 keep the warp's working set in shared memory (one warp per
+// CTA, as many CTAs per SM as fit); level 3 is global memory sized from |V| (a query that
+// reaches fewer than k objects may need to settle the whole graph).
+constexpr int NLEVELS = 4;
+const Caps kCaps[3] = {{1024, 256, 128, 64}, {2048, 512, 256, 256}, {16384, 4096, 4096, 2048}};
 
 Caps caps_for(int level, uint32_t V) {
-  if (level == 0) return kCaps0;
-  if (level == 1) return kCaps1;
-  uint32_t H = 1u << 14;
+  if (level < 3) return kCaps[level];
+  uint32_t H = 1u << 15;
   while (H < 2ull * V && H < (1u << 27)) H <<= 1;
   const uint32_t F = std::min<uint32_t>(H / 2, 1u << 22);
   return Caps{H, F, F, 8192};
 }
 
-bool g_attr_set[NLEVELS] = {false, false, false};
+bool g_attr_set = false;
+int g_blocks_per_sm[NLEVELS] = {0, 0, 0, 0};
 }  // namespace
 
 int expand_levels() { return NLEVELS; }
 
-uint32_t expand_max_k(int level) { return level == 0 ? 128 : (level == 1 ? 512 : 4096); }
+uint32_t expand_max_k(int level) { return caps_for(level, 1).C - 32; }
 
 size_t expand_warp_bytes(int level, uint32_t V) {
   const Caps c = caps_for(level, V);
@@ -462,7 +501,7 @@ size_t expand_warp_bytes(int level, uint32_t V) {
 void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
                    const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
                    uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist, void* scratch,
-                   uint32_t scratch_warps, cudaStream_t st) {
+                   uint32_t scratch_warps, int sm_count, cudaStream_t st) {
   if (n == 0) return;
   QParams P;
   P.g = g;
@@ -479,22 +518,25 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
   P.out_obj = out_obj;
   P.out_dist = out_dist;
   P.caps = caps_for(level, g.V);
+  P.warps_per_cta = 1;
   const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
-  if (level < 2) {
+  if (!g_attr_set) {
+    cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    g_attr_set = true;
+  }
+  if (level < NLEVELS - 1) {
     P.scratch = nullptr;
-    P.warps_per_cta = level == 0 ? kWarps0 : kWarps1;
-    const int smem = (int)(wbytes * P.warps_per_cta);
-    if (!g_attr_set[level]) {
-      cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-      g_attr_set[level] = true;
+    const int smem = (int)wbytes;
+    if (!g_blocks_per_sm[level]) {
+      int b = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand, 32, smem);
+      g_blocks_per_sm[level] = b > 0 ? b : 1;
     }
-    const uint32_t blocks = (n + P.warps_per_cta - 1) / P.warps_per_cta;
-    k_expand<<<blocks, 32 * P.warps_per_cta, smem, st>>>(P);
+    const uint32_t wave = (uint32_t)(sm_count * g_blocks_per_sm[level]);
+    k_expand<<<std::min<uint32_t>(n, wave), 32, smem, st>>>(P);
   } else {
     P.scratch = static_cast<unsigned char*>(scratch);
-    P.warps_per_cta = kWarps2;
-    const uint32_t blocks = std::min<uint32_t>((n + kWarps2 - 1) / kWarps2, std::max<uint32_t>(1, scratch_warps / kWarps2));
-    k_expand<<<blocks, 32 * kWarps2, 0, st>>>(P);
+    k_expand<<<std::min<uint32_t>(n, std::max<uint32_t>(1, scratch_warps)), 32, 0, st>>>(P);
   }
 }
 
