@@ -17,7 +17,7 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libggrid.so")
+LIB_PATH = os.environ.get("GGRID_LIB") or os.path.join(_PKG, "libggrid.so")
 
 GGRID_OK, GGRID_EINVAL, GGRID_ENOMEM, GGRID_ECUDA, GGRID_ENCCL, GGRID_EOVERFLOW = 0, -1, -2, -3, -4, -5
 PAD = 0xFFFFFFFF

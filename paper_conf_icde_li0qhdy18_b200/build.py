@@ -19,6 +19,11 @@ SOURCES = ["api.cu", "ingest.cu", "flush.cu", "knn.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUDE]
+# experiment hooks: extra nvcc flags and an alternative output path (default build unaffected)
+EXTRA = os.environ.get("GGRID_NVCC_FLAGS", "").split()
+if os.environ.get("GGRID_LIB_OUT"):
+    LIB = os.environ["GGRID_LIB_OUT"]
+    OBJDIR = LIB + ".objs"
 
 
 def _deps_mtime():
@@ -28,7 +33,7 @@ def _deps_mtime():
 
 def _compile(src: str, verbose: bool) -> str:
     obj = os.path.join(OBJDIR, src.replace(".cu", ".o"))
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
+    cmd = [NVCC, *ARCH, *FLAGS, *EXTRA, "-c", os.path.join(CSRC, src), "-o", obj]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -78,16 +78,28 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   return m;
 }
 
-__device__ __forceinline__ uint32_t vhash(uint32_t v) {
+#ifndef GG_HASH
+#define GG_HASH 2
+#endif
+#ifndef GG_H0
+#define GG_H0 1024
+#endif
+__device__ __forceinline__ uint32_t vhash(uint32_t v, uint32_t hmask) {
+#if GG_HASH == 1
+  return v;                                    // ids of a ball are Z-order clustered
+#elif GG_HASH == 2
+  return (v * 2654435761u) >> (32 - __popc(hmask));  // Fibonacci (high bits)
+#else
   uint32_t h = v * 2654435761u;
   return h ^ (h >> 15);
+#endif
 }
 
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
 __device__ __forceinline__ int tab_relax(unsigned long long* dtab, uint32_t hmask, uint32_t v,
                                          uint32_t d, bool& improved) {
   const unsigned long long nv = ((unsigned long long)v << 32) | d;
-  uint32_t sl = vhash(v) & hmask;
+  uint32_t sl = vhash(v, hmask) & hmask;
   volatile unsigned long long* vt = dtab;
 #pragma unroll 1
   for (int p = 0; p < MAXP; ++p) {
@@ -475,7 +487,7 @@ __global__ void k_expand(QParams P) {
 // CTA, as many CTAs per SM as fit); level 3 is global memory sized from |V| (a query that
 // reaches fewer than k objects may need to settle the whole graph).
 constexpr int NLEVELS = 4;
-const Caps kCaps[3] = {{1024, 256, 128, 64}, {2048, 512, 256, 256}, {16384, 4096, 4096, 2048}};
+const Caps kCaps[3] = {{GG_H0, 256, 128, 64}, {2048, 512, 256, 256}, {16384, 4096, 4096, 2048}};
 
 Caps caps_for(int level, uint32_t V) {
   if (level < 3) return kCaps[level];
