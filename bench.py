@@ -207,9 +207,16 @@ def run_ours(args, cfg_name):
     # ---- device-resident timed region -------------------------------------------------
     times = []
     st0 = None
+    from paper_conf_icde_li0qhdy18_b200 import dist as gdist
+
+    n_upd_step = cfg["n_objects"] * cfg["updates_per_object"]
     for s in range(args.warmup + args.steps):
-        u, q = step_inputs(s)
-        du = torch.from_numpy(u.view(np.int32)).to("cuda")
+        q = synth.queries(g, Q, seed=synth.SEED_QUERIES + 1000 * rank + s)
+        u = walk.ticks(cfg["updates_per_object"])  # every rank keeps the walk in step (untimed)
+        if rank == 0:  # the update stream arrives at rank 0 and is fanned out over NCCL
+            du = torch.from_numpy(u.view(np.int32)).to("cuda")
+        else:
+            du = torch.empty((n_upd_step, 4), dtype=torch.int32, device="cuda")
         dq = torch.from_numpy(q.view(np.int32)).to("cuda")
         with torch.cuda.stream(stream):
             l2.zero_()  # flush L2 between timed iterations (outside the events)
@@ -221,6 +228,9 @@ def run_ours(args, cfg_name):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
+        if world > 1:
+            with torch.cuda.stream(stream):
+                gdist.broadcast_updates(du, src=0)
         grid.ingest(du)
         grid.knn(dq, k, out_o, out_d)
         e1.record(stream)

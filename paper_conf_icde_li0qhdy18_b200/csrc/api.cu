@@ -163,7 +163,8 @@ struct ggrid_s {
 
   int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin) {
     CK(cudaMemsetAsync(&d_status->flush_work, 0, sizeof(unsigned int), stream));
-    launch(GGRID_K_FLUSH, [&] { launch_flush(g, s, out, out_top, begin, sm_count, stream); });
+    const uint32_t opc = (uint32_t)((h_status->n_live + n_cells - 1) / std::max(1u, n_cells));
+    launch(GGRID_K_FLUSH, [&] { launch_flush(g, s, out, out_top, begin, opc, sm_count, stream); });
     return GGRID_OK;
   }
 

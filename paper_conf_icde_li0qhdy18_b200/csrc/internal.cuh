@@ -121,8 +121,8 @@ void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int
 // Flush the cells flush_list[begin .. st->n_flush) writing compacted lists into `out`
 // (out == s.ar for a regular flush; a fresh arena for garbage collection).
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
-                  unsigned long long* out_top, uint32_t begin, int sm_count, cudaStream_t st);
-int flush_smem_bytes();
+                  unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
+                  int sm_count, cudaStream_t st);
 // Expansion (Alg. 5/6 semantics) for the queries qlist[0..n) at variant `level`.
 // Outcomes: answered (rows written), retried at the same level (retry_list, a needed cell
 // had cached updates) or promoted to the next level (promote_list, capacity overflow).
