@@ -41,9 +41,8 @@ METRIC = "kNN queries/sec incl. lazy flush at fixed update rate"
 
 # Algorithmic bytes per unit (restated in DESIGN.md §5)
 INGEST_BYTES_PER_UPDATE = 48          # 16 record + 4 arc->cell + 8 RED.MAX + 20 SoA write
-FLUSH_BYTES_PER_RECORD = 12           # obj + key
-FLUSH_BYTES_PER_WINNER = 12 + 8 + 24  # payload read + ot_key + compacted write
-FLUSH_BYTES_PER_VERTEX = 8            # v_obj index entry per vertex of a flushed cell
+FLUSH_BYTES_PER_RECORD = 12           # obj + key (ot_key match is an L1-resident gather)
+FLUSH_BYTES_PER_WINNER = 12 + 24 + 8 + 12  # payload read + compacted write + v_obj set + (next flush) clear
 # expansion: counted work (ggrid_stats expand_*), bytes each unit must move
 EXPAND_BYTES_PER_VERTEX = 8    # rowptr[u], rowptr[u+1]
 EXPAND_BYTES_PER_ARC = 8       # adj (dst, w)
@@ -262,7 +261,7 @@ def run_ours(args, cfg_name):
     expand_bytes = (dx["vertices"] * EXPAND_BYTES_PER_VERTEX + dx["arcs"] * EXPAND_BYTES_PER_ARC
                     + dx["harvested"] * EXPAND_BYTES_PER_HARVEST + dx["objects"] * EXPAND_BYTES_PER_OBJECT
                     + Q * K * (EXPAND_BYTES_PER_QUERY + 8 * k))
-    flush_bytes = rec * FLUSH_BYTES_PER_RECORD + win * FLUSH_BYTES_PER_WINNER + cells * cs * FLUSH_BYTES_PER_VERTEX
+    flush_bytes = rec * FLUSH_BYTES_PER_RECORD + win * FLUSH_BYTES_PER_WINNER
     kern = {
         "ingest": (ingest_ms, n_upd * K * INGEST_BYTES_PER_UPDATE,
                    kl["ingest_classify"] + kl["ingest_alloc"] + kl["ingest_scatter"]),

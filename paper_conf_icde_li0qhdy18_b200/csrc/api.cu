@@ -161,10 +161,10 @@ struct ggrid_s {
     return GGRID_OK;
   }
 
-  int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin) {
+  int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin, int full_vobj = 0) {
     CK(cudaMemsetAsync(&d_status->flush_work, 0, sizeof(unsigned int), stream));
     const uint32_t opc = (uint32_t)((h_status->n_live + n_cells - 1) / std::max(1u, n_cells));
-    launch(GGRID_K_FLUSH, [&] { launch_flush(g, s, out, out_top, begin, opc, sm_count, stream); });
+    launch(GGRID_K_FLUSH, [&] { launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, stream); });
     return GGRID_OK;
   }
 
@@ -200,7 +200,7 @@ int ggrid_s::gc() {
   epoch++;
   RC(set_status_u32(&d_status->n_flush, 0));
   launch(GGRID_K_OTHER, [&] { launch_mark_dirty(g, s, epoch, 1, stream); });
-  RC(flush_list_run(t, d_top, 0));
+  RC(flush_list_run(t, d_top, 0, /*full_vobj=*/1));
   unsigned long long top = 0;
   CK(cudaMemcpyAsync(&top, d_top, 8, cudaMemcpyDeviceToHost, stream));
   RC(sync());

@@ -221,7 +221,7 @@ __global__ void k_dump_cell(DevGraph g, DevState s, uint32_t c, uint32_t* obj, u
   uint32_t vb = c * g.cs;
   uint32_t ve = min(g.V, vb + g.cs);
   for (uint32_t v = vb + threadIdx.x; v < ve; v += blockDim.x) {
-    uint2 vo = s.v_obj[v];
+    uint2 vo = vobj_valid(s.v_obj[v], s.cell_comp[c]);
     for (uint32_t j = 0; j < vo.y; ++j) {
       uint32_t p = vo.x + j;
       uint32_t o = s.ar.obj[p];

@@ -122,7 +122,13 @@ void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int
 // (out == s.ar for a regular flush; a fresh arena for garbage collection).
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
-                  int sm_count, cudaStream_t st);
+                  int full_vobj, int sm_count, cudaStream_t st);
+
+// v_obj[v] = (start, n) is valid only if start lies inside the cell's current cleaned list
+// (lists only move up the arena between garbage collections, which rewrite every entry).
+__device__ __forceinline__ uint2 vobj_valid(uint2 vo, uint2 comp) {
+  return (vo.x >= comp.x && vo.x < comp.x + comp.y) ? vo : make_uint2(0, 0);
+}
 // Expansion (Alg. 5/6 semantics) for the queries qlist[0..n) at variant `level`.
 // Outcomes: answered (rows written), retried at the same level (retry_list, a needed cell
 // had cached updates) or promoted to the next level (promote_list, capacity overflow).

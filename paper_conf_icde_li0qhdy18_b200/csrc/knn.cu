@@ -242,7 +242,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       if (lane == 0) request_flush(s, c, P.epoch);
       return RETRY;
     }
-    const uint2 vo = s.v_obj[ei.x];
+    const uint2 vo = vobj_valid(s.v_obj[ei.x], s.cell_comp[c]);
     for (uint32_t j0 = 0; j0 < vo.y; j0 += 32) {
       const uint32_t j = j0 + lane;
       bool has = false;
@@ -292,7 +292,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
           dirty = true;
           request_flush(s, c, P.epoch);
         } else {
-          vo = s.v_obj[u];
+          vo = vobj_valid(s.v_obj[u], s.cell_comp[c]);
         }
       }
       if (__any_sync(FULL, dirty)) {

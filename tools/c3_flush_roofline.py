@@ -80,7 +80,7 @@ def main():
         rec = s1["records_flushed"] - s0["records_flushed"]
         win = s1["objects_written"] - s0["objects_written"]
         cells = s1["cells_flushed"] - s0["cells_flushed"]
-        alg = rec * 12 + win * 44 + cells * s1["cell_size"] * 8
+        alg = rec * 12 + win * 56  # DESIGN.md §4 (bench.py FLUSH_BYTES_*)
         rounds.append(dict(ingest_ms=ing_ms, flush_ms=s1["kernel_ms"]["flush"], rec=rec, win=win, cells=cells,
                            alg=alg, gc=s1["gc_runs"]))
     best = min(rounds, key=lambda x: x["flush_ms"])
