@@ -99,6 +99,9 @@ __device__ inline unsigned lanemask_lt() {
 // Request a flush of cell c in this knn epoch (deduplicated by the epoch stamp).
 __device__ inline void request_flush(const DevState& s, uint32_t c, uint32_t epoch) {
   if (s.cell_head[c] == NONE) return;
+  // plain read first: most requests of a batch hit an already-requested cell, so the
+  // contended atomic is only issued by the first few
+  if (*((volatile uint32_t*)&s.cell_req[c]) == epoch) return;
   if (atomicExch(&s.cell_req[c], epoch) != epoch) {
     unsigned i = atomicAdd(&s.st->n_flush, 1u);
     s.flush_list[i] = c;

@@ -13,8 +13,9 @@
 //     the distance).  Seeds follow reading R1 (d=0 -> D[src]=0, else D[dst]=w-d).
 //   * Each round walks the frontier in chunks of 32; the lanes whose D lies in the bucket
 //     [m, m+delta) (m = frontier minimum) relax their out-arcs lane-per-arc
-//     (warp-cooperative adjacency scan: a warp scan of the degrees, the chunk's arcs
-//     flattened into shared memory, one arc per lane).
+//     (warp-cooperative adjacency scan: a warp scan of the degrees flattens the chunk's
+//     arcs; each lane finds the owner of its arc with a start-bit mask, __fns and shuffles,
+//     no shared-memory staging).
 //   * Every vertex with D < m is final; its objects are harvested from the cell's cleaned
 //     list (v_obj index) as exact candidates dist = D[src(e_o)] + d_o (P@49436), objects on
 //     q's own arc ahead of q at d_o - d_q (reading R2), stale entries dropped by
@@ -34,7 +35,6 @@ namespace {
 
 enum { DONE = 0, RETRY = 1, OVERFLOW = 2 };
 constexpr int MAXP = 128;       // probe limit of the vertex table
-constexpr uint32_t ARCMAX = 128;  // flattened arcs per 32-vertex chunk (else binary search)
 
 struct Caps {
   uint32_t H, F, X, C;  // table slots (pow2), frontier, expanded list, candidates
@@ -49,15 +49,10 @@ struct WarpMem {
   uint32_t* exl;             // X
   uint32_t* fin;             // H/32
   uint32_t* listed;          // H/32
-  uint32_t* scan;            // 32
-  uint32_t* rp;              // 32
-  uint32_t* du;              // 32
-  uint32_t* own_arc;         // ARCMAX: arcs of the current chunk's active vertices
-  uint32_t* own_du;          // ARCMAX: D of each staged arc's source
 };
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 8ull * c.C + 4ull * (2ull * c.F + c.X + 2ull * (c.H / 32) + 96 + 2 * ARCMAX);
+  return 8ull * c.H + 8ull * c.C + 4ull * (2ull * c.F + c.X + 2ull * (c.H / 32));
 }
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
@@ -69,12 +64,7 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   m.front1 = p; p += c.F;
   m.exl = p; p += c.X;
   m.fin = p; p += c.H / 32;
-  m.listed = p; p += c.H / 32;
-  m.scan = p; p += 32;
-  m.rp = p; p += 32;
-  m.du = p; p += 32;
-  m.own_arc = p; p += ARCMAX;
-  m.own_du = p;
+  m.listed = p;
   return m;
 }
 
@@ -374,38 +364,26 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       }
       const uint32_t total = __shfl_sync(FULL, x, 31);
       c_arcs += total;
-      const bool staged = total <= ARCMAX;
-      if (staged) {
-        // flatten the chunk's arcs: lane j writes its deg arcs at [x - deg, x)
-        for (uint32_t e = 0; e < deg; ++e) {
-          m.own_arc[x - deg + e] = rp0 + e;
-          m.own_du[x - deg + e] = du;
-        }
-      } else {
-        m.scan[lane] = x;
-        m.rp[lane] = rp0;
-        m.du[lane] = du;
-      }
-      __syncwarp();
+      const uint32_t sj = x - deg;  // first flattened arc index of lane j's vertex
       for (uint32_t t0 = 0; t0 < total; t0 += 32) {
+        // owner of flattened arc t0+lane, without shared memory: the lanes whose arc range
+        // starts inside this window (bit mask by position, and by lane), plus the lane whose
+        // range covers the window start
+        const bool starts = deg != 0 && sj >= t0 && sj < t0 + 32;
+        const uint32_t smask = __reduce_or_sync(FULL, starts ? 1u << (sj - t0) : 0u);
+        const unsigned slanes = __ballot_sync(FULL, starts);
+        const unsigned before = __ballot_sync(FULL, deg != 0 && sj < t0);
+        const int carry_lane = before ? 31 - __clz(before) : 0;
         const uint32_t t = t0 + lane;
+        const int kth = __popc(smask & (0xffffffffu >> (31 - lane)));  // starts at or before t
+        const int owner = kth ? (int)__fns(slanes, 0, kth) : carry_lane;
+        const uint32_t o_rp = __shfl_sync(FULL, rp0, owner);
+        const uint32_t o_s = __shfl_sync(FULL, sj, owner);
+        const uint32_t dsrc = __shfl_sync(FULL, du, owner);
         bool has = false, ovf = false;
         uint32_t slot = 0;
         if (t < total) {
-          uint32_t arc, dsrc;
-          if (staged) {
-            arc = m.own_arc[t];
-            dsrc = m.own_du[t];
-          } else {  // high-degree chunk: binary-search the owner of arc t
-            int lo = 0, hi = 31;
-            while (lo < hi) {
-              const int mid = (lo + hi) >> 1;
-              if (m.scan[mid] > t) hi = mid; else lo = mid + 1;
-            }
-            const uint32_t excl = lo ? m.scan[lo - 1] : 0;
-            arc = m.rp[lo] + (t - excl);
-            dsrc = m.du[lo];
-          }
+          const uint32_t arc = o_rp + (t - o_s);
           const uint2 av = g.adj[arc];
           const unsigned long long nd = (unsigned long long)dsrc + av.y;
           if (nd < INF) {
