@@ -1,0 +1,107 @@
+"""Summarise a profiling pass (tools/profile_round.sh) into profiles/<tag>_*.
+
+    python tools/summarize_profiles.py r01
+
+Writes profiles/<tag>_summary.md (per-kernel ncu metrics, stall reasons, launch-list shares),
+profiles/<tag>_launches_C1.csv (the launch list), profiles/<tag>_<kernel>_raw.csv (ncu raw page
+of each full capture) and profiles/traffic_<cfg>.json (DRAM bytes per launch of each kernel,
+read by bench.py for the roofline `traffic` field).
+"""
+import collections
+import csv
+import json
+import os
+import shutil
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
+src = os.path.join(ROOT, "gpurun_out", f"prof_{tag}")
+dst = os.path.join(ROOT, "profiles")
+os.makedirs(dst, exist_ok=True)
+
+WANT = [
+    ("gpu__time_duration.sum", "duration"),
+    ("dram__bytes_read.sum", "DRAM read"),
+    ("dram__bytes_write.sum", "DRAM write"),
+    ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "DRAM throughput % of peak"),
+    ("lts__t_sector_hit_rate.pct", "L2 hit rate"),
+    ("l1tex__t_sector_hit_rate.pct", "L1 hit rate"),
+    ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps active % (achieved occupancy)"),
+    ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue slots busy %"),
+    ("smsp__inst_executed.sum", "warp instructions"),
+    ("launch__registers_per_thread", "registers/thread"),
+    ("launch__grid_size", "grid"),
+    ("launch__block_size", "block"),
+    ("launch__occupancy_limit_registers", "CTA limit (registers)"),
+    ("launch__occupancy_limit_shared_mem", "CTA limit (smem)"),
+]
+
+
+def raw_rows(path):
+    rows = list(csv.reader(open(path)))
+    hdr, units = rows[0], rows[1]
+    return [(hdr, units, r) for r in rows[2:]]
+
+
+lines = [f"# Profiling summary — round tag `{tag}`", "",
+         "Source: `tools/profile_round.sh` under gpurun on one B200 (ncu 2025, `--clock-control none`).",
+         "Raw pages: `profiles/%s_<capture>_raw.csv`; launch list: `profiles/%s_launches_C1.csv`." % (tag, tag), ""]
+traffic = {}
+for cap in ("expand_C1", "ingest_C1", "flush_C3"):
+    p = os.path.join(src, f"{cap}_raw.csv")
+    if not os.path.exists(p):
+        continue
+    shutil.copy(p, os.path.join(dst, f"{tag}_{cap}_raw.csv"))
+    for hdr, units, r in raw_rows(p):
+        name = r[hdr.index("Kernel Name")].split("(")[0]
+        lines.append(f"## `{name}` ({cap})")
+        lines.append("")
+        lines.append("| metric | value |")
+        lines.append("|---|---|")
+        for key, label in WANT:
+            if key in hdr:
+                i = hdr.index(key)
+                lines.append(f"| {label} (`{key}`) | {r[i]} {units[i]} |")
+        stalls = []
+        for i, k in enumerate(hdr):
+            if k.startswith("smsp__pcsamp_warps_issue_stalled_") and not k.endswith("_not_issued"):
+                try:
+                    stalls.append((float(r[i].replace(",", "")), k.replace("smsp__pcsamp_warps_issue_stalled_", "")))
+                except ValueError:
+                    pass
+        tot = sum(v for v, _ in stalls) or 1.0
+        top = ", ".join(f"{n} {100 * v / tot:.0f}%" for v, n in sorted(stalls, reverse=True)[:6])
+        lines.append(f"| warp stall samples (top) | {top} |")
+        lines.append("")
+        rd = float(r[hdr.index("dram__bytes_read.sum")].replace(",", ""))
+        wr = float(r[hdr.index("dram__bytes_write.sum")].replace(",", ""))
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+        rd *= scale.get(units[hdr.index("dram__bytes_read.sum")], 1)
+        wr *= scale.get(units[hdr.index("dram__bytes_write.sum")], 1)
+        kind = {"expand_C1": "expand", "ingest_C1": "ingest", "flush_C3": "flush"}[cap]
+        cfg = cap.split("_")[1]
+        traffic.setdefault(cfg, collections.defaultdict(float))[kind] += rd + wr
+
+ll = os.path.join(src, "launches_C1.csv")
+if os.path.exists(ll):
+    shutil.copy(ll, os.path.join(dst, f"{tag}_launches_C1.csv"))
+    rows = list(csv.reader(open(ll)))
+    hi = [i for i, r in enumerate(rows) if r and r[0] == "ID"][0]
+    h = rows[hi]
+    agg = collections.defaultdict(list)
+    for r in rows[hi + 1:]:
+        agg[r[h.index("Kernel Name")].split("(")[0]].append(float(r[h.index("Metric Value")].replace(",", "")))
+    tot = sum(sum(v) for k, v in agg.items() if "gg::" in k)
+    lines += ["## Launch list, default bench (C1), cold-cache serialised (`gpu__time_duration.sum`)", "",
+              "| kernel | launches | mean µs | share of library time |", "|---|---|---|---|"]
+    for k, v in sorted(agg.items(), key=lambda x: -sum(x[1])):
+        share = f"{100 * sum(v) / tot:.1f}%" if "gg::" in k else "(torch L2 flush, untimed)"
+        lines.append(f"| `{k}` | {len(v)} | {sum(v) / len(v) / 1e3:.1f} | {share} |")
+    lines.append("")
+
+open(os.path.join(dst, f"{tag}_summary.md"), "w").write("\n".join(lines) + "\n")
+for cfg, d in traffic.items():
+    # ingest capture holds 3 launches (classify, alloc, scatter) of one step: per-step bytes
+    json.dump({k: v for k, v in d.items()}, open(os.path.join(dst, f"traffic_{cfg}.json"), "w"), indent=1)
+print("\n".join(lines))
