@@ -177,8 +177,15 @@ def run_ours(args, cfg_name):
     if world > 1:
         import torch.distributed as dist
 
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        # one process per GPU over NCCL; BENCH_DIST_BACKEND=gloo lets the harness be exercised
+        # with several ranks sharing one GPU (a test mode, not a measurement)
+        backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")
+        dev_i = local % max(1, torch.cuda.device_count())
+        torch.cuda.set_device(dev_i)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev_i))
+        else:
+            dist.init_process_group(backend)
     else:
         torch.cuda.set_device(0)
     dev = torch.cuda.current_device()
