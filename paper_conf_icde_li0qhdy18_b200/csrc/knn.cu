@@ -366,17 +366,16 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       c_arcs += total;
       const uint32_t sj = x - deg;  // first flattened arc index of lane j's vertex
       for (uint32_t t0 = 0; t0 < total; t0 += 32) {
-        // owner of flattened arc t0+lane, without shared memory: the lanes whose arc range
-        // starts inside this window (bit mask by position, and by lane), plus the lane whose
-        // range covers the window start
-        const bool starts = deg != 0 && sj >= t0 && sj < t0 + 32;
-        const uint32_t smask = __reduce_or_sync(FULL, starts ? 1u << (sj - t0) : 0u);
-        const unsigned slanes = __ballot_sync(FULL, starts);
-        const unsigned before = __ballot_sync(FULL, deg != 0 && sj < t0);
-        const int carry_lane = before ? 31 - __clz(before) : 0;
+        // owner of flattened arc t = t0+lane without shared memory: the starts sj are
+        // non-decreasing over lanes, so the owner is the last lane with sj <= t (a lane after
+        // the owner starts at or past the owner's end); 5-step binary search over shuffles
         const uint32_t t = t0 + lane;
-        const int kth = __popc(smask & (0xffffffffu >> (31 - lane)));  // starts at or before t
-        const int owner = kth ? (int)__fns(slanes, 0, kth) : carry_lane;
+        int owner = 0;
+#pragma unroll
+        for (int step = 16; step >= 1; step >>= 1) {
+          const uint32_t sc = __shfl_sync(FULL, sj, owner + step);
+          if (sc <= t) owner += step;
+        }
         const uint32_t o_rp = __shfl_sync(FULL, rp0, owner);
         const uint32_t o_s = __shfl_sync(FULL, sj, owner);
         const uint32_t dsrc = __shfl_sync(FULL, du, owner);
