@@ -280,3 +280,88 @@ def test_c2_fla_k_sweep(gg):
     for k in (10, 20, 30, 40, 50):
         _assert_same(grid.knn(q, k), _oracle(g, upd, q, k, mode=oracle.EARLY), f"C2 k={k}")
     grid.close()
+
+
+# ------------------------------------------------------------ flush paths and bench config
+def test_flush_histogram_and_global_counter_paths(gg):
+    """cell_size > 4096 (per-vertex counters in global memory) and > 128 winners per cell
+    (counter + scan indexing instead of ranks)."""
+    g = synth.table_ii_graph("NY", scale=0.03)
+    upd = synth.RandomWalk(g, 3000, inject=True).ticks(6)
+    q = synth.queries(g, 200)
+    for cs in (5000, 2048):
+        grid = gg.GGrid(g, cs, max_objects=4096)
+        grid.ingest(upd)
+        _assert_same(grid.knn(q, 8), _oracle(g, upd, q, 8), f"cs={cs}")
+        grid.close()
+
+
+def test_flush_long_chains_and_overflow(gg):
+    """40 ingest batches without a query (chains longer than the 32-extent gather), and one
+    cell holding far more objects than the flush's winner staging (re-stream fallback)."""
+    g = synth.table_ii_graph("NY", scale=0.03)
+    grid = gg.GGrid(g, 64, max_objects=8192)
+    vcell = grid.vertex_cell()
+    # crowd 1500 objects onto the arcs leaving cell 0's vertices
+    hot = np.flatnonzero(vcell[g["src"]] == 0)
+    rng = np.random.default_rng(9)
+    n_hot = 1500
+    e = hot[rng.integers(0, len(hot), n_hot)].astype(np.uint32)
+    d = (rng.random(n_hot) * g["w"][e]).astype(np.uint32)
+    crowd = np.stack([np.arange(n_hot, dtype=np.uint32), e, d, np.zeros(n_hot, np.uint32)], 1)
+    walk = synth.RandomWalk(g, 600, obj_ids=np.arange(n_hot, n_hot + 600, dtype=np.uint32))
+    hist = [crowd]
+    grid.ingest(crowd)
+    for _ in range(40):
+        u = walk.tick()
+        hist.append(u)
+        grid.ingest(u)
+    allu = np.concatenate(hist)
+    q = synth.queries(g, 150)
+    q[:20, 0] = hot[:20]  # queries right at the crowded cell
+    q[:20, 1] = 0
+    _assert_same(grid.knn(q, 12), _oracle(g, allu, q, 12), "long chains + crowded cell")
+    grid.close()
+
+
+def test_bench_configuration_steady_state(gg):
+    """The launch configuration bench.py times (C1: NY graph, cell_size 1024, profile mode on a
+    caller stream, 1M updates + 10k queries per step): every query of the first step and 1,000
+    sampled queries of two further steps, bit-exact."""
+    import torch
+
+    g = synth.config_graph("C1")
+    walk = synth.RandomWalk(g, 10_000)
+    stream = torch.cuda.Stream()
+    grid = gg.GGrid(g, 1024, max_objects=10_000, profile=True, stream=stream.cuda_stream)
+    out_o = torch.empty((10_000, 10), dtype=torch.int32, device="cuda")
+    out_d = torch.empty((10_000, 10), dtype=torch.int32, device="cuda")
+    hist = []
+    for step in range(3):
+        u = walk.ticks(100)
+        hist.append(u)
+        q = synth.queries(g, 10_000, seed=synth.SEED_QUERIES + step)
+        grid.ingest(torch.from_numpy(u.view(np.int32)).cuda())
+        grid.knn(torch.from_numpy(q.view(np.int32)).cuda(), 10, out_o, out_d)
+        torch.cuda.synchronize()
+        go = out_o.cpu().numpy().view(np.uint32)
+        gd = out_d.cpu().numpy().view(np.uint32)
+        sel = np.arange(10_000) if step == 0 else np.random.default_rng(step).choice(10_000, 1000, replace=False)
+        ro, rd = _oracle(g, np.concatenate(hist), q[sel], 10)
+        _assert_same((go[sel], gd[sel]), (ro, rd), f"step {step}")
+    grid.close()
+
+
+def test_usa_shaped_sampled(gg):
+    """configs[3] shape at 1/10 scale (2.4M vertices, 5.8M arcs): 100k objects, 64 cached
+    updates each, 65,536 queries; 200 sampled rows against the oracle (EARLY) and 10 (FULL)."""
+    g = synth.table_ii_graph("USA", scale=0.1)
+    upd = synth.RandomWalk(g, 100_000).ticks(64)
+    grid = gg.GGrid(g, 1024, max_objects=100_000, log_capacity=8_000_000)
+    grid.ingest(upd)
+    q = synth.queries(g, 65536)
+    go, gd = grid.knn(q, 10)
+    sel = np.linspace(0, 65535, 200).astype(np.int64)
+    _assert_same((go[sel], gd[sel]), _oracle(g, upd, q[sel], 10, mode=oracle.EARLY), "USA/10 early")
+    _assert_same((go[sel[:10]], gd[sel[:10]]), _oracle(g, upd, q[sel[:10]], 10), "USA/10 full")
+    grid.close()
