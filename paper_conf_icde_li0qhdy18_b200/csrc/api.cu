@@ -325,23 +325,39 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   h->user_cell.resize(V);
   for (uint32_t v = 0; v < V; ++v) h->user_cell[v] = newid[v] / cell_size;
 
-  // ---- CSR over internal ids, inverted index (user edge -> src, w, dst)
+  // ---- CSR over internal ids, inverted index (user edge -> src, w, dst).  An arc of weight
+  // 2^32-1 can never lie on a path shorter than INF (R18), so it is left out of the CSR (its
+  // inverted-index entry stays: objects and queries on it are still valid locations).
+  constexpr uint32_t WMAX = 0xFFFFFFFFu;
   std::vector<uint32_t> rowptr((size_t)V + 1, 0);
-  for (uint32_t a = 0; a < A; ++a) rowptr[newid[gr->src[a]] + 1]++;
+  for (uint32_t a = 0; a < A; ++a)
+    if (gr->w[a] != WMAX) rowptr[newid[gr->src[a]] + 1]++;
   for (uint32_t v = 0; v < V; ++v) rowptr[v + 1] += rowptr[v];
-  std::vector<uint2> adj(A), einfo(A);
+  const uint32_t An = rowptr[V];
+  std::vector<uint2> adj(An), einfo(A);
   std::vector<uint32_t> edst(A);
   {
     std::vector<uint32_t> fill(rowptr.begin(), rowptr.end() - 1);
     uint64_t wsum = 0;
     for (uint32_t a = 0; a < A; ++a) {
       const uint32_t u = newid[gr->src[a]], v = newid[gr->dst[a]];
-      adj[fill[u]++] = make_uint2(v, gr->w[a]);
+      if (gr->w[a] != WMAX) adj[fill[u]++] = make_uint2(v, gr->w[a]);
       einfo[a] = make_uint2(u, gr->w[a]);
       edst[a] = v;
       wsum += gr->w[a];
     }
     h->delta = o.delta ? o.delta : (uint32_t)std::max<uint64_t>(1, A ? wsum / A : 1);
+  }
+  // ---- inline adjacency: 4 slots (dst, w) per vertex, one 32-byte record, so the expansion
+  // reads a vertex's arcs with one dependent load (road graphs: degree <= 4 almost always).
+  // w = 0: empty slot; a vertex with more than 4 arcs keeps 3 inline and slot 3 = (u, WMAX):
+  // "arcs 3.. of u are adj[rowptr[u]+3 .. rowptr[u+1])".
+  std::vector<uint2> vadj((size_t)V * 4, make_uint2(0, 0));
+  for (uint32_t u = 0; u < V; ++u) {
+    const uint32_t d = rowptr[u + 1] - rowptr[u];
+    const uint32_t inl = d <= 4 ? d : 3;
+    for (uint32_t j = 0; j < inl; ++j) vadj[(size_t)u * 4 + j] = adj[rowptr[u] + j];
+    if (d > 4) vadj[(size_t)u * 4 + 3] = make_uint2(u, WMAX);
   }
   // ---- cell adjacency (P@47172: c_i neighbours c_j if an arc goes from c_i to c_j)
   std::vector<uint64_t> cpairs;
@@ -360,22 +376,24 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
 
   // ---- device graph
   uint32_t *d_rowptr, *d_edst, *d_cptr, *d_cadj;
-  uint2 *d_adj, *d_einfo;
+  uint2 *d_adj, *d_einfo, *d_vadj;
   int rc;
   if ((rc = h->alloc(&d_rowptr, (size_t)V + 1, false))) return fail(rc);
-  if ((rc = h->alloc(&d_adj, A, false))) return fail(rc);
+  if ((rc = h->alloc(&d_adj, An, false))) return fail(rc);
+  if ((rc = h->alloc(&d_vadj, (size_t)V * 4, false))) return fail(rc);
   if ((rc = h->alloc(&d_einfo, A, false))) return fail(rc);
   if ((rc = h->alloc(&d_edst, A, false))) return fail(rc);
   if ((rc = h->alloc(&d_cptr, (size_t)h->n_cells + 1, false))) return fail(rc);
   if ((rc = h->alloc(&d_cadj, cadj.size(), false))) return fail(rc);
   if (cudaMemcpy(d_rowptr, rowptr.data(), rowptr.size() * 4, cudaMemcpyHostToDevice) ||
-      cudaMemcpy(d_adj, adj.data(), (size_t)A * 8, cudaMemcpyHostToDevice) ||
+      (An && cudaMemcpy(d_adj, adj.data(), (size_t)An * 8, cudaMemcpyHostToDevice)) ||
+      cudaMemcpy(d_vadj, vadj.data(), vadj.size() * 8, cudaMemcpyHostToDevice) ||
       cudaMemcpy(d_einfo, einfo.data(), (size_t)A * 8, cudaMemcpyHostToDevice) ||
       cudaMemcpy(d_edst, edst.data(), (size_t)A * 4, cudaMemcpyHostToDevice) ||
       cudaMemcpy(d_cptr, cptr.data(), cptr.size() * 4, cudaMemcpyHostToDevice) ||
       (cadj.size() && cudaMemcpy(d_cadj, cadj.data(), cadj.size() * 4, cudaMemcpyHostToDevice)))
     return fail(GGRID_ECUDA);
-  h->g = DevGraph{V, A, cell_size, h->n_cells, h->delta, d_rowptr, d_adj, d_einfo, d_edst, d_cptr, d_cadj};
+  h->g = DevGraph{V, A, cell_size, h->n_cells, h->delta, d_rowptr, d_adj, d_einfo, d_edst, d_cptr, d_cadj, d_vadj};
 
   // ---- dynamic state
   DevState& s = h->s;

@@ -57,6 +57,8 @@ struct DevGraph {
   const uint32_t* edst;      // [A]  user edge -> internal dst
   const uint32_t* cadj_ptr;  // [n_cells+1] cell adjacency (P@47172)
   const uint32_t* cadj;
+  const uint2* vadj;         // [4V] inline adjacency: up to 4 (dst, w) per vertex; w=0 empty,
+                             //      w=2^32-1: arcs 3.. of the vertex are in the CSR above
 };
 
 struct Arena {  // SoA record arena

@@ -10,20 +10,23 @@
 //
 //   * D lives in a per-warp shared-memory open-addressing table keyed by vertex; one
 //     64-bit word (v<<32 | dist) so relaxation is a single atomicMin (same key => min on
-//     the distance).  Seeds follow reading R1 (d=0 -> D[src]=0, else D[dst]=w-d).
-//   * Each round walks the frontier in chunks of 32; the lanes whose D lies in the bucket
-//     [m, m+delta) (m = frontier minimum) relax their out-arcs lane-per-arc
-//     (warp-cooperative adjacency scan: a warp scan of the degrees flattens the chunk's
-//     arcs; each lane finds the owner of its arc with a start-bit mask, __fns and shuffles,
-//     no shared-memory staging).
-//   * Every vertex with D < m is final; its objects are harvested from the cell's cleaned
-//     list (v_obj index) as exact candidates dist = D[src(e_o)] + d_o (P@49436), objects on
-//     q's own arc ahead of q at d_o - d_q (reading R2), stale entries dropped by
-//     key == ot_key.  Harvesting a vertex of a cell with cached updates requests that cell's
-//     flush and the query is retried next round (lazy cleaning, Alg. 4 lines 2-4).
-//   * Stop once k candidates have dist < m (every unharvested object is >= m): this is
-//     Def. 3's unresolved-vertex rule taken inclusively (reading R13) and Alg. 6's refinement
-//     fused into the same expansion.  Output: k smallest (dist<<32 | obj) (readings R5, R6).
+//     the distance), issued only when it improves.  Seeds follow reading R1 (d=0 ->
+//     D[src]=0, else D[dst]=w-d).
+//   * Each round walks the frontier in chunks of 32; the vertices whose D lies in the bucket
+//     [m, m+delta) (m = frontier minimum) are expanded 8 per window, lane = (vertex, slot):
+//     each lane reads one arc of its vertex's 32-byte inline adjacency record (graph grid,
+//     csrc/api.cu) — one dependent load per round, no degree scan.
+//   * A vertex's objects are harvested the first time it is expanded (its cell's cleaned
+//     list through the v_obj index, in the same memory round as its arcs) and kept as
+//     (D-table slot, offset, object): a candidate's distance D[src(e_o)] + d_o (P@49436) is
+//     re-read from the table when needed, so it is exact once the vertex is settled.
+//     Objects on q's own arc ahead of q are at d_o - d_q (reading R2); stale entries are
+//     dropped by key == ot_key.  Harvesting a vertex of a cell with cached updates requests
+//     that cell's flush and the query is retried next round (lazy cleaning, Alg. 4 l.2-4).
+//   * Stop once k candidates have dist < m (every object not yet harvested, or at an
+//     unsettled vertex, is >= m): Def. 3's unresolved-vertex rule taken inclusively
+//     (reading R13) and Alg. 6's refinement fused into the same expansion.  Output: the k
+//     smallest (dist<<32 | obj) (readings R5, R6).
 // Capacities are per variant ("level"); a query that overflows one is retried on the next.
 #include <algorithm>
 
@@ -34,25 +37,28 @@ namespace gg {
 namespace {
 
 enum { DONE = 0, RETRY = 1, OVERFLOW = 2 };
-constexpr int MAXP = 128;       // probe limit of the vertex table
+constexpr int MAXP = 128;                  // probe limit of the vertex table
+constexpr uint32_t SPECIAL = 0xFFFFFFFFu;  // candidate slot of a same-arc object
+constexpr uint32_t WMAX = 0xFFFFFFFFu;     // inline-adjacency overflow marker
 
 struct Caps {
-  uint32_t H, F, X, C;  // table slots (pow2), frontier, expanded list, candidates
+  uint32_t H, F, C;  // table slots (pow2), frontier, candidates
 };
 
 // byte layout of one warp's working memory
 struct WarpMem {
-  unsigned long long* dtab;  // H
-  unsigned long long* cand;  // C
+  unsigned long long* dtab;  // H: (v<<32 | D)
+  unsigned long long* cand;  // C: (slot<<32 | offset); at the end (dist<<32 | obj)
+  uint32_t* cobj;            // C: object ids
   uint32_t* front0;          // F
   uint32_t* front1;          // F
-  uint32_t* exl;             // X
-  uint32_t* fin;             // H/32
-  uint32_t* listed;          // H/32
+  uint32_t* fin;             // H/32: slot is in the frontier
+  uint32_t* listed;          // H/32: vertex expanded at least once (objects harvested)
+  uint32_t* act;             // 32: active slots of the current frontier chunk
 };
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 8ull * c.C + 4ull * (2ull * c.F + c.X + 2ull * (c.H / 32));
+  return 8ull * c.H + 12ull * c.C + 4ull * (2ull * c.F + 2ull * (c.H / 32) + 32);
 }
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
@@ -60,29 +66,19 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   m.dtab = reinterpret_cast<unsigned long long*>(base);
   m.cand = m.dtab + c.H;
   uint32_t* p = reinterpret_cast<uint32_t*>(m.cand + c.C);
+  m.cobj = p; p += c.C;
   m.front0 = p; p += c.F;
   m.front1 = p; p += c.F;
-  m.exl = p; p += c.X;
   m.fin = p; p += c.H / 32;
-  m.listed = p;
+  m.listed = p; p += c.H / 32;
+  m.act = p;
   return m;
 }
 
-#ifndef GG_HASH
-#define GG_HASH 2
-#endif
-#ifndef GG_H0
-#define GG_H0 1024
-#endif
+// Fibonacci hashing (high bits): ball vertex ids are Z-order clustered, so low-bit or
+// identity hashing makes long probe runs
 __device__ __forceinline__ uint32_t vhash(uint32_t v, uint32_t hmask) {
-#if GG_HASH == 1
-  return v;                                    // ids of a ball are Z-order clustered
-#elif GG_HASH == 2
-  return (v * 2654435761u) >> (32 - __popc(hmask));  // Fibonacci (high bits)
-#else
-  uint32_t h = v * 2654435761u;
-  return h ^ (h >> 15);
-#endif
+  return (v * 2654435761u) >> (32 - __popc(hmask));
 }
 
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
@@ -160,18 +156,25 @@ struct QParams {
   uint32_t warps_per_cta;
 };
 
-// Append one ballot's worth of candidates; when full, keep only the k best so far (a
-// dropped candidate has >= k better ones, so it can never be in the answer).
-__device__ __forceinline__ bool cand_push(const WarpMem& m, uint32_t& nc, uint32_t C, uint32_t k,
-                                          bool has, unsigned long long dk, int lane, unsigned lt) {
+// current distance of candidate i (exact once its source vertex is settled)
+__device__ __forceinline__ unsigned long long cand_dist(const WarpMem& m, uint32_t i) {
+  const unsigned long long a = m.cand[i];
+  const uint32_t slot = (uint32_t)(a >> 32), off = (uint32_t)a;
+  if (slot == SPECIAL) return off;
+  return (unsigned long long)(uint32_t)m.dtab[slot] + off;
+}
+
+// Append one ballot's worth of candidates (false: capacity exceeded)
+__device__ __forceinline__ bool cand_push(const WarpMem& m, uint32_t& nc, uint32_t C, bool has,
+                                          uint32_t slot, uint32_t off, uint32_t obj, unsigned lt) {
   const unsigned hm = __ballot_sync(0xffffffffu, has);
   if (!hm) return true;
-  if (nc + __popc(hm) > C) {
-    warp_sort(m.cand, nc, C, lane);
-    nc = min(nc, k);
-    if (nc + __popc(hm) > C) return false;
+  if (nc + __popc(hm) > C) return false;
+  if (has) {
+    const uint32_t i = nc + __popc(hm & lt);
+    m.cand[i] = ((unsigned long long)slot << 32) | off;
+    m.cobj[i] = obj;
   }
-  if (has) m.cand[nc + __popc(hm & lt)] = dk;
   nc += __popc(hm);
   return true;
 }
@@ -216,7 +219,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   }
   uint32_t* front = m.front0;
   uint32_t* nfront = m.front1;
-  uint32_t nf = 1, nx = 0, nc = 0;
+  uint32_t nf = 1, nc = 0;
   if (lane == 0) {
     bool imp;
     const int sl = tab_relax(m.dtab, hmask, seed_v, seed_d, imp);
@@ -236,17 +239,17 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
     for (uint32_t j0 = 0; j0 < vo.y; j0 += 32) {
       const uint32_t j = j0 + lane;
       bool has = false;
-      unsigned long long dk = 0;
+      uint32_t ob = 0, dd = 0;
       if (j < vo.y) {
         const uint32_t p = vo.x + j;
-        const uint32_t ob = s.ar.obj[p];
+        ob = s.ar.obj[p];
         const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
         if (oe == q.x && oo >= q.y && s.ar.key[p] == s.ot_key[ob]) {
           has = true;
-          dk = ((unsigned long long)(oo - q.y) << 32) | ob;
+          dd = oo - q.y;
         }
       }
-      if (!cand_push(m, nc, cp.C, k, has, dk, lane, lt)) return OVERFLOW;
+      if (!cand_push(m, nc, cp.C, has, SPECIAL, dd, ob, lt)) return OVERFLOW;
     }
     __syncwarp();
   }
@@ -258,73 +261,17 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
     // ---- 1. frontier minimum: every vertex with D < m is final -------------------------
     uint32_t ml = INF;
     for (uint32_t i = lane; i < nf; i += 32) ml = min(ml, (uint32_t)m.dtab[front[i]]);
-    const uint32_t mn = __reduce_min_sync(FULL, ml);
-    const uint32_t blo = nf ? mn : INF;
+    const uint32_t blo = nf ? __reduce_min_sync(FULL, ml) : INF;
 
-    // ---- 2. harvest the objects of the newly final vertices -----------------------------
-    uint32_t keep = 0;
-    for (uint32_t b0 = 0; b0 < nx; b0 += 32) {
-      const uint32_t i = b0 + lane;
-      const uint32_t sl = i < nx ? m.exl[i] : NONE;
-      const unsigned long long ent = sl != NONE ? m.dtab[sl] : EMPTY64;
-      const uint32_t d = (uint32_t)ent, u = (uint32_t)(ent >> 32);
-      const bool take = sl != NONE && (nf == 0 || d < blo);
-      const bool stay = sl != NONE && !take;
-      const unsigned smk = __ballot_sync(FULL, stay);
-      __syncwarp();
-      if (stay) m.exl[keep + __popc(smk & lt)] = sl;
-      keep += __popc(smk);
-      uint2 vo = make_uint2(0, 0);
-      bool dirty = false;
-      if (take) {
-        const uint32_t c = cell_of(u, g.cs);
-        if (s.cell_head[c] != NONE) {
-          dirty = true;
-          request_flush(s, c, P.epoch);
-        } else {
-          vo = vobj_valid(s.v_obj[u], s.cell_comp[c]);
-        }
-      }
-      if (__any_sync(FULL, dirty)) {
-        request_lookahead(P, m, front, nf, lane);
-        return RETRY;
-      }
-      c_harv += __popc(__ballot_sync(FULL, take));
-      const uint32_t most = __reduce_max_sync(FULL, vo.y);
-      if (most == 0) continue;
-      c_objs += __reduce_add_sync(FULL, vo.y);
-      for (uint32_t j = 0; j < most; ++j) {
-        bool has = false;
-        unsigned long long dk = 0;
-        if (j < vo.y) {
-          const uint32_t p = vo.x + j;
-          const uint32_t ob = s.ar.obj[p];
-          const unsigned long long kk = s.ar.key[p];
-          const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
-          const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
-          if (!same_ahead && kk == s.ot_key[ob]) {
-            const unsigned long long dd = (unsigned long long)d + oo;
-            if (dd < INF) {
-              has = true;
-              dk = (dd << 32) | ob;
-            }
-          }
-        }
-        if (!cand_push(m, nc, cp.C, k, has, dk, lane, lt)) return OVERFLOW;
-      }
-    }
-    nx = keep;
-    __syncwarp();
-
-    // ---- 3. termination: k candidates strictly closer than any unharvested object -------
+    // ---- 2. termination: k candidates strictly closer than anything not yet final -------
     if (nf == 0) break;
     if (nc >= k) {
       uint32_t cl = 0;
-      for (uint32_t i = lane; i < nc; i += 32) cl += (uint32_t)(m.cand[i] >> 32) < blo;
+      for (uint32_t i = lane; i < nc; i += 32) cl += cand_dist(m, i) < blo;
       if (__reduce_add_sync(FULL, cl) >= k) break;
     }
 
-    // ---- 4+5. walk the frontier; relax the out-arcs of the bucket [m, m + delta) ---------
+    // ---- 3. walk the frontier; expand the bucket [m, m + delta) -------------------------
     const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
     uint32_t nn = 0;
     for (uint32_t b0 = 0; b0 < nf; b0 += 32) {
@@ -336,76 +283,134 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       const unsigned rm = __ballot_sync(FULL, r);
       if (r) nfront[nn + __popc(rm & lt)] = sl;
       nn += __popc(rm);
-      bool newl = false;
-      uint32_t rp0 = 0, deg = 0, du = INF;
-      if (a) {
-        const uint32_t bit = 1u << (sl & 31);
-        atomicAnd(&m.fin[sl >> 5], ~bit);  // re-queued if improved from here on
-        newl = !(atomicOr(&m.listed[sl >> 5], bit) & bit);
-        const uint32_t u = (uint32_t)(ent >> 32);
-        // re-read D after clearing the frontier bit (an improvement in between re-queues u)
-        du = (uint32_t)m.dtab[sl];
-        rp0 = g.rowptr[u];
-        deg = g.rowptr[u + 1] - rp0;
-      }
-      const unsigned lm = __ballot_sync(FULL, newl);
-      if (nx + __popc(lm) > cp.X) return OVERFLOW;
-      if (newl) m.exl[nx + __popc(lm & lt)] = sl;
-      nx += __popc(lm);
       const unsigned am = __ballot_sync(FULL, a);
       if (!am) continue;
-      c_vert += __popc(am);
-
-      uint32_t x = deg;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, x, o);
-        if (lane >= o) x += y;
+      if (a) {
+        m.act[__popc(am & lt)] = sl;
+        atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));  // re-queued if improved from here on
       }
-      const uint32_t total = __shfl_sync(FULL, x, 31);
-      c_arcs += total;
-      const uint32_t sj = x - deg;  // first flattened arc index of lane j's vertex
-      for (uint32_t t0 = 0; t0 < total; t0 += 32) {
-        // owner of flattened arc t = t0+lane without shared memory: the starts sj are
-        // non-decreasing over lanes, so the owner is the last lane with sj <= t (a lane after
-        // the owner starts at or past the owner's end); 5-step binary search over shuffles
-        const uint32_t t = t0 + lane;
-        int owner = 0;
-#pragma unroll
-        for (int step = 16; step >= 1; step >>= 1) {
-          const uint32_t sc = __shfl_sync(FULL, sj, owner + step);
-          if (sc <= t) owner += step;
+      __syncwarp();
+      const uint32_t na = __popc(am);
+      c_vert += na;
+      // 8 vertices per window, lane = (vertex, arc slot)
+      for (uint32_t w0 = 0; w0 < na; w0 += 8) {
+        const uint32_t vi = w0 + (lane >> 2), s4 = lane & 3;
+        const bool vv = vi < na;
+        uint32_t vslot = 0, u = 0, du = INF;
+        uint2 arc = make_uint2(0, 0);
+        if (vv) {
+          vslot = m.act[vi];
+          const unsigned long long e2 = m.dtab[vslot];  // D re-read after the frontier bit
+          u = (uint32_t)(e2 >> 32);
+          du = (uint32_t)e2;
+          arc = g.vadj[(size_t)u * 4 + s4];
         }
-        const uint32_t o_rp = __shfl_sync(FULL, rp0, owner);
-        const uint32_t o_s = __shfl_sync(FULL, sj, owner);
-        const uint32_t dsrc = __shfl_sync(FULL, du, owner);
+        // first expansion of the vertex: its objects (same memory round as its arcs)
+        bool harv = false, dirty = false;
+        uint2 vo = make_uint2(0, 0);
+        if (vv && s4 == 0) {
+          const uint32_t bit = 1u << (vslot & 31);
+          if (!(atomicOr(&m.listed[vslot >> 5], bit) & bit)) {
+            harv = true;
+            const uint32_t c = cell_of(u, g.cs);
+            const uint32_t hd = s.cell_head[c];
+            const uint2 cc = s.cell_comp[c];
+            const uint2 v0 = s.v_obj[u];
+            if (hd != NONE) {
+              dirty = true;
+              request_flush(s, c, P.epoch);
+            } else {
+              vo = vobj_valid(v0, cc);
+            }
+          }
+        }
+        if (__any_sync(FULL, dirty)) {
+          request_lookahead(P, m, front, nf, lane);
+          return RETRY;
+        }
+        c_harv += __popc(__ballot_sync(FULL, harv));
+        // relax the inline arc
         bool has = false, ovf = false;
-        uint32_t slot = 0;
-        if (t < total) {
-          const uint32_t arc = o_rp + (t - o_s);
-          const uint2 av = g.adj[arc];
-          const unsigned long long nd = (unsigned long long)dsrc + av.y;
+        uint32_t nslot = 0;
+        const bool overflow_arcs = arc.y == WMAX;
+        if (arc.y != 0 && !overflow_arcs) {
+          const unsigned long long nd = (unsigned long long)du + arc.y;
           if (nd < INF) {
             bool imp;
-            const int rr = tab_relax(m.dtab, hmask, av.x, (uint32_t)nd, imp);
+            const int rr = tab_relax(m.dtab, hmask, arc.x, (uint32_t)nd, imp);
             if (rr < 0) {
               ovf = true;
             } else if (imp) {
               const uint32_t bit = 1u << (rr & 31);
               if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
                 has = true;
-                slot = (uint32_t)rr;
+                nslot = (uint32_t)rr;
               }
             }
           }
         }
+        c_arcs += __popc(__ballot_sync(FULL, arc.y != 0 && !overflow_arcs));
         if (__any_sync(FULL, ovf)) return OVERFLOW;
-        const unsigned hm = __ballot_sync(FULL, has);
+        unsigned hm = __ballot_sync(FULL, has);
         if (nn + __popc(hm) > cp.F) return OVERFLOW;
-        if (has) nfront[nn + __popc(hm & lt)] = slot;
+        if (has) nfront[nn + __popc(hm & lt)] = nslot;
         nn += __popc(hm);
+        // vertices with more than 4 arcs: the rest live in the CSR (rare on road graphs)
+        if (__any_sync(FULL, overflow_arcs)) {
+          uint32_t a0 = 0, a1 = 0;
+          if (overflow_arcs) {
+            a0 = g.rowptr[u] + 3;
+            a1 = g.rowptr[u + 1];
+          }
+          const uint32_t most = __reduce_max_sync(FULL, a1 - a0);
+          for (uint32_t j = 0; j < most; ++j) {
+            has = false;
+            ovf = false;
+            if (a0 + j < a1) {
+              const uint2 av = g.adj[a0 + j];
+              const unsigned long long nd = (unsigned long long)du + av.y;
+              if (nd < INF) {
+                bool imp;
+                const int rr = tab_relax(m.dtab, hmask, av.x, (uint32_t)nd, imp);
+                if (rr < 0) {
+                  ovf = true;
+                } else if (imp) {
+                  const uint32_t bit = 1u << (rr & 31);
+                  if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+                    has = true;
+                    nslot = (uint32_t)rr;
+                  }
+                }
+              }
+            }
+            c_arcs += __popc(__ballot_sync(FULL, a0 + j < a1));
+            if (__any_sync(FULL, ovf)) return OVERFLOW;
+            hm = __ballot_sync(FULL, has);
+            if (nn + __popc(hm) > cp.F) return OVERFLOW;
+            if (has) nfront[nn + __popc(hm & lt)] = nslot;
+            nn += __popc(hm);
+          }
+        }
+        // harvest the objects of the vertices expanded for the first time
+        const uint32_t most = __reduce_max_sync(FULL, vo.y);
+        if (most) {
+          c_objs += __reduce_add_sync(FULL, vo.y);
+          for (uint32_t j = 0; j < most; ++j) {
+            bool hc = false;
+            uint32_t ob = 0, oo = 0;
+            if (j < vo.y) {
+              const uint32_t p = vo.x + j;
+              ob = s.ar.obj[p];
+              const unsigned long long kk = s.ar.key[p];
+              const uint32_t oe = s.ar.edge[p];
+              oo = s.ar.off[p];
+              const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
+              hc = !same_ahead && kk == s.ot_key[ob];
+            }
+            if (!cand_push(m, nc, cp.C, hc, vslot, oo, ob, lt)) return OVERFLOW;
+          }
+        }
       }
-      __syncwarp();
     }
     uint32_t* tmp = front;
     front = nfront;
@@ -414,11 +419,16 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
     __syncwarp();
   }
 
-  // ---- 6. the k smallest (dist, obj) ------------------------------------------------------
+  // ---- 4. the k smallest (dist, obj) ------------------------------------------------------
+  for (uint32_t i = lane; i < nc; i += 32) {
+    const unsigned long long d = cand_dist(m, i);
+    m.cand[i] = d < INF ? ((d << 32) | m.cobj[i]) : EMPTY64;
+  }
+  __syncwarp();
   warp_sort(m.cand, nc, cp.C, lane);
   for (uint32_t r = lane; r < k; r += 32) {
-    const bool ok = r < nc;
-    const unsigned long long dk = ok ? m.cand[r] : EMPTY64;
+    const unsigned long long dk = r < nc ? m.cand[r] : EMPTY64;
+    const bool ok = dk != EMPTY64;
     P.out_obj[(size_t)qi * k + r] = ok ? (uint32_t)dk : GGRID_PAD;
     P.out_dist[(size_t)qi * k + r] = ok ? (uint32_t)(dk >> 32) : GGRID_PAD;
   }
@@ -464,14 +474,14 @@ __global__ void k_expand(QParams P) {
 // CTA, as many CTAs per SM as fit); level 3 is global memory sized from |V| (a query that
 // reaches fewer than k objects may need to settle the whole graph).
 constexpr int NLEVELS = 4;
-const Caps kCaps[3] = {{GG_H0, 256, 128, 64}, {2048, 512, 256, 256}, {16384, 4096, 4096, 2048}};
+const Caps kCaps[3] = {{1024, 256, 64}, {2048, 512, 256}, {16384, 4096, 2048}};
 
 Caps caps_for(int level, uint32_t V) {
   if (level < 3) return kCaps[level];
   uint32_t H = 1u << 15;
   while (H < 2ull * V && H < (1u << 27)) H <<= 1;
   const uint32_t F = std::min<uint32_t>(H / 2, 1u << 22);
-  return Caps{H, F, F, 8192};
+  return Caps{H, F, 8192};
 }
 
 bool g_attr_set = false;
