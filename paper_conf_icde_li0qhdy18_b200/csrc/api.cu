@@ -393,7 +393,10 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
       cudaMemcpy(d_cptr, cptr.data(), cptr.size() * 4, cudaMemcpyHostToDevice) ||
       (cadj.size() && cudaMemcpy(d_cadj, cadj.data(), cadj.size() * 4, cudaMemcpyHostToDevice)))
     return fail(GGRID_ECUDA);
-  h->g = DevGraph{V, A, cell_size, h->n_cells, h->delta, d_rowptr, d_adj, d_einfo, d_edst, d_cptr, d_cadj, d_vadj};
+  uint32_t cs_mul, cs_shift;
+  fastdiv_params(cell_size, cs_mul, cs_shift);
+  h->g = DevGraph{V,      A,       cell_size, h->n_cells, h->delta, cs_mul, cs_shift, d_rowptr,
+                  d_adj,  d_einfo, d_edst,    d_cptr,     d_cadj,   d_vadj};
 
   // ---- dynamic state
   DevState& s = h->s;

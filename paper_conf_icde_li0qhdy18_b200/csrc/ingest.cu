@@ -56,7 +56,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
       atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
       continue;
     }
-    const uint32_t c = cell_of(e.x, g.cs);
+    const uint32_t c = cellof(g, e.x);
     uint32_t h = (c * 2654435761u) >> 20;  // 12 bits
     volatile uint32_t* vc = h_cell;
     for (;;) {
@@ -138,7 +138,7 @@ __global__ void __launch_bounds__(256) k_ingest_scatter(const uint4* __restrict_
   if (i >= n) return;
   uint4 m = upd[i];
   uint2 vr = tmp[i];
-  uint32_t pos = s.bbase[cell_of(vr.x, g.cs)] + vr.y;
+  uint32_t pos = s.bbase[cellof(g, vr.x)] + vr.y;
   unsigned long long key = ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
   s.ar.obj[pos] = m.x;
   s.ar.key[pos] = key;
@@ -179,12 +179,12 @@ __global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint3
     atomicOr(&s.st->err, (unsigned)ERR_QUERY);
     return;
   }
-  uint32_t c = cell_of(e.x, g.cs);
+  uint32_t c = cellof(g, e.x);
   request_flush(s, c, epoch);
   if (neighbors) {
     for (uint32_t j = g.cadj_ptr[c]; j < g.cadj_ptr[c + 1]; ++j) request_flush(s, g.cadj[j], epoch);
   } else {
-    request_flush(s, cell_of(g.edst[qq.x], g.cs), epoch);
+    request_flush(s, cellof(g, g.edst[qq.x]), epoch);
   }
 }
 

@@ -51,6 +51,7 @@ struct DevStatus {
 
 struct DevGraph {
   uint32_t V, A, cs, n_cells, delta;
+  uint32_t cs_mul, cs_shift;  // v / cs by multiply-high (cs_mul = 0: cs is 2^cs_shift)
   const uint32_t* rowptr;    // [V+1] out-arc CSR by internal source
   const uint2* adj;          // [A]  (internal dst, w) in CSR order
   const uint2* einfo;        // [A]  user edge -> (internal src, w)
@@ -91,6 +92,26 @@ struct DevState {
 };
 
 __host__ __device__ inline uint32_t cell_of(uint32_t v, uint32_t cs) { return v / cs; }
+
+// cell(v) = v / cell_size without a hardware divide (Granlund-Montgomery round-up multiplier;
+// exact for every 32-bit v, checked against v / d in tests/test_abi.py's reference of it)
+inline void fastdiv_params(uint32_t d, uint32_t& mul, uint32_t& shift) {
+  if ((d & (d - 1)) == 0) {
+    mul = 0;
+    shift = 0;
+    while ((1u << shift) < d) ++shift;
+    return;
+  }
+  uint32_t l = 0;
+  while ((1ull << l) < d) ++l;  // ceil(log2 d)
+  mul = (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+  shift = l;
+}
+__device__ __forceinline__ uint32_t cellof(const DevGraph& g, uint32_t v) {
+  if (g.cs_mul == 0) return v >> g.cs_shift;
+  const uint32_t t = __umulhi(v, g.cs_mul);
+  return (t + ((v - t) >> 1)) >> (g.cs_shift - 1);
+}
 
 __device__ inline unsigned lanemask_lt() {
   unsigned m;

@@ -185,7 +185,7 @@ __device__ void request_lookahead(const QParams& P, const WarpMem& m, const uint
                                   uint32_t nf, int lane) {
   for (uint32_t i = lane; i < nf; i += 32) {
     const uint32_t v = (uint32_t)(m.dtab[front[i]] >> 32);
-    request_flush(P.s, cell_of(v, P.g.cs), P.epoch);
+    request_flush(P.s, cellof(P.g, v), P.epoch);
   }
 }
 
@@ -230,7 +230,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
 
   // objects on q's own arc ahead of q (reading R2); they are stored at vertex src(q.e)
   if (q.y > 0) {
-    const uint32_t c = cell_of(ei.x, g.cs);
+    const uint32_t c = cellof(g, ei.x);
     if (s.cell_head[c] != NONE) {
       if (lane == 0) request_flush(s, c, P.epoch);
       return RETRY;
@@ -305,30 +305,19 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
           du = (uint32_t)e2;
           arc = g.vadj[(size_t)u * 4 + s4];
         }
-        // first expansion of the vertex: its objects (same memory round as its arcs)
-        bool harv = false, dirty = false;
-        uint2 vo = make_uint2(0, 0);
+        // the vertex's object metadata: loads issued in the same memory round as its arcs,
+        // consumed after the relaxation (harvested on the vertex's first expansion only)
+        bool harv = false;
+        uint32_t hcell = 0, hd = NONE;
+        uint2 cc = make_uint2(0, 0), v0 = make_uint2(0, 0);
         if (vv && s4 == 0) {
+          hcell = cellof(g, u);
+          hd = s.cell_head[hcell];
+          cc = s.cell_comp[hcell];
+          v0 = s.v_obj[u];
           const uint32_t bit = 1u << (vslot & 31);
-          if (!(atomicOr(&m.listed[vslot >> 5], bit) & bit)) {
-            harv = true;
-            const uint32_t c = cell_of(u, g.cs);
-            const uint32_t hd = s.cell_head[c];
-            const uint2 cc = s.cell_comp[c];
-            const uint2 v0 = s.v_obj[u];
-            if (hd != NONE) {
-              dirty = true;
-              request_flush(s, c, P.epoch);
-            } else {
-              vo = vobj_valid(v0, cc);
-            }
-          }
+          harv = !(atomicOr(&m.listed[vslot >> 5], bit) & bit);
         }
-        if (__any_sync(FULL, dirty)) {
-          request_lookahead(P, m, front, nf, lane);
-          return RETRY;
-        }
-        c_harv += __popc(__ballot_sync(FULL, harv));
         // relax the inline arc
         bool has = false, ovf = false;
         uint32_t nslot = 0;
@@ -391,7 +380,16 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
             nn += __popc(hm);
           }
         }
-        // harvest the objects of the vertices expanded for the first time
+        // harvest the objects of the vertices expanded for the first time; a cell with cached
+        // updates must be cleaned first (lazy flush): request it and retry the query
+        const bool dirty = harv && hd != NONE;
+        if (dirty) request_flush(s, hcell, P.epoch);
+        if (__any_sync(FULL, dirty)) {
+          request_lookahead(P, m, front, nf, lane);
+          return RETRY;
+        }
+        c_harv += __popc(__ballot_sync(FULL, harv));
+        const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
         const uint32_t most = __reduce_max_sync(FULL, vo.y);
         if (most) {
           c_objs += __reduce_add_sync(FULL, vo.y);
