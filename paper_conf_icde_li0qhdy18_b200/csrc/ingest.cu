@@ -21,6 +21,7 @@ constexpr int CT = 256;            // threads
 constexpr int CPT = 8;             // updates per thread
 constexpr int CU = CT * CPT;       // updates per CTA
 constexpr int CH = 4096;           // hash slots (>= 2*CU)
+constexpr int SPT = 4;             // scatter: updates per thread
 
 __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
                                                         DevGraph g, DevState s,
@@ -36,20 +37,29 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
   const uint64_t base = (uint64_t)blockIdx.x * CU;
   int slot[CPT];
   uint32_t vs[CPT], lr[CPT];
+  // all CPT record loads in flight, then all CPT inverted-index gathers, then the hashing
+  uint4 mm[CPT];
+#pragma unroll
+  for (int j = 0; j < CPT; ++j) {
+    const uint64_t i = base + (uint64_t)j * CT + tid;
+    mm[j] = i < n ? __ldg(upd + i) : make_uint4(0, 0xFFFFFFFFu, 0, 0);  // re-read by scatter
+  }
+  uint2 ee[CPT];
+#pragma unroll
+  for (int j = 0; j < CPT; ++j) ee[j] = mm[j].y < g.A ? __ldg(g.einfo + mm[j].y) : make_uint2(0, 1);
 #pragma unroll
   for (int j = 0; j < CPT; ++j) {
     const uint64_t i = base + (uint64_t)j * CT + tid;
     slot[j] = -1;
     if (i >= n) continue;
-    const uint4 m = upd[i];
+    const uint4 m = mm[j];
+    const uint2 e = ee[j];
     unsigned bad = 0;
-    uint2 e = make_uint2(0, 1);
     if (m.x >= s.max_objects) bad |= ERR_OBJ;
     if (m.y >= g.A) {
       bad |= ERR_EDGE;
-    } else {
-      e = g.einfo[m.y];
-      if (m.z >= e.y) bad |= ERR_OFF;
+    } else if (m.z >= e.y) {
+      bad |= ERR_OFF;
     }
     if (bad) {
       atomicOr(&s.st->err, bad);
@@ -134,19 +144,37 @@ __global__ void __launch_bounds__(256) k_ingest_scatter(const uint4* __restrict_
                                                         uint32_t seq0, DevGraph g, DevState s,
                                                         const uint2* __restrict__ tmp) {
   if (s.st->err) return;
-  uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  uint4 m = upd[i];
-  uint2 vr = tmp[i];
-  uint32_t pos = s.bbase[cellof(g, vr.x)] + vr.y;
-  unsigned long long key = ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
-  s.ar.obj[pos] = m.x;
-  s.ar.key[pos] = key;
-  s.ar.vsrc[pos] = vr.x;
-  s.ar.off[pos] = m.z;
-  s.ar.edge[pos] = m.y;
-  unsigned long long old = atomicMax(&s.ot_key[m.x], key);
-  if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+  // SPT updates per thread (strided by the CTA, so every load is coalesced), all loads of a
+  // stage in flight before the dependent stage
+  const uint64_t base = (uint64_t)blockIdx.x * (256 * SPT) + threadIdx.x;
+  uint4 m[SPT];
+  uint2 vr[SPT];
+#pragma unroll
+  for (int j = 0; j < SPT; ++j) {
+    const uint64_t i = base + (uint64_t)j * 256;
+    if (i < n) {
+      m[j] = __ldcs(upd + i);
+      vr[j] = __ldcs(tmp + i);
+    }
+  }
+  uint32_t pos[SPT];
+#pragma unroll
+  for (int j = 0; j < SPT; ++j)
+    if (base + (uint64_t)j * 256 < n) pos[j] = s.bbase[cellof(g, vr[j].x)] + vr[j].y;
+#pragma unroll
+  for (int j = 0; j < SPT; ++j) {
+    const uint64_t i = base + (uint64_t)j * 256;
+    if (i >= n) continue;
+    const unsigned long long key =
+        ((unsigned long long)m[j].w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
+    s.ar.obj[pos[j]] = m[j].x;
+    s.ar.key[pos[j]] = key;
+    s.ar.vsrc[pos[j]] = vr[j].x;
+    s.ar.off[pos[j]] = m[j].z;
+    s.ar.edge[pos[j]] = m[j].y;
+    const unsigned long long old = atomicMax(&s.ot_key[m[j].x], key);
+    if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+  }
 }
 
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
@@ -159,7 +187,7 @@ void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st) 
 }
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st) {
-  unsigned blocks = (unsigned)((n + 255) / 256);
+  unsigned blocks = (unsigned)((n + 256 * SPT - 1) / (256 * SPT));
   k_ingest_scatter<<<blocks, 256, 0, st>>>(upd, n, seq0, g, s, tmp);
 }
 

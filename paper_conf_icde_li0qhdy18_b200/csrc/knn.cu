@@ -472,7 +472,13 @@ __global__ void k_expand(QParams P) {
 // CTA, as many CTAs per SM as fit); level 3 is global memory sized from |V| (a query that
 // reaches fewer than k objects may need to settle the whole graph).
 constexpr int NLEVELS = 4;
-const Caps kCaps[3] = {{1024, 256, 64}, {2048, 512, 256}, {16384, 4096, 2048}};
+#ifndef GG_H0
+#define GG_H0 1024  // level-0 vertex table (experiment hook: -DGG_H0=..., -DGG_F0=...)
+#endif
+#ifndef GG_F0
+#define GG_F0 128
+#endif
+const Caps kCaps[3] = {{GG_H0, GG_F0, 64}, {2048, 512, 256}, {16384, 4096, 2048}};
 
 Caps caps_for(int level, uint32_t V) {
   if (level < 3) return kCaps[level];
