@@ -136,6 +136,18 @@ int ggrid_build(const ggrid_graph* g, uint32_t cell_size, const ggrid_opts* opts
  * (log arena full even after garbage collection), ECUDA. */
 int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n);
 
+/* Pipelined ingest (the paper's pipelined transfer, P@45017-45625: the GPU works on one group
+ * of messages while the next is being received).  ggrid_ingest_stage starts copying n updates
+ * (host or device pointer; pinned host memory makes the copy asynchronous) into one of two
+ * device staging buffers on a dedicated copy stream and returns at once.  The caller must
+ * leave u untouched until the matching ggrid_ingest_commit returns.  ggrid_ingest_commit
+ * ingests the oldest staged batch with the semantics and errors of ggrid_ingest (arrival
+ * order = commit order).  A ggrid_knn issued between the two calls does not see the staged
+ * batch; its kernels overlap the copy.  Errors: EINVAL (stage with both buffers staged,
+ * commit with none staged, null u), ENOMEM, ECUDA. */
+int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n);
+int ggrid_ingest_commit(ggrid_t h);
+
 /* Answer n_q kNN queries (Def. 1, P@9206-9761; Alg. 4-6, P@44429-52751) on the snapshot
  * of all updates ingested before the call.  Row i of out_obj / out_dist (n_q*k each,
  * host or device pointers) holds the k nearest objects in ascending (dist, obj) order,

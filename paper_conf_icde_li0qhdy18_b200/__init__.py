@@ -23,7 +23,7 @@ GGRID_OK, GGRID_EINVAL, GGRID_ENOMEM, GGRID_ECUDA, GGRID_ENCCL, GGRID_EOVERFLOW 
 PAD = 0xFFFFFFFF
 KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "flush", "expand",
                 "expand_big", "other"]
-EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_flush_all",
+EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_flush_all",
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
            "ggrid_version"]
 
@@ -73,6 +73,8 @@ def lib():
         sig = {
             "ggrid_build": ([ctypes.POINTER(ggrid_graph), u32, ctypes.POINTER(ggrid_opts), ctypes.POINTER(P)], i32),
             "ggrid_ingest": ([P, P, u64], i32),
+            "ggrid_ingest_stage": ([P, P, u64], i32),
+            "ggrid_ingest_commit": ([P], i32),
             "ggrid_knn": ([P, P, u32, u32, P, P], i32),
             "ggrid_free": ([P], i32),
             "ggrid_strerror": ([i32], ctypes.c_char_p),
@@ -146,6 +148,17 @@ def ggrid_ingest(h, updates, n: int | None = None):
     _check(lib().ggrid_ingest(h, _ptr(u), cnt), "ggrid_ingest")
 
 
+def ggrid_ingest_stage(h, updates):
+    """Start the asynchronous copy of a batch (keep `updates` alive until the commit)."""
+    u = _u32(updates)
+    _check(lib().ggrid_ingest_stage(h, _ptr(u), int(u.shape[0])), "ggrid_ingest_stage")
+    return u
+
+
+def ggrid_ingest_commit(h):
+    _check(lib().ggrid_ingest_commit(h), "ggrid_ingest_commit")
+
+
 def ggrid_knn(h, queries, k: int, out_obj=None, out_dist=None):
     """Answer queries ((n, 2) u32 (edge, offset)); returns (out_obj, out_dist) of shape (n, k).
 
@@ -215,10 +228,21 @@ class GGrid:
 
     def __init__(self, graph: dict, cell_size: int, **opts):
         self.n_vertices = int(graph["n_vertices"])
+        self._staged = []
         self.h = ggrid_build(graph, cell_size, **opts)
 
     def ingest(self, updates):
         ggrid_ingest(self.h, updates)
+        return self
+
+    def ingest_stage(self, updates):
+        """Pipelined ingest: copy now, ingest at ingest_commit (P@45017-45625)."""
+        self._staged.append(ggrid_ingest_stage(self.h, updates))
+        return self
+
+    def ingest_commit(self):
+        ggrid_ingest_commit(self.h)
+        self._staged.pop(0)
         return self
 
     def knn(self, queries, k: int, out_obj=None, out_dist=None):

@@ -76,6 +76,23 @@ bool is_device_ptr(const void* p) {
   return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// pointer the kernels may dereference for p: p itself for device/managed memory, the mapped
+// device alias for pinned host memory, null for pageable host memory (must be copied)
+void* device_view(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) return const_cast<void*>(p);
+  if (a.type == cudaMemoryTypeHost && a.devicePointer) {
+    // offset of p inside its allocation maps 1:1 onto the device alias
+    return static_cast<char*>(a.devicePointer) +
+           (static_cast<const char*>(p) - static_cast<const char*>(a.hostPointer));
+  }
+  return nullptr;
+}
+
 }  // namespace
 
 struct ggrid_s {
@@ -92,9 +109,19 @@ struct ggrid_s {
   std::vector<void*> allocs;
   DevStatus* d_status = nullptr;
   DevStatus* h_status = nullptr;  // pinned
+  DevStatus* h_status_dev = nullptr;  // its mapped device alias (the kernels' store target)
   uint64_t seq_next = 0;
   uint32_t epoch = 0;
   DBuf upd_stage, tmp, q_stage, out_stage, lists, l2_scratch, dump_stage, gc_buf, misc;
+  // pipelined ingest: two staging buffers filled on a copy stream
+  struct Staged {
+    DBuf buf;
+    uint64_t n = 0;
+    cudaEvent_t done = nullptr;
+  };
+  Staged staged[2];
+  int stage_head = 0, n_staged = 0;
+  cudaStream_t copy_stream = nullptr;
   ggrid_stats_t stats{};
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending_ev;
   std::vector<cudaEvent_t> ev_pool;
@@ -139,9 +166,11 @@ struct ggrid_s {
     }
   }
 
-  // drain the stream, collect event timings, refresh the status mirror
+  // drain the stream, collect event timings, refresh the status mirror.  The mirror is written
+  // by a kernel through its mapped alias, not a D2H cudaMemcpy: a copy would share the copy
+  // engine with a staged ingest transfer and wait behind it.
   int sync() {
-    CK(cudaMemcpyAsync(h_status, d_status, sizeof(DevStatus), cudaMemcpyDeviceToHost, stream));
+    launch(GGRID_K_OTHER, [&] { launch_copy_words(d_status, h_status_dev, sizeof(DevStatus), stream); });
     CK(cudaStreamSynchronize(stream));
     for (auto& pe : pending_ev) {
       float ms = 0.f;
@@ -155,14 +184,18 @@ struct ggrid_s {
     return GGRID_OK;
   }
 
-  int set_status_u32(unsigned int* field, unsigned int v) {
-    CK(cudaMemsetAsync(field, 0, sizeof(unsigned int), stream));
-    if (v) CK(cudaMemcpyAsync(field, &v, sizeof v, cudaMemcpyHostToDevice, stream));
+  // device-side word stores (a kernel: never queued behind a staged copy on a copy engine)
+  int set_words(const WordSet& ws) {
+    launch(GGRID_K_OTHER, [&] { launch_set_words(ws, stream); });
     return GGRID_OK;
+  }
+  int set_status_u32(unsigned int* field, unsigned int v) {
+    WordSet ws;
+    ws.add(field, v);
+    return set_words(ws);
   }
 
   int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin, int full_vobj = 0) {
-    CK(cudaMemsetAsync(&d_status->flush_work, 0, sizeof(unsigned int), stream));
     const uint32_t opc = (uint32_t)((h_status->n_live + n_cells - 1) / std::max(1u, n_cells));
     launch(GGRID_K_FLUSH, [&] { launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, stream); });
     return GGRID_OK;
@@ -196,9 +229,13 @@ int ggrid_s::gc() {
   unsigned long long* d_top = nullptr;
   RC(misc.ensure(64));
   d_top = misc.as<unsigned long long>();
-  CK(cudaMemsetAsync(d_top, 0, 8, stream));
   epoch++;
-  RC(set_status_u32(&d_status->n_flush, 0));
+  {
+    WordSet ws;
+    ws.zero_range(reinterpret_cast<uint32_t*>(d_top), 2);
+    ws.add(&d_status->n_flush, 0);
+    RC(set_words(ws));
+  }
   launch(GGRID_K_OTHER, [&] { launch_mark_dirty(g, s, epoch, 1, stream); });
   RC(flush_list_run(t, d_top, 0, /*full_vobj=*/1));
   unsigned long long top = 0;
@@ -289,6 +326,9 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
     if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess)
       return fail(GGRID_ECUDA);
     h->own_stream = true;
+  }
+  if (cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking) != cudaSuccess) {
+    return fail(GGRID_ECUDA);
   }
   h->V = V;
   h->A = A;
@@ -428,6 +468,8 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   s.st = h->d_status;
   if (cudaMallocHost((void**)&h->h_status, sizeof(DevStatus)) != cudaSuccess) return fail(GGRID_ENOMEM);
   memset(h->h_status, 0, sizeof(DevStatus));
+  if (cudaHostGetDevicePointer((void**)&h->h_status_dev, h->h_status, 0) != cudaSuccess)
+    return fail(GGRID_ECUDA);
   h->stats.arena_capacity = cap;
   if (cudaDeviceSynchronize() != cudaSuccess) return fail(GGRID_ECUDA);
   *out = h;
@@ -437,10 +479,14 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
 int ggrid_free(ggrid_t h) {
   if (!h) return GGRID_OK;
   if (h->stream) cudaStreamSynchronize(h->stream);
+  if (h->copy_stream) cudaStreamSynchronize(h->copy_stream);
   for (void* p : h->allocs) cudaFree(p);
   for (DBuf* b : {&h->upd_stage, &h->tmp, &h->q_stage, &h->out_stage, &h->lists, &h->l2_scratch,
-                  &h->dump_stage, &h->gc_buf, &h->misc})
+                  &h->dump_stage, &h->gc_buf, &h->misc, &h->staged[0].buf, &h->staged[1].buf})
     b->release();
+  for (auto& sb : h->staged)
+    if (sb.done) cudaEventDestroy(sb.done);
+  if (h->copy_stream) cudaStreamDestroy(h->copy_stream);
   for (auto& pe : h->pending_ev) {
     cudaEventDestroy(pe.second.first);
     cudaEventDestroy(pe.second.second);
@@ -452,23 +498,19 @@ int ggrid_free(ggrid_t h) {
   return GGRID_OK;
 }
 
-int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
-  if (!h) return GGRID_EINVAL;
-  if (n == 0) return GGRID_OK;
-  if (!u) return GGRID_EINVAL;
+// ingest n updates already resident in device memory at d_u (the main stream must be
+// ordered after their arrival)
+static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
-  CK(cudaSetDevice(h->device));
   const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
   RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
-  const uint4* d_u = reinterpret_cast<const uint4*>(u);
-  if (!is_device_ptr(u)) {
-    RC(h->upd_stage.ensure(n * sizeof(uint4)));
-    CK(cudaMemcpyAsync(h->upd_stage.p, u, n * sizeof(uint4), cudaMemcpyHostToDevice, h->stream));
-    d_u = h->upd_stage.as<uint4>();
-  }
   RC(h->tmp.ensure(n * sizeof(uint2)));
-  unsigned int zero_bad[2] = {0u, 0xFFFFFFFFu};
-  CK(cudaMemcpyAsync(&h->d_status->err, zero_bad, 8, cudaMemcpyHostToDevice, h->stream));
+  {
+    WordSet ws;
+    ws.add(&h->d_status->err, 0u);
+    ws.add(&h->d_status->bad_index, 0xFFFFFFFFu);
+    RC(h->set_words(ws));
+  }
   const uint32_t seq0 = (uint32_t)h->seq_next;
   const DevGraph& g = h->g;
   const DevState& s = h->s;
@@ -486,21 +528,73 @@ int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
   return GGRID_OK;
 }
 
+int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
+  if (!h) return GGRID_EINVAL;
+  if (n == 0) return GGRID_OK;
+  if (!u) return GGRID_EINVAL;
+  if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
+  CK(cudaSetDevice(h->device));
+  const uint4* d_u = reinterpret_cast<const uint4*>(u);
+  if (!is_device_ptr(u)) {
+    RC(h->upd_stage.ensure(n * sizeof(uint4)));
+    CK(cudaMemcpyAsync(h->upd_stage.p, u, n * sizeof(uint4), cudaMemcpyHostToDevice, h->stream));
+    d_u = h->upd_stage.as<uint4>();
+  }
+  return ingest_device(h, d_u, n);
+}
+
+int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n) {
+  if (!h || (n && !u) || h->n_staged == 2) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  ggrid_s::Staged& sb = h->staged[(h->stage_head + h->n_staged) & 1];
+  if (!sb.done) CK(cudaEventCreateWithFlags(&sb.done, cudaEventDisableTiming));
+  sb.n = n;
+  if (n) {
+    // both buffers grow together: a cudaMalloc in the middle of a running pipeline stalls it
+    RC(h->staged[0].buf.ensure(n * sizeof(uint4)));
+    RC(h->staged[1].buf.ensure(n * sizeof(uint4)));
+    CK(cudaMemcpyAsync(sb.buf.p, u, n * sizeof(uint4), cudaMemcpyDefault, h->copy_stream));
+  }
+  CK(cudaEventRecord(sb.done, h->copy_stream));
+  h->n_staged++;
+  return GGRID_OK;
+}
+
+int ggrid_ingest_commit(ggrid_t h) {
+  if (!h || h->n_staged == 0) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  ggrid_s::Staged& sb = h->staged[h->stage_head];
+  h->stage_head ^= 1;
+  h->n_staged--;
+  CK(cudaStreamWaitEvent(h->stream, sb.done, 0));
+  if (sb.n == 0) return GGRID_OK;
+  return ingest_device(h, sb.buf.as<uint4>(), sb.n);
+}
+
 static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
                     uint32_t* out_dist) {
   CK(cudaSetDevice(h->device));
   cudaStream_t st = h->stream;
   // every flushed cell writes at most its live objects (+ alignment padding)
   RC(h->ensure_arena(h->flush_need(), 0));
-  const uint2* d_q = reinterpret_cast<const uint2*>(q);
-  if (!is_device_ptr(q)) {
+  // device and pinned (mapped) host buffers are used in place — pinned queries and answers
+  // cross PCIe inside the kernels and leave the copy engine to a staged ingest batch
+  // (ggrid_ingest_stage); pageable host buffers are copied
+  const uint2* d_q = static_cast<const uint2*>(device_view(q));
+  uint2* q_copy = nullptr;  // pinned queries: the seed kernel copies them into HBM
+  if (!d_q) {
     RC(h->q_stage.ensure((size_t)n_q * 8));
     CK(cudaMemcpyAsync(h->q_stage.p, q, (size_t)n_q * 8, cudaMemcpyHostToDevice, st));
     d_q = h->q_stage.as<uint2>();
+  } else if (!is_device_ptr(q)) {
+    RC(h->q_stage.ensure((size_t)n_q * 8));
+    q_copy = h->q_stage.as<uint2>();
   }
-  const bool dev_o = is_device_ptr(out_obj), dev_d = is_device_ptr(out_dist);
-  uint32_t* d_oo = out_obj;
-  uint32_t* d_od = out_dist;
+  uint32_t* v_oo = static_cast<uint32_t*>(device_view(out_obj));
+  uint32_t* v_od = static_cast<uint32_t*>(device_view(out_dist));
+  const bool dev_o = v_oo != nullptr, dev_d = v_od != nullptr;
+  uint32_t* d_oo = dev_o ? v_oo : out_obj;
+  uint32_t* d_od = dev_d ? v_od : out_dist;
   const size_t outn = (size_t)n_q * k;
   if (!dev_o || !dev_d) {
     RC(h->out_stage.ensure(outn * 8));
@@ -515,11 +609,17 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   h->epoch++;
   const uint32_t epoch = h->epoch;
   // reset err, n_flush, flush_work, n_next[*], flush_end, expand_work[*]
-  CK(cudaMemsetAsync(&h->d_status->err, 0, sizeof(unsigned), st));
-  CK(cudaMemsetAsync(&h->d_status->n_flush, 0, offsetof(DevStatus, round_end) - offsetof(DevStatus, n_flush), st));
+  {
+    WordSet ws;
+    ws.add(&h->d_status->err, 0u);
+    ws.zero_range(&h->d_status->n_flush,
+                  (int)((offsetof(DevStatus, round_end) - offsetof(DevStatus, n_flush)) / 4));
+    RC(h->set_words(ws));
+  }
   const DevGraph& g = h->g;
   const DevState& s = h->s;
-  h->launch(GGRID_K_SEED, [&] { launch_seed(d_q, n_q, g, s, epoch, h->seed_neighbors, st); });
+  h->launch(GGRID_K_SEED, [&] { launch_seed(d_q, n_q, g, s, epoch, h->seed_neighbors, q_copy, st); });
+  if (q_copy) d_q = q_copy;
 
   int lvl0 = 0;
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
@@ -531,8 +631,12 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   for (int round = 0;; ++round) {
     if (round > 100000) return GGRID_ECUDA;
     RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin));
-    CK(cudaMemsetAsync(h->d_status->n_next, 0, sizeof(h->d_status->n_next), st));
-    CK(cudaMemsetAsync(h->d_status->expand_work, 0, sizeof(h->d_status->expand_work), st));
+    if (round > 0) {  // round 0 was reset with the rest at the start
+      WordSet ws;
+      ws.zero_range(h->d_status->n_next, 4);
+      ws.zero_range(h->d_status->expand_work, 4);
+      RC(h->set_words(ws));
+    }
     for (int lvl = 0; lvl < L; ++lvl) {
       if (!n_in[lvl]) continue;
       void* scratch = nullptr;
@@ -568,9 +672,11 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
     cur ^= 1;
     if (!any) break;
   }
-  if (!dev_o) CK(cudaMemcpyAsync(out_obj, d_oo, outn * 4, cudaMemcpyDeviceToHost, st));
-  if (!dev_d) CK(cudaMemcpyAsync(out_dist, d_od, outn * 4, cudaMemcpyDeviceToHost, st));
-  RC(h->sync());
+  if (!dev_o || !dev_d) {  // (device / pinned outputs were written in place; the loop drained)
+    if (!dev_o) CK(cudaMemcpyAsync(out_obj, d_oo, outn * 4, cudaMemcpyDeviceToHost, st));
+    if (!dev_d) CK(cudaMemcpyAsync(out_dist, d_od, outn * 4, cudaMemcpyDeviceToHost, st));
+    RC(h->sync());
+  }
   h->stats.n_queries += n_q;
   h->stats.knn_calls++;
   return GGRID_OK;
@@ -612,7 +718,7 @@ int ggrid_cell_objects(ggrid_t h, uint32_t cell, uint32_t* obj, uint32_t* edge, 
   uint32_t* d_o = d_n + 4;
   uint32_t* d_e = d_o + cap;
   uint32_t* d_f = d_e + cap;
-  CK(cudaMemsetAsync(d_n, 0, 4, h->stream));
+  RC(h->set_status_u32(d_n, 0));
   h->launch(GGRID_K_OTHER, [&] { launch_dump_cell(h->g, h->s, cell, d_o, d_e, d_f, cap, d_n, h->stream); });
   uint32_t cnt = 0;
   CK(cudaMemcpyAsync(&cnt, d_n, 4, cudaMemcpyDeviceToHost, h->stream));

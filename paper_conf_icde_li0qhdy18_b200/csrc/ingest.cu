@@ -194,10 +194,14 @@ void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const De
 // ---------------------------------------------------------------------------------------
 // Alg. 4 line 1 (P@45660): c_q = getCell(q.e) and getNeighbors({c_q}) are cleaned first.
 __global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint32_t nq, DevGraph g,
-                                              DevState s, uint32_t epoch, int neighbors) {
+                                              DevState s, uint32_t epoch, int neighbors,
+                                              uint2* __restrict__ q_copy) {
   uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= nq) return;
   uint2 qq = q[i];
+  // queries in mapped host memory are read across PCIe once, here, and kept in HBM for the
+  // expansion (each warp re-reading its query over PCIe would queue behind a staged transfer)
+  if (q_copy) q_copy[i] = qq;
   if (qq.x >= g.A) {
     atomicOr(&s.st->err, (unsigned)ERR_QUERY);
     return;
@@ -217,9 +221,9 @@ __global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint3
 }
 
 void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s, uint32_t epoch,
-                 int neighbors, cudaStream_t st) {
+                 int neighbors, uint2* q_copy, cudaStream_t st) {
   if (nq == 0) return;
-  k_seed<<<(nq + 255) / 256, 256, 0, st>>>(q, nq, g, s, epoch, neighbors);
+  k_seed<<<(nq + 255) / 256, 256, 0, st>>>(q, nq, g, s, epoch, neighbors, q_copy);
 }
 
 // Every dirty cell (eager cleaning; all_cells additionally queues clean cells for GC).
@@ -269,4 +273,24 @@ void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t
   k_dump_cell<<<1, 256, 0, st>>>(g, s, c, obj, edge, off, cap, n_out);
 }
 
+}  // namespace gg
+
+namespace gg {
+__global__ void k_set_words(WordSet ws) {
+  if ((int)threadIdx.x < ws.n) *ws.p[threadIdx.x] = ws.v[threadIdx.x];
+}
+void launch_set_words(const WordSet& ws, cudaStream_t st) {
+  if (ws.n) k_set_words<<<1, 32, 0, st>>>(ws);
+}
+}  // namespace gg
+
+namespace gg {
+// status readback through mapped pinned memory: a kernel store, no copy engine involved
+__global__ void k_copy_words(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst, int n) {
+  for (int i = threadIdx.x; i < n; i += blockDim.x) dst[i] = src[i];
+}
+void launch_copy_words(const void* src, void* dst, size_t bytes, cudaStream_t st) {
+  k_copy_words<<<1, 64, 0, st>>>(static_cast<const uint32_t*>(src), static_cast<uint32_t*>(dst),
+                                 (int)(bytes / 4));
+}
 }  // namespace gg

@@ -135,13 +135,32 @@ __device__ inline void request_flush(const DevState& s, uint32_t c, uint32_t epo
 
 // Launchers (defined in the .cu files; called by api.cu).
 namespace gg {
+// Small device-side word stores (status counters).  A kernel, not cudaMemset/cudaMemcpy: those
+// can run on a copy engine and would queue behind a staged ingest transfer.
+struct WordSet {
+  static constexpr int N = 24;
+  uint32_t* p[N];
+  uint32_t v[N];
+  int n = 0;
+  void add(uint32_t* ptr, uint32_t val) {
+    p[n] = ptr;
+    v[n] = val;
+    ++n;
+  }
+  void zero_range(uint32_t* ptr, int words) {
+    for (int i = 0; i < words; ++i) add(ptr + i, 0u);
+  }
+};
+void launch_set_words(const WordSet& ws, cudaStream_t st);
+void launch_copy_words(const void* src, void* dst, size_t bytes, cudaStream_t st);
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
                             uint2* tmp, cudaStream_t st);
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st);
+// q_copy (nullable): also store the queries there (q in mapped host memory)
 void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s, uint32_t epoch,
-                 int neighbors, cudaStream_t st);
+                 int neighbors, uint2* q_copy, cudaStream_t st);
 void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int all_cells,
                        cudaStream_t st);
 // Flush the cells flush_list[begin .. st->n_flush) writing compacted lists into `out`

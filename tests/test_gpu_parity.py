@@ -365,3 +365,30 @@ def test_usa_shaped_sampled(gg):
     _assert_same((go[sel], gd[sel]), _oracle(g, upd, q[sel], 10, mode=oracle.EARLY), "USA/10 early")
     _assert_same((go[sel[:10]], gd[sel[:10]]), _oracle(g, upd, q[sel[:10]], 10), "USA/10 full")
     grid.close()
+
+
+def test_pipelined_ingest_stage_commit(gg):
+    """ggrid_ingest_stage/commit (P@45017-45625 pipelined transfer): a knn issued between
+    stage and commit answers on the snapshot without the staged batch; after the commit it
+    includes it; the stage/commit misuse errors."""
+    import torch
+
+    g = synth.table_ii_graph("NY", scale=0.03)
+    walk = synth.RandomWalk(g, 500, inject=True)
+    u1, u2, u3 = walk.ticks(3), walk.ticks(3), walk.ticks(3)
+    q = synth.queries(g, 100)
+    grid = gg.GGrid(g, 128, max_objects=512)
+    with pytest.raises(gg.GGridError):
+        grid.ingest_commit()  # nothing staged
+    grid.ingest(u1)
+    grid.ingest_stage(torch.from_numpy(u2.view(np.int32)).pin_memory())
+    grid.ingest_stage(u3)  # pageable host memory also works
+    with pytest.raises(gg.GGridError):
+        grid.ingest_stage(u3)  # both buffers staged
+    _assert_same(grid.knn(q, 6), _oracle(g, u1, q, 6), "before commit")
+    grid.ingest_commit()
+    _assert_same(grid.knn(q, 6), _oracle(g, np.concatenate([u1, u2]), q, 6), "after commit 1")
+    grid.ingest_commit()
+    _assert_same(grid.knn(q, 6), _oracle(g, np.concatenate([u1, u2, u3]), q, 6), "after commit 2")
+    assert grid.stats()["n_updates"] == len(u1) + len(u2) + len(u3)
+    grid.close()
