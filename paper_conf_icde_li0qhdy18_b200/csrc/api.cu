@@ -461,7 +461,7 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   if ((rc = h->alloc(&s.cell_comp, h->n_cells))) return fail(rc);
   s.vcnt = nullptr;
   if (cell_size > 4096 && (rc = h->alloc(&s.vcnt, V))) return fail(rc);
-  if ((rc = h->alloc(&s.bcount, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&s.bcount, (size_t)h->n_cells * BCOUNT_STRIDE))) return fail(rc);
   if ((rc = h->alloc(&s.bbase, h->n_cells))) return fail(rc);
   if ((rc = h->alloc(&s.flush_list, h->n_cells))) return fail(rc);
   if ((rc = h->alloc(&h->d_status, 1))) return fail(rc);
@@ -504,7 +504,7 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
   const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
   RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
-  RC(h->tmp.ensure(n * sizeof(uint2)));
+  RC(h->tmp.ensure(ingest_tmp_bytes(n)));
   {
     WordSet ws;
     ws.add(&h->d_status->err, 0u);

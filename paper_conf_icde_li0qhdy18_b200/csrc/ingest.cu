@@ -14,21 +14,28 @@
 
 namespace gg {
 
-// CTA-level aggregation: each CTA takes CU consecutive updates, counts them per cell in a
-// shared-memory hash (rank within the CTA), then claims one global range per distinct
+// CTA-level aggregation: each CTA takes CU consecutive updates (a tile), counts them per cell
+// in a shared-memory hash (rank within the CTA), then claims one global range per distinct
 // cell with a single atomicAdd on bcount[cell] (few cells => no hot-spot serialisation).
+// It also orders its tile by cell (hash slot): tmp[] holds, in that order, each update's
+// (source vertex, rank in the cell's batch extent) and perm[] its index in the tile, so the
+// scatter's consecutive threads write consecutive arena positions (runs per cell).
 constexpr int CT = 256;            // threads
 constexpr int CPT = 8;             // updates per thread
-constexpr int CU = CT * CPT;       // updates per CTA
+constexpr int CU = CT * CPT;       // updates per CTA (tile)
 constexpr int CH = 4096;           // hash slots (>= 2*CU)
-constexpr int SPT = 4;             // scatter: updates per thread
+constexpr int SPC = CH / CT;       // hash slots per thread in the scan
+static_assert(CU < 65536, "tile offsets and counts are packed in 16 bits");
 
 __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
                                                         DevGraph g, DevState s,
-                                                        uint2* __restrict__ tmp) {
-  __shared__ uint32_t h_cell[CH];
-  __shared__ uint32_t h_cnt[CH];
-  const int tid = threadIdx.x;
+                                                        uint2* __restrict__ tmp,
+                                                        uint16_t* __restrict__ perm) {
+  __shared__ __align__(16) uint32_t h_buf[2 * CH];
+  uint32_t* h_cell = h_buf;       // cell id; after the claim, the cell's global rank base
+  uint32_t* h_cnt = h_buf + CH;   // count; after the scan, (tile offset << 16) | count
+  __shared__ uint32_t w_sum[CT / 32];
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   for (int i = tid; i < CH; i += CT) {
     h_cell[i] = NONE;
     h_cnt[i] = 0;
@@ -83,25 +90,64 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
     lr[j] = atomicAdd(&h_cnt[h], 1u);
   }
   __syncthreads();
+  // exclusive scan of the slot counts = each cell's group offset in the tile's sorted order
+  {
+    uint32_t loc[SPC], sum = 0;
+#pragma unroll
+    for (int q = 0; q < SPC; ++q) {
+      loc[q] = sum;
+      sum += h_cnt[tid * SPC + q];
+    }
+    uint32_t x = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) w_sum[wid] = x;
+    __syncthreads();
+    uint32_t wpre = 0;
+    for (int w = 0; w < wid; ++w) wpre += w_sum[w];
+    const uint32_t excl = wpre + x - sum;
+#pragma unroll
+    for (int q = 0; q < SPC; ++q) h_cnt[tid * SPC + q] |= (excl + loc[q]) << 16;  // counts <= CU
+  }
   for (int i = tid; i < CH; i += CT) {
     const uint32_t c = h_cell[i];
-    if (c != NONE) h_cnt[i] = atomicAdd(&s.bcount[c], h_cnt[i]);
+    if (c != NONE) h_cell[i] = atomicAdd(&s.bcount[c * BCOUNT_STRIDE], h_cnt[i] & 0xFFFFu);
   }
   __syncthreads();
+  uint32_t si[CPT], rk[CPT];
 #pragma unroll
   for (int j = 0; j < CPT; ++j) {
     if (slot[j] < 0) continue;
-    const uint64_t i = base + (uint64_t)j * CT + tid;
-    tmp[i] = make_uint2(vs[j], h_cnt[slot[j]] + lr[j]);
+    si[j] = (h_cnt[slot[j]] >> 16) + lr[j];
+    rk[j] = h_cell[slot[j]] + lr[j];
+  }
+  __syncthreads();
+  // the tile in cell order, staged in the (now free) hash table, then written coalesced
+  uint2* stg = reinterpret_cast<uint2*>(h_buf);            // CU x 8 B
+  uint16_t* stp = reinterpret_cast<uint16_t*>(h_buf + CH);  // CU x 2 B
+#pragma unroll
+  for (int j = 0; j < CPT; ++j) {
+    if (slot[j] < 0) continue;
+    stg[si[j]] = make_uint2(vs[j], rk[j]);
+    stp[si[j]] = (uint16_t)(j * CT + tid);
+  }
+  __syncthreads();
+  const uint32_t nt = (n - base) < (uint64_t)CU ? (uint32_t)(n - base) : (uint32_t)CU;
+  for (uint32_t k = tid; k < nt; k += CT) {
+    tmp[base + k] = stg[k];
+    perm[base + k] = stp[k];
   }
 }
 
 __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
   uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
   const bool err = s.st->err != 0;
-  uint32_t cnt = (c < g.n_cells) ? s.bcount[c] : 0;
+  uint32_t cnt = (c < g.n_cells) ? s.bcount[c * BCOUNT_STRIDE] : 0;
   if (err) {
-    if (c < g.n_cells && cnt) s.bcount[c] = 0;
+    if (c < g.n_cells && cnt) s.bcount[c * BCOUNT_STRIDE] = 0;
     return;
   }
   unsigned lane = threadIdx.x & 31;
@@ -137,58 +183,93 @@ __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
   s.cell_head[c] = e;
   s.cell_pending[c] += cnt;
   s.bbase[c] = (uint32_t)start;
-  s.bcount[c] = 0;
+  s.bcount[c * BCOUNT_STRIDE] = 0;
 }
 
-__global__ void __launch_bounds__(256) k_ingest_scatter(const uint4* __restrict__ upd, uint64_t n,
-                                                        uint32_t seq0, DevGraph g, DevState s,
-                                                        const uint2* __restrict__ tmp) {
-  if (s.st->err) return;
-  // SPT updates per thread (strided by the CTA, so every load is coalesced), all loads of a
-  // stage in flight before the dependent stage
-  const uint64_t base = (uint64_t)blockIdx.x * (256 * SPT) + threadIdx.x;
-  uint4 m[SPT];
-  uint2 vr[SPT];
+// One CTA per classify tile.  The tile's updates are staged in shared memory (coalesced), then
+// thread k takes the k-th update in cell order: consecutive threads write consecutive
+// positions of a cell's extent (coalesced runs, few pages per warp store).
+__global__ void __launch_bounds__(CT) k_ingest_scatter(const uint4* __restrict__ upd, uint64_t n,
+                                                       uint32_t seq0, DevGraph g, DevState s,
+                                                       const uint2* __restrict__ tmp,
+                                                       const uint16_t* __restrict__ perm) {
+  __shared__ uint4 su[CU];
+  const int tid = threadIdx.x;
+  const uint64_t base = (uint64_t)blockIdx.x * CU;
+  const uint32_t nt = (n - base) < (uint64_t)CU ? (uint32_t)(n - base) : (uint32_t)CU;
+  // the tile's sorted (vertex, rank) and permutation (failed updates were left out: the
+  // batch is rejected below then)
+  uint2 vr[CPT];
+  uint32_t il[CPT];
 #pragma unroll
-  for (int j = 0; j < SPT; ++j) {
-    const uint64_t i = base + (uint64_t)j * 256;
-    if (i < n) {
-      m[j] = __ldcs(upd + i);
-      vr[j] = __ldcs(tmp + i);
+  for (int j = 0; j < CPT; ++j) {
+    const uint32_t k = (uint32_t)(j * CT + tid);
+    if (k < nt) {
+      su[k] = __ldcs(upd + base + k);
+      vr[j] = __ldcs(tmp + base + k);
+      il[j] = __ldcs(perm + base + k);
     }
   }
-  uint32_t pos[SPT];
+  if (*((volatile unsigned*)&s.st->err)) return;
+  __syncthreads();
+  // two halves of CPT/2 updates: every load of a half in flight before its stores, at half
+  // the registers (occupancy)
+  constexpr int HP = CPT / 2;
 #pragma unroll
-  for (int j = 0; j < SPT; ++j)
-    if (base + (uint64_t)j * 256 < n) pos[j] = s.bbase[cellof(g, vr[j].x)] + vr[j].y;
+  for (int hf = 0; hf < 2; ++hf) {
+    uint32_t pos[HP];
+    uint4 m[HP];
+    unsigned long long cur[HP];
 #pragma unroll
-  for (int j = 0; j < SPT; ++j) {
-    const uint64_t i = base + (uint64_t)j * 256;
-    if (i >= n) continue;
-    const unsigned long long key =
-        ((unsigned long long)m[j].w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
-    s.ar.obj[pos[j]] = m[j].x;
-    s.ar.key[pos[j]] = key;
-    s.ar.vsrc[pos[j]] = vr[j].x;
-    s.ar.off[pos[j]] = m[j].z;
-    s.ar.edge[pos[j]] = m[j].y;
-    const unsigned long long old = atomicMax(&s.ot_key[m[j].x], key);
-    if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+    for (int q = 0; q < HP; ++q) {
+      const int j = hf * HP + q;
+      const uint32_t k = (uint32_t)(j * CT + tid);
+      if (k < nt) {
+        m[q] = su[il[j]];
+        pos[q] = s.bbase[cellof(g, vr[j].x)] + vr[j].y;
+        cur[q] = __ldcg(s.ot_key + m[q].x);  // L2 value (the atomics' point of coherence)
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      const int j = hf * HP + q;
+      const uint32_t k = (uint32_t)(j * CT + tid);
+      if (k >= nt) continue;
+      const unsigned long long key =
+          ((unsigned long long)m[q].w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + il[j]));
+      s.ar.obj[pos[q]] = m[q].x;
+      s.ar.key[pos[q]] = key;
+      s.ar.vsrc[pos[q]] = vr[j].x;
+      s.ar.off[pos[q]] = m[q].z;
+      s.ar.edge[pos[q]] = m[q].y;
+      // ot_key only grows: a key below the value already seen needs no atomic; a live object
+      // takes a fire-and-forget RED.MAX; only an object seen without updates (0) needs the
+      // old value back, to count it live exactly once
+      if (cur[q] == 0ull) {
+        const unsigned long long old = atomicMax(&s.ot_key[m[q].x], key);
+        if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+      } else if (key > cur[q]) {
+        atomicMax(&s.ot_key[m[q].x], key);
+      }
+    }
   }
 }
 
+static uint16_t* perm_of(uint2* tmp, uint64_t n) { return reinterpret_cast<uint16_t*>(tmp + n); }
+size_t ingest_tmp_bytes(uint64_t n) { return (size_t)n * (sizeof(uint2) + sizeof(uint16_t)); }
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
                             uint2* tmp, cudaStream_t st) {
   unsigned blocks = (unsigned)((n + CU - 1) / CU);
-  k_ingest_classify<<<blocks, CT, 0, st>>>(upd, n, g, s, tmp);
+  k_ingest_classify<<<blocks, CT, 0, st>>>(upd, n, g, s, tmp, perm_of(tmp, n));
 }
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st) {
   k_ingest_alloc<<<(g.n_cells + 255) / 256, 256, 0, st>>>(g, s);
 }
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st) {
-  unsigned blocks = (unsigned)((n + 256 * SPT - 1) / (256 * SPT));
-  k_ingest_scatter<<<blocks, 256, 0, st>>>(upd, n, seq0, g, s, tmp);
+  unsigned blocks = (unsigned)((n + CU - 1) / CU);
+  k_ingest_scatter<<<blocks, CT, 0, st>>>(upd, n, seq0, g, s, tmp,
+                                          perm_of(const_cast<uint2*>(tmp), n));
 }
 
 // ---------------------------------------------------------------------------------------

@@ -20,6 +20,7 @@ namespace gg {
 constexpr uint32_t NONE = 0xFFFFFFFFu;
 constexpr uint32_t INF = 0xFFFFFFFFu;  // u32 distance "unreachable" (reading R18)
 constexpr unsigned long long EMPTY64 = ~0ull;
+constexpr uint32_t BCOUNT_STRIDE = 32;
 
 enum ErrBits : unsigned {
   ERR_OBJ = 1u,      // update obj >= max_objects
@@ -85,7 +86,8 @@ struct DevState {
   uint2* v_obj;            // [V] (arena start, count) of the objects at each vertex
   uint2* cell_comp;        // [n_cells] (arena start, count) of the cell's compacted list
   uint32_t* vcnt;          // [V] flush scratch, only when cell_size > 4096 (else null)
-  uint32_t* bcount;        // [n_cells] per-batch counts
+  uint32_t* bcount;        // [n_cells * BCOUNT_STRIDE] per-batch counts, one 128-byte line per
+                           // cell (same-line atomics from every ingest CTA serialise in L2)
   uint32_t* bbase;         // [n_cells] per-batch arena base
   uint32_t* flush_list;    // [n_cells]
   DevStatus* st;
@@ -155,6 +157,7 @@ void launch_set_words(const WordSet& ws, cudaStream_t st);
 void launch_copy_words(const void* src, void* dst, size_t bytes, cudaStream_t st);
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
                             uint2* tmp, cudaStream_t st);
+size_t ingest_tmp_bytes(uint64_t n);  // classify -> scatter scratch (tmp + perm)
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st);
