@@ -59,7 +59,13 @@ typedef struct ggrid_opts {
   uint32_t seed_neighbors; /* 0 = default on: flush c_q and its neighbour cells up
                               front (Alg. 4 line 1); 2 = off (c_q only)            */
   uint32_t profile;        /* 1 = time every kernel launch with CUDA events        */
-  uint32_t reserved;
+  uint32_t t_delta;        /* message expiry window t_Delta (P@20631-21157, sign
+                              corrected, reading R21): at cleaning time a
+                              cached extent (one ingest batch's messages for one
+                              cell) whose newest t is < t_now - t_delta is dropped
+                              unread; t_now = the largest t ingested so far.  Exact
+                              iff every object reports at least once per t_delta of
+                              arrival-ordered time.  0 = never expire.             */
   void* stream;            /* cudaStream_t to run on, or NULL (library stream)    */
 } ggrid_opts;
 
@@ -118,6 +124,9 @@ typedef struct ggrid_stats_t {
   uint32_t n_vertices;
   uint32_t n_arcs;
   uint32_t max_objects;
+  uint32_t t_delta;          /* opts.t_delta                                          */
+  uint32_t t_now;            /* largest t ingested so far                             */
+  uint64_t records_expired;  /* cached records dropped unread by t_delta expiry       */
 } ggrid_stats_t;
 
 /* Build the index (graph grid, P@11423-15818; object table P@15869; message lists

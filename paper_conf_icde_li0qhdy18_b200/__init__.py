@@ -44,7 +44,7 @@ class ggrid_opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("max_k", ctypes.c_uint32), ("max_objects", ctypes.c_uint32),
                 ("log_capacity", ctypes.c_uint64), ("delta", ctypes.c_uint32),
                 ("seed_neighbors", ctypes.c_uint32), ("profile", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32), ("stream", ctypes.c_void_p)]
+                ("t_delta", ctypes.c_uint32), ("stream", ctypes.c_void_p)]
 
 
 NK = 8
@@ -56,7 +56,8 @@ class ggrid_stats_t(ctypes.Structure):
                  "objects_written", "arena_used", "arena_capacity", "gc_runs", "launches", "expand_iterations",
                  "expand_vertices", "expand_arcs", "expand_harvested", "expand_objects"]] + [
         ("kernel_launches", ctypes.c_uint64 * NK), ("kernel_ms", ctypes.c_double * NK)] + [
-        (n, ctypes.c_uint32) for n in ["n_cells", "cell_size", "delta", "n_vertices", "n_arcs", "max_objects"]]
+        (n, ctypes.c_uint32) for n in ["n_cells", "cell_size", "delta", "n_vertices", "n_arcs", "max_objects",
+                                       "t_delta", "t_now"]] + [("records_expired", ctypes.c_uint64)]
 
 
 _lib = None
@@ -125,7 +126,7 @@ def _u32(a):
 # ------------------------------------------------------------------------ the C ABI names
 def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 256,
                 max_objects: int = 1 << 24, log_capacity: int = 0, delta: int = 0,
-                seed_neighbors: bool = True, profile: bool = False, stream=None):
+                seed_neighbors: bool = True, profile: bool = False, t_delta: int = 0, stream=None):
     """ggrid_build(graph, cell_size) -> handle (c_void_p).  graph: dict(n_vertices, src, dst, w[, x, y])."""
     src, dst, w = (np.ascontiguousarray(graph[k], np.uint32) for k in ("src", "dst", "w"))
     x = graph.get("x")
@@ -135,7 +136,7 @@ def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 25
     g = ggrid_graph(int(graph["n_vertices"]), len(src), src.ctypes.data, dst.ctypes.data, w.ctypes.data,
                     None if x is None else x.ctypes.data, None if y is None else y.ctypes.data)
     o = ggrid_opts(int(device), int(max_k), int(max_objects), int(log_capacity), int(delta),
-                   0 if seed_neighbors else 2, 1 if profile else 0, 0, stream)
+                   0 if seed_neighbors else 2, 1 if profile else 0, int(t_delta), stream)
     h = ctypes.c_void_p()
     _check(lib().ggrid_build(ctypes.byref(g), int(cell_size), ctypes.byref(o), ctypes.byref(h)), "ggrid_build")
     return h

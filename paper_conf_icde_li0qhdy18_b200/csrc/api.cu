@@ -103,6 +103,7 @@ struct ggrid_s {
   uint32_t V = 0, A = 0, cs = 1, n_cells = 0, delta = 1, max_k = 256, max_objects = 0;
   int seed_neighbors = 1;
   int profile = 0;
+  uint32_t t_delta = 0;  // message expiry window (0 = never)
   std::vector<uint32_t> user_cell;
   DevGraph g{};
   DevState s{};
@@ -112,7 +113,7 @@ struct ggrid_s {
   DevStatus* h_status_dev = nullptr;  // its mapped device alias (the kernels' store target)
   uint64_t seq_next = 0;
   uint32_t epoch = 0;
-  DBuf upd_stage, tmp, q_stage, out_stage, lists, l2_scratch, dump_stage, gc_buf, misc;
+  DBuf upd_stage, tmp, q_stage, out_stage, lists, l2_scratch, dump_stage, gc_buf, misc, flush_spill;
   // pipelined ingest: two staging buffers filled on a copy stream
   struct Staged {
     DBuf buf;
@@ -197,7 +198,16 @@ struct ggrid_s {
 
   int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin, int full_vobj = 0) {
     const uint32_t opc = (uint32_t)((h_status->n_live + n_cells - 1) / std::max(1u, n_cells));
-    launch(GGRID_K_FLUSH, [&] { launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, stream); });
+    uint32_t spill_cap = 0;
+    const size_t sb = flush_spill_bytes(g.cs, opc, sm_count, &spill_cap);
+    if (sb) RC(flush_spill.ensure(sb));
+    uint32_t* spill = sb ? flush_spill.as<uint32_t>() : nullptr;
+    // expiry (reading R21): drop extents whose newest t < t_now - t_delta
+    const uint32_t t_now = h_status->t_max;
+    const uint32_t t_cut = (t_delta && t_now > t_delta) ? t_now - t_delta : 0;
+    launch(GGRID_K_FLUSH, [&] {
+      launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, spill, spill_cap, t_cut, stream);
+    });
     return GGRID_OK;
   }
 
@@ -250,7 +260,8 @@ int ggrid_s::gc() {
   CK(cudaMemcpyAsync(&d_status->arena_top, &top, 8, cudaMemcpyHostToDevice, stream));
   RC(set_status_u32(&d_status->ext_top, 0));
   RC(sync());
-  gc_buf.release();
+  // gc_buf stays allocated (live-sized, small next to the arena): a cudaMalloc/cudaFree pair
+  // per collection costs milliseconds and synchronises the device
   stats.gc_runs++;
   return GGRID_OK;
 }
@@ -338,6 +349,7 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   h->max_objects = o.max_objects;
   h->seed_neighbors = o.seed_neighbors == 2 ? 0 : 1;
   h->profile = o.profile ? 1 : 0;
+  h->t_delta = o.t_delta;
 
   // ---- graph grid: Z-order of quantised coordinates, cells = runs of cell_size vertices
   std::vector<uint32_t> order(V);
@@ -453,6 +465,7 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   if ((rc = h->alloc(&s.x_start, s.ext_cap, false))) return fail(rc);
   if ((rc = h->alloc(&s.x_len, s.ext_cap, false))) return fail(rc);
   if ((rc = h->alloc(&s.x_next, s.ext_cap, false))) return fail(rc);
+  if ((rc = h->alloc(&s.x_tmax, s.ext_cap, false))) return fail(rc);
   if ((rc = h->alloc(&s.cell_head, h->n_cells, false))) return fail(rc);
   if (cudaMemset(s.cell_head, 0xFF, (size_t)h->n_cells * 4)) return fail(GGRID_ECUDA);
   if ((rc = h->alloc(&s.cell_pending, h->n_cells))) return fail(rc);
@@ -482,7 +495,8 @@ int ggrid_free(ggrid_t h) {
   if (h->copy_stream) cudaStreamSynchronize(h->copy_stream);
   for (void* p : h->allocs) cudaFree(p);
   for (DBuf* b : {&h->upd_stage, &h->tmp, &h->q_stage, &h->out_stage, &h->lists, &h->l2_scratch,
-                  &h->dump_stage, &h->gc_buf, &h->misc, &h->staged[0].buf, &h->staged[1].buf})
+                  &h->dump_stage, &h->gc_buf, &h->misc, &h->flush_spill, &h->staged[0].buf,
+                  &h->staged[1].buf})
     b->release();
   for (auto& sb : h->staged)
     if (sb.done) cudaEventDestroy(sb.done);
@@ -753,6 +767,9 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
   s.n_vertices = h->V;
   s.n_arcs = h->A;
   s.max_objects = h->max_objects;
+  s.t_delta = h->t_delta;
+  s.t_now = h->h_status->t_max;
+  s.records_expired = h->h_status->records_expired;
   *out = s;
   return GGRID_OK;
 }

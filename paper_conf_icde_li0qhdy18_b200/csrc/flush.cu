@@ -26,8 +26,9 @@
 //                       sorted by source vertex, v_obj set for the vertices holding objects,
 //                       cell marked clean) and gathers the extent list of cell i+2.
 // One CTA barrier per step.  Cells with more winners than the rank path handles, or GC's
-// full v_obj rewrite, take a counter + warp-scan path; a cell with more than WCAP winners is
-// re-streamed by the index warp.
+// full v_obj rewrite, take a counter + warp-scan path; the positions of winners beyond the
+// shared-memory staging (WCAP) spill to a per-CTA global area, and only a cell that overflows
+// that too is re-streamed by the index warp.
 #include <algorithm>
 
 #include "internal.cuh"
@@ -52,6 +53,7 @@ struct CellBuf {
   uint32_t c, head, has;  // cell id, chain head, this buffer holds a cell
   uint2 comp;             // previous cleaned list
   unsigned long long nrec;
+  unsigned long long nexp;  // records of extents dropped by t_delta expiry
   uint32_t n_win;
   uint32_t w_pos[WCAP];   // arena positions of the matched records
 };
@@ -72,12 +74,19 @@ __device__ __forceinline__ void stream_bar() { asm volatile("bar.sync 1, %0;" ::
 
 // Walk up to XMAX extents of a chain starting at e into buffer bf; the cleaned list `comp`
 // goes last.  One lane.
+// Extents whose newest message is older than t_cut are expired: skipped unread (the paper's
+// bucket discard at cleaning time, P@20631-21157, reading R21).
 template <class B>
-__device__ void walk_extents(B& bf, const DevState& s, uint32_t e, uint2 comp) {
+__device__ void walk_extents(B& bf, const DevState& s, uint32_t e, uint2 comp, uint32_t t_cut) {
   uint32_t n = 0, pre = 0;
-  unsigned long long nrec = 0;
+  unsigned long long nrec = 0, nexp = 0;
   while (e != NONE && n < XMAX) {
     const uint32_t st = s.x_start[e], ln = s.x_len[e], nxt = s.x_next[e];
+    if (t_cut && s.x_tmax[e] < t_cut) {
+      nexp += ln;
+      e = nxt;
+      continue;
+    }
     bf.xs[n] = st;
     bf.xl[n] = ln;
     bf.xpre[n] = pre;
@@ -102,6 +111,7 @@ __device__ void walk_extents(B& bf, const DevState& s, uint32_t e, uint2 comp) {
   bf.nx = n;
   bf.e_next = e;
   bf.nrec += nrec;
+  bf.nexp += nexp;
 }
 
 struct Grp {
@@ -135,7 +145,8 @@ __device__ __forceinline__ Grp load_group(const B& bf, const DevState& s, uint32
 
 // streaming warps: match the gathered extent list of buffer bf
 template <int WCAP, class B>
-__device__ __forceinline__ void stream_list(B& bf, const DevState& s, int sw, int lane, unsigned lt) {
+__device__ __forceinline__ void stream_list(B& bf, const DevState& s, int sw, int lane, unsigned lt,
+                                            uint32_t* __restrict__ spill, uint32_t spill_cap) {
   const unsigned long long* __restrict__ otk = s.ot_key;
   const uint32_t total = bf.xpre[bf.nx];
   int xj = 0;
@@ -159,7 +170,10 @@ __device__ __forceinline__ void stream_list(B& bf, const DevState& s, int sw, in
         if (lane == __ffs(hm) - 1) base = atomicAdd(&bf.n_win, (unsigned)__popc(hm));
         base = __shfl_sync(0xffffffffu, base, __ffs(hm) - 1);
         const uint32_t w = base + __popc(hm & lt);
-        if (hit && w < (uint32_t)WCAP) bf.w_pos[w] = cur.pos + j;
+        if (hit) {
+          if (w < (uint32_t)WCAP) bf.w_pos[w] = cur.pos + j;
+          else if (w - (uint32_t)WCAP < spill_cap) spill[w - WCAP] = cur.pos + j;
+        }
       }
     }
     cur = nxt;
@@ -188,17 +202,23 @@ __device__ uint32_t warp_exclusive_scan(uint32_t* a, uint32_t n, int lane) {
 // index warp: build R[c] for the cell of buffer bf (whose winners are known)
 template <int HCAP, int WCAP, class SM, class B>
 __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, const Arena& out,
-                           unsigned long long* out_top, int full_vobj, int lane) {
+                           unsigned long long* out_top, int full_vobj, int lane,
+                           const uint32_t* __restrict__ spill, uint32_t spill_cap, uint32_t t_cut) {
   const unsigned long long* __restrict__ otk = s.ot_key;
   const uint32_t c = bf.c, head = bf.head;
   const uint2 comp = bf.comp;
   const uint32_t n_win = bf.n_win;
-  const bool overflow = n_win > (uint32_t)WCAP;
+  // winners: staged in shared memory (<= WCAP), positions spilled to this buffer's global
+  // spill area (<= WCAP + spill_cap), else the cell's log is re-streamed (overflow)
+  const bool spilled = n_win > (uint32_t)WCAP && n_win - (uint32_t)WCAP <= spill_cap;
+  const bool overflow = n_win > (uint32_t)WCAP && !spilled;
+  const bool staged = !spilled && !overflow;
+  auto wpos = [&](uint32_t i) { return i < (uint32_t)WCAP ? bf.w_pos[i] : spill[i - WCAP]; };
   const uint32_t cbeg = c * g.cs;
   const uint32_t nvert = min(g.cs, g.V - cbeg);
   unsigned long long o0 = 0;
   if (lane == 0) o0 = atomicAdd(out_top, (n_win + 3u) & ~3ull);  // consumed after staging
-  if (!overflow) {
+  if (staged) {
     for (uint32_t i = lane; i < n_win; i += 32) {  // one gather round of the payload
       const uint32_t p = bf.w_pos[i];
       sm.w_vs[i] = s.ar.vsrc[p];
@@ -218,7 +238,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
   const uint32_t ob0 = (uint32_t)o0;
   // v_obj entries are self-validating (vobj_valid): only vertices holding objects now are
   // written; garbage collection (full_vobj) rewrites every vertex of the cell.
-  if (!overflow && n_win <= (uint32_t)RANKMAX && !full_vobj) {
+  if (staged && n_win <= (uint32_t)RANKMAX && !full_vobj) {
     // slot of a winner = its rank among the winners ordered by (source vertex, index)
     for (uint32_t i = lane; i < n_win; i += 32) {
       const uint32_t vi = sm.w_vs[i];
@@ -250,7 +270,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
         uint32_t sst, sln;
         if (e2 != NONE) {
           sst = s.x_start[e2];
-          sln = s.x_len[e2];
+          sln = (t_cut && s.x_tmax[e2] < t_cut) ? 0u : s.x_len[e2];
           e2 = s.x_next[e2];
         } else {
           sst = comp.x;
@@ -260,8 +280,20 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
         for (uint32_t r = lane; r < sln; r += 32) fn(sst + r);
       }
     };
-    if (!overflow) {
+    if (staged) {
       for (uint32_t i = lane; i < n_win; i += 32) atomicAdd(&cnt[sm.w_vs[i] - cbeg], 1u);
+    } else if (spilled) {
+      constexpr int U = 4;  // four winners per lane in flight
+      for (uint32_t i0 = lane; i0 < n_win; i0 += 32 * U) {
+        uint32_t p[U], vs[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) p[u] = i0 + u * 32 < n_win ? wpos(i0 + u * 32) : 0;
+#pragma unroll
+        for (int u = 0; u < U; ++u) vs[u] = i0 + u * 32 < n_win ? s.ar.vsrc[p[u]] : 0;
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+          if (i0 + u * 32 < n_win) atomicAdd(&cnt[vs[u] - cbeg], 1u);
+      }
     } else {
       for_each_record([&](uint32_t p) {
         if (s.ar.key[p] == otk[s.ar.obj[p]]) atomicAdd(&cnt[s.ar.vsrc[p] - cbeg], 1u);
@@ -276,7 +308,33 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
       if (full_vobj || en != b) s.v_obj[cbeg + i] = make_uint2(ob0 + b, en - b);
     }
     __syncwarp();
-    if (!overflow) {
+    if (spilled) {
+      constexpr int U = 4;
+      for (uint32_t i0 = lane; i0 < n_win; i0 += 32 * U) {
+        uint32_t p[U], ob[U], vs[U], of[U], ed[U];
+        unsigned long long kk[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) p[u] = i0 + u * 32 < n_win ? wpos(i0 + u * 32) : 0;
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          ob[u] = s.ar.obj[p[u]];
+          kk[u] = s.ar.key[p[u]];
+          vs[u] = s.ar.vsrc[p[u]];
+          of[u] = s.ar.off[p[u]];
+          ed[u] = s.ar.edge[p[u]];
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          if (i0 + u * 32 >= n_win) continue;
+          const uint32_t q = ob0 + atomicAdd(&cnt[vs[u] - cbeg], 1u);
+          out.obj[q] = ob[u];
+          out.key[q] = kk[u];
+          out.vsrc[q] = vs[u];
+          out.off[q] = of[u];
+          out.edge[q] = ed[u];
+        }
+      }
+    } else if (staged) {
       for (uint32_t i = lane; i < n_win; i += 32) {
         const uint32_t vs = sm.w_vs[i];
         const uint32_t q = ob0 + atomicAdd(&cnt[vs - cbeg], 1u);
@@ -309,13 +367,15 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
     atomicAdd(&s.st->objects_written, (unsigned long long)n_win);
     atomicAdd(&s.st->cells_flushed, 1ull);
     atomicAdd(&s.st->records_flushed, bf.nrec);
+    if (bf.nexp) atomicAdd(&s.st->records_expired, bf.nexp);
   }
 }
 
 template <int HCAP, int WCAP>
 __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
                                               unsigned long long* out_top, uint32_t begin,
-                                              int full_vobj) {
+                                              int full_vobj, uint32_t* spill, uint32_t spill_cap,
+                                              uint32_t t_cut) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   using SM = FlushSmem<HCAP, WCAP>;
   SM& sm = *reinterpret_cast<SM*>(smem_raw);
@@ -327,6 +387,10 @@ __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
   const uint32_t first_li = begin + blockIdx.x;
   const uint32_t n_mine = first_li < lend ? (lend - first_li + G - 1) / G : 0;
   const bool is_index = wid == SW;
+  // this CTA's spill area of buffer k % NBUF
+  auto spill_of = [&](uint32_t k) {
+    return spill + ((size_t)blockIdx.x * NBUF + k % NBUF) * spill_cap;
+  };
 
   // index-warp lane 0 gathers cells ahead of the stream; the next cell's list entry, chain
   // head and cleaned list are loaded one gather ahead
@@ -336,6 +400,7 @@ __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
     auto& bf = sm.b[k % NBUF];
     bf.n_win = 0;
     bf.nrec = 0;
+    bf.nexp = 0;
     bf.has = k < n_mine;
     if (!bf.has) {
       bf.nx = 0;
@@ -353,7 +418,7 @@ __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
     bf.c = c;
     bf.head = head;
     bf.comp = comp;
-    walk_extents(bf, s, head, comp);
+    walk_extents(bf, s, head, comp, t_cut);
   };
 
   if (is_index && lane == 0 && n_mine) {
@@ -370,16 +435,18 @@ __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
       auto& bf = sm.b[k % NBUF];
       if (k < n_mine) {
         for (;;) {
-          stream_list<WCAP>(bf, s, wid, lane, lt);
+          stream_list<WCAP>(bf, s, wid, lane, lt, spill_of(k), spill_cap);
           if (bf.comp_done) break;
           // chains longer than XMAX extents: the streaming warps gather the next part
           stream_bar();
-          if (tid == 0) walk_extents(bf, s, bf.e_next, bf.comp);
+          if (tid == 0) walk_extents(bf, s, bf.e_next, bf.comp, t_cut);
           stream_bar();
         }
       }
     } else {
-      if (k >= 1) index_cell<HCAP, WCAP>(sm, sm.b[(k - 1) % NBUF], g, s, out, out_top, full_vobj, lane);
+      if (k >= 1)
+        index_cell<HCAP, WCAP>(sm, sm.b[(k - 1) % NBUF], g, s, out, out_top, full_vobj, lane,
+                               spill_of(k - 1), spill_cap, t_cut);
       if (lane == 0) gather(k + 2);
       __syncwarp();
     }
@@ -388,8 +455,17 @@ __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
 }
 
 template <int HCAP, int WCAP>
+int blocks_per_sm_t();
+template <int HCAP, int WCAP>
 void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned long long* out_top,
-              uint32_t begin, int full_vobj, int sm_count, cudaStream_t st) {
+              uint32_t begin, int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap,
+              uint32_t t_cut, cudaStream_t st) {
+  const int blocks_per_sm = blocks_per_sm_t<HCAP, WCAP>();
+  k_flush<HCAP, WCAP><<<sm_count * blocks_per_sm, FT, sizeof(FlushSmem<HCAP, WCAP>), st>>>(
+      g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
+}
+template <int HCAP, int WCAP>
+int blocks_per_sm_t() {
   static int blocks_per_sm = 0;
   const int smem = (int)sizeof(FlushSmem<HCAP, WCAP>);
   if (blocks_per_sm == 0) {
@@ -403,25 +479,53 @@ void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned l
     cudaFuncSetAttribute(k_flush<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
     blocks_per_sm = b;
   }
-  k_flush<HCAP, WCAP><<<sm_count * blocks_per_sm, FT, smem, st>>>(g, s, out, out_top, begin, full_vobj);
+  return blocks_per_sm;
 }
 }  // namespace
 
+// the variant for a given cell size and average objects per cell: staging sized for ~2x the
+// live objects of an average cell (more winners spill their positions to global memory)
+static int flush_variant(uint32_t cs, uint32_t objects_per_cell) {
+  const int h = cs <= 1024 ? 0 : 1;
+  const int w = objects_per_cell <= 64 ? 0 : objects_per_cell <= 256 ? 1 : 2;
+  return w * 2 + h;
+}
+static const uint32_t kWcap[3] = {128, 512, 2048};
+
+size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, uint32_t* cap) {
+  const int v = flush_variant(cs, objects_per_cell);
+  const uint32_t wcap = kWcap[v / 2];
+  // room for 4x the average cell beyond the staging (a cell with more is re-streamed)
+  uint32_t want = 0;
+  if (4ull * objects_per_cell > wcap) {
+    want = 1024;
+    while (want < 4ull * objects_per_cell - wcap && want < (1u << 20)) want <<= 1;
+  }
+  *cap = want;
+  if (!want) return 0;
+  int bps = 0;
+  switch (v) {
+    case 0: bps = blocks_per_sm_t<1024, 128>(); break;
+    case 1: bps = blocks_per_sm_t<4096, 128>(); break;
+    case 2: bps = blocks_per_sm_t<1024, 512>(); break;
+    case 3: bps = blocks_per_sm_t<4096, 512>(); break;
+    case 4: bps = blocks_per_sm_t<1024, 2048>(); break;
+    default: bps = blocks_per_sm_t<4096, 2048>(); break;
+  }
+  return (size_t)sm_count * bps * NBUF * want * sizeof(uint32_t);
+}
+
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
-                  int full_vobj, int sm_count, cudaStream_t st) {
-  // staging sized for ~2x the live objects of an average cell (more winners fall back to a
-  // re-streaming pass of the index warp)
-  const bool small_h = g.cs <= 1024;
-  if (objects_per_cell <= 64) {
-    if (small_h) launch_t<1024, 128>(g, s, out, out_top, begin, full_vobj, sm_count, st);
-    else launch_t<4096, 128>(g, s, out, out_top, begin, full_vobj, sm_count, st);
-  } else if (objects_per_cell <= 256) {
-    if (small_h) launch_t<1024, 512>(g, s, out, out_top, begin, full_vobj, sm_count, st);
-    else launch_t<4096, 512>(g, s, out, out_top, begin, full_vobj, sm_count, st);
-  } else {
-    if (small_h) launch_t<1024, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, st);
-    else launch_t<4096, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, st);
+                  int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap, uint32_t t_cut,
+                  cudaStream_t st) {
+  switch (flush_variant(g.cs, objects_per_cell)) {
+    case 0: launch_t<1024, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
+    case 1: launch_t<4096, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
+    case 2: launch_t<1024, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
+    case 3: launch_t<4096, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
+    case 4: launch_t<1024, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
+    default: launch_t<4096, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
   }
 }
 

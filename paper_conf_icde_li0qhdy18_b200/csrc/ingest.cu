@@ -26,22 +26,26 @@ constexpr int CU = CT * CPT;       // updates per CTA (tile)
 constexpr int CH = 4096;           // hash slots (>= 2*CU)
 constexpr int SPC = CH / CT;       // hash slots per thread in the scan
 static_assert(CU < 65536, "tile offsets and counts are packed in 16 bits");
+constexpr int CLASSIFY_SMEM = (3 * CH + CT / 32) * 4;
 
 __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
                                                         DevGraph g, DevState s,
                                                         uint2* __restrict__ tmp,
                                                         uint16_t* __restrict__ perm) {
-  __shared__ __align__(16) uint32_t h_buf[2 * CH];
-  uint32_t* h_cell = h_buf;       // cell id; after the claim, the cell's global rank base
-  uint32_t* h_cnt = h_buf + CH;   // count; after the scan, (tile offset << 16) | count
-  __shared__ uint32_t w_sum[CT / 32];
+  extern __shared__ __align__(16) uint32_t h_buf[];  // CLASSIFY_SMEM bytes
+  uint32_t* h_cell = h_buf;           // cell id; after the claim, the cell's global rank base
+  uint32_t* h_cnt = h_buf + CH;       // count; after the scan, (tile offset << 16) | count
+  uint32_t* h_tmax = h_buf + 2 * CH;  // newest t per cell (the extent's zeta.t)
+  uint32_t* w_sum = h_buf + 3 * CH;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   for (int i = tid; i < CH; i += CT) {
     h_cell[i] = NONE;
     h_cnt[i] = 0;
+    h_tmax[i] = 0;
   }
   __syncthreads();
   const uint64_t base = (uint64_t)blockIdx.x * CU;
+  uint32_t tl = 0;  // this thread's newest t
   int slot[CPT];
   uint32_t vs[CPT], lr[CPT];
   // all CPT record loads in flight, then all CPT inverted-index gathers, then the hashing
@@ -88,7 +92,11 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
     slot[j] = (int)h;
     vs[j] = e.x;
     lr[j] = atomicAdd(&h_cnt[h], 1u);
+    atomicMax(&h_tmax[h], m.w);
+    tl = max(tl, m.w);
   }
+  tl = __reduce_max_sync(0xffffffffu, tl);
+  if (lane == 0 && tl) atomicMax(&s.st->t_max, tl);
   __syncthreads();
   // exclusive scan of the slot counts = each cell's group offset in the tile's sorted order
   {
@@ -114,7 +122,10 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
   }
   for (int i = tid; i < CH; i += CT) {
     const uint32_t c = h_cell[i];
-    if (c != NONE) h_cell[i] = atomicAdd(&s.bcount[c * BCOUNT_STRIDE], h_cnt[i] & 0xFFFFu);
+    if (c != NONE) {
+      atomicMax(&s.bcount[c * BCOUNT_STRIDE + 1], h_tmax[i]);
+      h_cell[i] = atomicAdd(&s.bcount[c * BCOUNT_STRIDE], h_cnt[i] & 0xFFFFu);
+    }
   }
   __syncthreads();
   uint32_t si[CPT], rk[CPT];
@@ -147,7 +158,10 @@ __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
   const bool err = s.st->err != 0;
   uint32_t cnt = (c < g.n_cells) ? s.bcount[c * BCOUNT_STRIDE] : 0;
   if (err) {
-    if (c < g.n_cells && cnt) s.bcount[c * BCOUNT_STRIDE] = 0;
+    if (c < g.n_cells && cnt) {
+      s.bcount[c * BCOUNT_STRIDE] = 0;
+      s.bcount[c * BCOUNT_STRIDE + 1] = 0;
+    }
     return;
   }
   unsigned lane = threadIdx.x & 31;
@@ -179,6 +193,8 @@ __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
   }
   s.x_start[e] = (uint32_t)start;
   s.x_len[e] = cnt;
+  s.x_tmax[e] = s.bcount[c * BCOUNT_STRIDE + 1];
+  s.bcount[c * BCOUNT_STRIDE + 1] = 0;
   s.x_next[e] = s.cell_head[c];
   s.cell_head[c] = e;
   s.cell_pending[c] += cnt;
@@ -259,8 +275,13 @@ static uint16_t* perm_of(uint2* tmp, uint64_t n) { return reinterpret_cast<uint1
 size_t ingest_tmp_bytes(uint64_t n) { return (size_t)n * (sizeof(uint2) + sizeof(uint16_t)); }
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
                             uint2* tmp, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_ingest_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, CLASSIFY_SMEM);
+    attr = true;
+  }
   unsigned blocks = (unsigned)((n + CU - 1) / CU);
-  k_ingest_classify<<<blocks, CT, 0, st>>>(upd, n, g, s, tmp, perm_of(tmp, n));
+  k_ingest_classify<<<blocks, CT, CLASSIFY_SMEM, st>>>(upd, n, g, s, tmp, perm_of(tmp, n));
 }
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st) {
   k_ingest_alloc<<<(g.n_cells + 255) / 256, 256, 0, st>>>(g, s);

@@ -38,10 +38,12 @@ struct DevStatus {
   unsigned long long objects_written;
   unsigned long long cells_flushed;
   unsigned long long ex_iters, ex_vertices, ex_arcs, ex_harvested, ex_objects;  // expansion work
+  unsigned long long records_expired;  // dropped unread by t_delta expiry
   unsigned int ext_top;     // next free extent
   unsigned int err;         // ErrBits
   unsigned int bad_index;   // smallest offending index (ingest)
   unsigned int n_live;      // objects with at least one update
+  unsigned int t_max;       // largest t ingested (t_now of the expiry rule)
   unsigned int n_flush;     // entries in flush_list
   unsigned int flush_work;  // persistent flush work counter
   unsigned int n_next[4];   // per expansion level: queries queued for the next round
@@ -79,6 +81,7 @@ struct DevState {
   uint32_t* x_start;  // extents
   uint32_t* x_len;
   uint32_t* x_next;
+  uint32_t* x_tmax;   // newest t of the extent's messages (zeta.t, P@20743)
   uint32_t ext_cap;
   uint32_t* cell_head;     // newest pending extent or NONE (NONE = clean)
   uint32_t* cell_pending;  // cached records not yet cleaned
@@ -86,8 +89,9 @@ struct DevState {
   uint2* v_obj;            // [V] (arena start, count) of the objects at each vertex
   uint2* cell_comp;        // [n_cells] (arena start, count) of the cell's compacted list
   uint32_t* vcnt;          // [V] flush scratch, only when cell_size > 4096 (else null)
-  uint32_t* bcount;        // [n_cells * BCOUNT_STRIDE] per-batch counts, one 128-byte line per
-                           // cell (same-line atomics from every ingest CTA serialise in L2)
+  uint32_t* bcount;        // [n_cells * BCOUNT_STRIDE] per-batch count ([0]) and newest t ([1]),
+                           // one 128-byte line per cell (same-line atomics from every ingest
+                           // CTA serialise in L2)
   uint32_t* bbase;         // [n_cells] per-batch arena base
   uint32_t* flush_list;    // [n_cells]
   DevStatus* st;
@@ -168,9 +172,14 @@ void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int
                        cudaStream_t st);
 // Flush the cells flush_list[begin .. st->n_flush) writing compacted lists into `out`
 // (out == s.ar for a regular flush; a fresh arena for garbage collection).
+// spill: per-CTA global staging of winner positions beyond shared memory, sized by
+// flush_spill_bytes (which also returns its per-buffer capacity; 0 = none needed)
+size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, uint32_t* cap);
+// t_cut: extents whose newest t is below it are expired (dropped unread); 0 = none
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
-                  int full_vobj, int sm_count, cudaStream_t st);
+                  int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap, uint32_t t_cut,
+                  cudaStream_t st);
 
 // v_obj[v] = (start, n) is valid only if start lies inside the cell's current cleaned list
 // (lists only move up the arena between garbage collections, which rewrite every entry).

@@ -324,6 +324,91 @@ def test_flush_long_chains_and_overflow(gg):
     grid.close()
 
 
+def test_flush_spill_paths(gg):
+    """Many objects per cell (the wider staging variant): one cell with more winners than the
+    shared-memory staging (positions spill to global memory), one beyond the spill area too
+    (re-stream), plus a random walk; GC (full v_obj rewrite) over the same state."""
+    g = synth.table_ii_graph("NY", scale=0.03)
+    grid = gg.GGrid(g, 64, max_objects=30_000, log_capacity=120_000)  # small: forces GC
+    vcell = grid.vertex_cell()
+    rng = np.random.default_rng(11)
+    parts, oid = [], 0
+    for cell, n_hot in ((0, 900), (1, 3000)):
+        hot = np.flatnonzero(vcell[g["src"]] == cell)
+        e = hot[rng.integers(0, len(hot), n_hot)].astype(np.uint32)
+        d = (rng.random(n_hot) * g["w"][e]).astype(np.uint32)
+        parts.append(np.stack([np.arange(oid, oid + n_hot, dtype=np.uint32), e, d,
+                               np.full(n_hot, 5, np.uint32)], 1))
+        oid += n_hot
+    walk = synth.RandomWalk(g, 18_000, obj_ids=np.arange(oid, oid + 18_000, dtype=np.uint32))
+    hist = parts + [walk.ticks(3)]
+    for u in hist:
+        grid.ingest(u)
+    q = synth.queries(g, 200)
+    for i, cell in enumerate((0, 1)):
+        hot = np.flatnonzero(vcell[g["src"]] == cell)
+        q[20 * i:20 * i + 20, 0] = hot[:20]
+        q[20 * i:20 * i + 20, 1] = 0
+    allu = np.concatenate(hist)
+    _assert_same(grid.knn(q, 40), _oracle(g, allu, q, 40), "spill + re-stream")
+    u = walk.ticks(2)
+    allu = np.concatenate([allu, u])
+    grid.ingest(u)
+    grid.flush_all()
+    _assert_same(grid.knn(q, 40), _oracle(g, allu, q, 40), "after flush_all")
+    st = grid.stats()
+    assert st["kernel_launches"]["flush"] >= 2 and st["gc_runs"] >= 1, st
+    grid.close()
+
+
+def test_expiry_honoured_is_exact(gg):
+    """t_delta expiry (P@20631-21157, reading R21) when every object reports within t_delta:
+    extents older than t_now - t_delta are dropped unread and the answers stay exact."""
+    g = synth.table_ii_graph("NY", scale=0.05)
+    walk = synth.RandomWalk(g, 3000)  # every object reports once per tick (t = tick*1000+U[0,999])
+    grid = gg.GGrid(g, 256, max_objects=3000, t_delta=2000)
+    hist = []
+    for tick in range(12):
+        u = walk.tick()
+        hist.append(u)
+        grid.ingest(u)
+        if tick == 5:  # clean some cells midway
+            grid.knn(synth.queries(g, 20, seed=5), 5)
+    q = synth.queries(g, 300)
+    allu = np.concatenate(hist)
+    _assert_same(grid.knn(q, 16), _oracle(g, allu, q, 16), "expiry, honoured")
+    st = grid.stats()
+    assert st["t_now"] == int(allu[:, 3].max()) and st["t_delta"] == 2000
+    assert st["records_expired"] > 0, st
+    grid.flush_all()
+    _assert_same(grid.knn(q, 16), _oracle(g, allu, q, 16), "expiry, after flush_all")
+    grid.close()
+
+
+def test_expiry_drops_silent_objects(gg):
+    """An object silent for longer than t_delta (the paper's reporting assumption violated,
+    P@20935) disappears when its cached extent expires; without expiry it stays."""
+    g = synth.table_ii_graph("NY", scale=0.05)
+    walk = synth.RandomWalk(g, 800, obj_ids=np.arange(1, 801, dtype=np.uint32))
+    e0 = np.uint32(17)
+    silent = np.array([[0, e0, 0, 0]], np.uint32)  # object 0 at t = 0, alone in its batch
+    ticks = []
+    for _ in range(6):
+        u = walk.tick()
+        u[:, 3] += 1000  # the walk starts at t = 1000
+        ticks.append(u)
+    q = np.array([[e0, 0]], np.uint32)  # right at object 0
+    for t_delta, expect_silent in ((0, True), (2000, False)):
+        grid = gg.GGrid(g, 256, max_objects=801, t_delta=t_delta)
+        for u in [silent] + ticks:
+            grid.ingest(u)
+        go, gd = grid.knn(q, 5)
+        ref_upd = np.concatenate(([silent] if expect_silent else []) + ticks)
+        _assert_same((go, gd), _oracle(g, ref_upd, q, 5), f"t_delta={t_delta}")
+        assert (0 in go[0]) == expect_silent
+        grid.close()
+
+
 def test_bench_configuration_steady_state(gg):
     """The launch configuration bench.py times (C1: NY graph, cell_size 1024, profile mode on a
     caller stream, 1M updates + 10k queries per step): every query of the first step and 1,000

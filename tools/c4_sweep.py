@@ -25,6 +25,7 @@ import synth  # noqa: E402
 from synth.device_walk import DeviceRandomWalk  # noqa: E402
 
 SEQ_LIMIT = (1 << 32) - 1
+TRACE = os.environ.get("C4_TRACE")
 
 
 def run_one(g, gname, n_obj, r, Q, k, cell_size, max_steps, l2):
@@ -49,6 +50,12 @@ def run_one(g, gname, n_obj, r, Q, k, cell_size, max_steps, l2):
         l2.zero_()
         torch.cuda.synchronize()
         grid.stats_reset()
+        st0 = grid.stats()
+        prof = None
+        if TRACE and s == n_steps:
+            from torch.profiler import ProfilerActivity, profile
+            prof = profile(activities=[ProfilerActivity.CUDA, ProfilerActivity.CPU])
+            prof.__enter__()
         e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
         e0.record()
         grid.ingest(u)
@@ -56,7 +63,15 @@ def run_one(g, gname, n_obj, r, Q, k, cell_size, max_steps, l2):
         grid.knn(q, k, out_o, out_d)
         e2.record()
         torch.cuda.synchronize()
+        if prof is not None:
+            prof.__exit__(None, None, None)
+            evs = sorted((e.time_range.start, e.time_range.end, e.name[:70]) for e in prof.events())
+            with open(TRACE, "w") as f:
+                for a, b, nm in evs:
+                    f.write(f"{a - evs[0][0]:10.1f} {b - evs[0][0]:10.1f} {b - a:8.1f}  {nm}\n")
         st = grid.stats()
+        for key in ("records_flushed", "cells_flushed", "objects_written", "knn_rounds", "gc_runs"):
+            st[key] -= st0[key]
         if s == 0:
             continue
         km = st["kernel_ms"]
@@ -89,6 +104,8 @@ def main():
     ap.add_argument("--cell-size", type=int, default=1024)
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--max-updates", type=float, default=1.0e9, help="skip combos above this")
+    ap.add_argument("--max-ticks", type=float, default=2.0e4,
+                    help="skip combos whose step needs more walk ticks (generator time)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "c4_sweep.jsonl"))
     a = ap.parse_args()
     l2 = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -97,7 +114,8 @@ def main():
             g = synth.config_graph(cfg)
             for n_obj in [int(float(x)) for x in a.objects.split(",")]:
                 for r in [int(float(x)) for x in a.r.split(",")]:
-                    if r * a.queries > a.max_updates:
+                    if r * a.queries > a.max_updates or r * a.queries / n_obj > a.max_ticks:
+                        print(f"{cfg} |O|={n_obj:>8} r={r:>6}: skipped (generator budget)", flush=True)
                         continue
                     res = run_one(g, cfg, n_obj, r, a.queries, a.k, a.cell_size, a.steps, l2)
                     f.write(json.dumps(res) + "\n")
