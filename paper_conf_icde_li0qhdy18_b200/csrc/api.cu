@@ -635,7 +635,13 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   h->launch(GGRID_K_SEED, [&] { launch_seed(d_q, n_q, g, s, epoch, h->seed_neighbors, q_copy, st); });
   if (q_copy) d_q = q_copy;
 
+  // starting level: k must fit the candidate list, and the vertex table should hold the
+  // expected ball (k objects at the current density need ~k |V| / |O| vertices; the table
+  // also holds the frontier and stays below ~1/3 load).  A guess only: a query that
+  // overflows is promoted, the answer does not depend on it.
   int lvl0 = 0;
+  const double ball = (double)k * h->V / std::max(1u, h->h_status->n_live);
+  while (lvl0 < L - 2 && (k > expand_max_k(lvl0) || 3.0 * ball > expand_table_slots(lvl0))) lvl0++;
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
   std::vector<uint32_t> n_in(L, 0);
   n_in[lvl0] = n_q;
@@ -647,8 +653,8 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
     RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin));
     if (round > 0) {  // round 0 was reset with the rest at the start
       WordSet ws;
-      ws.zero_range(h->d_status->n_next, 4);
-      ws.zero_range(h->d_status->expand_work, 4);
+      ws.zero_range(h->d_status->n_next, EXPAND_LEVELS);
+      ws.zero_range(h->d_status->expand_work, EXPAND_LEVELS);
       RC(h->set_words(ws));
     }
     for (int lvl = 0; lvl < L; ++lvl) {

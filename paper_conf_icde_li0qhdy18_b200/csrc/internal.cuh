@@ -21,6 +21,7 @@ constexpr uint32_t NONE = 0xFFFFFFFFu;
 constexpr uint32_t INF = 0xFFFFFFFFu;  // u32 distance "unreachable" (reading R18)
 constexpr unsigned long long EMPTY64 = ~0ull;
 constexpr uint32_t BCOUNT_STRIDE = 32;
+constexpr int EXPAND_LEVELS = 5;  // capacity ladder of the expansion (csrc/knn.cu)
 
 enum ErrBits : unsigned {
   ERR_OBJ = 1u,      // update obj >= max_objects
@@ -46,9 +47,9 @@ struct DevStatus {
   unsigned int t_max;       // largest t ingested (t_now of the expiry rule)
   unsigned int n_flush;     // entries in flush_list
   unsigned int flush_work;  // persistent flush work counter
-  unsigned int n_next[4];   // per expansion level: queries queued for the next round
+  unsigned int n_next[EXPAND_LEVELS];   // per expansion level: queries queued for the next round
   unsigned int flush_end;   // n_flush as seen by the last flush launch
-  unsigned int expand_work[4];  // per-level dynamic work counters of the expand launches
+  unsigned int expand_work[EXPAND_LEVELS];  // per-level dynamic work counters of the expand launches
   unsigned int round_end;   // (marks the end of the per-round reset region)
 };
 
@@ -194,6 +195,7 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
                    uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist, void* scratch,
                    uint32_t scratch_warps, int sm_count, cudaStream_t st);
 int expand_levels();
+uint32_t expand_table_slots(int level);  // vertex-table capacity H of a level
 uint32_t expand_max_k(int level);
 size_t expand_warp_bytes(int level, uint32_t V);
 void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t* obj,

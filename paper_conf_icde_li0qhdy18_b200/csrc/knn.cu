@@ -468,20 +468,21 @@ __global__ void k_expand(QParams P) {
   }
 }
 
-// Capacity ladder.  Levels 0-2 keep the warp's working set in shared memory (one warp per
-// CTA, as many CTAs per SM as fit); level 3 is global memory sized from |V| (a query that
-// reaches fewer than k objects may need to settle the whole graph).
-constexpr int NLEVELS = 4;
+// Capacity ladder.  Levels 0-3 keep the warp's working set in shared memory (one warp per
+// CTA, as many CTAs per SM as fit: ~10, 24, 45 and 190 KB per warp); level 4 is global memory
+// sized from |V| (a query that reaches fewer than k objects may need to settle the whole
+// graph).
+constexpr int NLEVELS = EXPAND_LEVELS;
 #ifndef GG_H0
 #define GG_H0 1024  // level-0 vertex table (experiment hook: -DGG_H0=..., -DGG_F0=...)
 #endif
 #ifndef GG_F0
 #define GG_F0 128
 #endif
-const Caps kCaps[3] = {{GG_H0, GG_F0, 64}, {2048, 512, 256}, {16384, 4096, 2048}};
+const Caps kCaps[NLEVELS - 1] = {{GG_H0, GG_F0, 64}, {2048, 512, 256}, {4096, 1024, 256}, {16384, 4096, 2048}};
 
 Caps caps_for(int level, uint32_t V) {
-  if (level < 3) return kCaps[level];
+  if (level < NLEVELS - 1) return kCaps[level];
   uint32_t H = 1u << 15;
   while (H < 2ull * V && H < (1u << 27)) H <<= 1;
   const uint32_t F = std::min<uint32_t>(H / 2, 1u << 22);
@@ -489,10 +490,12 @@ Caps caps_for(int level, uint32_t V) {
 }
 
 bool g_attr_set = false;
-int g_blocks_per_sm[NLEVELS] = {0, 0, 0, 0};
+int g_blocks_per_sm[NLEVELS] = {};
 }  // namespace
 
 int expand_levels() { return NLEVELS; }
+
+uint32_t expand_table_slots(int level) { return caps_for(level, 1).H; }
 
 uint32_t expand_max_k(int level) { return caps_for(level, 1).C - 32; }
 
