@@ -167,6 +167,47 @@ int ggrid_ingest_commit(ggrid_t h);
 int ggrid_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
               uint32_t* out_dist);
 
+/* ---- cell-ownership sharding across ranks (one process per GPU) ------------
+ *
+ * ggrid_shard makes this handle rank `rank` of `n_ranks` (<= 64): it owns the contiguous
+ * Z-order range of cells c with floor(c * n_ranks / n_cells) == rank.  Every rank ingests the
+ * full update stream (the object table stays replicated, so the validity test of reading R8
+ * holds everywhere) but keeps message logs and cleaned lists only for its own cells.  Must be
+ * called before the first ingest.  Errors: EINVAL (ranges, or updates already ingested).
+ *
+ * An exact kNN answer then takes one request/reply exchange (orchestrated by the caller over
+ * NCCL; paper_conf_icde_li0qhdy18_b200/dist.py):
+ *   1. the owner of the query's cell (ggrid_query_owner) runs ggrid_knn_ex with out_remote:
+ *      its k nearest among its own objects, and the mask of ranks whose cells the expansion
+ *      entered before it stopped;
+ *   2. each masked rank runs ggrid_knn_ex with bound = the owner's k-th distance (PAD if the
+ *      owner found fewer than k): its own objects within that radius (inclusive), k at most;
+ *   3. ggrid_merge_topk merges the owner's list and the replies.
+ * Exactness: every object of the global answer is within the owner's k-th distance l; such
+ * an object lies at a vertex the owner's expansion settled (all vertices closer than its
+ * stopping radius > l), so its cell's owner is in the mask, and that owner's bounded answer
+ * contains it (fewer than k of its own objects precede it). */
+int ggrid_shard(ggrid_t h, uint32_t n_ranks, uint32_t rank);
+
+/* Owner rank of each query: the rank owning the cell of the query arc's source vertex (where
+ * objects on the query's own arc are indexed).  q, out_rank: host or device. */
+int ggrid_query_owner(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t* out_rank);
+
+/* ggrid_knn with two optional arguments (NULL = as ggrid_knn):
+ *   bound      n_q u32, host or device: return only objects at distance <= bound[i] (rows
+ *              padded with GGRID_PAD beyond), and stop expanding past it;
+ *   out_remote n_q u64, host or device: bit r set iff the expansion of query i entered a
+ *              cell owned by rank r != this rank (sharded handles; 0 otherwise). */
+int ggrid_knn_ex(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, const uint32_t* bound,
+                 uint32_t* out_obj, uint32_t* out_dist, uint64_t* out_remote);
+
+/* Merge n_lists (<= 32) per-query answer lists, each ascending in (dist, obj) and padded with
+ * GGRID_PAD, laid out [n_lists][n_q][k] (lists_obj / lists_dist), into the k smallest
+ * (dist, obj) per query (the final first-k of the candidate union, P@49436-49765, P@51679).
+ * Lists must be disjoint in objects.  Host or device pointers. */
+int ggrid_merge_topk(ggrid_t h, uint32_t n_lists, uint32_t n_q, uint32_t k, const uint32_t* lists_obj,
+                     const uint32_t* lists_dist, uint32_t* out_obj, uint32_t* out_dist);
+
 /* Release every resource of h (NULL is accepted). */
 int ggrid_free(ggrid_t h);
 

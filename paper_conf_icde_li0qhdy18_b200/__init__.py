@@ -25,7 +25,7 @@ KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "fl
                 "expand_big", "other"]
 EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_flush_all",
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
-           "ggrid_version"]
+           "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk"]
 
 
 class GGridError(RuntimeError):
@@ -86,6 +86,10 @@ def lib():
             "ggrid_vertex_cell": ([P, P], i32),
             "ggrid_zvalue": ([u32, u32], u64),
             "ggrid_version": ([], ctypes.c_char_p),
+            "ggrid_shard": ([P, u32, u32], i32),
+            "ggrid_query_owner": ([P, P, u32, P], i32),
+            "ggrid_knn_ex": ([P, P, u32, u32, P, P, P, P], i32),
+            "ggrid_merge_topk": ([P, u32, u32, u32, P, P, P, P], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -175,6 +179,50 @@ def ggrid_knn(h, queries, k: int, out_obj=None, out_dist=None):
     return out_obj, out_dist
 
 
+def ggrid_knn_ex(h, queries, k: int, bound=None, out_obj=None, out_dist=None, out_remote=None):
+    """ggrid_knn with an optional per-query distance bound (n,) u32 and per-query remote-rank
+    masks (n,) u64 (pass an array/tensor, or True for a new numpy array).  Returns
+    (out_obj, out_dist, out_remote)."""
+    q = _u32(queries)
+    nq = int(q.shape[0])
+    if out_obj is None:
+        out_obj = np.empty((nq, k), np.uint32)
+    if out_dist is None:
+        out_dist = np.empty((nq, k), np.uint32)
+    if out_remote is True:
+        out_remote = np.empty(nq, np.uint64)
+    b = None if bound is None else _u32(bound)
+    _check(lib().ggrid_knn_ex(h, _ptr(q), nq, int(k), _ptr(b), _ptr(out_obj), _ptr(out_dist), _ptr(out_remote)),
+           "ggrid_knn_ex")
+    return out_obj, out_dist, out_remote
+
+
+def ggrid_shard(h, n_ranks: int, rank: int):
+    _check(lib().ggrid_shard(h, int(n_ranks), int(rank)), "ggrid_shard")
+
+
+def ggrid_query_owner(h, queries, out_rank=None):
+    q = _u32(queries)
+    nq = int(q.shape[0])
+    if out_rank is None:
+        out_rank = np.empty(nq, np.uint32)
+    _check(lib().ggrid_query_owner(h, _ptr(q), nq, _ptr(out_rank)), "ggrid_query_owner")
+    return out_rank
+
+
+def ggrid_merge_topk(h, lists_obj, lists_dist, out_obj=None, out_dist=None):
+    """lists_obj / lists_dist: (n_lists, n_q, k) u32; returns (out_obj, out_dist) (n_q, k)."""
+    lo, ld = _u32(lists_obj), _u32(lists_dist)
+    L, nq, k = (int(x) for x in lo.shape)
+    if out_obj is None:
+        out_obj = np.empty((nq, k), np.uint32)
+    if out_dist is None:
+        out_dist = np.empty((nq, k), np.uint32)
+    _check(lib().ggrid_merge_topk(h, L, nq, k, _ptr(lo), _ptr(ld), _ptr(out_obj), _ptr(out_dist)),
+           "ggrid_merge_topk")
+    return out_obj, out_dist
+
+
 def ggrid_free(h):
     if h:
         lib().ggrid_free(h)
@@ -248,6 +296,19 @@ class GGrid:
 
     def knn(self, queries, k: int, out_obj=None, out_dist=None):
         return ggrid_knn(self.h, queries, k, out_obj, out_dist)
+
+    def knn_ex(self, queries, k: int, bound=None, out_obj=None, out_dist=None, out_remote=None):
+        return ggrid_knn_ex(self.h, queries, k, bound, out_obj, out_dist, out_remote)
+
+    def shard(self, n_ranks: int, rank: int):
+        ggrid_shard(self.h, n_ranks, rank)
+        return self
+
+    def query_owner(self, queries, out_rank=None):
+        return ggrid_query_owner(self.h, queries, out_rank)
+
+    def merge_topk(self, lists_obj, lists_dist, out_obj=None, out_dist=None):
+        return ggrid_merge_topk(self.h, lists_obj, lists_dist, out_obj, out_dist)
 
     def flush_all(self):
         ggrid_flush_all(self.h)

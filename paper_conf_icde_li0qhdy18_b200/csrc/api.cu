@@ -113,7 +113,8 @@ struct ggrid_s {
   DevStatus* h_status_dev = nullptr;  // its mapped device alias (the kernels' store target)
   uint64_t seq_next = 0;
   uint32_t epoch = 0;
-  DBuf upd_stage, tmp, q_stage, out_stage, lists, l2_scratch, dump_stage, gc_buf, misc, flush_spill;
+  DBuf upd_stage, tmp, q_stage, out_stage, lists, l2_scratch, dump_stage, gc_buf, misc, flush_spill,
+      bound_stage, remote_stage, merge_stage;
   // pipelined ingest: two staging buffers filled on a copy stream
   struct Staged {
     DBuf buf;
@@ -350,6 +351,8 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   h->seed_neighbors = o.seed_neighbors == 2 ? 0 : 1;
   h->profile = o.profile ? 1 : 0;
   h->t_delta = o.t_delta;
+  h->s.n_ranks = 1;
+  h->s.rank = 0;
 
   // ---- graph grid: Z-order of quantised coordinates, cells = runs of cell_size vertices
   std::vector<uint32_t> order(V);
@@ -495,7 +498,8 @@ int ggrid_free(ggrid_t h) {
   if (h->copy_stream) cudaStreamSynchronize(h->copy_stream);
   for (void* p : h->allocs) cudaFree(p);
   for (DBuf* b : {&h->upd_stage, &h->tmp, &h->q_stage, &h->out_stage, &h->lists, &h->l2_scratch,
-                  &h->dump_stage, &h->gc_buf, &h->misc, &h->flush_spill, &h->staged[0].buf,
+                  &h->dump_stage, &h->gc_buf, &h->misc, &h->flush_spill, &h->bound_stage,
+                  &h->remote_stage, &h->merge_stage, &h->staged[0].buf,
                   &h->staged[1].buf})
     b->release();
   for (auto& sb : h->staged)
@@ -586,9 +590,30 @@ int ggrid_ingest_commit(ggrid_t h) {
 }
 
 static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
-                    uint32_t* out_dist) {
+                    uint32_t* out_dist, const uint32_t* bound = nullptr,
+                    uint64_t* out_remote = nullptr) {
   CK(cudaSetDevice(h->device));
   cudaStream_t st = h->stream;
+  // optional per-query bound (host or device) and remote-rank masks (sharded mode)
+  const uint32_t* d_bound = nullptr;
+  if (bound) {
+    d_bound = static_cast<const uint32_t*>(device_view(bound));
+    if (!d_bound) {
+      RC(h->bound_stage.ensure((size_t)n_q * 4));
+      CK(cudaMemcpyAsync(h->bound_stage.p, bound, (size_t)n_q * 4, cudaMemcpyHostToDevice, st));
+      d_bound = h->bound_stage.as<uint32_t>();
+    }
+  }
+  unsigned long long* d_remote = nullptr;
+  bool remote_copy = false;
+  if (out_remote) {
+    d_remote = static_cast<unsigned long long*>(device_view(out_remote));
+    if (!d_remote) {
+      RC(h->remote_stage.ensure((size_t)n_q * 8));
+      d_remote = h->remote_stage.as<unsigned long long>();
+      remote_copy = true;
+    }
+  }
   // every flushed cell writes at most its live objects (+ alignment padding)
   RC(h->ensure_arena(h->flush_need(), 0));
   // device and pinned (mapped) host buffers are used in place — pinned queries and answers
@@ -674,7 +699,8 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
       const uint32_t nn = n_in[lvl];
       const int kind = lvl == 0 ? GGRID_K_EXPAND : GGRID_K_EXPAND_BIG;
       h->launch(kind, [&] {
-        launch_expand(lvl, d_q, qlist, nn, k, g, s, epoch, retry, promote, d_oo, d_od, scratch, sw, h->sm_count, st);
+        launch_expand(lvl, d_q, qlist, nn, k, g, s, epoch, retry, promote, d_oo, d_od, d_bound, d_remote,
+                      scratch, sw, h->sm_count, st);
       });
     }
     RC(h->sync());
@@ -692,9 +718,10 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
     cur ^= 1;
     if (!any) break;
   }
-  if (!dev_o || !dev_d) {  // (device / pinned outputs were written in place; the loop drained)
+  if (!dev_o || !dev_d || remote_copy) {  // (device / pinned outputs were written in place)
     if (!dev_o) CK(cudaMemcpyAsync(out_obj, d_oo, outn * 4, cudaMemcpyDeviceToHost, st));
     if (!dev_d) CK(cudaMemcpyAsync(out_dist, d_od, outn * 4, cudaMemcpyDeviceToHost, st));
+    if (remote_copy) CK(cudaMemcpyAsync(out_remote, d_remote, (size_t)n_q * 8, cudaMemcpyDeviceToHost, st));
     RC(h->sync());
   }
   h->stats.n_queries += n_q;
@@ -708,6 +735,75 @@ int ggrid_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_
   if (n_q == 0) return GGRID_OK;
   if (!q || !out_obj || !out_dist) return GGRID_EINVAL;
   return knn_impl(h, q, n_q, k, out_obj, out_dist);
+}
+
+int ggrid_knn_ex(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, const uint32_t* bound,
+                 uint32_t* out_obj, uint32_t* out_dist, uint64_t* out_remote) {
+  if (!h || k == 0 || k > h->max_k) return GGRID_EINVAL;
+  if (n_q == 0) return GGRID_OK;
+  if (!q || !out_obj || !out_dist) return GGRID_EINVAL;
+  return knn_impl(h, q, n_q, k, out_obj, out_dist, bound, out_remote);
+}
+
+int ggrid_shard(ggrid_t h, uint32_t n_ranks, uint32_t rank) {
+  if (!h || n_ranks == 0 || n_ranks > 64 || rank >= n_ranks || n_ranks > h->n_cells) return GGRID_EINVAL;
+  if (h->seq_next != 0) return GGRID_EINVAL;  // ownership is fixed before the first update
+  h->s.n_ranks = n_ranks;
+  h->s.rank = rank;
+  return GGRID_OK;
+}
+
+int ggrid_query_owner(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t* out_rank) {
+  if (!h || (n_q && (!q || !out_rank))) return GGRID_EINVAL;
+  if (n_q == 0) return GGRID_OK;
+  CK(cudaSetDevice(h->device));
+  const uint2* d_q = static_cast<const uint2*>(device_view(q));
+  if (!d_q) {
+    RC(h->q_stage.ensure((size_t)n_q * 8));
+    CK(cudaMemcpyAsync(h->q_stage.p, q, (size_t)n_q * 8, cudaMemcpyHostToDevice, h->stream));
+    d_q = h->q_stage.as<uint2>();
+  }
+  uint32_t* d_o = static_cast<uint32_t*>(device_view(out_rank));
+  const bool copy = d_o == nullptr;
+  if (copy) {
+    RC(h->misc.ensure(std::max<size_t>(64, (size_t)n_q * 4)));
+    d_o = h->misc.as<uint32_t>();
+  }
+  h->launch(GGRID_K_OTHER, [&] { launch_query_owner(d_q, n_q, h->g, h->s, d_o, h->stream); });
+  if (copy) CK(cudaMemcpyAsync(out_rank, d_o, (size_t)n_q * 4, cudaMemcpyDeviceToHost, h->stream));
+  return h->sync();
+}
+
+int ggrid_merge_topk(ggrid_t h, uint32_t n_lists, uint32_t n_q, uint32_t k, const uint32_t* lists_obj,
+                     const uint32_t* lists_dist, uint32_t* out_obj, uint32_t* out_dist) {
+  if (!h || n_lists == 0 || n_lists > 32 || k == 0) return GGRID_EINVAL;
+  if (n_q == 0) return GGRID_OK;
+  if (!lists_obj || !lists_dist || !out_obj || !out_dist) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  cudaStream_t st = h->stream;
+  const size_t in_n = (size_t)n_lists * n_q * k, out_n = (size_t)n_q * k;
+  const uint32_t* d_lo = static_cast<const uint32_t*>(device_view(lists_obj));
+  const uint32_t* d_ld = static_cast<const uint32_t*>(device_view(lists_dist));
+  uint32_t* d_oo = static_cast<uint32_t*>(device_view(out_obj));
+  uint32_t* d_od = static_cast<uint32_t*>(device_view(out_dist));
+  const bool c_in = !d_lo || !d_ld, c_out = !d_oo || !d_od;
+  RC(h->merge_stage.ensure((c_in ? in_n * 8 : 0) + (c_out ? out_n * 8 : 0) + 16));
+  uint32_t* sp = h->merge_stage.as<uint32_t>();
+  if (c_in) {
+    CK(cudaMemcpyAsync(sp, lists_obj, in_n * 4, cudaMemcpyDefault, st));
+    CK(cudaMemcpyAsync(sp + in_n, lists_dist, in_n * 4, cudaMemcpyDefault, st));
+    d_lo = sp;
+    d_ld = sp + in_n;
+    sp += 2 * in_n;
+  }
+  uint32_t* w_o = c_out ? sp : d_oo;
+  uint32_t* w_d = c_out ? sp + out_n : d_od;
+  h->launch(GGRID_K_OTHER, [&] { launch_merge_topk(n_lists, n_q, k, d_lo, d_ld, w_o, w_d, st); });
+  if (c_out) {
+    CK(cudaMemcpyAsync(out_obj, w_o, out_n * 4, cudaMemcpyDefault, st));
+    CK(cudaMemcpyAsync(out_dist, w_d, out_n * 4, cudaMemcpyDefault, st));
+  }
+  return h->sync();
 }
 
 int ggrid_flush_all(ggrid_t h) {

@@ -26,6 +26,7 @@ constexpr int CU = CT * CPT;       // updates per CTA (tile)
 constexpr int CH = 4096;           // hash slots (>= 2*CU)
 constexpr int SPC = CH / CT;       // hash slots per thread in the scan
 static_assert(CU < 65536, "tile offsets and counts are packed in 16 bits");
+constexpr uint32_t REMOTE_CELL = 0xFFFFFFFEu;  // classify: pseudo-cell of other ranks' updates
 constexpr int CLASSIFY_SMEM = (3 * CH + CT / 32) * 4;
 
 __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
@@ -77,7 +78,11 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
       atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
       continue;
     }
-    const uint32_t c = cellof(g, e.x);
+    // updates of cells another rank owns (sharded mode) are grouped under one pseudo-cell:
+    // no record here, only the object-table update (in the scatter, after validation)
+    const uint32_t c0 = cellof(g, e.x);
+    const bool remote = s.n_ranks > 1 && owner_of(c0, g.n_cells, s.n_ranks) != s.rank;
+    const uint32_t c = remote ? REMOTE_CELL : c0;
     uint32_t h = (c * 2654435761u) >> 20;  // 12 bits
     volatile uint32_t* vc = h_cell;
     for (;;) {
@@ -122,7 +127,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
   }
   for (int i = tid; i < CH; i += CT) {
     const uint32_t c = h_cell[i];
-    if (c != NONE) {
+    if (c != NONE && c != REMOTE_CELL) {
       atomicMax(&s.bcount[c * BCOUNT_STRIDE + 1], h_tmax[i]);
       h_cell[i] = atomicAdd(&s.bcount[c * BCOUNT_STRIDE], h_cnt[i] & 0xFFFFu);
     }
@@ -133,7 +138,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
   for (int j = 0; j < CPT; ++j) {
     if (slot[j] < 0) continue;
     si[j] = (h_cnt[slot[j]] >> 16) + lr[j];
-    rk[j] = h_cell[slot[j]] + lr[j];
+    rk[j] = h_cell[slot[j]] == REMOTE_CELL ? NONE : h_cell[slot[j]] + lr[j];
   }
   __syncthreads();
   // the tile in cell order, staged in the (now free) hash table, then written coalesced
@@ -242,7 +247,7 @@ __global__ void __launch_bounds__(CT) k_ingest_scatter(const uint4* __restrict__
       const uint32_t k = (uint32_t)(j * CT + tid);
       if (k < nt) {
         m[q] = su[il[j]];
-        pos[q] = s.bbase[cellof(g, vr[j].x)] + vr[j].y;
+        pos[q] = vr[j].y == NONE ? NONE : s.bbase[cellof(g, vr[j].x)] + vr[j].y;
         cur[q] = __ldcg(s.ot_key + m[q].x);  // L2 value (the atomics' point of coherence)
       }
     }
@@ -253,11 +258,13 @@ __global__ void __launch_bounds__(CT) k_ingest_scatter(const uint4* __restrict__
       if (k >= nt) continue;
       const unsigned long long key =
           ((unsigned long long)m[q].w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + il[j]));
-      s.ar.obj[pos[q]] = m[q].x;
-      s.ar.key[pos[q]] = key;
-      s.ar.vsrc[pos[q]] = vr[j].x;
-      s.ar.off[pos[q]] = m[q].z;
-      s.ar.edge[pos[q]] = m[q].y;
+      if (pos[q] != NONE) {  // (NONE: a cell another rank owns)
+        s.ar.obj[pos[q]] = m[q].x;
+        s.ar.key[pos[q]] = key;
+        s.ar.vsrc[pos[q]] = vr[j].x;
+        s.ar.off[pos[q]] = m[q].z;
+        s.ar.edge[pos[q]] = m[q].y;
+      }
       // ot_key only grows: a key below the value already seen needs no atomic; a live object
       // takes a fire-and-forget RED.MAX; only an object seen without updates (0) needs the
       // old value back, to count it live exactly once
@@ -394,5 +401,53 @@ __global__ void k_copy_words(const uint32_t* __restrict__ src, uint32_t* __restr
 void launch_copy_words(const void* src, void* dst, size_t bytes, cudaStream_t st) {
   k_copy_words<<<1, 64, 0, st>>>(static_cast<const uint32_t*>(src), static_cast<uint32_t*>(dst),
                                  (int)(bytes / 4));
+}
+}  // namespace gg
+
+namespace gg {
+// owner rank of each query (cell of its arc's source vertex; sharded mode routing)
+__global__ void k_query_owner(const uint2* __restrict__ q, uint32_t nq, DevGraph g, DevState s,
+                              uint32_t* __restrict__ out) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nq) return;
+  const uint32_t e = q[i].x;
+  out[i] = e < g.A ? owner_of(cellof(g, g.einfo[e].x), g.n_cells, s.n_ranks) : 0u;
+}
+void launch_query_owner(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s,
+                        uint32_t* out_rank, cudaStream_t st) {
+  if (nq) k_query_owner<<<(nq + 255) / 256, 256, 0, st>>>(q, nq, g, s, out_rank);
+}
+
+// One warp per query: lane l < n_lists holds the head of list l; k rounds of a warp arg-min on
+// (dist, obj) (the final first-k of the candidate union, P@49436-49765 / P@51679).
+__global__ void k_merge_topk(uint32_t n_lists, uint32_t n_q, uint32_t k,
+                             const uint32_t* __restrict__ lobj, const uint32_t* __restrict__ ldist,
+                             uint32_t* __restrict__ out_obj, uint32_t* __restrict__ out_dist) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t qi = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (qi >= n_q) return;
+  const size_t row = (size_t)qi * k;
+  const size_t stride = (size_t)n_q * k;
+  uint32_t head = 0;
+  auto key_at = [&](uint32_t h) -> unsigned long long {
+    if (lane >= n_lists || h >= k) return EMPTY64;
+    const size_t p = lane * stride + row + h;
+    return ((unsigned long long)ldist[p] << 32) | lobj[p];
+  };
+  unsigned long long cur = key_at(head);
+  for (uint32_t r = 0; r < k; ++r) {
+    const uint32_t dmin = __reduce_min_sync(0xffffffffu, (uint32_t)(cur >> 32));
+    const uint32_t omin = __reduce_min_sync(0xffffffffu, (uint32_t)(cur >> 32) == dmin ? (uint32_t)cur : 0xFFFFFFFFu);
+    const unsigned long long best = ((unsigned long long)dmin << 32) | omin;
+    if (lane == 0) {
+      out_obj[row + r] = best == EMPTY64 ? GGRID_PAD : omin;
+      out_dist[row + r] = best == EMPTY64 ? GGRID_PAD : dmin;
+    }
+    if (best != EMPTY64 && cur == best) cur = key_at(++head);  // (lists are disjoint)
+  }
+}
+void launch_merge_topk(uint32_t n_lists, uint32_t n_q, uint32_t k, const uint32_t* lobj,
+                       const uint32_t* ldist, uint32_t* out_obj, uint32_t* out_dist, cudaStream_t st) {
+  if (n_q) k_merge_topk<<<(n_q + 7) / 8, 256, 0, st>>>(n_lists, n_q, k, lobj, ldist, out_obj, out_dist);
 }
 }  // namespace gg

@@ -96,7 +96,14 @@ struct DevState {
   uint32_t* bbase;         // [n_cells] per-batch arena base
   uint32_t* flush_list;    // [n_cells]
   DevStatus* st;
+  // cell ownership across ranks: rank r owns the contiguous Z-order range of
+  // cells c with floor(c * n_ranks / n_cells) == r; only owned cells keep logs and lists
+  uint32_t n_ranks, rank;
 };
+
+__host__ __device__ inline uint32_t owner_of(uint32_t c, uint32_t n_cells, uint32_t n_ranks) {
+  return (uint32_t)(((unsigned long long)c * n_ranks) / n_cells);
+}
 
 __host__ __device__ inline uint32_t cell_of(uint32_t v, uint32_t cs) { return v / cs; }
 
@@ -162,6 +169,12 @@ void launch_set_words(const WordSet& ws, cudaStream_t st);
 void launch_copy_words(const void* src, void* dst, size_t bytes, cudaStream_t st);
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
                             uint2* tmp, cudaStream_t st);
+// owner rank of each query's cell (cell of the query arc's source vertex)
+void launch_query_owner(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s,
+                        uint32_t* out_rank, cudaStream_t st);
+// k-way merge of n_lists ascending (dist, obj) lists per query, layout [n_lists][n_q][k]
+void launch_merge_topk(uint32_t n_lists, uint32_t n_q, uint32_t k, const uint32_t* lobj,
+                       const uint32_t* ldist, uint32_t* out_obj, uint32_t* out_dist, cudaStream_t st);
 size_t ingest_tmp_bytes(uint64_t n);  // classify -> scatter scratch (tmp + perm)
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
@@ -190,9 +203,13 @@ __device__ __forceinline__ uint2 vobj_valid(uint2 vo, uint2 comp) {
 // Expansion (Alg. 5/6 semantics) for the queries qlist[0..n) at variant `level`.
 // Outcomes: answered (rows written), retried at the same level (retry_list, a needed cell
 // had cached updates) or promoted to the next level (promote_list, capacity overflow).
+// bound (nullable): per-query inclusive distance limit (objects farther are not returned and
+// the search stops beyond it); remote (nullable): per-query bitmask of the ranks owning cells
+// the search expanded into (sharded mode)
 void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
                    const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
-                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist, void* scratch,
+                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist,
+                   const uint32_t* bound, unsigned long long* remote, void* scratch,
                    uint32_t scratch_warps, int sm_count, cudaStream_t st);
 int expand_levels();
 uint32_t expand_table_slots(int level);  // vertex-table capacity H of a level

@@ -151,6 +151,8 @@ struct QParams {
   uint32_t* promote_list;   // next level, next round
   uint32_t* out_obj;
   uint32_t* out_dist;
+  const uint32_t* bound;          // per-query inclusive distance limit, or null
+  unsigned long long* remote;     // per-query mask of other ranks' cells reached, or null
   Caps caps;
   unsigned char* scratch;   // global working memory (last level) or null (shared)
   uint32_t warps_per_cta;
@@ -209,6 +211,15 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   if (q.x >= g.A) return DONE;   // invalid query: reported by the seed kernel (EINVAL)
   const uint2 ei = g.einfo[q.x];  // (internal src, w)
   if (q.y >= ei.y) return DONE;
+  // sharded mode: objects only from this rank's cells; the owners of other cells the search
+  // expands into are collected (they are asked for their objects within the final radius)
+  const uint32_t lim = P.bound ? P.bound[qi] : INF;
+  const bool track = P.remote != nullptr && s.n_ranks > 1;
+  unsigned long long rmask = 0;
+  if (track) {
+    const uint32_t o = owner_of(cellof(g, ei.x), g.n_cells, s.n_ranks);
+    if (o != s.rank) rmask |= 1ull << o;  // same-arc objects ahead of q live at src(q.e)
+  }
   uint32_t seed_v, seed_d;
   if (q.y == 0) {
     seed_v = ei.x;
@@ -265,6 +276,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
 
     // ---- 2. termination: k candidates strictly closer than anything not yet final -------
     if (nf == 0) break;
+    if (blo > lim) break;  // every object not yet harvested is beyond the caller's bound
     if (nc >= k) {
       uint32_t cl = 0;
       for (uint32_t i = lane; i < nc; i += 32) cl += cand_dist(m, i) < blo;
@@ -389,6 +401,12 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
           return RETRY;
         }
         c_harv += __popc(__ballot_sync(FULL, harv));
+        if (track) {
+          const uint32_t o = harv ? owner_of(hcell, g.n_cells, s.n_ranks) : s.rank;
+          const unsigned long long b = o != s.rank ? 1ull << o : 0ull;
+          rmask |= ((unsigned long long)__reduce_or_sync(FULL, (uint32_t)(b >> 32)) << 32) |
+                   __reduce_or_sync(FULL, (uint32_t)b);
+        }
         const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
         const uint32_t most = __reduce_max_sync(FULL, vo.y);
         if (most) {
@@ -426,10 +444,11 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   warp_sort(m.cand, nc, cp.C, lane);
   for (uint32_t r = lane; r < k; r += 32) {
     const unsigned long long dk = r < nc ? m.cand[r] : EMPTY64;
-    const bool ok = dk != EMPTY64;
+    const bool ok = dk != EMPTY64 && (uint32_t)(dk >> 32) <= lim;
     P.out_obj[(size_t)qi * k + r] = ok ? (uint32_t)dk : GGRID_PAD;
     P.out_dist[(size_t)qi * k + r] = ok ? (uint32_t)(dk >> 32) : GGRID_PAD;
   }
+  if (lane == 0 && P.remote) P.remote[qi] = rmask;
   if (lane == 0) {
     atomicAdd(&s.st->ex_iters, (unsigned long long)c_iter);
     atomicAdd(&s.st->ex_vertices, (unsigned long long)c_vert);
@@ -506,7 +525,8 @@ size_t expand_warp_bytes(int level, uint32_t V) {
 
 void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
                    const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
-                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist, void* scratch,
+                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist,
+                   const uint32_t* bound, unsigned long long* remote, void* scratch,
                    uint32_t scratch_warps, int sm_count, cudaStream_t st) {
   if (n == 0) return;
   QParams P;
@@ -523,6 +543,8 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
   P.promote_list = promote_list;
   P.out_obj = out_obj;
   P.out_dist = out_dist;
+  P.bound = bound;
+  P.remote = remote;
   P.caps = caps_for(level, g.V);
   P.warps_per_cta = 1;
   const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
