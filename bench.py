@@ -194,8 +194,11 @@ def run_ours(args, cfg_name):
     g = synth.config_graph(cfg_name)
     walk = synth.RandomWalk(g, cfg["n_objects"])
     stream = torch.cuda.Stream()
+    shard = world > 1 and args.parallel == "shard"
     grid = gg.GGrid(g, args.cell_size or cfg["cell_size"], max_objects=cfg["n_objects"], profile=True,
                     log_capacity=args.log_capacity, delta=args.delta, stream=stream.cuda_stream)
+    if shard:  # cell-ownership sharding: logs of own cells only
+        grid.shard(world, rank)
     out_o = torch.empty((Q, k), dtype=torch.int32, device="cuda")
     out_d = torch.empty((Q, k), dtype=torch.int32, device="cuda")
     l2 = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
@@ -216,6 +219,7 @@ def run_ours(args, cfg_name):
     from paper_conf_icde_li0qhdy18_b200 import dist as gdist
 
     n_upd_step = cfg["n_objects"] * cfg["updates_per_object"]
+    remote_requests = 0
     for s in range(args.warmup + args.steps):
         q = synth.queries(g, Q, seed=synth.SEED_QUERIES + 1000 * rank + s)
         u = walk.ticks(cfg["updates_per_object"])  # every rank keeps the walk in step (untimed)
@@ -238,7 +242,12 @@ def run_ours(args, cfg_name):
             with torch.cuda.stream(stream):
                 gdist.broadcast_updates(du, src=0)
         grid.ingest(du)
-        grid.knn(dq, k, out_o, out_d)
+        if shard:  # owner search + bounded requests/replies + merge, all ordered on `stream`
+            with torch.cuda.stream(stream):
+                out_o, out_d, n_req = gdist.sharded_knn(grid, dq, k, world, rank)
+                remote_requests += n_req if s >= args.warmup else 0
+        else:
+            grid.knn(dq, k, out_o, out_d)
         e1.record(stream)
         e1.synchronize()
         if s >= args.warmup:
@@ -298,6 +307,19 @@ def run_ours(args, cfg_name):
     grid.close()
     grid = gg.GGrid(g, args.cell_size or cfg["cell_size"], max_objects=cfg["n_objects"],
                     log_capacity=args.log_capacity, delta=args.delta)
+    if shard:
+        grid.shard(world, rank)
+    dq_e = torch.empty((Q, 2), dtype=torch.int32, device="cuda")
+
+    def e2e_knn(hq):
+        if not shard:
+            grid.knn(hq, k, h_o, h_d)  # pinned queries/answers used in place (zero-copy)
+            return
+        dq_e.copy_(hq, non_blocking=True)
+        o, d_, _ = gdist.sharded_knn(grid, dq_e, k, world, rank)
+        h_o.copy_(o, non_blocking=True)
+        h_d.copy_(d_, non_blocking=True)
+        torch.cuda.current_stream().synchronize()
     h_o = torch.empty((Q, k), dtype=torch.int32).pin_memory()
     h_d = torch.empty((Q, k), dtype=torch.int32).pin_memory()
     n_e2e = max(1, args.e2e_steps)
@@ -310,7 +332,7 @@ def run_ours(args, cfg_name):
     for s in range(w_e2e):  # warm-up steps
         grid.ingest_stage(hus[s])
         grid.ingest_commit()
-        grid.knn(hqs[s], k, h_o, h_d)
+        e2e_knn(hqs[s])
     hus, hqs = hus[w_e2e:], hqs[w_e2e:]
     hus.insert(0, None)
     hqs.insert(0, None)
@@ -326,7 +348,7 @@ def run_ours(args, cfg_name):
         grid.ingest_commit()
         if s + 1 <= n_e2e:
             grid.ingest_stage(hus[s + 1])  # overlaps the queries below
-        grid.knn(hqs[s], k, h_o, h_d)
+        e2e_knn(hqs[s])
     e2e_total = time.perf_counter() - t0
     if trace is not None:
         trace.__exit__(None, None, None)
@@ -357,10 +379,12 @@ def run_ours(args, cfg_name):
                            "n_vertices": int(g["n_vertices"]), "n_arcs": int(len(g["src"])),
                            "objects": cfg["n_objects"], "updates_per_step": n_upd, "queries_per_step_per_gpu": Q,
                            "k": k, "cell_size": cs, "l2": "flushed between timed steps (256 MB write)",
-                           "parallelism": f"replicas x{world}, queries sharded"},
+                           "parallelism": (f"cell-ownership shards x{world} (one request/reply exchange per batch)"
+                                           if shard else f"replicas x{world}, queries sharded")},
                 "updates_per_s": updates_per_s, "per_kernel": per_kernel, "roofline": roofline,
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(st1["launches"]), "clocks": clk,
                 "knn_rounds_per_step": (st1["knn_rounds"] - st0["knn_rounds"]) / K,
+                "remote_requests_per_step_rank0": remote_requests / K if shard else None,
                 "expand_work_per_query": {n: v / (Q * K) for n, v in dx.items()}, "delta": st1["delta"]}
         print(json.dumps(line), flush=True)
     grid.close()
@@ -382,6 +406,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=12)
     ap.add_argument("--ref-sample", type=int, default=400)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--parallel", default="shard", choices=["shard", "replicas"],
+                    help="N>1 layout: cell-ownership shards (SURVEY 8(e)) or full replicas")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference" or os.environ.get("BENCH_ALLOW_SHORT"), "W >= 3"
     if args.impl == "reference":

@@ -1,8 +1,11 @@
 """Multi-GPU plumbing over torch.distributed.
 
-One process per GPU.  Every rank holds a full replica of the index; the update stream is
-broadcast from the rank that receives it (NCCL over NVLink on GPUs, gloo in CPU tests) and
-query batches are sharded into contiguous ranges, so the query phase needs no collective.
+One process per GPU.  The update stream is broadcast from the rank that receives it (NCCL over
+NVLink on GPUs, gloo in CPU tests).  Two layouts:
+  * cell-ownership sharding (default): each rank's handle keeps the logs of its
+    own cells only; queries are answered with one request/reply exchange (sharded_knn below);
+  * replicas: every rank holds the whole index and answers its own contiguous share of the
+    queries with no collective in the query phase.
 Only host-side orchestration lives here; all per-query and per-update work runs in
 libggrid.so on each rank's GPU.
 """
@@ -116,20 +119,28 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
     dev = queries.device
     n = int(queries.shape[0])
     i32 = torch.int32
+
+    def ready():
+        # the library runs on its own stream: inputs made by torch ops (or collectives, which
+        # torch orders on its current stream) must be complete before a library call
+        if dev.type == "cuda":
+            torch.cuda.current_stream(dev).synchronize()
+
     idx = torch.arange(n, dtype=i32, device=dev)
     if routed:
         mine, src_counts = torch.cat([queries, idx[:, None]], 1), None
     else:
         owner = torch.empty(n, dtype=i32, device=dev)
+        ready()
         grid.query_owner(queries, owner)
         order, counts = _group_by(owner, world)
         mine, src_counts = _a2a(torch.cat([queries, idx[:, None]], 1)[order], counts, world)
-        back_order = order
     m = int(mine.shape[0])
     q_m = mine[:, :2].contiguous()
     own_o = torch.empty((m, k), dtype=i32, device=dev)
     own_d = torch.empty((m, k), dtype=i32, device=dev)
     mask = torch.empty(m, dtype=torch.int64, device=dev)
+    ready()
     grid.knn_ex(q_m, k, None, own_o, own_d, mask)
     # requests: (edge, offset, bound, local row) to every rank in the mask
     bits = ((mask[:, None] >> torch.arange(world, device=dev, dtype=torch.int64)[None, :]) & 1).bool()
@@ -139,9 +150,9 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
     got, got_counts = _a2a(req[order_r], counts_r, world)
     rep_o = torch.empty((int(got.shape[0]), k), dtype=i32, device=dev)
     rep_d = torch.empty_like(rep_o)
-    grid.knn_ex(got[:, :2].contiguous(), k, got[:, 2].contiguous(), rep_o, rep_d)
-    rep_src = torch.repeat_interleave(torch.arange(world, device=dev),
-                                      torch.tensor(got_counts, device=dev))
+    got_q, got_b = got[:, :2].contiguous(), got[:, 2].contiguous()
+    ready()
+    grid.knn_ex(got_q, k, got_b, rep_o, rep_d)
     replies, _ = _a2a(torch.cat([rep_o, rep_d, got[:, 3:4], torch.full_like(got[:, 3:4], rank)], 1),
                       got_counts, world)
     # dense [world][m][k] lists: own list at slot `rank`, the reply of rank t at slot t
@@ -156,8 +167,8 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
         ld[r_t, r_q] = replies[:, k:2 * k]
     fo = torch.empty((m, k), dtype=i32, device=dev)
     fd = torch.empty((m, k), dtype=i32, device=dev)
+    ready()
     grid.merge_topk(lo, ld, fo, fd)
-    del rep_src
     if routed:
         return fo, fd, int(req.shape[0])
     # answers back to the ranks the queries came from, into their original rows
@@ -167,5 +178,4 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
     rows = ans[:, 2 * k].long()
     out_o[rows] = ans[:, :k]
     out_d[rows] = ans[:, k:2 * k]
-    del back_order
     return out_o, out_d, int(req.shape[0])
