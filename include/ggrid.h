@@ -208,6 +208,36 @@ int ggrid_knn_ex(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, cons
 int ggrid_merge_topk(ggrid_t h, uint32_t n_lists, uint32_t n_q, uint32_t k, const uint32_t* lists_obj,
                      const uint32_t* lists_dist, uint32_t* out_obj, uint32_t* out_dist);
 
+/* ---- prior-art comparison path (not used by ggrid_knn) -------------------
+ *
+ * The paper's message cleaning (Alg. 2 steps 2-4 with Alg. 3 GPU_X_Shuffle and GPU_Collect,
+ * P@19259-30196) run on this GPU over the message lists of every cell (cached extents and
+ * cleaned lists), read-only: buckets of bucket_size messages, one thread per bucket, bundles of
+ * 2^eta threads (eta 4 or 5) resolving same-object messages by cache-and-shuffle (reading R23),
+ * then the intermediate table T[object][bundle] written with mu(eta) rounds of "write if newer"
+ * (write_mode 0, as printed) or until no lane is newer (write_mode 1), then per object the
+ * newest message over the bundles.  out_edge / out_off (nullable; max_objects entries, host or
+ * device) receive each object's collected location (GGRID_PAD if none).  T needs
+ * max_objects x ceil(buckets / 2^eta) x 16 bytes; ENOMEM beyond 48 GiB. */
+typedef struct ggrid_prior_art_result {
+  double ms_prepare;        /* bucket table + T reset (CUDA events)                       */
+  double ms_shuffle;        /* Alg. 3 over every bucket                                   */
+  double ms_collect;        /* GPU_Collect                                                */
+  uint64_t n_buckets;
+  uint64_t n_bundles;
+  uint64_t table_bytes;     /* T                                                          */
+  uint64_t objects_found;   /* objects with a message in the lists                        */
+  uint64_t objects_wrong;   /* of those, collected message != the object's newest (key)  */
+} ggrid_prior_art_result;
+int ggrid_prior_art_clean(ggrid_t h, uint32_t eta, uint32_t bucket_size, uint32_t write_mode,
+                          uint32_t* out_edge, uint32_t* out_off, ggrid_prior_art_result* res);
+
+/* Test hook: Step 1 (cache-and-shuffle, reading R23) of Alg. 3 on one bundle of 2^eta lanes
+ * holding messages (obj[i], key[i]) (host arrays); out_obj / out_key receive the message each
+ * lane holds afterwards. */
+int ggrid_prior_art_bundle(const uint32_t* obj, const uint64_t* key, uint32_t eta, uint32_t* out_obj,
+                           uint64_t* out_key);
+
 /* Release every resource of h (NULL is accepted). */
 int ggrid_free(ggrid_t h);
 

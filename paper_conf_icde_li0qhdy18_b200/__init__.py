@@ -25,7 +25,8 @@ KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "fl
                 "expand_big", "other"]
 EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_flush_all",
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
-           "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk"]
+           "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk",
+           "ggrid_prior_art_clean", "ggrid_prior_art_bundle"]
 
 
 class GGridError(RuntimeError):
@@ -60,6 +61,11 @@ class ggrid_stats_t(ctypes.Structure):
                                        "t_delta", "t_now"]] + [("records_expired", ctypes.c_uint64)]
 
 
+class ggrid_prior_art_result(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_double) for n in ["ms_prepare", "ms_shuffle", "ms_collect"]] + [
+        (n, ctypes.c_uint64) for n in ["n_buckets", "n_bundles", "table_bytes", "objects_found", "objects_wrong"]]
+
+
 _lib = None
 
 
@@ -90,6 +96,8 @@ def lib():
             "ggrid_query_owner": ([P, P, u32, P], i32),
             "ggrid_knn_ex": ([P, P, u32, u32, P, P, P, P], i32),
             "ggrid_merge_topk": ([P, u32, u32, u32, P, P, P, P], i32),
+            "ggrid_prior_art_clean": ([P, u32, u32, u32, P, P, ctypes.POINTER(ggrid_prior_art_result)], i32),
+            "ggrid_prior_art_bundle": ([P, P, u32, P, P], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -223,6 +231,30 @@ def ggrid_merge_topk(h, lists_obj, lists_dist, out_obj=None, out_dist=None):
     return out_obj, out_dist
 
 
+def ggrid_prior_art_clean(h, eta: int = 5, bucket_size: int = 128, write_mode: int = 0,
+                          max_objects: int | None = None):
+    """The paper's message cleaning (Alg. 2-3 + GPU_Collect) as a read-only comparison pass.
+    Returns (result dict, edge, off) — edge/off per object (PAD: none) if max_objects given."""
+    r = ggrid_prior_art_result()
+    e = o = None
+    if max_objects:
+        e = np.empty(max_objects, np.uint32)
+        o = np.empty(max_objects, np.uint32)
+    _check(lib().ggrid_prior_art_clean(h, int(eta), int(bucket_size), int(write_mode), _ptr(e), _ptr(o),
+                                       ctypes.byref(r)), "ggrid_prior_art_clean")
+    return {f: getattr(r, f) for f, _ in ggrid_prior_art_result._fields_}, e, o
+
+
+def ggrid_prior_art_bundle(obj, key, eta: int):
+    """Alg. 3 Step 1 (cache-and-shuffle) on one bundle; returns (obj, key) per lane after it."""
+    ob = np.ascontiguousarray(obj, np.uint32)
+    ky = np.ascontiguousarray(key, np.uint64)
+    oo = np.empty_like(ob)
+    ok = np.empty_like(ky)
+    _check(lib().ggrid_prior_art_bundle(_ptr(ob), _ptr(ky), int(eta), _ptr(oo), _ptr(ok)), "ggrid_prior_art_bundle")
+    return oo, ok
+
+
 def ggrid_free(h):
     if h:
         lib().ggrid_free(h)
@@ -309,6 +341,10 @@ class GGrid:
 
     def merge_topk(self, lists_obj, lists_dist, out_obj=None, out_dist=None):
         return ggrid_merge_topk(self.h, lists_obj, lists_dist, out_obj, out_dist)
+
+    def prior_art_clean(self, eta: int = 5, bucket_size: int = 128, write_mode: int = 0, locations: bool = False):
+        return ggrid_prior_art_clean(self.h, eta, bucket_size, write_mode,
+                                     self.stats()["max_objects"] if locations else None)
 
     def flush_all(self):
         ggrid_flush_all(self.h)

@@ -806,6 +806,102 @@ int ggrid_merge_topk(ggrid_t h, uint32_t n_lists, uint32_t n_q, uint32_t k, cons
   return h->sync();
 }
 
+int ggrid_prior_art_clean(ggrid_t h, uint32_t eta, uint32_t bucket_size, uint32_t write_mode,
+                          uint32_t* out_edge, uint32_t* out_off, ggrid_prior_art_result* res) {
+  if (!h || (eta != 4 && eta != 5) || bucket_size == 0 || bucket_size > 4096 || write_mode > 1)
+    return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  cudaStream_t st = h->stream;
+  RC(h->sync());
+  const uint32_t nc = h->n_cells;
+  DBuf cnt, off, scan_tmp, buckets, table, oe, counts;
+  auto release = [&] {
+    for (DBuf* b : {&cnt, &off, &scan_tmp, &buckets, &table, &oe, &counts}) b->release();
+  };
+  cudaEvent_t ev[4];
+  for (auto& e : ev) CK(cudaEventCreate(&e));
+  auto done = [&](int rc) {
+    release();
+    for (auto& e : ev) cudaEventDestroy(e);
+    return rc;
+  };
+  if (cnt.ensure((size_t)(nc + 1) * 4) || off.ensure((size_t)(nc + 1) * 4) || counts.ensure(16))
+    return done(GGRID_ENOMEM);
+  const size_t sb = prior_art_scan_bytes(nc + 1);
+  if (scan_tmp.ensure(sb)) return done(GGRID_ENOMEM);
+  CK(cudaEventRecord(ev[0], st));
+  launch_pa_count(h->g, h->s, bucket_size, cnt.as<uint32_t>(), st);
+  if (launch_pa_scan(scan_tmp.p, sb, cnt.as<uint32_t>(), off.as<uint32_t>(), nc + 1, st)) return done(GGRID_ECUDA);
+  uint32_t n_buckets = 0;
+  CK(cudaMemcpyAsync(&n_buckets, off.as<uint32_t>() + nc, 4, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  const uint32_t n_bundles = (n_buckets + (1u << eta) - 1) >> eta;
+  const uint64_t tbytes = (uint64_t)h->max_objects * std::max(1u, n_bundles) * 16;
+  if (tbytes > (48ull << 30)) return done(GGRID_ENOMEM);
+  if (buckets.ensure((size_t)std::max(1u, n_buckets) * prior_art_bucket_bytes()) || table.ensure(tbytes))
+    return done(GGRID_ENOMEM);
+  launch_pa_fill(h->g, h->s, bucket_size, off.as<uint32_t>(), buckets.p, st);
+  CK(cudaMemsetAsync(table.p, 0xFF, tbytes, st));
+  CK(cudaMemsetAsync(counts.p, 0, 16, st));
+  CK(cudaEventRecord(ev[1], st));
+  launch_pa_shuffle(h->s, buckets.p, n_buckets, bucket_size, (int)eta, (int)write_mode, n_bundles, table.p, st);
+  CK(cudaEventRecord(ev[2], st));
+  uint32_t* d_e = out_edge ? static_cast<uint32_t*>(device_view(out_edge)) : nullptr;
+  uint32_t* d_o = out_off ? static_cast<uint32_t*>(device_view(out_off)) : nullptr;
+  const bool ce = out_edge && !d_e, co = out_off && !d_o;
+  if ((ce || co) && oe.ensure((size_t)h->max_objects * 8)) return done(GGRID_ENOMEM);
+  if (ce) d_e = oe.as<uint32_t>();
+  if (co) d_o = oe.as<uint32_t>() + h->max_objects;
+  launch_pa_collect(h->s, h->max_objects, std::max(1u, n_bundles), table.p, d_e, d_o,
+                    counts.as<unsigned long long>(), st);
+  CK(cudaEventRecord(ev[3], st));
+  unsigned long long hc[2] = {0, 0};
+  CK(cudaMemcpyAsync(hc, counts.p, 16, cudaMemcpyDeviceToHost, st));
+  if (ce) CK(cudaMemcpyAsync(out_edge, d_e, (size_t)h->max_objects * 4, cudaMemcpyDeviceToHost, st));
+  if (co) CK(cudaMemcpyAsync(out_off, d_o, (size_t)h->max_objects * 4, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  CK(cudaGetLastError());
+  h->stats.launches += 5;
+  if (res) {
+    float a = 0, b = 0, c = 0;
+    cudaEventElapsedTime(&a, ev[0], ev[1]);
+    cudaEventElapsedTime(&b, ev[1], ev[2]);
+    cudaEventElapsedTime(&c, ev[2], ev[3]);
+    res->ms_prepare = a;
+    res->ms_shuffle = b;
+    res->ms_collect = c;
+    res->n_buckets = n_buckets;
+    res->n_bundles = n_bundles;
+    res->table_bytes = tbytes;
+    res->objects_found = hc[0];
+    res->objects_wrong = hc[1];
+  }
+  return done(GGRID_OK);
+}
+
+int ggrid_prior_art_bundle(const uint32_t* obj, const uint64_t* key, uint32_t eta, uint32_t* out_obj,
+                           uint64_t* out_key) {
+  if (!obj || !key || !out_obj || !out_key || (eta != 4 && eta != 5)) return GGRID_EINVAL;
+  const uint32_t n = 1u << eta;
+  DBuf b;
+  if (b.ensure((size_t)n * 24)) return GGRID_ENOMEM;
+  uint32_t* d_o = b.as<uint32_t>();
+  unsigned long long* d_k = reinterpret_cast<unsigned long long*>(d_o + 2 * n);
+  uint32_t* d_oo = d_o + n;
+  unsigned long long* d_ok = d_k + n;
+  int rc = GGRID_OK;
+  if (cudaMemcpy(d_o, obj, n * 4, cudaMemcpyHostToDevice) || cudaMemcpy(d_k, key, n * 8, cudaMemcpyHostToDevice))
+    rc = GGRID_ECUDA;
+  if (!rc) {
+    launch_pa_bundle(d_o, d_k, (int)eta, d_oo, d_ok, 0);
+    if (cudaMemcpy(out_obj, d_oo, n * 4, cudaMemcpyDeviceToHost) ||
+        cudaMemcpy(out_key, d_ok, n * 8, cudaMemcpyDeviceToHost))
+      rc = GGRID_ECUDA;
+  }
+  b.release();
+  return rc;
+}
+
 int ggrid_flush_all(ggrid_t h) {
   if (!h) return GGRID_EINVAL;
   CK(cudaSetDevice(h->device));

@@ -211,6 +211,20 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
                    uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist,
                    const uint32_t* bound, unsigned long long* remote, void* scratch,
                    uint32_t scratch_warps, int sm_count, cudaStream_t st);
+// prior-art comparison path (csrc/prior_art.cu)
+int prior_art_mu(int eta);
+size_t prior_art_scan_bytes(uint32_t n);
+size_t prior_art_bucket_bytes();
+void launch_pa_count(const DevGraph& g, const DevState& s, uint32_t bsize, uint32_t* cnt, cudaStream_t st);
+int launch_pa_scan(void* tmp, size_t tmp_bytes, const uint32_t* cnt, uint32_t* off, uint32_t n, cudaStream_t st);
+void launch_pa_fill(const DevGraph& g, const DevState& s, uint32_t bsize, const uint32_t* off, void* out,
+                    cudaStream_t st);
+void launch_pa_shuffle(const DevState& s, const void* bk, uint32_t n_buckets, uint32_t bsize, int eta,
+                       int write_mode, uint32_t n_bundles, void* T, cudaStream_t st);
+void launch_pa_collect(const DevState& s, uint32_t max_objects, uint32_t n_bundles, const void* T,
+                       uint32_t* out_edge, uint32_t* out_off, unsigned long long* counts, cudaStream_t st);
+void launch_pa_bundle(const uint32_t* obj, const unsigned long long* key, int eta, uint32_t* out_obj,
+                      unsigned long long* out_key, cudaStream_t st);
 int expand_levels();
 uint32_t expand_table_slots(int level);  // vertex-table capacity H of a level
 uint32_t expand_max_k(int level);
