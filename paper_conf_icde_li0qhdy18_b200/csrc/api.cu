@@ -104,6 +104,7 @@ struct ggrid_s {
   int seed_neighbors = 1;
   int profile = 0;
   uint32_t t_delta = 0;  // message expiry window (0 = never)
+  uint32_t max_cell_degree = 0;  // most neighbour cells of any cell
   std::vector<uint32_t> user_cell;
   DevGraph g{};
   DevState s{};
@@ -197,7 +198,8 @@ struct ggrid_s {
     return set_words(ws);
   }
 
-  int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin, int full_vobj = 0) {
+  int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin, int full_vobj = 0,
+                     uint32_t max_cells = 0) {
     const uint32_t opc = (uint32_t)((h_status->n_live + n_cells - 1) / std::max(1u, n_cells));
     uint32_t spill_cap = 0;
     const size_t sb = flush_spill_bytes(g.cs, opc, sm_count, &spill_cap);
@@ -207,7 +209,8 @@ struct ggrid_s {
     const uint32_t t_now = h_status->t_max;
     const uint32_t t_cut = (t_delta && t_now > t_delta) ? t_now - t_delta : 0;
     launch(GGRID_K_FLUSH, [&] {
-      launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, spill, spill_cap, t_cut, stream);
+      launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, spill, spill_cap, t_cut, max_cells,
+                   stream);
     });
     return GGRID_OK;
   }
@@ -427,7 +430,10 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
     cptr[(cpairs[i] >> 32) + 1]++;
     cadj[i] = (uint32_t)cpairs[i];
   }
-  for (uint32_t c = 0; c < h->n_cells; ++c) cptr[c + 1] += cptr[c];
+  for (uint32_t c = 0; c < h->n_cells; ++c) {
+    h->max_cell_degree = std::max(h->max_cell_degree, cptr[c + 1]);
+    cptr[c + 1] += cptr[c];
+  }
 
   // ---- device graph
   uint32_t *d_rowptr, *d_edst, *d_cptr, *d_cadj;
@@ -675,7 +681,10 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   uint32_t flush_begin = 0;
   for (int round = 0;; ++round) {
     if (round > 100000) return GGRID_ECUDA;
-    RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin));
+    // round 0 cleans what the seed requested: c_q and its neighbour cells per query
+    const uint64_t seeded = (uint64_t)n_q * (h->seed_neighbors ? h->max_cell_degree + 1 : 2);
+    RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin, 0,
+                         round == 0 ? (uint32_t)std::min<uint64_t>(seeded, 1u << 30) : 0));
     if (round > 0) {  // round 0 was reset with the rest at the start
       WordSet ws;
       ws.zero_range(h->d_status->n_next, EXPAND_LEVELS);

@@ -459,9 +459,11 @@ int blocks_per_sm_t();
 template <int HCAP, int WCAP>
 void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned long long* out_top,
               uint32_t begin, int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap,
-              uint32_t t_cut, cudaStream_t st) {
+              uint32_t t_cut, uint32_t max_ctas, cudaStream_t st) {
   const int blocks_per_sm = blocks_per_sm_t<HCAP, WCAP>();
-  k_flush<HCAP, WCAP><<<sm_count * blocks_per_sm, FT, sizeof(FlushSmem<HCAP, WCAP>), st>>>(
+  uint32_t grid = (uint32_t)(sm_count * blocks_per_sm);
+  if (max_ctas && max_ctas < grid) grid = max_ctas;  // few cells to clean: fewer idle CTAs
+  k_flush<HCAP, WCAP><<<grid, FT, sizeof(FlushSmem<HCAP, WCAP>), st>>>(
       g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
 }
 template <int HCAP, int WCAP>
@@ -518,14 +520,14 @@ size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, u
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
                   int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap, uint32_t t_cut,
-                  cudaStream_t st) {
+                  uint32_t max_ctas, cudaStream_t st) {
   switch (flush_variant(g.cs, objects_per_cell)) {
-    case 0: launch_t<1024, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
-    case 1: launch_t<4096, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
-    case 2: launch_t<1024, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
-    case 3: launch_t<4096, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
-    case 4: launch_t<1024, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
-    default: launch_t<4096, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, st); break;
+    case 0: launch_t<1024, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
+    case 1: launch_t<4096, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
+    case 2: launch_t<1024, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
+    case 3: launch_t<4096, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
+    case 4: launch_t<1024, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
+    default: launch_t<4096, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
   }
 }
 

@@ -42,7 +42,7 @@ constexpr uint32_t SPECIAL = 0xFFFFFFFFu;  // candidate slot of a same-arc objec
 constexpr uint32_t WMAX = 0xFFFFFFFFu;     // inline-adjacency overflow marker
 
 struct Caps {
-  uint32_t H, F, C;  // table slots (pow2), frontier, candidates
+  uint32_t H, F, C;  // table slots, frontier, candidates
 };
 
 // byte layout of one warp's working memory
@@ -58,7 +58,7 @@ struct WarpMem {
 };
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 12ull * c.C + 4ull * (2ull * c.F + 2ull * (c.H / 32) + 32);
+  return 8ull * c.H + 12ull * c.C + 4ull * (2ull * c.F + 2ull * ((c.H + 31) / 32) + 32);
 }
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
@@ -69,23 +69,21 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   m.cobj = p; p += c.C;
   m.front0 = p; p += c.F;
   m.front1 = p; p += c.F;
-  m.fin = p; p += c.H / 32;
-  m.listed = p; p += c.H / 32;
+  m.fin = p; p += (c.H + 31) / 32;
+  m.listed = p; p += (c.H + 31) / 32;
   m.act = p;
   return m;
 }
 
-// Fibonacci hashing (high bits): ball vertex ids are Z-order clustered, so low-bit or
-// identity hashing makes long probe runs
-__device__ __forceinline__ uint32_t vhash(uint32_t v, uint32_t hmask) {
-  return (v * 2654435761u) >> (32 - __popc(hmask));
-}
+// Fibonacci hashing (high bits, scaled to any table size H): ball vertex ids are Z-order
+// clustered, so low-bit or identity hashing makes long probe runs
+__device__ __forceinline__ uint32_t vhash(uint32_t v, uint32_t H) { return __umulhi(v * 2654435761u, H); }
 
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
-__device__ __forceinline__ int tab_relax(unsigned long long* dtab, uint32_t hmask, uint32_t v,
+__device__ __forceinline__ int tab_relax(unsigned long long* dtab, uint32_t H, uint32_t v,
                                          uint32_t d, bool& improved) {
   const unsigned long long nv = ((unsigned long long)v << 32) | d;
-  uint32_t sl = vhash(v, hmask) & hmask;
+  uint32_t sl = vhash(v, H);
   volatile unsigned long long* vt = dtab;
 #pragma unroll 1
   for (int p = 0; p < MAXP; ++p) {
@@ -107,7 +105,7 @@ __device__ __forceinline__ int tab_relax(unsigned long long* dtab, uint32_t hmas
       }
       if ((uint32_t)(old >> 32) == v) continue;  // same vertex inserted meanwhile: re-read
     }
-    sl = (sl + 1) & hmask;
+    sl = sl + 1 == H ? 0 : sl + 1;
   }
   improved = false;
   return -1;
@@ -196,12 +194,12 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   const DevGraph& g = P.g;
   const DevState& s = P.s;
   const Caps& cp = P.caps;
-  const uint32_t hmask = cp.H - 1;
+  const uint32_t H = cp.H;
   const uint32_t k = P.k;
   const unsigned lt = lanemask_lt();
 
   for (uint32_t i = lane; i < cp.H; i += 32) m.dtab[i] = EMPTY64;
-  for (uint32_t i = lane; i < cp.H / 32; i += 32) {
+  for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) {
     m.fin[i] = 0;
     m.listed[i] = 0;
   }
@@ -233,7 +231,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   uint32_t nf = 1, nc = 0;
   if (lane == 0) {
     bool imp;
-    const int sl = tab_relax(m.dtab, hmask, seed_v, seed_d, imp);
+    const int sl = tab_relax(m.dtab, H, seed_v, seed_d, imp);
     front[0] = (uint32_t)sl;
     m.fin[sl >> 5] |= 1u << (sl & 31);
   }
@@ -338,7 +336,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
           const unsigned long long nd = (unsigned long long)du + arc.y;
           if (nd < INF) {
             bool imp;
-            const int rr = tab_relax(m.dtab, hmask, arc.x, (uint32_t)nd, imp);
+            const int rr = tab_relax(m.dtab, H, arc.x, (uint32_t)nd, imp);
             if (rr < 0) {
               ovf = true;
             } else if (imp) {
@@ -372,7 +370,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
               const unsigned long long nd = (unsigned long long)du + av.y;
               if (nd < INF) {
                 bool imp;
-                const int rr = tab_relax(m.dtab, hmask, av.x, (uint32_t)nd, imp);
+                const int rr = tab_relax(m.dtab, H, av.x, (uint32_t)nd, imp);
                 if (rr < 0) {
                   ovf = true;
                 } else if (imp) {
@@ -487,6 +485,332 @@ __global__ void k_expand(QParams P) {
   }
 }
 
+// ---------------------------------------------------------------------------------------------
+// CTA-per-query variant: the same expansion with W warps cooperating on one query (block-wide
+// shared-memory table, atomically appended frontier and candidates, barriers between the
+// phases of a round).  Used where one warp is too narrow: balls of thousands of vertices (the
+// larger levels, whose per-query tables would otherwise leave one or a few warps per SM) and
+// small batches, where the single query's latency is the metric ("G-Grid (L)", P@61891).
+struct CtaShared {
+  uint32_t nf, nn, na, nc;
+  uint32_t flags;  // 1: retry (dirty cell met), 2: overflow
+  uint32_t red[32];
+  unsigned long long redl[32];
+};
+constexpr uint32_t FL_RETRY = 1, FL_OVF = 2;
+
+template <int W>
+__device__ __forceinline__ uint32_t block_min(uint32_t v, CtaShared& sh) {
+  v = __reduce_min_sync(0xffffffffu, v);
+  __syncthreads();
+  if ((threadIdx.x & 31) == 0) sh.red[threadIdx.x >> 5] = v;
+  __syncthreads();
+  uint32_t r = sh.red[0];
+#pragma unroll
+  for (int w = 1; w < W; ++w) r = min(r, sh.red[w]);
+  return r;
+}
+template <int W>
+__device__ __forceinline__ uint32_t block_sum(uint32_t v, CtaShared& sh) {
+  v = __reduce_add_sync(0xffffffffu, v);
+  __syncthreads();
+  if ((threadIdx.x & 31) == 0) sh.red[threadIdx.x >> 5] = v;
+  __syncthreads();
+  uint32_t r = 0;
+#pragma unroll
+  for (int w = 0; w < W; ++w) r += sh.red[w];
+  return r;
+}
+
+// block bitonic sort of a[0..n) ascending (n padded to a power of two <= cap)
+template <int W>
+__device__ void block_sort(unsigned long long* a, uint32_t n, uint32_t cap) {
+  constexpr uint32_t T = W * 32;
+  uint32_t n2 = 1;
+  while (n2 < n) n2 <<= 1;
+  if (n2 > cap) n2 = cap;
+  for (uint32_t i = n + threadIdx.x; i < n2; i += T) a[i] = EMPTY64;
+  __syncthreads();
+  for (uint32_t size = 2; size <= n2; size <<= 1) {
+    for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+      for (uint32_t i = threadIdx.x; i < n2 / 2; i += T) {
+        const uint32_t lo = 2 * i - (i & (stride - 1));
+        const uint32_t hi = lo + stride;
+        const bool asc = (lo & size) == 0;
+        const unsigned long long x = a[lo], y = a[hi];
+        if ((x > y) == asc) {
+          a[lo] = y;
+          a[hi] = x;
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
+template <int W>
+__device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, uint32_t qi) {
+  constexpr uint32_t T = W * 32;
+  const uint32_t tid = threadIdx.x;
+  const DevGraph& g = P.g;
+  const DevState& s = P.s;
+  const Caps& cp = P.caps;
+  const uint32_t H = cp.H;
+  const uint32_t k = P.k;
+
+  for (uint32_t i = tid; i < H; i += T) m.dtab[i] = EMPTY64;
+  for (uint32_t i = tid; i < (H + 31) / 32; i += T) {
+    m.fin[i] = 0;
+    m.listed[i] = 0;
+  }
+  if (tid == 0) {
+    sh.nf = 0;
+    sh.nc = 0;
+    sh.flags = 0;
+  }
+  __syncthreads();
+
+  const uint2 q = P.q[qi];
+  if (q.x >= g.A) return DONE;
+  const uint2 ei = g.einfo[q.x];
+  if (q.y >= ei.y) return DONE;
+  const uint32_t lim = P.bound ? P.bound[qi] : INF;
+  const bool track = P.remote != nullptr && s.n_ranks > 1;
+  unsigned long long rmask = 0;  // (per thread; OR-reduced at the end)
+  if (track) {
+    const uint32_t o = owner_of(cellof(g, ei.x), g.n_cells, s.n_ranks);
+    if (o != s.rank) rmask |= 1ull << o;
+  }
+  if (tid == 0) {
+    const uint32_t seed_v = q.y == 0 ? ei.x : g.edst[q.x];
+    const uint32_t seed_d = q.y == 0 ? 0u : ei.y - q.y;
+    bool imp;
+    const int sl = tab_relax(m.dtab, H, seed_v, seed_d, imp);
+    m.front0[0] = (uint32_t)sl;
+    m.fin[sl >> 5] |= 1u << (sl & 31);
+    sh.nf = 1;
+  }
+  // objects on q's own arc ahead of q (reading R2), stored at vertex src(q.e)
+  if (q.y > 0) {
+    const uint32_t c = cellof(g, ei.x);
+    if (s.cell_head[c] != NONE) {
+      if (tid == 0) request_flush(s, c, P.epoch);
+      __syncthreads();
+      return RETRY;
+    }
+    const uint2 vo = vobj_valid(s.v_obj[ei.x], s.cell_comp[c]);
+    for (uint32_t j = tid; j < vo.y; j += T) {
+      const uint32_t p = vo.x + j;
+      const uint32_t ob = s.ar.obj[p];
+      const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
+      if (oe == q.x && oo >= q.y && s.ar.key[p] == s.ot_key[ob]) {
+        const uint32_t i = atomicAdd(&sh.nc, 1u);
+        if (i < cp.C) {
+          m.cand[i] = ((unsigned long long)SPECIAL << 32) | (oo - q.y);
+          m.cobj[i] = ob;
+        }
+      }
+    }
+  }
+  __syncthreads();
+  if (sh.nc > cp.C) return OVERFLOW;
+
+  uint32_t* front = m.front0;
+  uint32_t* nfront = m.front1;
+  uint32_t c_iter = 0, c_vert = 0, c_arcs = 0, c_harv = 0, c_objs = 0;
+  for (;;) {
+    ++c_iter;
+    const uint32_t nf = sh.nf;
+    uint32_t ml = INF;
+    for (uint32_t i = tid; i < nf; i += T) ml = min(ml, (uint32_t)m.dtab[front[i]]);
+    const uint32_t blo = block_min<W>(ml, sh);
+    if (nf == 0 || blo > lim) break;
+    const uint32_t nc0 = sh.nc;
+    if (nc0 >= k) {
+      uint32_t cl = 0;
+      for (uint32_t i = tid; i < nc0; i += T) cl += cand_dist(m, i) < blo;
+      if (block_sum<W>(cl, sh) >= k) break;
+    }
+    // partition the frontier: the bucket [m, m + delta) is expanded, the rest re-queued
+    const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
+    if (tid == 0) {
+      sh.na = 0;
+      sh.nn = 0;
+    }
+    __syncthreads();
+    for (uint32_t i = tid; i < nf; i += T) {
+      const uint32_t sl = front[i];
+      if ((uint32_t)m.dtab[sl] < bhi) {
+        m.act[atomicAdd(&sh.na, 1u)] = sl;  // (act has F entries: na <= nf <= F)
+        atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
+      } else {
+        nfront[atomicAdd(&sh.nn, 1u)] = sl;
+      }
+    }
+    __syncthreads();
+    const uint32_t na = sh.na;
+    if (tid == 0) c_vert += na;
+    // expand: lane = (vertex, arc slot), T/4 vertices per window
+    for (uint32_t w0 = 0; w0 < na; w0 += T / 4) {
+      const uint32_t vi = w0 + (tid >> 2), s4 = tid & 3;
+      if (vi < na) {
+        const uint32_t vslot = m.act[vi];
+        const unsigned long long e2 = m.dtab[vslot];  // D re-read after the frontier bit
+        const uint32_t u = (uint32_t)(e2 >> 32), du = (uint32_t)e2;
+        const uint2 arc = g.vadj[(size_t)u * 4 + s4];
+        bool harv = false;
+        uint32_t hcell = 0, hd = NONE;
+        uint2 cc = make_uint2(0, 0), v0 = make_uint2(0, 0);
+        if (s4 == 0) {
+          hcell = cellof(g, u);
+          hd = s.cell_head[hcell];
+          cc = s.cell_comp[hcell];
+          v0 = s.v_obj[u];
+          const uint32_t bit = 1u << (vslot & 31);
+          harv = !(atomicOr(&m.listed[vslot >> 5], bit) & bit);
+        }
+        auto relax = [&](uint32_t dst, uint32_t w) {
+          ++c_arcs;
+          const unsigned long long nd = (unsigned long long)du + w;
+          if (nd >= INF) return;
+          bool imp;
+          const int rr = tab_relax(m.dtab, H, dst, (uint32_t)nd, imp);
+          if (rr < 0) {
+            atomicOr(&sh.flags, FL_OVF);
+          } else if (imp) {
+            const uint32_t bit = 1u << (rr & 31);
+            if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+              const uint32_t p = atomicAdd(&sh.nn, 1u);
+              if (p < cp.F) nfront[p] = (uint32_t)rr;
+              else atomicOr(&sh.flags, FL_OVF);
+            }
+          }
+        };
+        if (arc.y == WMAX) {  // more than 4 arcs: slot 3 continues in the CSR
+          for (uint32_t a = g.rowptr[u] + 3; a < g.rowptr[u + 1]; ++a) {
+            const uint2 av = g.adj[a];
+            relax(av.x, av.y);
+          }
+        } else if (arc.y != 0) {
+          relax(arc.x, arc.y);
+        }
+        if (harv) {
+          ++c_harv;
+          if (track) {
+            const uint32_t o = owner_of(hcell, g.n_cells, s.n_ranks);
+            if (o != s.rank) rmask |= 1ull << o;
+          }
+          if (hd != NONE) {  // cached updates: lazy flush, then retry
+            request_flush(s, hcell, P.epoch);
+            atomicOr(&sh.flags, FL_RETRY);
+          } else {
+            const uint2 vo = vobj_valid(v0, cc);
+            c_objs += vo.y;
+            for (uint32_t j = 0; j < vo.y; ++j) {
+              const uint32_t p = vo.x + j;
+              const uint32_t ob = s.ar.obj[p];
+              const unsigned long long kk = s.ar.key[p];
+              const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
+              const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
+              if (!same_ahead && kk == s.ot_key[ob]) {
+                const uint32_t i = atomicAdd(&sh.nc, 1u);
+                if (i < cp.C) {
+                  m.cand[i] = ((unsigned long long)vslot << 32) | oo;
+                  m.cobj[i] = ob;
+                } else {
+                  atomicOr(&sh.flags, FL_OVF);
+                }
+              }
+            }
+          }
+        }
+      }
+      __syncthreads();
+      const uint32_t fl = sh.flags;
+      if (fl & FL_OVF) return OVERFLOW;
+      if (fl & FL_RETRY) {
+        for (uint32_t i = tid; i < nf; i += T)
+          request_flush(s, cellof(g, (uint32_t)(m.dtab[front[i]] >> 32)), P.epoch);
+        return RETRY;
+      }
+    }
+    uint32_t* tmp = front;
+    front = nfront;
+    nfront = tmp;
+    if (tid == 0) sh.nf = sh.nn;
+    __syncthreads();
+  }
+
+  // the k smallest (dist, obj)
+  const uint32_t nc = sh.nc;
+  for (uint32_t i = tid; i < nc; i += T) {
+    const unsigned long long d = cand_dist(m, i);
+    m.cand[i] = d < INF ? ((d << 32) | m.cobj[i]) : EMPTY64;
+  }
+  __syncthreads();
+  block_sort<W>(m.cand, nc, cp.C);
+  for (uint32_t r = tid; r < k; r += T) {
+    const unsigned long long dk = r < nc ? m.cand[r] : EMPTY64;
+    const bool ok = dk != EMPTY64 && (uint32_t)(dk >> 32) <= lim;
+    P.out_obj[(size_t)qi * k + r] = ok ? (uint32_t)dk : GGRID_PAD;
+    P.out_dist[(size_t)qi * k + r] = ok ? (uint32_t)(dk >> 32) : GGRID_PAD;
+  }
+  if (P.remote) {
+    unsigned long long x = rmask;
+    x = ((unsigned long long)__reduce_or_sync(0xffffffffu, (uint32_t)(x >> 32)) << 32) |
+        __reduce_or_sync(0xffffffffu, (uint32_t)x);
+    if ((tid & 31) == 0) sh.redl[tid >> 5] = x;
+    __syncthreads();
+    if (tid == 0) {
+      unsigned long long r = 0;
+      for (int w = 0; w < W; ++w) r |= sh.redl[w];
+      P.remote[qi] = r;
+    }
+  }
+  const uint32_t sa = block_sum<W>(c_arcs, sh), sh_ = block_sum<W>(c_harv, sh), so = block_sum<W>(c_objs, sh);
+  if (tid == 0) {
+    atomicAdd(&s.st->ex_iters, (unsigned long long)c_iter);
+    atomicAdd(&s.st->ex_vertices, (unsigned long long)c_vert);
+    atomicAdd(&s.st->ex_arcs, (unsigned long long)sa);
+    atomicAdd(&s.st->ex_harvested, (unsigned long long)sh_);
+    atomicAdd(&s.st->ex_objects, (unsigned long long)so);
+  }
+  __syncthreads();
+  return DONE;
+}
+
+constexpr int CTA_W = 8;  // warps per query in the CTA variant
+
+__global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ CtaShared sh;
+  __shared__ uint32_t qslot;
+  // shared memory: the level's working set, then the round's active list (F entries; the
+  // warp kernel's 32-entry act list is per frontier chunk)
+  const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
+  WarpMem m = carve(smem_raw, P.caps);
+  m.act = reinterpret_cast<uint32_t*>(smem_raw + wbytes);
+  for (;;) {  // persistent: queries fetched dynamically
+    if (threadIdx.x == 0) qslot = atomicAdd(&P.s.st->expand_work[P.level], 1u);
+    __syncthreads();
+    const uint32_t li = qslot;
+    __syncthreads();
+    if (li >= P.n) break;
+    const uint32_t qi = P.qlist ? P.qlist[li] : li;
+    const int r = run_query_cta<CTA_W>(P, m, sh, qi);
+    if (threadIdx.x == 0 && r != DONE) {
+      if (r == RETRY) {
+        P.retry_list[atomicAdd(&P.s.st->n_next[P.level], 1u)] = qi;
+      } else if (P.level < P.last_level) {
+        P.promote_list[atomicAdd(&P.s.st->n_next[P.level + 1], 1u)] = qi;
+      } else {
+        atomicOr(&P.s.st->err, (unsigned)ERR_FAIL);
+      }
+    }
+    __syncthreads();
+  }
+}
+
 // Capacity ladder.  Levels 0-3 keep the warp's working set in shared memory (one warp per
 // CTA, as many CTAs per SM as fit: ~10, 24, 45 and 190 KB per warp); level 4 is global memory
 // sized from |V| (a query that reaches fewer than k objects may need to settle the whole
@@ -551,6 +875,26 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
   if (!g_attr_set) {
     cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     g_attr_set = true;
+  }
+  // CTA-per-query for the big shared-memory levels, and for small batches at any of them
+  const bool cta = level < NLEVELS - 1 && (level >= 2 || n <= (uint32_t)sm_count);
+  if (cta) {
+    P.scratch = nullptr;
+    const int smem = (int)(wbytes + 4ull * P.caps.F);
+    static bool attr = false;
+    static int bps[NLEVELS] = {};
+    if (!attr) {
+      cudaFuncSetAttribute(k_expand_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024 + 16 * 1024);
+      attr = true;
+    }
+    if (!bps[level]) {
+      int b = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand_cta, CTA_W * 32, smem);
+      bps[level] = b > 0 ? b : 1;
+    }
+    const uint32_t wave = (uint32_t)(sm_count * bps[level]);
+    k_expand_cta<<<std::min<uint32_t>(n, wave), CTA_W * 32, smem, st>>>(P);
+    return;
   }
   if (level < NLEVELS - 1) {
     P.scratch = nullptr;

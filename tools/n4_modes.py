@@ -37,6 +37,11 @@ def run(g, f, mode, Q, k, L, steps, warm, n_obj, cell_size, l2):
     o1 = torch.empty((1, k), dtype=torch.int32, device="cuda")
     d1 = torch.empty_like(o1)
     grid.ingest(walk.tick())
+    # single-query response times on an index without profile-mode events (each event pair
+    # around a launch adds microseconds), fed the same update stream
+    lwalk = synth.RandomWalk(g, n_obj)
+    lgrid = gg.GGrid(g, cell_size, max_objects=n_obj, stream=stream.cuda_stream)
+    lgrid.ingest(lwalk.tick())
     rows, lat_dev, lat_host = [], [], []
     for s in range(warm + steps):
         u = torch.from_numpy(walk.ticks(f).view(np.int32)).cuda()
@@ -60,11 +65,11 @@ def run(g, f, mode, Q, k, L, steps, warm, n_obj, cell_size, l2):
             rows.append(dict(unit_ms=e[0].elapsed_time(e[3]), ingest_ms=e[0].elapsed_time(e[1]),
                              eager_flush_ms=e[1].elapsed_time(e[2]), knn_ms=e[2].elapsed_time(e[3]),
                              k_flush_ms=km["flush"], k_expand_ms=km["expand"] + km["expand_big"]))
-        # single-query response times on a fresh ingest (cells dirty again)
+        # single-query response times after a fresh ingest (cells dirty again)
         if L and s >= warm:
-            grid.ingest(torch.from_numpy(walk.ticks(f).view(np.int32)).cuda())
+            lgrid.ingest(torch.from_numpy(lwalk.ticks(f).view(np.int32)).cuda())
             if mode == "eager":
-                grid.flush_all()
+                lgrid.flush_all()
             q1 = torch.from_numpy(synth.queries(g, L, seed=99_000 + s).view(np.int32)).cuda()
             for i in range(L):
                 a = torch.cuda.Event(enable_timing=True)
@@ -72,12 +77,13 @@ def run(g, f, mode, Q, k, L, steps, warm, n_obj, cell_size, l2):
                 torch.cuda.synchronize()
                 t0 = time.perf_counter()
                 a.record(stream)
-                grid.knn(q1[i:i + 1], k, o1, d1)
+                lgrid.knn(q1[i:i + 1], k, o1, d1)
                 b.record(stream)
                 b.synchronize()
                 lat_host.append(time.perf_counter() - t0)
                 lat_dev.append(a.elapsed_time(b))
     grid.close()
+    lgrid.close()
     med = {key: float(np.median([r[key] for r in rows])) for key in rows[0]}
     res = dict(mode=mode, f=f, objects=n_obj, Q=Q, k=k, updates_per_unit=f * n_obj, steps=steps, **med)
     res["amortised_us_per_query"] = 1e3 * med["unit_ms"] / Q
