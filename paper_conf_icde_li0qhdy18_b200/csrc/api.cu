@@ -595,6 +595,9 @@ int ggrid_ingest_commit(ggrid_t h) {
   return ingest_device(h, sb.buf.as<uint4>(), sb.n);
 }
 
+#ifndef GG_BALL_FACTOR
+#define GG_BALL_FACTOR 2.0  // vertex-table slots per expected ball vertex (experiment hook)
+#endif
 static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
                     uint32_t* out_dist, const uint32_t* bound = nullptr,
                     uint64_t* out_remote = nullptr) {
@@ -672,7 +675,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   // overflows is promoted, the answer does not depend on it.
   int lvl0 = 0;
   const double ball = (double)k * h->V / std::max(1u, h->h_status->n_live);
-  while (lvl0 < L - 2 && (k > expand_max_k(lvl0) || 3.0 * ball > expand_table_slots(lvl0))) lvl0++;
+  while (lvl0 < L - 2 && (k > expand_max_k(lvl0) || GG_BALL_FACTOR * ball > expand_table_slots(lvl0))) lvl0++;
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
   std::vector<uint32_t> n_in(L, 0);
   n_in[lvl0] = n_q;

@@ -780,6 +780,9 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
 }
 
 constexpr int CTA_W = 8;  // warps per query in the CTA variant
+#ifndef GG_CTA_LEVEL
+#define GG_CTA_LEVEL 1  // first level run CTA-per-query (experiment hook; level 0 stays per-warp)
+#endif
 
 __global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -811,10 +814,11 @@ __global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
   }
 }
 
-// Capacity ladder.  Levels 0-3 keep the warp's working set in shared memory (one warp per
-// CTA, as many CTAs per SM as fit: ~10, 24, 45 and 190 KB per warp); level 4 is global memory
-// sized from |V| (a query that reaches fewer than k objects may need to settle the whole
-// graph).
+// Capacity ladder.  Levels 0-4 keep the query's working set in shared memory (~10, 24, 45, 95
+// and 190 KB): level 0 one warp per query (as many single-warp CTAs per SM as fit), levels 1-4
+// one 8-warp CTA per query (k_expand_cta; measured faster from level 1 up, slower at level 0);
+// level 5 is global memory sized from |V| (a query that reaches fewer than k objects may need
+// to settle the whole graph).
 constexpr int NLEVELS = EXPAND_LEVELS;
 #ifndef GG_H0
 #define GG_H0 1024  // level-0 vertex table (experiment hook: -DGG_H0=..., -DGG_F0=...)
@@ -822,7 +826,8 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 #ifndef GG_F0
 #define GG_F0 128
 #endif
-const Caps kCaps[NLEVELS - 1] = {{GG_H0, GG_F0, 64}, {2048, 512, 256}, {4096, 1024, 256}, {16384, 4096, 2048}};
+const Caps kCaps[NLEVELS - 1] = {
+    {GG_H0, GG_F0, 64}, {2048, 512, 256}, {4096, 1024, 256}, {8192, 2048, 512}, {16384, 4096, 2048}};
 
 Caps caps_for(int level, uint32_t V) {
   if (level < NLEVELS - 1) return kCaps[level];
@@ -877,7 +882,7 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
     g_attr_set = true;
   }
   // CTA-per-query for the big shared-memory levels, and for small batches at any of them
-  const bool cta = level < NLEVELS - 1 && (level >= 2 || n <= (uint32_t)sm_count);
+  const bool cta = level < NLEVELS - 1 && (level >= GG_CTA_LEVEL || n <= (uint32_t)sm_count);
   if (cta) {
     P.scratch = nullptr;
     const int smem = (int)(wbytes + 4ull * P.caps.F);
