@@ -55,6 +55,8 @@ struct CellBuf {
   unsigned long long nrec;
   unsigned long long nexp;  // records of extents dropped by t_delta expiry
   uint32_t n_win;
+  uint32_t spill_cap;     // this buffer's global spill area (winners beyond WCAP)
+  uint32_t* spill;
   uint32_t w_pos[WCAP];   // arena positions of the matched records
 };
 
@@ -145,8 +147,7 @@ __device__ __forceinline__ Grp load_group(const B& bf, const DevState& s, uint32
 
 // streaming warps: match the gathered extent list of buffer bf
 template <int WCAP, class B>
-__device__ __forceinline__ void stream_list(B& bf, const DevState& s, int sw, int lane, unsigned lt,
-                                            uint32_t* __restrict__ spill, uint32_t spill_cap) {
+__device__ __forceinline__ void stream_list(B& bf, const DevState& s, int sw, int lane, unsigned lt) {
   const unsigned long long* __restrict__ otk = s.ot_key;
   const uint32_t total = bf.xpre[bf.nx];
   int xj = 0;
@@ -172,7 +173,7 @@ __device__ __forceinline__ void stream_list(B& bf, const DevState& s, int sw, in
         const uint32_t w = base + __popc(hm & lt);
         if (hit) {
           if (w < (uint32_t)WCAP) bf.w_pos[w] = cur.pos + j;
-          else if (w - (uint32_t)WCAP < spill_cap) spill[w - WCAP] = cur.pos + j;
+          else if (w - (uint32_t)WCAP < bf.spill_cap) bf.spill[w - WCAP] = cur.pos + j;  // (rare)
         }
       }
     }
@@ -309,7 +310,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
     }
     __syncwarp();
     if (spilled) {
-      constexpr int U = 4;
+      constexpr int U = 2;  // (the kernel's register count is set by its widest path)
       for (uint32_t i0 = lane; i0 < n_win; i0 += 32 * U) {
         uint32_t p[U], ob[U], vs[U], of[U], ed[U];
         unsigned long long kk[U];
@@ -401,6 +402,8 @@ __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
     bf.n_win = 0;
     bf.nrec = 0;
     bf.nexp = 0;
+    bf.spill = spill_of(k);
+    bf.spill_cap = spill_cap;
     bf.has = k < n_mine;
     if (!bf.has) {
       bf.nx = 0;
@@ -435,7 +438,7 @@ __global__ void __launch_bounds__(FT) k_flush(DevGraph g, DevState s, Arena out,
       auto& bf = sm.b[k % NBUF];
       if (k < n_mine) {
         for (;;) {
-          stream_list<WCAP>(bf, s, wid, lane, lt, spill_of(k), spill_cap);
+          stream_list<WCAP>(bf, s, wid, lane, lt);
           if (bf.comp_done) break;
           // chains longer than XMAX extents: the streaming warps gather the next part
           stream_bar();
