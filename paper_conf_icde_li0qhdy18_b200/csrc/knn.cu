@@ -53,12 +53,13 @@ struct WarpMem {
   uint32_t* front0;          // F
   uint32_t* front1;          // F
   uint32_t* fin;             // H/32: slot is in the frontier
-  uint32_t* listed;          // H/32: vertex expanded at least once (objects harvested)
-  uint32_t* act;             // 32: active slots of the current frontier chunk
+  uint32_t* act;             // F: the round's active slots (the bucket being expanded)
+  uint8_t* listed;           // H: vertex expanded at least once (objects harvested); a vertex is
+                             //    in one round's active list at most once, so plain stores
 };
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 12ull * c.C + 4ull * (2ull * c.F + 2ull * ((c.H + 31) / 32) + 32);
+  return 8ull * c.H + 12ull * c.C + 4ull * (3ull * c.F + (c.H + 31) / 32) + ((c.H + 3) & ~3u);
 }
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
@@ -70,8 +71,8 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   m.front0 = p; p += c.F;
   m.front1 = p; p += c.F;
   m.fin = p; p += (c.H + 31) / 32;
-  m.listed = p; p += (c.H + 31) / 32;
-  m.act = p;
+  m.act = p; p += c.F;
+  m.listed = reinterpret_cast<uint8_t*>(p);
   return m;
 }
 
@@ -199,10 +200,8 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   const unsigned lt = lanemask_lt();
 
   for (uint32_t i = lane; i < cp.H; i += 32) m.dtab[i] = EMPTY64;
-  for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) {
-    m.fin[i] = 0;
-    m.listed[i] = 0;
-  }
+  for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) m.fin[i] = 0;
+  for (uint32_t i = lane; i < (cp.H + 3) / 4; i += 32) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
   __syncwarp();
 
   const uint2 q = P.q[qi];
@@ -263,16 +262,20 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
     __syncwarp();
   }
 
-  // work counters (warp-uniform), published once per answered query
+  // work counters: c_iter / c_vert warp-uniform, the others per lane (reduced at the end)
   uint32_t c_iter = 0, c_vert = 0, c_arcs = 0, c_harv = 0, c_objs = 0;
+  // frontier minimum, maintained across rounds: the next frontier holds the re-queued
+  // entries (their D read at partition) and every vertex improved during the round (each
+  // improvement's new D is seen here), so min over those is exact
+  uint32_t blo = seed_d;
+  struct Win {
+    uint32_t vslot, u, hcell, hd;
+    uint2 arc, cc, v0;
+    bool vv, harv;
+  };
   for (;;) {
     ++c_iter;
-    // ---- 1. frontier minimum: every vertex with D < m is final -------------------------
-    uint32_t ml = INF;
-    for (uint32_t i = lane; i < nf; i += 32) ml = min(ml, (uint32_t)m.dtab[front[i]]);
-    const uint32_t blo = nf ? __reduce_min_sync(FULL, ml) : INF;
-
-    // ---- 2. termination: k candidates strictly closer than anything not yet final -------
+    // ---- 1. termination: k candidates strictly closer than anything not yet final ---------
     if (nf == 0) break;
     if (blo > lim) break;  // every object not yet harvested is beyond the caller's bound
     if (nc >= k) {
@@ -281,9 +284,9 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       if (__reduce_add_sync(FULL, cl) >= k) break;
     }
 
-    // ---- 3. walk the frontier; expand the bucket [m, m + delta) -------------------------
+    // ---- 2. partition the frontier: the bucket [m, m + delta) into act, the rest re-queued --
     const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
-    uint32_t nn = 0;
+    uint32_t nn = 0, na = 0, mn = INF;
     for (uint32_t b0 = 0; b0 < nf; b0 += 32) {
       const uint32_t i = b0 + lane;
       const uint32_t sl = i < nf ? front[i] : NONE;
@@ -291,147 +294,151 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       const bool a = sl != NONE && (uint32_t)ent < bhi;
       const bool r = sl != NONE && !a;
       const unsigned rm = __ballot_sync(FULL, r);
-      if (r) nfront[nn + __popc(rm & lt)] = sl;
+      if (r) {
+        nfront[nn + __popc(rm & lt)] = sl;
+        mn = min(mn, (uint32_t)ent);
+      }
       nn += __popc(rm);
       const unsigned am = __ballot_sync(FULL, a);
-      if (!am) continue;
       if (a) {
-        m.act[__popc(am & lt)] = sl;
+        m.act[na + __popc(am & lt)] = sl;
         atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));  // re-queued if improved from here on
       }
-      __syncwarp();
-      const uint32_t na = __popc(am);
-      c_vert += na;
-      // 8 vertices per window, lane = (vertex, arc slot)
-      for (uint32_t w0 = 0; w0 < na; w0 += 8) {
-        const uint32_t vi = w0 + (lane >> 2), s4 = lane & 3;
-        const bool vv = vi < na;
-        uint32_t vslot = 0, u = 0, du = INF;
-        uint2 arc = make_uint2(0, 0);
-        if (vv) {
-          vslot = m.act[vi];
-          const unsigned long long e2 = m.dtab[vslot];  // D re-read after the frontier bit
-          u = (uint32_t)(e2 >> 32);
-          du = (uint32_t)e2;
-          arc = g.vadj[(size_t)u * 4 + s4];
-        }
-        // the vertex's object metadata: loads issued in the same memory round as its arcs,
-        // consumed after the relaxation (harvested on the vertex's first expansion only)
-        bool harv = false;
-        uint32_t hcell = 0, hd = NONE;
-        uint2 cc = make_uint2(0, 0), v0 = make_uint2(0, 0);
-        if (vv && s4 == 0) {
-          hcell = cellof(g, u);
-          hd = s.cell_head[hcell];
-          cc = s.cell_comp[hcell];
-          v0 = s.v_obj[u];
-          const uint32_t bit = 1u << (vslot & 31);
-          harv = !(atomicOr(&m.listed[vslot >> 5], bit) & bit);
-        }
-        // relax the inline arc
-        bool has = false, ovf = false;
-        uint32_t nslot = 0;
-        const bool overflow_arcs = arc.y == WMAX;
-        if (arc.y != 0 && !overflow_arcs) {
-          const unsigned long long nd = (unsigned long long)du + arc.y;
-          if (nd < INF) {
-            bool imp;
-            const int rr = tab_relax(m.dtab, H, arc.x, (uint32_t)nd, imp);
-            if (rr < 0) {
-              ovf = true;
-            } else if (imp) {
-              const uint32_t bit = 1u << (rr & 31);
-              if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
-                has = true;
-                nslot = (uint32_t)rr;
-              }
-            }
-          }
-        }
-        c_arcs += __popc(__ballot_sync(FULL, arc.y != 0 && !overflow_arcs));
-        if (__any_sync(FULL, ovf)) return OVERFLOW;
-        unsigned hm = __ballot_sync(FULL, has);
-        if (nn + __popc(hm) > cp.F) return OVERFLOW;
-        if (has) nfront[nn + __popc(hm & lt)] = nslot;
-        nn += __popc(hm);
-        // vertices with more than 4 arcs: the rest live in the CSR (rare on road graphs)
-        if (__any_sync(FULL, overflow_arcs)) {
-          uint32_t a0 = 0, a1 = 0;
-          if (overflow_arcs) {
-            a0 = g.rowptr[u] + 3;
-            a1 = g.rowptr[u + 1];
-          }
-          const uint32_t most = __reduce_max_sync(FULL, a1 - a0);
-          for (uint32_t j = 0; j < most; ++j) {
-            has = false;
-            ovf = false;
-            if (a0 + j < a1) {
-              const uint2 av = g.adj[a0 + j];
-              const unsigned long long nd = (unsigned long long)du + av.y;
-              if (nd < INF) {
-                bool imp;
-                const int rr = tab_relax(m.dtab, H, av.x, (uint32_t)nd, imp);
-                if (rr < 0) {
-                  ovf = true;
-                } else if (imp) {
-                  const uint32_t bit = 1u << (rr & 31);
-                  if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
-                    has = true;
-                    nslot = (uint32_t)rr;
-                  }
-                }
-              }
-            }
-            c_arcs += __popc(__ballot_sync(FULL, a0 + j < a1));
-            if (__any_sync(FULL, ovf)) return OVERFLOW;
-            hm = __ballot_sync(FULL, has);
-            if (nn + __popc(hm) > cp.F) return OVERFLOW;
-            if (has) nfront[nn + __popc(hm & lt)] = nslot;
-            nn += __popc(hm);
-          }
-        }
-        // harvest the objects of the vertices expanded for the first time; a cell with cached
-        // updates must be cleaned first (lazy flush): request it and retry the query
-        const bool dirty = harv && hd != NONE;
-        if (dirty) request_flush(s, hcell, P.epoch);
-        if (__any_sync(FULL, dirty)) {
-          request_lookahead(P, m, front, nf, lane);
-          return RETRY;
-        }
-        c_harv += __popc(__ballot_sync(FULL, harv));
-        if (track) {
-          const uint32_t o = harv ? owner_of(hcell, g.n_cells, s.n_ranks) : s.rank;
-          const unsigned long long b = o != s.rank ? 1ull << o : 0ull;
-          rmask |= ((unsigned long long)__reduce_or_sync(FULL, (uint32_t)(b >> 32)) << 32) |
-                   __reduce_or_sync(FULL, (uint32_t)b);
-        }
-        const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
-        const uint32_t most = __reduce_max_sync(FULL, vo.y);
-        if (most) {
-          c_objs += __reduce_add_sync(FULL, vo.y);
-          for (uint32_t j = 0; j < most; ++j) {
-            bool hc = false;
-            uint32_t ob = 0, oo = 0;
-            if (j < vo.y) {
-              const uint32_t p = vo.x + j;
-              ob = s.ar.obj[p];
-              const unsigned long long kk = s.ar.key[p];
-              const uint32_t oe = s.ar.edge[p];
-              oo = s.ar.off[p];
-              const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
-              hc = !same_ahead && kk == s.ot_key[ob];
-            }
-            if (!cand_push(m, nc, cp.C, hc, vslot, oo, ob, lt)) return OVERFLOW;
-          }
+      na += __popc(am);
+    }
+    __syncwarp();
+    c_vert += na;
+
+    // ---- 3. expand: 8 vertices per window, lane = (vertex, arc slot); the next window's
+    //         global loads (inline arcs, object metadata) are issued before this window's
+    //         relaxations
+    auto load_win = [&](uint32_t w0) {
+      Win w;
+      const uint32_t vi = w0 + (lane >> 2), s4 = lane & 3;
+      w.vv = vi < na;
+      w.vslot = 0;
+      w.u = 0;
+      w.arc = make_uint2(0, 0);
+      w.harv = false;
+      w.hcell = 0;
+      w.hd = NONE;
+      w.cc = make_uint2(0, 0);
+      w.v0 = make_uint2(0, 0);
+      if (w.vv) {
+        w.vslot = m.act[vi];
+        w.u = (uint32_t)(m.dtab[w.vslot] >> 32);
+        w.arc = g.vadj[(size_t)w.u * 4 + s4];
+        if (s4 == 0) {
+          w.hcell = cellof(g, w.u);
+          w.hd = s.cell_head[w.hcell];
+          w.cc = s.cell_comp[w.hcell];
+          w.v0 = s.v_obj[w.u];
+          w.harv = !m.listed[w.vslot];
+          if (w.harv) m.listed[w.vslot] = 1;
         }
       }
+      return w;
+    };
+    Win cur = load_win(0);
+    for (uint32_t w0 = 0; w0 < na; w0 += 8) {
+      const Win nxt = load_win(w0 + 8);  // (all lanes out of range past the last window)
+      // D re-read now: an earlier window may have improved it (the frontier bit was cleared
+      // at partition, so such an improvement also re-queued the vertex)
+      const uint32_t du = cur.vv ? (uint32_t)m.dtab[cur.vslot] : INF;
+      bool has = false, ovf = false;
+      uint32_t nslot = 0;
+      auto relax = [&](uint32_t dst, uint32_t w) {
+        ++c_arcs;
+        const unsigned long long nd = (unsigned long long)du + w;
+        if (nd >= INF) return;
+        bool imp;
+        const int rr = tab_relax(m.dtab, H, dst, (uint32_t)nd, imp);
+        if (rr < 0) {
+          ovf = true;
+        } else if (imp) {
+          mn = min(mn, (uint32_t)nd);
+          const uint32_t bit = 1u << (rr & 31);
+          if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+            has = true;
+            nslot = (uint32_t)rr;
+          }
+        }
+      };
+      const bool overflow_arcs = cur.arc.y == WMAX;
+      if (cur.arc.y != 0 && !overflow_arcs) relax(cur.arc.x, cur.arc.y);
+      if (__any_sync(FULL, ovf)) return OVERFLOW;
+      unsigned hm = __ballot_sync(FULL, has);
+      if (nn + __popc(hm) > cp.F) return OVERFLOW;
+      if (has) nfront[nn + __popc(hm & lt)] = nslot;
+      nn += __popc(hm);
+      // vertices with more than 4 arcs: the rest live in the CSR (rare on road graphs)
+      if (__any_sync(FULL, overflow_arcs)) {
+        uint32_t a0 = 0, a1 = 0;
+        if (overflow_arcs) {
+          a0 = g.rowptr[cur.u] + 3;
+          a1 = g.rowptr[cur.u + 1];
+        }
+        const uint32_t most = __reduce_max_sync(FULL, a1 - a0);
+        for (uint32_t j = 0; j < most; ++j) {
+          has = false;
+          ovf = false;
+          if (a0 + j < a1) {
+            const uint2 av = g.adj[a0 + j];
+            relax(av.x, av.y);
+          }
+          if (__any_sync(FULL, ovf)) return OVERFLOW;
+          hm = __ballot_sync(FULL, has);
+          if (nn + __popc(hm) > cp.F) return OVERFLOW;
+          if (has) nfront[nn + __popc(hm & lt)] = nslot;
+          nn += __popc(hm);
+        }
+      }
+      // harvest the objects of the vertices expanded for the first time; a cell with cached
+      // updates must be cleaned first (lazy flush): request it and retry the query
+      const bool dirty = cur.harv && cur.hd != NONE;
+      if (dirty) request_flush(s, cur.hcell, P.epoch);
+      if (__any_sync(FULL, dirty)) {
+        request_lookahead(P, m, front, nf, lane);
+        return RETRY;
+      }
+      c_harv += cur.harv;
+      if (track) {
+        const uint32_t o = cur.harv ? owner_of(cur.hcell, g.n_cells, s.n_ranks) : s.rank;
+        const unsigned long long bm = o != s.rank ? 1ull << o : 0ull;
+        rmask |= ((unsigned long long)__reduce_or_sync(FULL, (uint32_t)(bm >> 32)) << 32) |
+                 __reduce_or_sync(FULL, (uint32_t)bm);
+      }
+      const uint2 vo = cur.harv ? vobj_valid(cur.v0, cur.cc) : make_uint2(0, 0);
+      const uint32_t most = __reduce_max_sync(FULL, vo.y);
+      if (most) {
+        c_objs += vo.y;
+        for (uint32_t j = 0; j < most; ++j) {
+          bool hc = false;
+          uint32_t ob = 0, oo = 0;
+          if (j < vo.y) {
+            const uint32_t p = vo.x + j;
+            ob = s.ar.obj[p];
+            const unsigned long long kk = s.ar.key[p];
+            const uint32_t oe = s.ar.edge[p];
+            oo = s.ar.off[p];
+            const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
+            hc = !same_ahead && kk == s.ot_key[ob];
+          }
+          if (!cand_push(m, nc, cp.C, hc, cur.vslot, oo, ob, lt)) return OVERFLOW;
+        }
+      }
+      cur = nxt;
     }
     uint32_t* tmp = front;
     front = nfront;
     nfront = tmp;
     nf = nn;
+    blo = __reduce_min_sync(FULL, mn);
     __syncwarp();
   }
+  c_arcs = __reduce_add_sync(FULL, c_arcs);
+  c_harv = __reduce_add_sync(FULL, c_harv);
+  c_objs = __reduce_add_sync(FULL, c_objs);
 
   // ---- 4. the k smallest (dist, obj) ------------------------------------------------------
   for (uint32_t i = lane; i < nc; i += 32) {
@@ -559,10 +566,8 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
   const uint32_t k = P.k;
 
   for (uint32_t i = tid; i < H; i += T) m.dtab[i] = EMPTY64;
-  for (uint32_t i = tid; i < (H + 31) / 32; i += T) {
-    m.fin[i] = 0;
-    m.listed[i] = 0;
-  }
+  for (uint32_t i = tid; i < (H + 31) / 32; i += T) m.fin[i] = 0;
+  for (uint32_t i = tid; i < (H + 3) / 4; i += T) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
   if (tid == 0) {
     sh.nf = 0;
     sh.nc = 0;
@@ -666,8 +671,8 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
           hd = s.cell_head[hcell];
           cc = s.cell_comp[hcell];
           v0 = s.v_obj[u];
-          const uint32_t bit = 1u << (vslot & 31);
-          harv = !(atomicOr(&m.listed[vslot >> 5], bit) & bit);
+          harv = !m.listed[vslot];  // (one thread per active vertex per round)
+          if (harv) m.listed[vslot] = 1;
         }
         auto relax = [&](uint32_t dst, uint32_t w) {
           ++c_arcs;
@@ -788,11 +793,7 @@ __global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ CtaShared sh;
   __shared__ uint32_t qslot;
-  // shared memory: the level's working set, then the round's active list (F entries; the
-  // warp kernel's 32-entry act list is per frontier chunk)
-  const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
-  WarpMem m = carve(smem_raw, P.caps);
-  m.act = reinterpret_cast<uint32_t*>(smem_raw + wbytes);
+  const WarpMem m = carve(smem_raw, P.caps);
   for (;;) {  // persistent: queries fetched dynamically
     if (threadIdx.x == 0) qslot = atomicAdd(&P.s.st->expand_work[P.level], 1u);
     __syncthreads();
@@ -885,11 +886,11 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
   const bool cta = level < NLEVELS - 1 && (level >= GG_CTA_LEVEL || n <= (uint32_t)sm_count);
   if (cta) {
     P.scratch = nullptr;
-    const int smem = (int)(wbytes + 4ull * P.caps.F);
+    const int smem = (int)wbytes;
     static bool attr = false;
     static int bps[NLEVELS] = {};
     if (!attr) {
-      cudaFuncSetAttribute(k_expand_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024 + 16 * 1024);
+      cudaFuncSetAttribute(k_expand_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
       attr = true;
     }
     if (!bps[level]) {
