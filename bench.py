@@ -50,6 +50,13 @@ EXPAND_BYTES_PER_HARVEST = 12  # cell_head (dirty check) + v_obj (start, count)
 EXPAND_BYTES_PER_OBJECT = 28   # obj, key, edge, off + ot_key (validity)
 EXPAND_BYTES_PER_QUERY = 16    # query (edge, off) + inverted index (src, w)
 
+# opts.profile masks (include/ggrid.h): bit 0 = every launch kind, bit k+1 = kind k.  A timed
+# launch costs ~3-4 us of device idle time per event, so the timed steps time only the
+# dominant kernel (the expansion, GGRID_K_EXPAND = 5 / GGRID_K_EXPAND_BIG = 6); the
+# per-kernel split comes from extra, untimed breakdown steps with every launch timed.
+PROFILE_ALL = 1
+PROFILE_EXPAND = (2 << 5) | (2 << 6)
+
 
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
@@ -195,8 +202,9 @@ def run_ours(args, cfg_name):
     walk = synth.RandomWalk(g, cfg["n_objects"])
     stream = torch.cuda.Stream()
     shard = world > 1 and args.parallel == "shard"
-    grid = gg.GGrid(g, args.cell_size or cfg["cell_size"], max_objects=cfg["n_objects"], profile=True,
-                    log_capacity=args.log_capacity, delta=args.delta, stream=stream.cuda_stream)
+    grid = gg.GGrid(g, args.cell_size or cfg["cell_size"], max_objects=cfg["n_objects"], profile=PROFILE_EXPAND,
+                    log_capacity=args.log_capacity, delta=args.delta, stream=stream.cuda_stream,
+                    async_ingest=True)
     if shard:  # cell-ownership sharding: logs of own cells only
         grid.shard(world, rank)
     out_o = torch.empty((Q, k), dtype=torch.int32, device="cuda")
@@ -220,7 +228,8 @@ def run_ours(args, cfg_name):
 
     n_upd_step = cfg["n_objects"] * cfg["updates_per_object"]
     remote_requests = 0
-    for s in range(args.warmup + args.steps):
+    n_break = max(3, min(args.steps, 10))  # breakdown steps (every launch timed), after the timed ones
+    for s in range(args.warmup + args.steps + n_break):
         q = synth.queries(g, Q, seed=synth.SEED_QUERIES + 1000 * rank + s)
         u = walk.ticks(cfg["updates_per_object"])  # every rank keeps the walk in step (untimed)
         if rank == 0:  # the update stream arrives at rank 0 and is fanned out over NCCL
@@ -228,15 +237,24 @@ def run_ours(args, cfg_name):
         else:
             du = torch.empty((n_upd_step, 4), dtype=torch.int32, device="cuda")
         dq = torch.from_numpy(q.view(np.int32)).to("cuda")
-        with torch.cuda.stream(stream):
-            l2.zero_()  # flush L2 between timed iterations (outside the events)
         barrier()
         if s == args.warmup:
             grid.stats_reset()
             st0 = grid.stats()
             clocks = ClockSampler(dev)
+        if s == args.warmup + args.steps:  # end of the timed steps
+            clk = clocks.stop()
+            grid.sync()  # (raises a deferred ingest error, if any)
+            st1 = grid.stats()
+            grid.set_profile(PROFILE_ALL)
+            grid.stats_reset()
+            sb0 = grid.stats()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            # flush L2 between timed iterations (outside the events); the host queues the
+            # step's launches while the device is still writing it
+            l2.zero_()
         e0.record(stream)
         if world > 1:
             with torch.cuda.stream(stream):
@@ -245,16 +263,16 @@ def run_ours(args, cfg_name):
         if shard:  # owner search + bounded requests/replies + merge, all ordered on `stream`
             with torch.cuda.stream(stream):
                 out_o, out_d, n_req = gdist.sharded_knn(grid, dq, k, world, rank)
-                remote_requests += n_req if s >= args.warmup else 0
+                remote_requests += n_req if args.warmup <= s < args.warmup + args.steps else 0
         else:
             grid.knn(dq, k, out_o, out_d)
         e1.record(stream)
         e1.synchronize()
-        if s >= args.warmup:
+        if args.warmup <= s < args.warmup + args.steps:
             times.append(e0.elapsed_time(e1))
     barrier()
-    clk = clocks.stop()
-    st1 = grid.stats()
+    grid.sync()
+    sb1 = grid.stats()
     total_ms = sum(times)
     if world > 1:
         t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
@@ -264,37 +282,46 @@ def run_ours(args, cfg_name):
     value = world * Q * K / (total_ms / 1e3)
     n_upd = cfg["n_objects"] * cfg["updates_per_object"]
 
-    # ---- per-kernel roofline from the profile-mode events of the timed region -----------
+    # ---- per-kernel roofline ----------------------------------------------------------------
+    # split: the breakdown steps (every launch timed); the dominant kernel's achieved rate: its
+    # CUDA events inside the timed steps when it is the expansion (timed there), else the split
     peak, peak_kind = load_peaks()
-    kms = st1["kernel_ms"]
-    kl = st1["kernel_launches"]
-    ingest_ms = kms["ingest_classify"] + kms["ingest_alloc"] + kms["ingest_scatter"]
-    rec = st1["records_flushed"] - st0["records_flushed"]
-    win = st1["objects_written"] - st0["objects_written"]
-    cells = st1["cells_flushed"] - st0["cells_flushed"]
     cs = st1["cell_size"]
-    dx = {n: st1["expand_" + n] - st0["expand_" + n] for n in ("iterations", "vertices", "arcs", "harvested", "objects")}
-    expand_bytes = (dx["vertices"] * EXPAND_BYTES_PER_VERTEX + dx["arcs"] * EXPAND_BYTES_PER_ARC
-                    + dx["harvested"] * EXPAND_BYTES_PER_HARVEST + dx["objects"] * EXPAND_BYTES_PER_OBJECT
-                    + Q * K * (EXPAND_BYTES_PER_QUERY + 8 * k))
-    flush_bytes = rec * FLUSH_BYTES_PER_RECORD + win * FLUSH_BYTES_PER_WINNER
-    kern = {
-        "ingest": (ingest_ms, n_upd * K * INGEST_BYTES_PER_UPDATE,
-                   kl["ingest_classify"] + kl["ingest_alloc"] + kl["ingest_scatter"]),
-        "flush": (kms["flush"], flush_bytes, kl["flush"]),
-        "expand": (kms["expand"] + kms["expand_big"], expand_bytes, kl["expand"] + kl["expand_big"]),
-    }
+
+    def kernels(a, b, nsteps):
+        kms, kl = b["kernel_ms"], b["kernel_launches"]
+        rec = b["records_flushed"] - a["records_flushed"]
+        win = b["objects_written"] - a["objects_written"]
+        dx = {n: b["expand_" + n] - a["expand_" + n] for n in ("iterations", "vertices", "arcs", "harvested", "objects")}
+        expand_bytes = (dx["vertices"] * EXPAND_BYTES_PER_VERTEX + dx["arcs"] * EXPAND_BYTES_PER_ARC
+                        + dx["harvested"] * EXPAND_BYTES_PER_HARVEST + dx["objects"] * EXPAND_BYTES_PER_OBJECT
+                        + Q * nsteps * (EXPAND_BYTES_PER_QUERY + 8 * k))
+        kern = {
+            "ingest": (kms["ingest_classify"] + kms["ingest_alloc"] + kms["ingest_scatter"],
+                       n_upd * nsteps * INGEST_BYTES_PER_UPDATE,
+                       kl["ingest_classify"] + kl["ingest_alloc"] + kl["ingest_scatter"]),
+            "flush": (kms["flush"], rec * FLUSH_BYTES_PER_RECORD + win * FLUSH_BYTES_PER_WINNER, kl["flush"]),
+            "expand": (kms["expand"] + kms["expand_big"], expand_bytes, kl["expand"] + kl["expand_big"]),
+        }
+        return kern, dx
+
+    kern, _ = kernels(sb0, sb1, n_break)
+    kern_t, dx = kernels(st0, st1, K)
+    ingest_ms = kern["ingest"][0] * K / n_break  # ingest time of K steps, from the split
     dom = max(kern, key=lambda n: kern[n][0])
-    dms, dbytes, dl = kern[dom]
+    dms, dbytes, dl = kern_t[dom] if dom == "expand" else kern[dom]
     achieved = dbytes / (dms / 1e3) / 1e9 if dms > 0 else 0.0
-    per_kernel = {n: {"ms_total": v[0], "launches": v[2], "alg_bytes": v[1],
+    per_kernel = {n: {"ms_per_step": v[0] / n_break, "launches_per_step": v[2] / n_break,
+                      "alg_bytes_per_step": v[1] / n_break,
                       "gbs": (v[1] / (v[0] / 1e3) / 1e9) if v[0] > 0 else 0.0} for n, v in kern.items()}
+    per_kernel["source"] = f"{n_break} breakdown steps after the timed ones, every launch timed"
     traffic = None
     tp = os.path.join(ROOT, "profiles", f"traffic_{cfg_name}.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get(dom)
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic, "kernel": dom, "peak_source": peak_kind}
+                "traffic": traffic, "kernel": dom, "peak_source": peak_kind,
+                "launch_ms": dms / max(1, dl), "timed_in": "timed steps" if dom == "expand" else "breakdown steps"}
     updates_per_s = n_upd * K / (ingest_ms / 1e3) if ingest_ms > 0 else None
 
     # ---- e2e through the public API with pinned host buffers -------------------------------
@@ -306,7 +333,7 @@ def run_ours(args, cfg_name):
     # costs ~50 us), warmed by the same stream of steps
     grid.close()
     grid = gg.GGrid(g, args.cell_size or cfg["cell_size"], max_objects=cfg["n_objects"],
-                    log_capacity=args.log_capacity, delta=args.delta)
+                    log_capacity=args.log_capacity, delta=args.delta, async_ingest=True)
     if shard:
         grid.shard(world, rank)
     dq_e = torch.empty((Q, 2), dtype=torch.int32, device="cuda")
@@ -349,6 +376,7 @@ def run_ours(args, cfg_name):
         if s + 1 <= n_e2e:
             grid.ingest_stage(hus[s + 1])  # overlaps the queries below
         e2e_knn(hqs[s])
+    grid.sync()  # (the last step's answers were read back inside knn already)
     e2e_total = time.perf_counter() - t0
     if trace is not None:
         trace.__exit__(None, None, None)

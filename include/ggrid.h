@@ -58,7 +58,10 @@ typedef struct ggrid_opts {
   uint32_t delta;          /* expansion bucket width; 0 = mean arc weight          */
   uint32_t seed_neighbors; /* 0 = default on: flush c_q and its neighbour cells up
                               front (Alg. 4 line 1); 2 = off (c_q only)            */
-  uint32_t profile;        /* 1 = time every kernel launch with CUDA events        */
+  uint32_t profile;        /* time kernel launches with CUDA events (kernel_ms):
+                              bit 0 = every kind, bit k+1 = kind k (GGRID_K_*) only.
+                              Each timed launch costs a few microseconds of device
+                              idle time between kernels.                           */
   uint32_t t_delta;        /* message expiry window t_Delta (P@20631-21157, sign
                               corrected, reading R21): at cleaning time a
                               cached extent (one ingest batch's messages for one
@@ -67,6 +70,14 @@ typedef struct ggrid_opts {
                               iff every object reports at least once per t_delta of
                               arrival-ordered time.  0 = never expire.             */
   void* stream;            /* cudaStream_t to run on, or NULL (library stream)    */
+  uint32_t async_ingest;   /* 1 = ggrid_ingest / ggrid_ingest_commit return once
+                              the batch's kernels are queued on the stream (no
+                              host round trip).  Validation still happens, on the
+                              device, and still rejects the whole batch; the error
+                              (EINVAL, or ENOMEM) is reported later, by the next
+                              ggrid_sync or ggrid_ingest call.  A rejected batch
+                              leaves its seq range unused.  Ignored (synchronous)
+                              when t_delta != 0.  0 = default, synchronous.         */
 } ggrid_opts;
 
 typedef struct ggrid_s* ggrid_t;
@@ -117,7 +128,7 @@ typedef struct ggrid_stats_t {
   uint64_t expand_harvested; /* settled vertices whose object lists were read        */
   uint64_t expand_objects;   /* object entries read while harvesting                 */
   uint64_t kernel_launches[GGRID_NK];
-  double kernel_ms[GGRID_NK];/* summed CUDA-event device time (opts.profile = 1)     */
+  double kernel_ms[GGRID_NK];/* summed CUDA-event device time (kinds opts.profile times) */
   uint32_t n_cells;
   uint32_t cell_size;
   uint32_t delta;
@@ -238,6 +249,11 @@ int ggrid_prior_art_clean(ggrid_t h, uint32_t eta, uint32_t bucket_size, uint32_
 int ggrid_prior_art_bundle(const uint32_t* obj, const uint64_t* key, uint32_t eta, uint32_t* out_obj,
                            uint64_t* out_key);
 
+/* Drain the handle's stream.  Returns the deferred error of an asynchronous ingest batch
+ * (opts.async_ingest) that was rejected since the last report, else GGRID_OK; the error is
+ * reported once. */
+int ggrid_sync(ggrid_t h);
+
 /* Release every resource of h (NULL is accepted). */
 int ggrid_free(ggrid_t h);
 
@@ -245,6 +261,9 @@ int ggrid_free(ggrid_t h);
 const char* ggrid_strerror(int rc);
 
 /* ---- test / bench hooks -------------------------------------------------------- */
+
+/* Change opts.profile (the kinds of kernel launches timed with CUDA events) after build. */
+int ggrid_set_profile(ggrid_t h, uint32_t mask);
 
 /* Eager message cleaning of every cell with cached updates (lazy == eager invariant). */
 int ggrid_flush_all(ggrid_t h);

@@ -23,7 +23,7 @@ GGRID_OK, GGRID_EINVAL, GGRID_ENOMEM, GGRID_ECUDA, GGRID_ENCCL, GGRID_EOVERFLOW 
 PAD = 0xFFFFFFFF
 KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "flush", "expand",
                 "expand_big", "other"]
-EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_flush_all",
+EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_sync", "ggrid_set_profile", "ggrid_flush_all",
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
            "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk",
            "ggrid_prior_art_clean", "ggrid_prior_art_bundle"]
@@ -45,7 +45,7 @@ class ggrid_opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("max_k", ctypes.c_uint32), ("max_objects", ctypes.c_uint32),
                 ("log_capacity", ctypes.c_uint64), ("delta", ctypes.c_uint32),
                 ("seed_neighbors", ctypes.c_uint32), ("profile", ctypes.c_uint32),
-                ("t_delta", ctypes.c_uint32), ("stream", ctypes.c_void_p)]
+                ("t_delta", ctypes.c_uint32), ("stream", ctypes.c_void_p), ("async_ingest", ctypes.c_uint32)]
 
 
 NK = 8
@@ -86,6 +86,8 @@ def lib():
             "ggrid_free": ([P], i32),
             "ggrid_strerror": ([i32], ctypes.c_char_p),
             "ggrid_flush_all": ([P], i32),
+            "ggrid_sync": ([P], i32),
+            "ggrid_set_profile": ([P, u32], i32),
             "ggrid_cell_objects": ([P, u32, P, P, P, u32, ctypes.POINTER(u32)], i32),
             "ggrid_stats": ([P, ctypes.POINTER(ggrid_stats_t)], i32),
             "ggrid_stats_reset": ([P], i32),
@@ -138,7 +140,8 @@ def _u32(a):
 # ------------------------------------------------------------------------ the C ABI names
 def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 256,
                 max_objects: int = 1 << 24, log_capacity: int = 0, delta: int = 0,
-                seed_neighbors: bool = True, profile: bool = False, t_delta: int = 0, stream=None):
+                seed_neighbors: bool = True, profile: bool = False, t_delta: int = 0, stream=None,
+                async_ingest: bool = False):
     """ggrid_build(graph, cell_size) -> handle (c_void_p).  graph: dict(n_vertices, src, dst, w[, x, y])."""
     src, dst, w = (np.ascontiguousarray(graph[k], np.uint32) for k in ("src", "dst", "w"))
     x = graph.get("x")
@@ -148,7 +151,8 @@ def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 25
     g = ggrid_graph(int(graph["n_vertices"]), len(src), src.ctypes.data, dst.ctypes.data, w.ctypes.data,
                     None if x is None else x.ctypes.data, None if y is None else y.ctypes.data)
     o = ggrid_opts(int(device), int(max_k), int(max_objects), int(log_capacity), int(delta),
-                   0 if seed_neighbors else 2, 1 if profile else 0, int(t_delta), stream)
+                   0 if seed_neighbors else 2, int(profile), int(t_delta), stream,
+                   1 if async_ingest else 0)
     h = ctypes.c_void_p()
     _check(lib().ggrid_build(ctypes.byref(g), int(cell_size), ctypes.byref(o), ctypes.byref(h)), "ggrid_build")
     return h
@@ -159,6 +163,16 @@ def ggrid_ingest(h, updates, n: int | None = None):
     u = _u32(updates)
     cnt = int(u.shape[0]) if n is None else int(n)
     _check(lib().ggrid_ingest(h, _ptr(u), cnt), "ggrid_ingest")
+
+
+def ggrid_sync(h):
+    """Drain the stream; raises the deferred error of a rejected asynchronous ingest batch."""
+    _check(lib().ggrid_sync(h), "ggrid_sync")
+
+
+def ggrid_set_profile(h, mask: int):
+    """Kinds of launches timed with CUDA events: bit 0 = all, bit k+1 = kind k (K_*)."""
+    _check(lib().ggrid_set_profile(h, int(mask)), "ggrid_set_profile")
 
 
 def ggrid_ingest_stage(h, updates):
@@ -314,6 +328,14 @@ class GGrid:
 
     def ingest(self, updates):
         ggrid_ingest(self.h, updates)
+        return self
+
+    def sync(self):
+        ggrid_sync(self.h)
+        return self
+
+    def set_profile(self, mask: int):
+        ggrid_set_profile(self.h, mask)
         return self
 
     def ingest_stage(self, updates):

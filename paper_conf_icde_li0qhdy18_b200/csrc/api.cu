@@ -102,8 +102,14 @@ struct ggrid_s {
   int sm_count = 148;
   uint32_t V = 0, A = 0, cs = 1, n_cells = 0, delta = 1, max_k = 256, max_objects = 0;
   int seed_neighbors = 1;
-  int profile = 0;
+  uint32_t profile = 0;  // opts.profile: bit 0 = every kind, bit k+1 = kind k
   uint32_t t_delta = 0;  // message expiry window (0 = never)
+  // asynchronous ingest (opts.async_ingest): ggrid_ingest returns once its kernels are queued.
+  // Until the next sync the status mirror is stale by the batches queued since; these bound
+  // what they can have added (records incl. extent padding, extents, newly live objects).
+  int async_ingest = 0;
+  uint64_t pend_records = 0, pend_updates = 0;
+  uint32_t pend_ext = 0;
   uint32_t max_cell_degree = 0;  // most neighbour cells of any cell
   std::vector<uint32_t> user_cell;
   DevGraph g{};
@@ -120,7 +126,8 @@ struct ggrid_s {
   struct Staged {
     DBuf buf;
     uint64_t n = 0;
-    cudaEvent_t done = nullptr;
+    cudaEvent_t done = nullptr;      // copy finished (copy stream)
+    cudaEvent_t consumed = nullptr;  // its ingest kernels finished reading it (main stream)
   };
   Staged staged[2];
   int stage_head = 0, n_staged = 0;
@@ -158,7 +165,7 @@ struct ggrid_s {
   void launch(int kind, F&& f) {
     stats.launches++;
     stats.kernel_launches[kind]++;
-    if (profile) {
+    if (profile & (1u | (2u << kind))) {
       cudaEvent_t a = get_event(), b = get_event();
       cudaEventRecord(a, stream);
       f();
@@ -175,6 +182,8 @@ struct ggrid_s {
   int sync() {
     launch(GGRID_K_OTHER, [&] { launch_copy_words(d_status, h_status_dev, sizeof(DevStatus), stream); });
     CK(cudaStreamSynchronize(stream));
+    pend_records = pend_updates = 0;
+    pend_ext = 0;
     for (auto& pe : pending_ev) {
       float ms = 0.f;
       if (cudaEventElapsedTime(&ms, pe.second.first, pe.second.second) == cudaSuccess)
@@ -200,7 +209,7 @@ struct ggrid_s {
 
   int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin, int full_vobj = 0,
                      uint32_t max_cells = 0) {
-    const uint32_t opc = (uint32_t)((h_status->n_live + n_cells - 1) / std::max(1u, n_cells));
+    const uint32_t opc = (uint32_t)((n_live_hi() + n_cells - 1) / std::max(1u, n_cells));
     uint32_t spill_cap = 0;
     const size_t sb = flush_spill_bytes(g.cs, opc, sm_count, &spill_cap);
     if (sb) RC(flush_spill.ensure(sb));
@@ -217,10 +226,26 @@ struct ggrid_s {
 
   int gc();
   int ensure_arena(uint64_t need_records, uint32_t need_ext);
+  // upper bound of the objects live on the device (exact after a sync)
+  uint64_t n_live_hi() const {
+    return std::min<uint64_t>(max_objects, (uint64_t)h_status->n_live + pend_updates);
+  }
   // upper bound of the records a flush of every dirty cell can write: each live object is
   // valid in exactly one cell, plus <= 3 padding records per cell (dirty cells <= extents)
   uint64_t flush_need() const {
-    return (uint64_t)h_status->n_live + 4ull * std::min<uint64_t>(n_cells, h_status->ext_top) + 16;
+    return n_live_hi() + 4ull * std::min<uint64_t>(n_cells, (uint64_t)h_status->ext_top + pend_ext) + 16;
+  }
+  // the deferred error of an asynchronous ingest batch, as of the last sync (then cleared)
+  int take_deferred() {
+    const unsigned e = h_status->err_deferred | (async_ingest ? h_status->ingest_err : 0u);
+    if (!e) return GGRID_OK;
+    WordSet ws;
+    ws.add(&d_status->err_deferred, 0u);
+    ws.add(&d_status->ingest_err, 0u);
+    RC(set_words(ws));
+    h_status->err_deferred = 0;
+    h_status->ingest_err = 0;
+    return (e & (ERR_OBJ | ERR_EDGE | ERR_OFF)) ? GGRID_EINVAL : GGRID_ENOMEM;
   }
 };
 
@@ -271,10 +296,10 @@ int ggrid_s::gc() {
 }
 
 int ggrid_s::ensure_arena(uint64_t need_records, uint32_t need_ext) {
-  const bool fits_a = h_status->arena_top + need_records <= s.ar.cap;
-  const bool fits_e = (uint64_t)h_status->ext_top + need_ext <= s.ext_cap;
+  const bool fits_a = h_status->arena_top + pend_records + need_records <= s.ar.cap;
+  const bool fits_e = (uint64_t)h_status->ext_top + pend_ext + need_ext <= s.ext_cap;
   if (fits_a && fits_e) return GGRID_OK;
-  RC(gc());
+  RC(gc());  // (syncs first: the pending bounds are resolved)
   if (h_status->arena_top + need_records > s.ar.cap) return GGRID_ENOMEM;
   if ((uint64_t)h_status->ext_top + need_ext > s.ext_cap) return GGRID_ENOMEM;
   return GGRID_OK;
@@ -352,8 +377,10 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   h->max_k = o.max_k;
   h->max_objects = o.max_objects;
   h->seed_neighbors = o.seed_neighbors == 2 ? 0 : 1;
-  h->profile = o.profile ? 1 : 0;
+  h->profile = o.profile;
   h->t_delta = o.t_delta;
+  // the expiry cut reads t_now on the host, so expiry keeps ingest synchronous
+  h->async_ingest = (o.async_ingest && !o.t_delta) ? 1 : 0;
   h->s.n_ranks = 1;
   h->s.rank = 0;
 
@@ -508,8 +535,10 @@ int ggrid_free(ggrid_t h) {
                   &h->remote_stage, &h->merge_stage, &h->staged[0].buf,
                   &h->staged[1].buf})
     b->release();
-  for (auto& sb : h->staged)
+  for (auto& sb : h->staged) {
     if (sb.done) cudaEventDestroy(sb.done);
+    if (sb.consumed) cudaEventDestroy(sb.consumed);
+  }
   if (h->copy_stream) cudaStreamDestroy(h->copy_stream);
   for (auto& pe : h->pending_ev) {
     cudaEventDestroy(pe.second.first);
@@ -526,12 +555,17 @@ int ggrid_free(ggrid_t h) {
 // ordered after their arrival)
 static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
+  if (h->async_ingest) RC(h->take_deferred());  // an earlier batch was rejected
   const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
   RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
   RC(h->tmp.ensure(ingest_tmp_bytes(n)));
   {
     WordSet ws;
-    ws.add(&h->d_status->err, 0u);
+    if (h->async_ingest) {  // the previous batch's error bits move to err_deferred (ggrid_sync)
+      ws.fold_dst = &h->d_status->err_deferred;
+      ws.fold_src = &h->d_status->ingest_err;
+    }
+    ws.add(&h->d_status->ingest_err, 0u);
     ws.add(&h->d_status->bad_index, 0xFFFFFFFFu);
     RC(h->set_words(ws));
   }
@@ -543,8 +577,18 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   h->launch(GGRID_K_INGEST_CLASSIFY, [&] { launch_ingest_classify(d_u, n, g, s, tmp, st); });
   h->launch(GGRID_K_INGEST_ALLOC, [&] { launch_ingest_alloc(g, s, st); });
   h->launch(GGRID_K_INGEST_SCATTER, [&] { launch_ingest_scatter(d_u, n, seq0, g, s, tmp, st); });
+  if (h->async_ingest) {
+    // no host round trip: a rejected batch (checked on the device, all or nothing) keeps its
+    // seq range unused, which changes no answer (only the order of keys matters)
+    h->pend_records += n + 3ull * ext_need;
+    h->pend_ext += ext_need;
+    h->pend_updates += n;
+    h->seq_next += n;
+    h->stats.n_updates = h->seq_next;
+    return GGRID_OK;
+  }
   RC(h->sync());
-  const unsigned err = h->h_status->err;
+  const unsigned err = h->h_status->ingest_err;
   if (err & (ERR_OBJ | ERR_EDGE | ERR_OFF)) return GGRID_EINVAL;
   if (err & ERR_ARENA) return GGRID_ENOMEM;
   h->seq_next += n;
@@ -572,7 +616,13 @@ int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n) {
   CK(cudaSetDevice(h->device));
   ggrid_s::Staged& sb = h->staged[(h->stage_head + h->n_staged) & 1];
   if (!sb.done) CK(cudaEventCreateWithFlags(&sb.done, cudaEventDisableTiming));
+  if (!sb.consumed) {
+    CK(cudaEventCreateWithFlags(&sb.consumed, cudaEventDisableTiming));
+    CK(cudaEventRecord(sb.consumed, h->stream));
+  }
   sb.n = n;
+  // an asynchronous ingest of this buffer's previous batch may still be reading it
+  CK(cudaStreamWaitEvent(h->copy_stream, sb.consumed, 0));
   if (n) {
     // both buffers grow together: a cudaMalloc in the middle of a running pipeline stalls it
     RC(h->staged[0].buf.ensure(n * sizeof(uint4)));
@@ -592,7 +642,9 @@ int ggrid_ingest_commit(ggrid_t h) {
   h->n_staged--;
   CK(cudaStreamWaitEvent(h->stream, sb.done, 0));
   if (sb.n == 0) return GGRID_OK;
-  return ingest_device(h, sb.buf.as<uint4>(), sb.n);
+  const int rc = ingest_device(h, sb.buf.as<uint4>(), sb.n);
+  CK(cudaEventRecord(sb.consumed, h->stream));
+  return rc;
 }
 
 #ifndef GG_BALL_FACTOR
@@ -674,7 +726,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   // also holds the frontier and stays below ~1/3 load).  A guess only: a query that
   // overflows is promoted, the answer does not depend on it.
   int lvl0 = 0;
-  const double ball = (double)k * h->V / std::max(1u, h->h_status->n_live);
+  const double ball = (double)k * h->V / (double)std::max<uint64_t>(1, h->n_live_hi());
   while (lvl0 < L - 2 && (k > expand_max_k(lvl0) || GG_BALL_FACTOR * ball > expand_table_slots(lvl0))) lvl0++;
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
   std::vector<uint32_t> n_in(L, 0);
@@ -912,6 +964,20 @@ int ggrid_prior_art_bundle(const uint32_t* obj, const uint64_t* key, uint32_t et
   }
   b.release();
   return rc;
+}
+
+int ggrid_set_profile(ggrid_t h, uint32_t mask) {
+  if (!h) return GGRID_EINVAL;
+  RC(h->sync());  // (collects the events of the previous mode)
+  h->profile = mask;
+  return GGRID_OK;
+}
+
+int ggrid_sync(ggrid_t h) {
+  if (!h) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  RC(h->sync());
+  return h->take_deferred();
 }
 
 int ggrid_flush_all(ggrid_t h) {

@@ -74,7 +74,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
       bad |= ERR_OFF;
     }
     if (bad) {
-      atomicOr(&s.st->err, bad);
+      atomicOr(&s.st->ingest_err, bad);
       atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
       continue;
     }
@@ -160,7 +160,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
 
 __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
   uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
-  const bool err = s.st->err != 0;
+  const bool err = s.st->ingest_err != 0;
   uint32_t cnt = (c < g.n_cells) ? s.bcount[c * BCOUNT_STRIDE] : 0;
   if (err) {
     if (c < g.n_cells && cnt) {
@@ -193,7 +193,7 @@ __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
   unsigned long long start = base + (incl - alloc);
   unsigned e = ebase + __popc(nonempty & lanemask_lt());
   if (start + alloc > s.ar.cap || e >= s.ext_cap) {  // host pre-checks make this unreachable
-    atomicOr(&s.st->err, (unsigned)ERR_ARENA);
+    atomicOr(&s.st->ingest_err, (unsigned)ERR_ARENA);
     return;
   }
   s.x_start[e] = (uint32_t)start;
@@ -231,7 +231,7 @@ __global__ void __launch_bounds__(CT) k_ingest_scatter(const uint4* __restrict__
       il[j] = __ldcs(perm + base + k);
     }
   }
-  if (*((volatile unsigned*)&s.st->err)) return;
+  if (*((volatile unsigned*)&s.st->ingest_err)) return;
   __syncthreads();
   // two halves of CPT/2 updates: every load of a half in flight before its stores, at half
   // the registers (occupancy)
@@ -386,10 +386,12 @@ void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t
 
 namespace gg {
 __global__ void k_set_words(WordSet ws) {
+  if (ws.fold_dst && threadIdx.x == 0) *ws.fold_dst |= *ws.fold_src;
+  __syncwarp();
   if ((int)threadIdx.x < ws.n) *ws.p[threadIdx.x] = ws.v[threadIdx.x];
 }
 void launch_set_words(const WordSet& ws, cudaStream_t st) {
-  if (ws.n) k_set_words<<<1, 32, 0, st>>>(ws);
+  if (ws.n || ws.fold_dst) k_set_words<<<1, 32, 0, st>>>(ws);
 }
 }  // namespace gg
 

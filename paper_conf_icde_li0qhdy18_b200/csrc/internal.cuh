@@ -41,7 +41,9 @@ struct DevStatus {
   unsigned long long ex_iters, ex_vertices, ex_arcs, ex_harvested, ex_objects;  // expansion work
   unsigned long long records_expired;  // dropped unread by t_delta expiry
   unsigned int ext_top;     // next free extent
-  unsigned int err;         // ErrBits
+  unsigned int err;         // ErrBits of the current knn / flush / gc call
+  unsigned int ingest_err;  // ErrBits of the current ingest batch (classify / alloc / scatter)
+  unsigned int err_deferred;  // ingest_err of earlier asynchronous batches, not yet reported
   unsigned int bad_index;   // smallest offending index (ingest)
   unsigned int n_live;      // objects with at least one update
   unsigned int t_max;       // largest t ingested (t_now of the expiry rule)
@@ -156,6 +158,9 @@ struct WordSet {
   uint32_t* p[N];
   uint32_t v[N];
   int n = 0;
+  // optional, applied before the stores: *fold_dst |= *fold_src (error bits carried over)
+  uint32_t* fold_dst = nullptr;
+  const uint32_t* fold_src = nullptr;
   void add(uint32_t* ptr, uint32_t val) {
     p[n] = ptr;
     v[n] = val;

@@ -37,7 +37,7 @@ def test_library_exports_every_declared_symbol(gg):
 def test_struct_layouts_match_header(gg):
     # sizes the header implies on LP64
     assert ctypes.sizeof(gg.ggrid_graph) == 8 + 5 * 8
-    assert ctypes.sizeof(gg.ggrid_opts) == 4 + 4 + 4 + 4 + 8 + 4 * 4 + 8
+    assert ctypes.sizeof(gg.ggrid_opts) == 4 + 4 + 4 + 4 + 8 + 4 * 4 + 8 + 4 + 4  # async_ingest + tail padding
     assert ctypes.sizeof(gg.ggrid_stats_t) == 16 * 8 + 8 * 8 + 8 * 8 + 8 * 4 + 8
 
 

@@ -255,6 +255,55 @@ def test_garbage_collection_keeps_answers(gg):
     grid.close()
 
 
+def test_async_ingest_deferred_errors(gg):
+    """opts.async_ingest: ggrid_ingest returns without a host round trip; a bad batch is still
+    rejected whole on the device and its EINVAL surfaces once, at the next ggrid_sync (or the
+    next ggrid_ingest); answers are the oracle's on the accepted batches."""
+    g = synth.lattice_graph(8, 8, 1, 4)
+    grid = gg.GGrid(g, 16, max_objects=32, max_k=8, async_ingest=True)
+    walk = synth.RandomWalk(g, 20, inject=True)
+    good = [walk.ticks(2)]
+    grid.ingest(good[0])
+    bad = np.concatenate([good[0][:5], np.array([[1, len(g["src"]), 0, 0]], np.uint32)])
+    grid.ingest(bad)  # accepted for now: validated on the device
+    q = synth.queries(g, 10)
+    _assert_same(grid.knn(q, 4), _oracle(g, good[0], q, 4), "rejected batch not visible")
+    with pytest.raises(gg.GGridError) as e:
+        grid.sync()
+    assert e.value.rc == gg.GGRID_EINVAL
+    grid.sync()  # reported once
+    # the next ingest reports a deferred error instead of the sync
+    grid.ingest(np.array([[40, 0, 0, 0]], np.uint32))
+    grid.knn(q, 4)  # (syncs: the mirror now holds the rejection)
+    with pytest.raises(gg.GGridError) as e:
+        grid.ingest(walk.ticks(1))
+    assert e.value.rc == gg.GGRID_EINVAL
+    good.append(walk.ticks(2))
+    grid.ingest(good[-1])
+    grid.sync()
+    _assert_same(grid.knn(q, 4), _oracle(g, np.concatenate(good), q, 4), "after deferred errors")
+    grid.close()
+
+
+def test_async_ingest_streams_and_gc(gg):
+    """Asynchronous ingest across many batches with no sync in between, under arena pressure
+    (garbage collection must see the pending batches' records): bit-exact at every query."""
+    g = synth.table_ii_graph("NY", scale=0.03)
+    walk = synth.RandomWalk(g, 800, inject=True)
+    grid = gg.GGrid(g, 128, max_objects=1024, log_capacity=12_000, async_ingest=True)
+    hist = []
+    for r in range(10):
+        for _ in range(3):  # several batches queued back to back
+            u = walk.ticks(1)
+            hist.append(u)
+            grid.ingest(u)
+        q = synth.queries(g, 50, seed=70 + r)
+        _assert_same(grid.knn(q, 6), _oracle(g, np.concatenate(hist), q, 6), f"round {r}")
+    grid.sync()
+    assert grid.stats()["gc_runs"] > 0
+    grid.close()
+
+
 # ----------------------------------------------------------------- BASELINE-scale configs
 def test_c1_ny_bit_exact(gg):
     """configs[1] at full size: NY-shaped graph, 10k objects, 1M cached updates, k=10;
