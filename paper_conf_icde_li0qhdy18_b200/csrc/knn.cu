@@ -8,10 +8,11 @@
 // here.  This kernel computes the same exact answer with one bounded, label-correcting
 // delta-stepping expansion per query that never leaves the GPU:
 //
-//   * D lives in a per-warp shared-memory open-addressing table keyed by vertex; one
-//     64-bit word (v<<32 | dist) so relaxation is a single atomicMin (same key => min on
-//     the distance), issued only when it improves.  Seeds follow reading R1 (d=0 ->
-//     D[src]=0, else D[dst]=w-d).
+//   * D lives in a per-warp shared-memory open-addressing table keyed by vertex: a u32 key
+//     array (a new vertex is claimed with a 32-bit atomicCAS) beside a u32 distance array
+//     (relaxation = native 32-bit shared atomicMin, issued only when it improves; a 64-bit
+//     (v<<32 | d) word would need a CAS loop: shared memory has no 64-bit min).  Seeds
+//     follow reading R1 (d=0 -> D[src]=0, else D[dst]=w-d).
 //   * Each round walks the frontier in chunks of 32; the vertices whose D lies in the bucket
 //     [m, m+delta) (m = frontier minimum) are expanded 8 per window, lane = (vertex, slot):
 //     each lane reads one arc of its vertex's 32-byte inline adjacency record (graph grid,
@@ -47,7 +48,8 @@ struct Caps {
 
 // byte layout of one warp's working memory
 struct WarpMem {
-  unsigned long long* dtab;  // H: (v<<32 | D)
+  uint32_t* key;             // H: vertex of the slot (EMPTY32 = free)
+  uint32_t* dist;            // H: its tentative distance D
   unsigned long long* cand;  // C: (slot<<32 | offset); at the end (dist<<32 | obj)
   uint32_t* cobj;            // C: object ids
   uint32_t* front0;          // F
@@ -64,9 +66,10 @@ __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   WarpMem m;
-  m.dtab = reinterpret_cast<unsigned long long*>(base);
-  m.cand = m.dtab + c.H;
+  m.cand = reinterpret_cast<unsigned long long*>(base);
   uint32_t* p = reinterpret_cast<uint32_t*>(m.cand + c.C);
+  m.key = p; p += c.H;
+  m.dist = p; p += c.H;
   m.cobj = p; p += c.C;
   m.front0 = p; p += c.F;
   m.front1 = p; p += c.F;
@@ -80,31 +83,27 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
 // clustered, so low-bit or identity hashing makes long probe runs
 __device__ __forceinline__ uint32_t vhash(uint32_t v, uint32_t H) { return __umulhi(v * 2654435761u, H); }
 
+constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^32-1)
+
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
-__device__ __forceinline__ int tab_relax(unsigned long long* dtab, uint32_t H, uint32_t v,
-                                         uint32_t d, bool& improved) {
-  const unsigned long long nv = ((unsigned long long)v << 32) | d;
+__device__ __forceinline__ int tab_relax(const WarpMem& m, uint32_t H, uint32_t v, uint32_t d,
+                                         bool& improved) {
   uint32_t sl = vhash(v, H);
-  volatile unsigned long long* vt = dtab;
+  volatile uint32_t* vk = m.key;
 #pragma unroll 1
   for (int p = 0; p < MAXP; ++p) {
-    unsigned long long cur = vt[sl];
-    if ((uint32_t)(cur >> 32) == v) {
-      if ((uint32_t)cur <= d) {  // not an improvement (e.g. the twin arc back): no atomic
+    uint32_t cur = vk[sl];
+    if (cur == EMPTY32) {
+      cur = atomicCAS(&m.key[sl], EMPTY32, v);
+      if (cur == EMPTY32) cur = v;  // claimed (its distance is still INF)
+    }
+    if (cur == v) {
+      if (((volatile uint32_t*)m.dist)[sl] <= d) {  // not an improvement (e.g. the twin arc back)
         improved = false;
         return (int)sl;
       }
-      const unsigned long long old = atomicMin(&dtab[sl], nv);
-      improved = (uint32_t)old > d;
+      improved = atomicMin(&m.dist[sl], d) > d;
       return (int)sl;
-    }
-    if (cur == EMPTY64) {
-      const unsigned long long old = atomicCAS(&dtab[sl], EMPTY64, nv);
-      if (old == EMPTY64) {
-        improved = true;
-        return (int)sl;
-      }
-      if ((uint32_t)(old >> 32) == v) continue;  // same vertex inserted meanwhile: re-read
     }
     sl = sl + 1 == H ? 0 : sl + 1;
   }
@@ -162,7 +161,7 @@ __device__ __forceinline__ unsigned long long cand_dist(const WarpMem& m, uint32
   const unsigned long long a = m.cand[i];
   const uint32_t slot = (uint32_t)(a >> 32), off = (uint32_t)a;
   if (slot == SPECIAL) return off;
-  return (unsigned long long)(uint32_t)m.dtab[slot] + off;
+  return (unsigned long long)m.dist[slot] + off;
 }
 
 // Append one ballot's worth of candidates (false: capacity exceeded)
@@ -185,7 +184,7 @@ __device__ __forceinline__ bool cand_push(const WarpMem& m, uint32_t& nc, uint32
 __device__ void request_lookahead(const QParams& P, const WarpMem& m, const uint32_t* front,
                                   uint32_t nf, int lane) {
   for (uint32_t i = lane; i < nf; i += 32) {
-    const uint32_t v = (uint32_t)(m.dtab[front[i]] >> 32);
+    const uint32_t v = m.key[front[i]];
     request_flush(P.s, cellof(P.g, v), P.epoch);
   }
 }
@@ -199,7 +198,10 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   const uint32_t k = P.k;
   const unsigned lt = lanemask_lt();
 
-  for (uint32_t i = lane; i < cp.H; i += 32) m.dtab[i] = EMPTY64;
+  for (uint32_t i = lane; i < cp.H; i += 32) {
+    m.key[i] = EMPTY32;
+    m.dist[i] = INF;
+  }
   for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) m.fin[i] = 0;
   for (uint32_t i = lane; i < (cp.H + 3) / 4; i += 32) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
   __syncwarp();
@@ -230,7 +232,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   uint32_t nf = 1, nc = 0;
   if (lane == 0) {
     bool imp;
-    const int sl = tab_relax(m.dtab, H, seed_v, seed_d, imp);
+    const int sl = tab_relax(m, H, seed_v, seed_d, imp);
     front[0] = (uint32_t)sl;
     m.fin[sl >> 5] |= 1u << (sl & 31);
   }
@@ -290,13 +292,13 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
     for (uint32_t b0 = 0; b0 < nf; b0 += 32) {
       const uint32_t i = b0 + lane;
       const uint32_t sl = i < nf ? front[i] : NONE;
-      const unsigned long long ent = sl != NONE ? m.dtab[sl] : EMPTY64;
-      const bool a = sl != NONE && (uint32_t)ent < bhi;
+      const uint32_t ent = sl != NONE ? m.dist[sl] : INF;
+      const bool a = sl != NONE && ent < bhi;
       const bool r = sl != NONE && !a;
       const unsigned rm = __ballot_sync(FULL, r);
       if (r) {
         nfront[nn + __popc(rm & lt)] = sl;
-        mn = min(mn, (uint32_t)ent);
+        mn = min(mn, ent);
       }
       nn += __popc(rm);
       const unsigned am = __ballot_sync(FULL, a);
@@ -326,7 +328,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       w.v0 = make_uint2(0, 0);
       if (w.vv) {
         w.vslot = m.act[vi];
-        w.u = (uint32_t)(m.dtab[w.vslot] >> 32);
+        w.u = m.key[w.vslot];
         w.arc = g.vadj[(size_t)w.u * 4 + s4];
         if (s4 == 0) {
           w.hcell = cellof(g, w.u);
@@ -344,7 +346,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       const Win nxt = load_win(w0 + 8);  // (all lanes out of range past the last window)
       // D re-read now: an earlier window may have improved it (the frontier bit was cleared
       // at partition, so such an improvement also re-queued the vertex)
-      const uint32_t du = cur.vv ? (uint32_t)m.dtab[cur.vslot] : INF;
+      const uint32_t du = cur.vv ? m.dist[cur.vslot] : INF;
       bool has = false, ovf = false;
       uint32_t nslot = 0;
       auto relax = [&](uint32_t dst, uint32_t w) {
@@ -352,7 +354,7 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
         const unsigned long long nd = (unsigned long long)du + w;
         if (nd >= INF) return;
         bool imp;
-        const int rr = tab_relax(m.dtab, H, dst, (uint32_t)nd, imp);
+        const int rr = tab_relax(m, H, dst, (uint32_t)nd, imp);
         if (rr < 0) {
           ovf = true;
         } else if (imp) {
@@ -565,7 +567,10 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
   const uint32_t H = cp.H;
   const uint32_t k = P.k;
 
-  for (uint32_t i = tid; i < H; i += T) m.dtab[i] = EMPTY64;
+  for (uint32_t i = tid; i < H; i += T) {
+    m.key[i] = EMPTY32;
+    m.dist[i] = INF;
+  }
   for (uint32_t i = tid; i < (H + 31) / 32; i += T) m.fin[i] = 0;
   for (uint32_t i = tid; i < (H + 3) / 4; i += T) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
   if (tid == 0) {
@@ -590,7 +595,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
     const uint32_t seed_v = q.y == 0 ? ei.x : g.edst[q.x];
     const uint32_t seed_d = q.y == 0 ? 0u : ei.y - q.y;
     bool imp;
-    const int sl = tab_relax(m.dtab, H, seed_v, seed_d, imp);
+    const int sl = tab_relax(m, H, seed_v, seed_d, imp);
     m.front0[0] = (uint32_t)sl;
     m.fin[sl >> 5] |= 1u << (sl & 31);
     sh.nf = 1;
@@ -627,7 +632,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
     ++c_iter;
     const uint32_t nf = sh.nf;
     uint32_t ml = INF;
-    for (uint32_t i = tid; i < nf; i += T) ml = min(ml, (uint32_t)m.dtab[front[i]]);
+    for (uint32_t i = tid; i < nf; i += T) ml = min(ml, m.dist[front[i]]);
     const uint32_t blo = block_min<W>(ml, sh);
     if (nf == 0 || blo > lim) break;
     const uint32_t nc0 = sh.nc;
@@ -645,7 +650,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
     __syncthreads();
     for (uint32_t i = tid; i < nf; i += T) {
       const uint32_t sl = front[i];
-      if ((uint32_t)m.dtab[sl] < bhi) {
+      if (m.dist[sl] < bhi) {
         m.act[atomicAdd(&sh.na, 1u)] = sl;  // (act has F entries: na <= nf <= F)
         atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
       } else {
@@ -660,8 +665,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
       const uint32_t vi = w0 + (tid >> 2), s4 = tid & 3;
       if (vi < na) {
         const uint32_t vslot = m.act[vi];
-        const unsigned long long e2 = m.dtab[vslot];  // D re-read after the frontier bit
-        const uint32_t u = (uint32_t)(e2 >> 32), du = (uint32_t)e2;
+        const uint32_t u = m.key[vslot], du = m.dist[vslot];  // D re-read after the frontier bit
         const uint2 arc = g.vadj[(size_t)u * 4 + s4];
         bool harv = false;
         uint32_t hcell = 0, hd = NONE;
@@ -679,7 +683,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
           const unsigned long long nd = (unsigned long long)du + w;
           if (nd >= INF) return;
           bool imp;
-          const int rr = tab_relax(m.dtab, H, dst, (uint32_t)nd, imp);
+          const int rr = tab_relax(m, H, dst, (uint32_t)nd, imp);
           if (rr < 0) {
             atomicOr(&sh.flags, FL_OVF);
           } else if (imp) {
@@ -735,7 +739,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
       if (fl & FL_OVF) return OVERFLOW;
       if (fl & FL_RETRY) {
         for (uint32_t i = tid; i < nf; i += T)
-          request_flush(s, cellof(g, (uint32_t)(m.dtab[front[i]] >> 32)), P.epoch);
+          request_flush(s, cellof(g, m.key[front[i]]), P.epoch);
         return RETRY;
       }
     }
