@@ -315,6 +315,8 @@ def run_ours(args, cfg_name):
                       "alg_bytes_per_step": v[1] / n_break,
                       "gbs": (v[1] / (v[0] / 1e3) / 1e9) if v[0] > 0 else 0.0} for n, v in kern.items()}
     per_kernel["source"] = f"{n_break} breakdown steps after the timed ones, every launch timed"
+    per_kernel["expand"]["level0_ms_per_step"] = sb1["kernel_ms"]["expand"] / n_break
+    per_kernel["expand"]["higher_levels_ms_per_step"] = sb1["kernel_ms"]["expand_big"] / n_break
     traffic = None
     tp = os.path.join(ROOT, "profiles", f"traffic_{cfg_name}.json")
     if os.path.exists(tp):
@@ -413,7 +415,9 @@ def run_ours(args, cfg_name):
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(st1["launches"]), "clocks": clk,
                 "knn_rounds_per_step": (st1["knn_rounds"] - st0["knn_rounds"]) / K,
                 "remote_requests_per_step_rank0": remote_requests / K if shard else None,
-                "expand_work_per_query": {n: v / (Q * K) for n, v in dx.items()}, "delta": st1["delta"]}
+                "expand_work_per_query": {n: v / (Q * K) for n, v in dx.items()}, "delta": st1["delta"],
+                "expand_promotions_per_step": (st1["expand_promotions"] - st0["expand_promotions"]) / K,
+                "expand_retries_per_step": (st1["expand_retries"] - st0["expand_retries"]) / K}
         print(json.dumps(line), flush=True)
     grid.close()
     if world > 1:

@@ -138,6 +138,8 @@ typedef struct ggrid_stats_t {
   uint32_t t_delta;          /* opts.t_delta                                          */
   uint32_t t_now;            /* largest t ingested so far                             */
   uint64_t records_expired;  /* cached records dropped unread by t_delta expiry       */
+  uint64_t expand_promotions;/* query runs that overflowed a capacity level (rerun on the next) */
+  uint64_t expand_retries;   /* query runs stopped by a cell with cached updates (rerun after its flush) */
 } ggrid_stats_t;
 
 /* Build the index (graph grid, P@11423-15818; object table P@15869; message lists

@@ -731,6 +731,10 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
   std::vector<uint32_t> n_in(L, 0);
   n_in[lvl0] = n_q;
+  // the level above the starting one runs in the same round, right behind it, on the queries
+  // the starting level promotes (counted on the device): an overflow costs no extra round
+  // (a host round trip).  Deeper promotions wait for the next round.
+  const int chain = lvl0 + 1 < L - 1 ? lvl0 + 1 : -1;
   std::vector<const uint32_t*> in_list(L, nullptr);
   int cur = 0;
   uint32_t flush_begin = 0;
@@ -740,14 +744,16 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
     const uint64_t seeded = (uint64_t)n_q * (h->seed_neighbors ? h->max_cell_degree + 1 : 2);
     RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin, 0,
                          round == 0 ? (uint32_t)std::min<uint64_t>(seeded, 1u << 30) : 0));
-    if (round > 0) {  // round 0 was reset with the rest at the start
+    if (round > 0) {  // round 0 was reset with the rest at the start (n_cur[chain] = n_in = 0)
       WordSet ws;
       ws.zero_range(h->d_status->n_next, EXPAND_LEVELS);
       ws.zero_range(h->d_status->expand_work, EXPAND_LEVELS);
+      if (chain >= 0) ws.add(&h->d_status->n_cur[chain], n_in[chain]);
       RC(h->set_words(ws));
     }
     for (int lvl = 0; lvl < L; ++lvl) {
-      if (!n_in[lvl]) continue;
+      const bool chained = lvl == chain && n_in[lvl0] > 0;
+      if (!n_in[lvl] && !chained) continue;
       void* scratch = nullptr;
       uint32_t sw = 0;
       if (lvl == L - 1) {
@@ -758,13 +764,18 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
         scratch = h->l2_scratch.p;
       }
       uint32_t* retry = list(cur ^ 1, lvl);
-      uint32_t* promote = lvl + 1 < L ? list(cur ^ 1, lvl + 1) : nullptr;
-      const uint32_t* qlist = in_list[lvl];
-      const uint32_t nn = n_in[lvl];
+      // promotions out of the starting level go to the chained level's list of this round
+      // (after its own n_in entries), others to the next round
+      const bool to_chain = lvl == lvl0 && chain >= 0;
+      uint32_t* promote = lvl + 1 < L ? list(to_chain ? cur : cur ^ 1, lvl + 1) : nullptr;
+      uint32_t* promote_count = to_chain ? &h->d_status->n_cur[chain] : &h->d_status->n_next[std::min(lvl + 1, L - 1)];
+      const uint32_t* qlist = chained ? list(cur, lvl) : in_list[lvl];
+      const uint32_t nn = chained ? n_q : n_in[lvl];
+      const uint32_t* n_dev = chained ? &h->d_status->n_cur[chain] : nullptr;
       const int kind = lvl == 0 ? GGRID_K_EXPAND : GGRID_K_EXPAND_BIG;
       h->launch(kind, [&] {
-        launch_expand(lvl, d_q, qlist, nn, k, g, s, epoch, retry, promote, d_oo, d_od, d_bound, d_remote,
-                      scratch, sw, h->sm_count, st);
+        launch_expand(lvl, d_q, qlist, nn, n_dev, k, g, s, epoch, retry, promote, promote_count, d_oo, d_od,
+                      d_bound, d_remote, scratch, sw, h->sm_count, st);
       });
     }
     RC(h->sync());
@@ -1046,6 +1057,8 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
   s.t_delta = h->t_delta;
   s.t_now = h->h_status->t_max;
   s.records_expired = h->h_status->records_expired;
+  s.expand_promotions = h->h_status->ex_promoted;
+  s.expand_retries = h->h_status->ex_retried;
   *out = s;
   return GGRID_OK;
 }

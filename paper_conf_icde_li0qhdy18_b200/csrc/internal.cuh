@@ -40,6 +40,7 @@ struct DevStatus {
   unsigned long long cells_flushed;
   unsigned long long ex_iters, ex_vertices, ex_arcs, ex_harvested, ex_objects;  // expansion work
   unsigned long long records_expired;  // dropped unread by t_delta expiry
+  unsigned long long ex_promoted, ex_retried;  // expansion outcomes: capacity overflow / dirty cell
   unsigned int ext_top;     // next free extent
   unsigned int err;         // ErrBits of the current knn / flush / gc call
   unsigned int ingest_err;  // ErrBits of the current ingest batch (classify / alloc / scatter)
@@ -52,6 +53,7 @@ struct DevStatus {
   unsigned int n_next[EXPAND_LEVELS];   // per expansion level: queries queued for the next round
   unsigned int flush_end;   // n_flush as seen by the last flush launch
   unsigned int expand_work[EXPAND_LEVELS];  // per-level dynamic work counters of the expand launches
+  unsigned int n_cur[EXPAND_LEVELS];  // per level: queries of the current round (chained level)
   unsigned int round_end;   // (marks the end of the per-round reset region)
 };
 
@@ -212,9 +214,11 @@ __device__ __forceinline__ uint2 vobj_valid(uint2 vo, uint2 comp) {
 // bound (nullable): per-query inclusive distance limit (objects farther are not returned and
 // the search stops beyond it); remote (nullable): per-query bitmask of the ranks owning cells
 // the search expanded into (sharded mode)
-void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
-                   const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
-                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist,
+// n_dev (nullable): the query count is read on the device (a level chained behind the level
+// below in the same round); promote_count: the counter that indexes promote_list.
+void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, const uint32_t* n_dev,
+                   uint32_t k, const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
+                   uint32_t* promote_list, uint32_t* promote_count, uint32_t* out_obj, uint32_t* out_dist,
                    const uint32_t* bound, unsigned long long* remote, void* scratch,
                    uint32_t scratch_warps, int sm_count, cudaStream_t st);
 // prior-art comparison path (csrc/prior_art.cu)

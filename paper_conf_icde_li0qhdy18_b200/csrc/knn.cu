@@ -141,12 +141,14 @@ struct QParams {
   const uint2* q;
   const uint32_t* qlist;
   uint32_t n;
+  const uint32_t* n_dev;    // (non-null: the count is read on the device at kernel start)
   uint32_t k;
   uint32_t epoch;
   int level;
   int last_level;
   uint32_t* retry_list;     // same level, next round
-  uint32_t* promote_list;   // next level, next round
+  uint32_t* promote_list;   // next level (this round when chained, else the next round)
+  uint32_t* promote_count;  // its counter
   uint32_t* out_obj;
   uint32_t* out_dist;
   const uint32_t* bound;          // per-query inclusive distance limit, or null
@@ -186,6 +188,20 @@ __device__ void request_lookahead(const QParams& P, const WarpMem& m, const uint
   for (uint32_t i = lane; i < nf; i += 32) {
     const uint32_t v = m.key[front[i]];
     request_flush(P.s, cellof(P.g, v), P.epoch);
+  }
+}
+
+// a query not answered at this level: retried here next round (a needed cell had cached
+// updates), or promoted to the next level (capacity overflow)
+__device__ void finish_undone(const QParams& P, uint32_t qi, int r) {
+  if (r == RETRY) {
+    atomicAdd(&P.s.st->ex_retried, 1ull);
+    P.retry_list[atomicAdd(&P.s.st->n_next[P.level], 1u)] = qi;
+  } else if (P.level < P.last_level) {
+    atomicAdd(&P.s.st->ex_promoted, 1ull);
+    P.promote_list[atomicAdd(P.promote_count, 1u)] = qi;
+  } else {
+    atomicOr(&P.s.st->err, (unsigned)ERR_FAIL);
   }
 }
 
@@ -474,22 +490,16 @@ __global__ void k_expand(QParams P) {
   const uint32_t gw = blockIdx.x * P.warps_per_cta + warp;
   unsigned char* base = P.scratch ? P.scratch + (size_t)gw * wbytes : smem_raw + (size_t)warp * wbytes;
   const WarpMem m = carve(base, P.caps);
+  const uint32_t n = P.n_dev ? *(volatile const uint32_t*)P.n_dev : P.n;
+  if (n == 0) return;  // (a chained level with nothing promoted: no contended work counter)
   for (;;) {  // persistent: queries fetched dynamically
     uint32_t li = 0;
     if (lane == 0) li = atomicAdd(&P.s.st->expand_work[P.level], 1u);
     li = __shfl_sync(0xffffffffu, li, 0);
-    if (li >= P.n) break;
+    if (li >= n) break;
     const uint32_t qi = P.qlist ? P.qlist[li] : li;
     const int r = run_query(P, m, qi, lane);
-    if (lane == 0 && r != DONE) {
-      if (r == RETRY) {
-        P.retry_list[atomicAdd(&P.s.st->n_next[P.level], 1u)] = qi;
-      } else if (P.level < P.last_level) {
-        P.promote_list[atomicAdd(&P.s.st->n_next[P.level + 1], 1u)] = qi;
-      } else {
-        atomicOr(&P.s.st->err, (unsigned)ERR_FAIL);
-      }
-    }
+    if (lane == 0 && r != DONE) finish_undone(P, qi, r);
     __syncwarp();
   }
 }
@@ -798,23 +808,17 @@ __global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
   __shared__ CtaShared sh;
   __shared__ uint32_t qslot;
   const WarpMem m = carve(smem_raw, P.caps);
+  const uint32_t n = P.n_dev ? *(volatile const uint32_t*)P.n_dev : P.n;
+  if (n == 0) return;  // (a chained level with nothing promoted: no contended work counter)
   for (;;) {  // persistent: queries fetched dynamically
     if (threadIdx.x == 0) qslot = atomicAdd(&P.s.st->expand_work[P.level], 1u);
     __syncthreads();
     const uint32_t li = qslot;
     __syncthreads();
-    if (li >= P.n) break;
+    if (li >= n) break;
     const uint32_t qi = P.qlist ? P.qlist[li] : li;
     const int r = run_query_cta<CTA_W>(P, m, sh, qi);
-    if (threadIdx.x == 0 && r != DONE) {
-      if (r == RETRY) {
-        P.retry_list[atomicAdd(&P.s.st->n_next[P.level], 1u)] = qi;
-      } else if (P.level < P.last_level) {
-        P.promote_list[atomicAdd(&P.s.st->n_next[P.level + 1], 1u)] = qi;
-      } else {
-        atomicOr(&P.s.st->err, (unsigned)ERR_FAIL);
-      }
-    }
+    if (threadIdx.x == 0 && r != DONE) finish_undone(P, qi, r);
     __syncthreads();
   }
 }
@@ -829,7 +833,7 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 #define GG_H0 1024  // level-0 vertex table (experiment hook: -DGG_H0=..., -DGG_F0=...)
 #endif
 #ifndef GG_F0
-#define GG_F0 128
+#define GG_F0 96
 #endif
 const Caps kCaps[NLEVELS - 1] = {
     {GG_H0, GG_F0, 64}, {2048, 512, 256}, {4096, 1024, 256}, {8192, 2048, 512}, {16384, 4096, 2048}};
@@ -857,24 +861,26 @@ size_t expand_warp_bytes(int level, uint32_t V) {
   return (warpmem_bytes(c) + 15) & ~size_t(15);
 }
 
-void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, uint32_t k,
-                   const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
-                   uint32_t* promote_list, uint32_t* out_obj, uint32_t* out_dist,
+void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, const uint32_t* n_dev,
+                   uint32_t k, const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
+                   uint32_t* promote_list, uint32_t* promote_count, uint32_t* out_obj, uint32_t* out_dist,
                    const uint32_t* bound, unsigned long long* remote, void* scratch,
                    uint32_t scratch_warps, int sm_count, cudaStream_t st) {
-  if (n == 0) return;
+  if (n == 0) return;  // (with n_dev: an upper bound of the device count)
   QParams P;
   P.g = g;
   P.s = s;
   P.q = q;
   P.qlist = qlist;
   P.n = n;
+  P.n_dev = n_dev;
   P.k = k;
   P.epoch = epoch;
   P.level = level;
   P.last_level = NLEVELS - 1;
   P.retry_list = retry_list;
   P.promote_list = promote_list;
+  P.promote_count = promote_count;
   P.out_obj = out_obj;
   P.out_dist = out_dist;
   P.bound = bound;
