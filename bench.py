@@ -358,6 +358,15 @@ def run_ours(args, cfg_name):
         u, q = step_inputs(10_000 + s)
         hus.append(torch.from_numpy(u.view(np.int32)).pin_memory())
         hqs.append(torch.from_numpy(q.view(np.int32)).pin_memory())
+    # one untimed DMA from every pinned input buffer (a producer would reuse a fixed set of
+    # pinned buffers; the first DMA from a freshly pinned allocation is measurably slower)
+    scratch_u = torch.empty_like(hus[0], device="cuda")
+    scratch_q = torch.empty_like(hqs[0], device="cuda")
+    for hu, hq in zip(hus, hqs):
+        scratch_u.copy_(hu)
+        scratch_q.copy_(hq)
+    torch.cuda.synchronize()
+    del scratch_u, scratch_q
     for s in range(w_e2e):  # warm-up steps
         grid.ingest_stage(hus[s])
         grid.ingest_commit()
@@ -372,12 +381,19 @@ def run_ours(args, cfg_name):
         trace = profile(activities=[ProfilerActivity.CUDA, ProfilerActivity.CPU])
         trace.__enter__()
     t0 = time.perf_counter()
+    tst = []
     grid.ingest_stage(hus[1])
     for s in range(1, n_e2e + 1):
         grid.ingest_commit()
         if s + 1 <= n_e2e:
             grid.ingest_stage(hus[s + 1])  # overlaps the queries below
         e2e_knn(hqs[s])
+        tst.append(time.perf_counter())
+    if os.environ.get("BENCH_E2E_DEBUG"):
+        print("e2e step ms:", [round(1e3 * (b - a), 3) for a, b in zip([t0] + tst[:-1], tst)], file=sys.stderr)
+        sd = grid.stats()
+        print("e2e stats:", {k: sd[k] for k in ("gc_runs", "knn_rounds", "knn_calls", "expand_promotions",
+                                                "expand_retries", "arena_used", "arena_capacity")}, file=sys.stderr)
     grid.sync()  # (the last step's answers were read back inside knn already)
     e2e_total = time.perf_counter() - t0
     if trace is not None:
