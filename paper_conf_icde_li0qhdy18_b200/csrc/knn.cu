@@ -90,25 +90,27 @@ __device__ __forceinline__ int tab_relax(const WarpMem& m, uint32_t H, uint32_t 
                                          bool& improved) {
   uint32_t sl = vhash(v, H);
   volatile uint32_t* vk = m.key;
+  // find or claim v's slot (one exit; the distance update below is out of the probe loop)
 #pragma unroll 1
-  for (int p = 0; p < MAXP; ++p) {
+  for (int p = 0;; ++p) {
     uint32_t cur = vk[sl];
     if (cur == EMPTY32) {
       cur = atomicCAS(&m.key[sl], EMPTY32, v);
       if (cur == EMPTY32) cur = v;  // claimed (its distance is still INF)
     }
-    if (cur == v) {
-      if (((volatile uint32_t*)m.dist)[sl] <= d) {  // not an improvement (e.g. the twin arc back)
-        improved = false;
-        return (int)sl;
-      }
-      improved = atomicMin(&m.dist[sl], d) > d;
-      return (int)sl;
+    if (cur == v) break;
+    if (p + 1 == MAXP) {
+      improved = false;
+      return -1;
     }
     sl = sl + 1 == H ? 0 : sl + 1;
   }
-  improved = false;
-  return -1;
+  if (((volatile uint32_t*)m.dist)[sl] <= d) {  // not an improvement (e.g. the twin arc back)
+    improved = false;
+  } else {
+    improved = atomicMin(&m.dist[sl], d) > d;
+  }
+  return (int)sl;
 }
 
 // warp bitonic sort of a[0..n) ascending (n padded to a power of two <= cap)
@@ -384,13 +386,20 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
       };
       const bool overflow_arcs = cur.arc.y == WMAX;
       if (cur.arc.y != 0 && !overflow_arcs) relax(cur.arc.x, cur.arc.y);
-      if (__any_sync(FULL, ovf)) return OVERFLOW;
+      // harvest the objects of the vertices expanded for the first time; a cell with cached
+      // updates must be cleaned first (lazy flush): request it and retry the query
+      const bool dirty = cur.harv && cur.hd != NONE;
+      const uint2 vo = cur.harv ? vobj_valid(cur.v0, cur.cc) : make_uint2(0, 0);
+      // one warp vote for every rare event of the window
+      const uint32_t ev = __reduce_or_sync(FULL, (ovf ? 1u : 0u) | (overflow_arcs ? 2u : 0u) |
+                                                     (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
+      if (ev & 1u) return OVERFLOW;
       unsigned hm = __ballot_sync(FULL, has);
       if (nn + __popc(hm) > cp.F) return OVERFLOW;
       if (has) nfront[nn + __popc(hm & lt)] = nslot;
       nn += __popc(hm);
       // vertices with more than 4 arcs: the rest live in the CSR (rare on road graphs)
-      if (__any_sync(FULL, overflow_arcs)) {
+      if (ev & 2u) {
         uint32_t a0 = 0, a1 = 0;
         if (overflow_arcs) {
           a0 = g.rowptr[cur.u] + 3;
@@ -411,11 +420,8 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
           nn += __popc(hm);
         }
       }
-      // harvest the objects of the vertices expanded for the first time; a cell with cached
-      // updates must be cleaned first (lazy flush): request it and retry the query
-      const bool dirty = cur.harv && cur.hd != NONE;
-      if (dirty) request_flush(s, cur.hcell, P.epoch);
-      if (__any_sync(FULL, dirty)) {
+      if (ev & 4u) {
+        if (dirty) request_flush(s, cur.hcell, P.epoch);
         request_lookahead(P, m, front, nf, lane);
         return RETRY;
       }
@@ -426,9 +432,8 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
         rmask |= ((unsigned long long)__reduce_or_sync(FULL, (uint32_t)(bm >> 32)) << 32) |
                  __reduce_or_sync(FULL, (uint32_t)bm);
       }
-      const uint2 vo = cur.harv ? vobj_valid(cur.v0, cur.cc) : make_uint2(0, 0);
-      const uint32_t most = __reduce_max_sync(FULL, vo.y);
-      if (most) {
+      if (ev & 8u) {
+        const uint32_t most = __reduce_max_sync(FULL, vo.y);
         c_objs += vo.y;
         for (uint32_t j = 0; j < most; ++j) {
           bool hc = false;
