@@ -207,7 +207,7 @@ __device__ void finish_undone(const QParams& P, uint32_t qi, int r) {
   }
 }
 
-__device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int lane) {
+__device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int lane) {
   const unsigned FULL = 0xffffffffu;
   const DevGraph& g = P.g;
   const DevState& s = P.s;
@@ -487,13 +487,18 @@ __device__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int la
   return DONE;
 }
 
+// SMEM: the working memory is this CTA's shared memory (levels 0..L-2), else per-warp global
+// scratch (the last level).  Two instantiations, so that every table access of the shared one
+// compiles to LDS/STS/ATOMS with 32-bit addresses (one pointer that may be either space makes
+// them generic 64-bit LD/ST/ATOM, measured ~10% slower overall).
+template <bool SMEM>
 __global__ void k_expand(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
   const uint32_t warp = threadIdx.x >> 5;
   const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
   const uint32_t gw = blockIdx.x * P.warps_per_cta + warp;
-  unsigned char* base = P.scratch ? P.scratch + (size_t)gw * wbytes : smem_raw + (size_t)warp * wbytes;
+  unsigned char* base = SMEM ? smem_raw + (size_t)warp * wbytes : P.scratch + (size_t)gw * wbytes;
   const WarpMem m = carve(base, P.caps);
   const uint32_t n = P.n_dev ? *(volatile const uint32_t*)P.n_dev : P.n;
   if (n == 0) return;  // (a chained level with nothing promoted: no contended work counter)
@@ -894,7 +899,7 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
   P.warps_per_cta = 1;
   const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
   if (!g_attr_set) {
-    cudaFuncSetAttribute(k_expand, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     g_attr_set = true;
   }
   // CTA-per-query for the big shared-memory levels, and for small batches at any of them
@@ -922,14 +927,14 @@ void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n,
     const int smem = (int)wbytes;
     if (!g_blocks_per_sm[level]) {
       int b = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand, 32, smem);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32, smem);
       g_blocks_per_sm[level] = b > 0 ? b : 1;
     }
     const uint32_t wave = (uint32_t)(sm_count * g_blocks_per_sm[level]);
-    k_expand<<<std::min<uint32_t>(n, wave), 32, smem, st>>>(P);
+    k_expand<true><<<std::min<uint32_t>(n, wave), 32, smem, st>>>(P);
   } else {
     P.scratch = static_cast<unsigned char*>(scratch);
-    k_expand<<<std::min<uint32_t>(n, std::max<uint32_t>(1, scratch_warps)), 32, 0, st>>>(P);
+    k_expand<false><<<std::min<uint32_t>(n, std::max<uint32_t>(1, scratch_warps)), 32, 0, st>>>(P);
   }
 }
 
