@@ -170,6 +170,18 @@ int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n);
 int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n);
 int ggrid_ingest_commit(ggrid_t h);
 
+/* Pipelined queries, the same two-deep staging for query batches: ggrid_query_stage starts
+ * copying n_q queries (host or device pointer) into a device staging buffer on the copy
+ * stream, behind any batch staged before it, and returns at once (keep q untouched until the
+ * matching ggrid_knn_commit returns).  ggrid_knn_commit answers the oldest staged batch with
+ * the semantics and errors of ggrid_knn, and stores its size in *n_q (nullable).  A staged
+ * copy competes with nothing on the device: the seed kernel reads HBM instead of reading
+ * pinned host queries across PCIe while a staged update batch saturates the link.
+ * Errors: EINVAL (stage with both buffers staged, commit with none staged, k, null outputs),
+ * ENOMEM, ECUDA. */
+int ggrid_query_stage(ggrid_t h, const ggrid_query* q, uint32_t n_q);
+int ggrid_knn_commit(ggrid_t h, uint32_t k, uint32_t* out_obj, uint32_t* out_dist, uint32_t* n_q);
+
 /* Answer n_q kNN queries (Def. 1, P@9206-9761; Alg. 4-6, P@44429-52751) on the snapshot
  * of all updates ingested before the call.  Row i of out_obj / out_dist (n_q*k each,
  * host or device pointers) holds the k nearest objects in ascending (dist, obj) order,

@@ -23,7 +23,7 @@ GGRID_OK, GGRID_EINVAL, GGRID_ENOMEM, GGRID_ECUDA, GGRID_ENCCL, GGRID_EOVERFLOW 
 PAD = 0xFFFFFFFF
 KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "flush", "expand",
                 "expand_big", "other"]
-EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_sync", "ggrid_set_profile", "ggrid_flush_all",
+EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_query_stage", "ggrid_knn_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_sync", "ggrid_set_profile", "ggrid_flush_all",
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
            "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk",
            "ggrid_prior_art_clean", "ggrid_prior_art_bundle"]
@@ -83,6 +83,8 @@ def lib():
             "ggrid_ingest": ([P, P, u64], i32),
             "ggrid_ingest_stage": ([P, P, u64], i32),
             "ggrid_ingest_commit": ([P], i32),
+            "ggrid_query_stage": ([P, P, u32], i32),
+            "ggrid_knn_commit": ([P, u32, P, P, P], i32),
             "ggrid_knn": ([P, P, u32, u32, P, P], i32),
             "ggrid_free": ([P], i32),
             "ggrid_strerror": ([i32], ctypes.c_char_p),
@@ -185,6 +187,21 @@ def ggrid_ingest_stage(h, updates):
 
 def ggrid_ingest_commit(h):
     _check(lib().ggrid_ingest_commit(h), "ggrid_ingest_commit")
+
+
+def ggrid_query_stage(h, queries):
+    """Start the asynchronous copy of a query batch (keep `queries` alive until knn_commit)."""
+    q = _u32(queries)
+    _check(lib().ggrid_query_stage(h, _ptr(q), int(q.shape[0])), "ggrid_query_stage")
+    return q
+
+
+def ggrid_knn_commit(h, k: int, out_obj, out_dist):
+    """Answer the oldest staged query batch into out_obj / out_dist (preallocated, (n, k))."""
+    n = ctypes.c_uint32(0)
+    _check(lib().ggrid_knn_commit(h, int(k), _ptr(out_obj), _ptr(out_dist), ctypes.byref(n)),
+           "ggrid_knn_commit")
+    return out_obj, out_dist
 
 
 def ggrid_knn(h, queries, k: int, out_obj=None, out_dist=None):
@@ -325,6 +342,7 @@ class GGrid:
     def __init__(self, graph: dict, cell_size: int, **opts):
         self.n_vertices = int(graph["n_vertices"])
         self._staged = []
+        self._qstaged = []
         self.h = ggrid_build(graph, cell_size, **opts)
 
     def ingest(self, updates):
@@ -351,6 +369,16 @@ class GGrid:
 
     def knn(self, queries, k: int, out_obj=None, out_dist=None):
         return ggrid_knn(self.h, queries, k, out_obj, out_dist)
+
+    def query_stage(self, queries):
+        """Pipelined queries: copy now, answer at knn_commit."""
+        self._qstaged.append(ggrid_query_stage(self.h, queries))
+        return self
+
+    def knn_commit(self, k: int, out_obj, out_dist):
+        r = ggrid_knn_commit(self.h, k, out_obj, out_dist)
+        self._qstaged.pop(0)
+        return r
 
     def knn_ex(self, queries, k: int, bound=None, out_obj=None, out_dist=None, out_remote=None):
         return ggrid_knn_ex(self.h, queries, k, bound, out_obj, out_dist, out_remote)

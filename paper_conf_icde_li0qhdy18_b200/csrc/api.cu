@@ -131,7 +131,10 @@ struct ggrid_s {
   };
   Staged staged[2];
   int stage_head = 0, n_staged = 0;
+  Staged qstaged[2];  // staged query batches (ggrid_query_stage / ggrid_knn_commit)
+  int qstage_head = 0, n_qstaged = 0;
   cudaStream_t copy_stream = nullptr;
+  DBuf chain_ring;  // queries promoted into the chained level (NONE = not yet written)
   ggrid_stats_t stats{};
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending_ev;
   std::vector<cudaEvent_t> ev_pool;
@@ -163,13 +166,17 @@ struct ggrid_s {
   // every kernel launch goes through here: counted, and timed in profile mode
   template <class F>
   void launch(int kind, F&& f) {
+    launch_on(kind, stream, f);
+  }
+  template <class F>
+  void launch_on(int kind, cudaStream_t on, F&& f) {
     stats.launches++;
     stats.kernel_launches[kind]++;
     if (profile & (1u | (2u << kind))) {
       cudaEvent_t a = get_event(), b = get_event();
-      cudaEventRecord(a, stream);
+      cudaEventRecord(a, on);
       f();
-      cudaEventRecord(b, stream);
+      cudaEventRecord(b, on);
       pending_ev.push_back({kind, {a, b}});
     } else {
       f();
@@ -533,13 +540,14 @@ int ggrid_free(ggrid_t h) {
   for (DBuf* b : {&h->upd_stage, &h->tmp, &h->q_stage, &h->out_stage, &h->lists, &h->l2_scratch,
                   &h->dump_stage, &h->gc_buf, &h->misc, &h->flush_spill, &h->bound_stage,
                   &h->remote_stage, &h->merge_stage, &h->staged[0].buf,
-                  &h->staged[1].buf})
+                  &h->staged[1].buf, &h->qstaged[0].buf, &h->qstaged[1].buf, &h->chain_ring})
     b->release();
-  for (auto& sb : h->staged) {
-    if (sb.done) cudaEventDestroy(sb.done);
-    if (sb.consumed) cudaEventDestroy(sb.consumed);
+  for (ggrid_s::Staged* sb : {&h->staged[0], &h->staged[1], &h->qstaged[0], &h->qstaged[1]}) {
+    if (sb->done) cudaEventDestroy(sb->done);
+    if (sb->consumed) cudaEventDestroy(sb->consumed);
   }
   if (h->copy_stream) cudaStreamDestroy(h->copy_stream);
+
   for (auto& pe : h->pending_ev) {
     cudaEventDestroy(pe.second.first);
     cudaEventDestroy(pe.second.second);
@@ -611,26 +619,42 @@ int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
   return ingest_device(h, d_u, n);
 }
 
-int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n) {
-  if (!h || (n && !u) || h->n_staged == 2) return GGRID_EINVAL;
-  CK(cudaSetDevice(h->device));
-  ggrid_s::Staged& sb = h->staged[(h->stage_head + h->n_staged) & 1];
+// copy n records of `bytes_each` from src into the next free buffer of a two-deep staging
+// ring on the copy stream (the paper's pipelined transfer, P@45017-45625)
+static int stage_into(ggrid_t h, ggrid_s::Staged* ring, int head, int count, const void* src, uint64_t n,
+                      size_t bytes_each) {
+  ggrid_s::Staged& sb = ring[(head + count) & 1];
   if (!sb.done) CK(cudaEventCreateWithFlags(&sb.done, cudaEventDisableTiming));
   if (!sb.consumed) {
     CK(cudaEventCreateWithFlags(&sb.consumed, cudaEventDisableTiming));
     CK(cudaEventRecord(sb.consumed, h->stream));
   }
   sb.n = n;
-  // an asynchronous ingest of this buffer's previous batch may still be reading it
+  // the kernels of this buffer's previous batch may still be reading it
   CK(cudaStreamWaitEvent(h->copy_stream, sb.consumed, 0));
   if (n) {
     // both buffers grow together: a cudaMalloc in the middle of a running pipeline stalls it
-    RC(h->staged[0].buf.ensure(n * sizeof(uint4)));
-    RC(h->staged[1].buf.ensure(n * sizeof(uint4)));
-    CK(cudaMemcpyAsync(sb.buf.p, u, n * sizeof(uint4), cudaMemcpyDefault, h->copy_stream));
+    RC(ring[0].buf.ensure(n * bytes_each));
+    RC(ring[1].buf.ensure(n * bytes_each));
+    CK(cudaMemcpyAsync(sb.buf.p, src, n * bytes_each, cudaMemcpyDefault, h->copy_stream));
   }
   CK(cudaEventRecord(sb.done, h->copy_stream));
+  return GGRID_OK;
+}
+
+int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n) {
+  if (!h || (n && !u) || h->n_staged == 2) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  RC(stage_into(h, h->staged, h->stage_head, h->n_staged, u, n, sizeof(uint4)));
   h->n_staged++;
+  return GGRID_OK;
+}
+
+int ggrid_query_stage(ggrid_t h, const ggrid_query* q, uint32_t n_q) {
+  if (!h || (n_q && !q) || h->n_qstaged == 2) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  RC(stage_into(h, h->qstaged, h->qstage_head, h->n_qstaged, q, n_q, sizeof(uint2)));
+  h->n_qstaged++;
   return GGRID_OK;
 }
 
@@ -733,10 +757,19 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
   std::vector<uint32_t> n_in(L, 0);
   n_in[lvl0] = n_q;
-  // the level above the starting one runs in the same round, right behind it, on the queries
-  // the starting level promotes (counted on the device): an overflow costs no extra round
-  // (a host round trip).  Deeper promotions wait for the next round.
+  // The level above the starting one runs in the same round BESIDE it (a programmatic
+  // dependent launch on the same stream, on SM space the starting level leaves free): it takes
+  // the queries the starting level promotes as soon as they are written, so a rare overflow
+  // costs neither an extra round (a host round trip) nor a serial tail after the starting
+  // level.  Deeper promotions wait for the next round.
   const int chain = lvl0 + 1 < L - 1 ? lvl0 + 1 : -1;
+  if (chain >= 0) {
+    const size_t need = (size_t)n_q * 4;
+    if (h->chain_ring.n < need) {
+      RC(h->chain_ring.ensure(need));
+      CK(cudaMemsetAsync(h->chain_ring.p, 0xFF, h->chain_ring.n, st));  // all NONE
+    }
+  }
   std::vector<const uint32_t*> in_list(L, nullptr);
   int cur = 0;
   uint32_t flush_begin = 0;
@@ -746,38 +779,74 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
     const uint64_t seeded = (uint64_t)n_q * (h->seed_neighbors ? h->max_cell_degree + 1 : 2);
     RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin, 0,
                          round == 0 ? (uint32_t)std::min<uint64_t>(seeded, 1u << 30) : 0));
-    if (round > 0) {  // round 0 was reset with the rest at the start (n_cur[chain] = n_in = 0)
+    if (round > 0) {  // round 0 was reset with the rest at the start
       WordSet ws;
       ws.zero_range(h->d_status->n_next, EXPAND_LEVELS);
       ws.zero_range(h->d_status->expand_work, EXPAND_LEVELS);
-      if (chain >= 0) ws.add(&h->d_status->n_cur[chain], n_in[chain]);
+      ws.add(&h->d_status->n_chain, 0u);
+      ws.add(&h->d_status->l0_exited, 0u);
       RC(h->set_words(ws));
     }
+    const bool conc = chain >= 0 && n_in[lvl0] > 0;
+    const uint32_t grid_c = conc ? std::min<uint32_t>(expand_grid(chain, n_q, h->sm_count), n_in[chain] + 16) : 0;
+    uint32_t grid0 = 0;
+    if (conc) {  // leave room for the chained level's CTAs (so they are resident from the start)
+      const uint32_t full = expand_grid(lvl0, n_in[lvl0], h->sm_count);
+      const size_t b0 = expand_warp_bytes(lvl0, h->V) + 1024, bc = expand_warp_bytes(chain, h->V) + 1024;
+      const uint32_t reserve = (uint32_t)(grid_c * ((bc + b0 - 1) / b0));
+      grid0 = full > reserve + h->sm_count ? full - reserve : full;
+    }
+    auto base = [&](int lvl) {
+      ExpandLaunch E;
+      E.level = lvl;
+      E.q = d_q;
+      E.qlist = in_list[lvl];
+      E.n = n_in[lvl];
+      E.k = k;
+      E.epoch = epoch;
+      E.retry_list = list(cur ^ 1, lvl);
+      E.promote_list = lvl + 1 < L ? list(cur ^ 1, lvl + 1) : nullptr;
+      E.promote_count = &h->d_status->n_next[std::min(lvl + 1, L - 1)];
+      E.out_obj = d_oo;
+      E.out_dist = d_od;
+      E.bound = d_bound;
+      E.remote = d_remote;
+      return E;
+    };
     for (int lvl = 0; lvl < L; ++lvl) {
-      const bool chained = lvl == chain && n_in[lvl0] > 0;
-      if (!n_in[lvl] && !chained) continue;
-      void* scratch = nullptr;
-      uint32_t sw = 0;
+      if (!n_in[lvl] || (conc && lvl == chain)) continue;
+      ExpandLaunch E = base(lvl);
       if (lvl == L - 1) {
         const size_t wb = expand_warp_bytes(lvl, h->V);
-        sw = (uint32_t)std::max<size_t>(1, std::min<size_t>(64, (size_t(2) << 30) / wb));
-        sw = std::min<uint32_t>(sw, n_in[lvl]);
-        RC(h->l2_scratch.ensure(wb * sw));
-        scratch = h->l2_scratch.p;
+        E.scratch_warps = (uint32_t)std::max<size_t>(1, std::min<size_t>(64, (size_t(2) << 30) / wb));
+        E.scratch_warps = std::min<uint32_t>(E.scratch_warps, n_in[lvl]);
+        RC(h->l2_scratch.ensure(wb * E.scratch_warps));
+        E.scratch = h->l2_scratch.p;
       }
-      uint32_t* retry = list(cur ^ 1, lvl);
-      // promotions out of the starting level go to the chained level's list of this round
-      // (after its own n_in entries), others to the next round
-      const bool to_chain = lvl == lvl0 && chain >= 0;
-      uint32_t* promote = lvl + 1 < L ? list(to_chain ? cur : cur ^ 1, lvl + 1) : nullptr;
-      uint32_t* promote_count = to_chain ? &h->d_status->n_cur[chain] : &h->d_status->n_next[std::min(lvl + 1, L - 1)];
-      const uint32_t* qlist = chained ? list(cur, lvl) : in_list[lvl];
-      const uint32_t nn = chained ? n_q : n_in[lvl];
-      const uint32_t* n_dev = chained ? &h->d_status->n_cur[chain] : nullptr;
+      if (conc && lvl == lvl0) {  // promotions go to the chained level running beside
+        E.promote_list = h->chain_ring.as<uint32_t>();
+        E.promote_count = &h->d_status->n_chain;
+        E.exited = &h->d_status->l0_exited;
+        E.grid = grid0;
+        E.trigger = true;
+      }
       const int kind = lvl == 0 ? GGRID_K_EXPAND : GGRID_K_EXPAND_BIG;
       h->launch(kind, [&] {
-        launch_expand(lvl, d_q, qlist, nn, n_dev, k, g, s, epoch, retry, promote, promote_count, d_oo, d_od,
-                      d_bound, d_remote, scratch, sw, h->sm_count, st);
+        launch_expand(E, g, s, h->sm_count, st);
+        if (conc && lvl == lvl0) {  // the chained level, started while the starting level runs
+          // (inside the same profile-event pair: an event between the two would end the overlap,
+          // so in profile mode the pair times the whole expansion phase)
+          ExpandLaunch C = base(chain);
+          C.chain_in = h->chain_ring.as<uint32_t>();
+          C.chain_cap = n_q;
+          C.wait_exited = &h->d_status->l0_exited;
+          C.wait_total = grid0;
+          C.grid = grid_c;
+          C.pdl = true;
+          h->stats.launches++;
+          h->stats.kernel_launches[GGRID_K_EXPAND_BIG]++;
+          launch_expand(C, g, s, h->sm_count, st);
+        }
       });
     }
     RC(h->sync());
@@ -804,6 +873,21 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   h->stats.n_queries += n_q;
   h->stats.knn_calls++;
   return GGRID_OK;
+}
+
+int ggrid_knn_commit(ggrid_t h, uint32_t k, uint32_t* out_obj, uint32_t* out_dist, uint32_t* n_q) {
+  if (!h || h->n_qstaged == 0 || k == 0 || k > h->max_k) return GGRID_EINVAL;
+  ggrid_s::Staged& sb = h->qstaged[h->qstage_head];
+  if (n_q) *n_q = (uint32_t)sb.n;
+  if (sb.n && (!out_obj || !out_dist)) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  h->qstage_head ^= 1;
+  h->n_qstaged--;
+  CK(cudaStreamWaitEvent(h->stream, sb.done, 0));
+  int rc = GGRID_OK;
+  if (sb.n) rc = knn_impl(h, sb.buf.as<ggrid_query>(), (uint32_t)sb.n, k, out_obj, out_dist);
+  CK(cudaEventRecord(sb.consumed, h->stream));
+  return rc;
 }
 
 int ggrid_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,

@@ -53,7 +53,8 @@ struct DevStatus {
   unsigned int n_next[EXPAND_LEVELS];   // per expansion level: queries queued for the next round
   unsigned int flush_end;   // n_flush as seen by the last flush launch
   unsigned int expand_work[EXPAND_LEVELS];  // per-level dynamic work counters of the expand launches
-  unsigned int n_cur[EXPAND_LEVELS];  // per level: queries of the current round (chained level)
+  unsigned int n_chain;     // queries the starting level promoted into the chained level this round
+  unsigned int l0_exited;   // CTAs of the starting level's launch that have exited this round
   unsigned int round_end;   // (marks the end of the per-round reset region)
 };
 
@@ -214,13 +215,37 @@ __device__ __forceinline__ uint2 vobj_valid(uint2 vo, uint2 comp) {
 // bound (nullable): per-query inclusive distance limit (objects farther are not returned and
 // the search stops beyond it); remote (nullable): per-query bitmask of the ranks owning cells
 // the search expanded into (sharded mode)
-// n_dev (nullable): the query count is read on the device (a level chained behind the level
-// below in the same round); promote_count: the counter that indexes promote_list.
-void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, const uint32_t* n_dev,
-                   uint32_t k, const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
-                   uint32_t* promote_list, uint32_t* promote_count, uint32_t* out_obj, uint32_t* out_dist,
-                   const uint32_t* bound, unsigned long long* remote, void* scratch,
-                   uint32_t scratch_warps, int sm_count, cudaStream_t st);
+struct ExpandLaunch {
+  int level = 0;
+  const uint2* q = nullptr;
+  const uint32_t* qlist = nullptr;  // (null: query i is qlist entry i)
+  uint32_t n = 0;                   // queries in qlist
+  uint32_t k = 0;
+  uint32_t epoch = 0;
+  uint32_t* retry_list = nullptr;   // this level, next round (counter: n_next[level])
+  uint32_t* promote_list = nullptr; // next level
+  uint32_t* promote_count = nullptr;
+  uint32_t* out_obj = nullptr;
+  uint32_t* out_dist = nullptr;
+  const uint32_t* bound = nullptr;
+  unsigned long long* remote = nullptr;
+  void* scratch = nullptr;          // the last level's global working memory
+  uint32_t scratch_warps = 0;
+  // concurrency of a chained level with the level below it (same round, two streams):
+  uint32_t* exited = nullptr;       // the lower level: each CTA counts itself out here
+  const uint32_t* chain_in = nullptr;  // the chained level: queries promoted by the lower level,
+                                       // appended after the n of qlist (entries NONE until written;
+                                       // taken entries are reset to NONE)
+  uint32_t chain_cap = 0;
+  const uint32_t* wait_exited = nullptr;  // ... done when *wait_exited == wait_total
+  uint32_t wait_total = 0;
+  uint32_t grid = 0;                // 0: the default (expand_grid)
+  bool trigger = false;             // let the next kernel of the stream start now (PDL)
+  bool pdl = false;                 // launched as a programmatic dependent of the previous kernel
+};
+// CTAs launch_expand uses for n queries at `level`
+uint32_t expand_grid(int level, uint32_t n, int sm_count);
+void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st);
 // prior-art comparison path (csrc/prior_art.cu)
 int prior_art_mu(int eta);
 size_t prior_art_scan_bytes(uint32_t n);

@@ -143,7 +143,6 @@ struct QParams {
   const uint2* q;
   const uint32_t* qlist;
   uint32_t n;
-  const uint32_t* n_dev;    // (non-null: the count is read on the device at kernel start)
   uint32_t k;
   uint32_t epoch;
   int level;
@@ -158,7 +157,27 @@ struct QParams {
   Caps caps;
   unsigned char* scratch;   // global working memory (last level) or null (shared)
   uint32_t warps_per_cta;
+  uint32_t* exited;               // (see ExpandLaunch)
+  uint32_t* chain_in;
+  uint32_t chain_cap;
+  const uint32_t* wait_exited;
+  uint32_t wait_total;
+  int trigger;
 };
+
+// programmatic dependent launch: the next kernel of the stream may start right away (it
+// depends on this one only through the promotion ring and the exit counter)
+__device__ __forceinline__ void pdl_trigger(const QParams& P) {
+  if (P.trigger) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
+// a CTA of a lower level leaving: publishes its promotions to a concurrent chained level
+__device__ __forceinline__ void count_exit(const QParams& P) {
+  if (P.exited) {
+    __threadfence();
+    atomicAdd(P.exited, 1u);
+  }
+}
 
 // current distance of candidate i (exact once its source vertex is settled)
 __device__ __forceinline__ unsigned long long cand_dist(const WarpMem& m, uint32_t i) {
@@ -500,18 +519,18 @@ __global__ void k_expand(QParams P) {
   const uint32_t gw = blockIdx.x * P.warps_per_cta + warp;
   unsigned char* base = SMEM ? smem_raw + (size_t)warp * wbytes : P.scratch + (size_t)gw * wbytes;
   const WarpMem m = carve(base, P.caps);
-  const uint32_t n = P.n_dev ? *(volatile const uint32_t*)P.n_dev : P.n;
-  if (n == 0) return;  // (a chained level with nothing promoted: no contended work counter)
+  pdl_trigger(P);
   for (;;) {  // persistent: queries fetched dynamically
     uint32_t li = 0;
     if (lane == 0) li = atomicAdd(&P.s.st->expand_work[P.level], 1u);
     li = __shfl_sync(0xffffffffu, li, 0);
-    if (li >= n) break;
+    if (li >= P.n) break;
     const uint32_t qi = P.qlist ? P.qlist[li] : li;
     const int r = run_query(P, m, qi, lane);
     if (lane == 0 && r != DONE) finish_undone(P, qi, r);
     __syncwarp();
   }
+  if (lane == 0) count_exit(P);
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -818,19 +837,43 @@ __global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
   __shared__ CtaShared sh;
   __shared__ uint32_t qslot;
   const WarpMem m = carve(smem_raw, P.caps);
-  const uint32_t n = P.n_dev ? *(volatile const uint32_t*)P.n_dev : P.n;
-  if (n == 0) return;  // (a chained level with nothing promoted: no contended work counter)
+  pdl_trigger(P);
   for (;;) {  // persistent: queries fetched dynamically
-    if (threadIdx.x == 0) qslot = atomicAdd(&P.s.st->expand_work[P.level], 1u);
+    if (threadIdx.x == 0) {
+      const uint32_t li = atomicAdd(&P.s.st->expand_work[P.level], 1u);
+      uint32_t qi = NONE;
+      if (li < P.n) {
+        qi = P.qlist ? P.qlist[li] : li;
+      } else if (P.chain_in && li - P.n < P.chain_cap) {
+        // a chained level running beside the level below: take the next promoted query as
+        // soon as it is written, until every CTA below has exited (promotions published)
+        volatile uint32_t* slot = P.chain_in + (li - P.n);
+        for (;;) {
+          uint32_t v = *slot;
+          if (v == NONE && *(volatile const uint32_t*)P.wait_exited == P.wait_total) {
+            __threadfence();
+            v = *slot;
+            if (v == NONE) break;
+          }
+          if (v != NONE) {
+            qi = v;
+            *slot = NONE;  // (the ring is all-NONE again when the level has drained it)
+            break;
+          }
+          __nanosleep(1000);
+        }
+      }
+      qslot = qi;
+    }
     __syncthreads();
-    const uint32_t li = qslot;
+    const uint32_t qi = qslot;
     __syncthreads();
-    if (li >= n) break;
-    const uint32_t qi = P.qlist ? P.qlist[li] : li;
+    if (qi == NONE) break;
     const int r = run_query_cta<CTA_W>(P, m, sh, qi);
     if (threadIdx.x == 0 && r != DONE) finish_undone(P, qi, r);
     __syncthreads();
   }
+  if (threadIdx.x == 0) count_exit(P);
 }
 
 // Capacity ladder.  Levels 0-4 keep the query's working set in shared memory (~10, 24, 45, 95
@@ -856,8 +899,6 @@ Caps caps_for(int level, uint32_t V) {
   return Caps{H, F, 8192};
 }
 
-bool g_attr_set = false;
-int g_blocks_per_sm[NLEVELS] = {};
 }  // namespace
 
 int expand_levels() { return NLEVELS; }
@@ -871,70 +912,86 @@ size_t expand_warp_bytes(int level, uint32_t V) {
   return (warpmem_bytes(c) + 15) & ~size_t(15);
 }
 
-void launch_expand(int level, const uint2* q, const uint32_t* qlist, uint32_t n, const uint32_t* n_dev,
-                   uint32_t k, const DevGraph& g, const DevState& s, uint32_t epoch, uint32_t* retry_list,
-                   uint32_t* promote_list, uint32_t* promote_count, uint32_t* out_obj, uint32_t* out_dist,
-                   const uint32_t* bound, unsigned long long* remote, void* scratch,
-                   uint32_t scratch_warps, int sm_count, cudaStream_t st) {
-  if (n == 0) return;  // (with n_dev: an upper bound of the device count)
+// CTA-per-query for the big shared-memory levels, and for small batches at any of them
+static bool use_cta(int level, uint32_t n, int sm_count) {
+  return level < NLEVELS - 1 && (level >= GG_CTA_LEVEL || n <= (uint32_t)sm_count);
+}
+
+// resident CTAs per SM of a shared-memory level's kernel (occupancy calculator, cached)
+static uint32_t blocks_per_sm(int level, bool cta) {
+  static int bps[2][NLEVELS] = {};
+  int& b = bps[cta ? 1 : 0][level];
+  if (!b) {
+    const int smem = (int)expand_warp_bytes(level, 1);
+    if (cta) {
+      cudaFuncSetAttribute(k_expand_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand_cta, CTA_W * 32, smem);
+    } else {
+      cudaFuncSetAttribute(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32, smem);
+    }
+    if (b <= 0) b = 1;
+  }
+  return (uint32_t)b;
+}
+
+uint32_t expand_grid(int level, uint32_t n, int sm_count) {
+  if (level == NLEVELS - 1) return 0;  // (global scratch: sized by the caller's scratch warps)
+  return std::min<uint32_t>(n, (uint32_t)sm_count * blocks_per_sm(level, use_cta(level, n, sm_count)));
+}
+
+void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st) {
+  const int level = L.level;
+  if (L.n == 0 && !L.chain_in) return;
   QParams P;
   P.g = g;
   P.s = s;
-  P.q = q;
-  P.qlist = qlist;
-  P.n = n;
-  P.n_dev = n_dev;
-  P.k = k;
-  P.epoch = epoch;
+  P.q = L.q;
+  P.qlist = L.qlist;
+  P.n = L.n;
+  P.k = L.k;
+  P.epoch = L.epoch;
   P.level = level;
   P.last_level = NLEVELS - 1;
-  P.retry_list = retry_list;
-  P.promote_list = promote_list;
-  P.promote_count = promote_count;
-  P.out_obj = out_obj;
-  P.out_dist = out_dist;
-  P.bound = bound;
-  P.remote = remote;
+  P.retry_list = L.retry_list;
+  P.promote_list = L.promote_list;
+  P.promote_count = L.promote_count;
+  P.out_obj = L.out_obj;
+  P.out_dist = L.out_dist;
+  P.bound = L.bound;
+  P.remote = L.remote;
   P.caps = caps_for(level, g.V);
   P.warps_per_cta = 1;
-  const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
-  if (!g_attr_set) {
-    cudaFuncSetAttribute(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    g_attr_set = true;
-  }
-  // CTA-per-query for the big shared-memory levels, and for small batches at any of them
-  const bool cta = level < NLEVELS - 1 && (level >= GG_CTA_LEVEL || n <= (uint32_t)sm_count);
-  if (cta) {
-    P.scratch = nullptr;
-    const int smem = (int)wbytes;
-    static bool attr = false;
-    static int bps[NLEVELS] = {};
-    if (!attr) {
-      cudaFuncSetAttribute(k_expand_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
-      attr = true;
-    }
-    if (!bps[level]) {
-      int b = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand_cta, CTA_W * 32, smem);
-      bps[level] = b > 0 ? b : 1;
-    }
-    const uint32_t wave = (uint32_t)(sm_count * bps[level]);
-    k_expand_cta<<<std::min<uint32_t>(n, wave), CTA_W * 32, smem, st>>>(P);
+  P.scratch = nullptr;
+  P.exited = L.exited;
+  P.chain_in = const_cast<uint32_t*>(L.chain_in);
+  P.chain_cap = L.chain_cap;
+  P.wait_exited = L.wait_exited;
+  P.wait_total = L.wait_total;
+  P.trigger = L.trigger ? 1 : 0;
+  const int smem = (int)expand_warp_bytes(level, g.V);
+  if (level == NLEVELS - 1) {
+    P.scratch = static_cast<unsigned char*>(L.scratch);
+    k_expand<false><<<std::min<uint32_t>(L.n, std::max<uint32_t>(1, L.scratch_warps)), 32, 0, st>>>(P);
     return;
   }
-  if (level < NLEVELS - 1) {
-    P.scratch = nullptr;
-    const int smem = (int)wbytes;
-    if (!g_blocks_per_sm[level]) {
-      int b = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32, smem);
-      g_blocks_per_sm[level] = b > 0 ? b : 1;
-    }
-    const uint32_t wave = (uint32_t)(sm_count * g_blocks_per_sm[level]);
-    k_expand<true><<<std::min<uint32_t>(n, wave), 32, smem, st>>>(P);
+  const bool cta = L.chain_in != nullptr || use_cta(level, L.n, sm_count);
+  const uint32_t grid = L.grid ? L.grid : std::max<uint32_t>(1, expand_grid(level, L.n, sm_count));
+  blocks_per_sm(level, cta);  // (sets the shared-memory attribute)
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(cta ? CTA_W * 32 : 32);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = L.pdl ? 1 : 0;
+  if (cta) {
+    cudaLaunchKernelEx(&cfg, k_expand_cta, P);
   } else {
-    P.scratch = static_cast<unsigned char*>(scratch);
-    k_expand<false><<<std::min<uint32_t>(n, std::max<uint32_t>(1, scratch_warps)), 32, 0, st>>>(P);
+    cudaLaunchKernelEx(&cfg, k_expand<true>, P);
   }
 }
 

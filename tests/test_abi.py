@@ -38,7 +38,7 @@ def test_struct_layouts_match_header(gg):
     # sizes the header implies on LP64
     assert ctypes.sizeof(gg.ggrid_graph) == 8 + 5 * 8
     assert ctypes.sizeof(gg.ggrid_opts) == 4 + 4 + 4 + 4 + 8 + 4 * 4 + 8 + 4 + 4  # async_ingest + tail padding
-    assert ctypes.sizeof(gg.ggrid_stats_t) == 16 * 8 + 8 * 8 + 8 * 8 + 8 * 4 + 8
+    assert ctypes.sizeof(gg.ggrid_stats_t) == 16 * 8 + 8 * 8 + 8 * 8 + 8 * 4 + 8 + 2 * 8  # + promotions, retries
 
 
 def test_zvalue_worked_example(gg):

@@ -526,3 +526,34 @@ def test_pipelined_ingest_stage_commit(gg):
     _assert_same(grid.knn(q, 6), _oracle(g, np.concatenate([u1, u2, u3]), q, 6), "after commit 2")
     assert grid.stats()["n_updates"] == len(u1) + len(u2) + len(u3)
     grid.close()
+
+
+def test_pipelined_queries_stage_commit(gg):
+    """ggrid_query_stage / ggrid_knn_commit (two-deep query staging on the copy stream),
+    interleaved with staged update batches: every committed batch answers the snapshot of the
+    updates committed before it, bit-exact."""
+    import torch
+
+    g = synth.table_ii_graph("NY", scale=0.03)
+    walk = synth.RandomWalk(g, 500, inject=True)
+    grid = gg.GGrid(g, 128, max_objects=512, async_ingest=True)
+    ups = [walk.ticks(2) for _ in range(5)]
+    qs = [synth.queries(g, 40 + 7 * i, seed=300 + i) for i in range(5)]
+    hu = [torch.from_numpy(u.view(np.int32)).pin_memory() for u in ups]
+    hq = [torch.from_numpy(q.view(np.int32)).pin_memory() for q in qs]
+    k = 5
+    grid.ingest_stage(hu[0])
+    grid.query_stage(hq[0])
+    for s in range(5):
+        grid.ingest_commit()
+        if s + 1 < 5:
+            grid.ingest_stage(hu[s + 1])
+            grid.query_stage(hq[s + 1])
+        o = torch.empty((len(qs[s]), k), dtype=torch.int32).pin_memory()
+        d = torch.empty((len(qs[s]), k), dtype=torch.int32).pin_memory()
+        grid.knn_commit(k, o, d)
+        ref = _oracle(g, np.concatenate(ups[: s + 1]), qs[s], k)
+        _assert_same((o.numpy().view(np.uint32), d.numpy().view(np.uint32)), ref, f"batch {s}")
+    with pytest.raises(gg.GGridError):
+        grid.knn_commit(k, o, d)  # nothing staged
+    grid.close()

@@ -31,6 +31,13 @@ hqs = [torch.from_numpy(synth.queries(g, Q, seed=100 + i).view(np.int32)).pin_me
 if args.variant == "rev":
     hus = hus[:3] + hus[3:][::-1]
     hqs = hqs[:3] + hqs[3:][::-1]
+if "warm" in args.variant:  # one DMA from every pinned buffer first
+    su = torch.empty_like(hus[0], device="cuda")
+    sq = torch.empty_like(hqs[0], device="cuda")
+    for a, b in zip(hus, hqs):
+        su.copy_(a)
+        sq.copy_(b)
+    torch.cuda.synchronize()
 h_o = torch.empty((Q, k), dtype=torch.int32).pin_memory()
 h_d = torch.empty((Q, k), dtype=torch.int32).pin_memory()
 for s in range(3):
@@ -40,13 +47,27 @@ for s in range(3):
 torch.cuda.synchronize()
 t0 = time.perf_counter()
 ts = []
+parts = []
+qs = "qstage" in args.variant
 grid.ingest_stage(hus[3])
+if qs:
+    grid.query_stage(hqs[3])
 for s in range(3, 3 + n):
+    a = time.perf_counter()
     grid.ingest_commit()
-    if s + 1 < 3 + n or args.variant == "extra":
+    b = time.perf_counter()
+    if s + 1 < 3 + n or "extra" in args.variant:
         grid.ingest_stage(hus[s + 1])
-    grid.knn(hqs[s], k, h_o, h_d)
-    if args.variant == "sync":
+        if qs:
+            grid.query_stage(hqs[s + 1])
+    c = time.perf_counter()
+    if qs:
+        grid.knn_commit(k, h_o, h_d)
+    else:
+        grid.knn(hqs[s], k, h_o, h_d)
+    if "sync" in args.variant:
         grid.sync()
     ts.append(time.perf_counter())
+    parts.append((round(1e3 * (b - a), 3), round(1e3 * (c - b), 3), round(1e3 * (ts[-1] - c), 3)))
 print(args.variant, "step ms:", [round(1e3 * (b - a), 3) for a, b in zip([t0] + ts[:-1], ts)])
+print("  (commit, stage, knn) ms:", parts[-4:])
