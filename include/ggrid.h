@@ -78,6 +78,13 @@ typedef struct ggrid_opts {
                               ggrid_sync or ggrid_ingest call.  A rejected batch
                               leaves its seq range unused.  Ignored (synchronous)
                               when t_delta != 0.  0 = default, synchronous.         */
+  uint32_t ingest_kernels; /* 0 = default: a batch that fits one resident wave
+                              (<= 8,192 updates per SM and few enough distinct cells
+                              per SM tile for shared memory) is ingested by ONE
+                              cooperative launch (classify, extent allocation and
+                              scatter separated by grid barriers), larger batches by
+                              three launches; 3 = always the three launches.  Both
+                              produce the same index state.                        */
 } ggrid_opts;
 
 typedef struct ggrid_s* ggrid_t;

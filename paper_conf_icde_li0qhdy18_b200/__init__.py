@@ -45,7 +45,8 @@ class ggrid_opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("max_k", ctypes.c_uint32), ("max_objects", ctypes.c_uint32),
                 ("log_capacity", ctypes.c_uint64), ("delta", ctypes.c_uint32),
                 ("seed_neighbors", ctypes.c_uint32), ("profile", ctypes.c_uint32),
-                ("t_delta", ctypes.c_uint32), ("stream", ctypes.c_void_p), ("async_ingest", ctypes.c_uint32)]
+                ("t_delta", ctypes.c_uint32), ("stream", ctypes.c_void_p), ("async_ingest", ctypes.c_uint32),
+                ("ingest_kernels", ctypes.c_uint32)]
 
 
 NK = 8
@@ -144,7 +145,7 @@ def _u32(a):
 def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 256,
                 max_objects: int = 1 << 24, log_capacity: int = 0, delta: int = 0,
                 seed_neighbors: bool = True, profile: bool = False, t_delta: int = 0, stream=None,
-                async_ingest: bool = False):
+                async_ingest: bool = False, ingest_kernels: int = 0):
     """ggrid_build(graph, cell_size) -> handle (c_void_p).  graph: dict(n_vertices, src, dst, w[, x, y])."""
     src, dst, w = (np.ascontiguousarray(graph[k], np.uint32) for k in ("src", "dst", "w"))
     x = graph.get("x")
@@ -155,7 +156,7 @@ def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 25
                     None if x is None else x.ctypes.data, None if y is None else y.ctypes.data)
     o = ggrid_opts(int(device), int(max_k), int(max_objects), int(log_capacity), int(delta),
                    0 if seed_neighbors else 2, int(profile), int(t_delta), stream,
-                   1 if async_ingest else 0)
+                   1 if async_ingest else 0, int(ingest_kernels))
     h = ctypes.c_void_p()
     _check(lib().ggrid_build(ctypes.byref(g), int(cell_size), ctypes.byref(o), ctypes.byref(h)), "ggrid_build")
     return h

@@ -108,6 +108,7 @@ struct ggrid_s {
   // Until the next sync the status mirror is stale by the batches queued since; these bound
   // what they can have added (records incl. extent padding, extents, newly live objects).
   int async_ingest = 0;
+  int fused_ingest = 1;  // opts.ingest_kernels: one cooperative launch when the batch fits
   uint64_t pend_records = 0, pend_updates = 0;
   uint32_t pend_ext = 0;
   uint32_t max_cell_degree = 0;  // most neighbour cells of any cell
@@ -388,6 +389,7 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   h->t_delta = o.t_delta;
   // the expiry cut reads t_now on the host, so expiry keeps ingest synchronous
   h->async_ingest = (o.async_ingest && !o.t_delta) ? 1 : 0;
+  h->fused_ingest = o.ingest_kernels == 3 ? 0 : 1;
   h->s.n_ranks = 1;
   h->s.rank = 0;
 
@@ -566,9 +568,12 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   if (h->async_ingest) RC(h->take_deferred());  // an earlier batch was rejected
   const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
   RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
-  RC(h->tmp.ensure(ingest_tmp_bytes(n)));
+  IngestPlan fp;
+  const bool fused = h->fused_ingest && ingest_fused_plan(n, h->n_cells, h->sm_count, &fp);
+  if (!fused) RC(h->tmp.ensure(ingest_tmp_bytes(n)));
   {
     WordSet ws;
+    if (fused) ws.add(&h->d_status->ingest_bar, 0u);
     if (h->async_ingest) {  // the previous batch's error bits move to err_deferred (ggrid_sync)
       ws.fold_dst = &h->d_status->err_deferred;
       ws.fold_src = &h->d_status->ingest_err;
@@ -582,9 +587,15 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   const DevState& s = h->s;
   uint2* tmp = h->tmp.as<uint2>();
   cudaStream_t st = h->stream;
-  h->launch(GGRID_K_INGEST_CLASSIFY, [&] { launch_ingest_classify(d_u, n, g, s, tmp, st); });
-  h->launch(GGRID_K_INGEST_ALLOC, [&] { launch_ingest_alloc(g, s, st); });
-  h->launch(GGRID_K_INGEST_SCATTER, [&] { launch_ingest_scatter(d_u, n, seq0, g, s, tmp, st); });
+  if (fused) {  // one cooperative launch (counted and timed as the classify kind)
+    cudaError_t le = cudaSuccess;
+    h->launch(GGRID_K_INGEST_CLASSIFY, [&] { le = launch_ingest_fused(d_u, n, seq0, g, s, fp, st); });
+    CK(le);
+  } else {
+    h->launch(GGRID_K_INGEST_CLASSIFY, [&] { launch_ingest_classify(d_u, n, g, s, tmp, st); });
+    h->launch(GGRID_K_INGEST_ALLOC, [&] { launch_ingest_alloc(g, s, st); });
+    h->launch(GGRID_K_INGEST_SCATTER, [&] { launch_ingest_scatter(d_u, n, seq0, g, s, tmp, st); });
+  }
   if (h->async_ingest) {
     // no host round trip: a rejected batch (checked on the device, all or nothing) keeps its
     // seq range unused, which changes no answer (only the order of keys matters)

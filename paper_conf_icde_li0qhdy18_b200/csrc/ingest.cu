@@ -10,6 +10,8 @@
 //   scatter  : writes the SoA record and RED.MAX-es (t<<32|seq) into ot_key[o].
 // No tombstones: a record is valid iff its key equals ot_key[obj] (reading R8/R9), which
 // also makes out-of-order arrivals harmless.
+#include <algorithm>
+
 #include "internal.cuh"
 
 namespace gg {
@@ -158,9 +160,9 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
   }
 }
 
-__global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
-  uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
-  const bool err = s.st->ingest_err != 0;
+// This batch's extent of cell c (a full warp calls it, c >= n_cells allowed: no cell): carved
+// out of the bump arena (warp-aggregated), linked at the head of the cell's chain.
+__device__ __forceinline__ void alloc_cell_warp(const DevGraph& g, const DevState& s, uint32_t c, bool err) {
   uint32_t cnt = (c < g.n_cells) ? s.bcount[c * BCOUNT_STRIDE] : 0;
   if (err) {
     if (c < g.n_cells && cnt) {
@@ -205,6 +207,10 @@ __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
   s.cell_pending[c] += cnt;
   s.bbase[c] = (uint32_t)start;
   s.bcount[c * BCOUNT_STRIDE] = 0;
+}
+
+__global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
+  alloc_cell_warp(g, s, blockIdx.x * blockDim.x + threadIdx.x, s.st->ingest_err != 0);
 }
 
 // One CTA per classify tile.  The tile's updates are staged in shared memory (coalesced), then
@@ -298,6 +304,241 @@ void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const De
   unsigned blocks = (unsigned)((n + CU - 1) / CU);
   k_ingest_scatter<<<blocks, CT, 0, st>>>(upd, n, seq0, g, s, tmp,
                                           perm_of(const_cast<uint2*>(tmp), n));
+}
+
+// ---------------------------------------------------------------------------------------
+// Single-launch ingest for a batch that fits one resident wave: the classify, alloc and
+// scatter phases above as one persistent cooperative kernel (one 1,024-thread CTA per SM)
+// with two grid barriers between them.  Each CTA keeps its tile's cell hash, cell order and
+// permutation in shared memory across the barriers (no tmp/perm round trip through HBM, no
+// launch gaps, no tail wave); the scatter re-reads the tile's records from L2.
+constexpr int FT = 1024;                // threads per CTA
+constexpr int FPT = 8;                  // updates per thread at most
+constexpr uint32_t FUSED_TILE = FT * FPT;
+constexpr uint32_t FUSED_CH_MAX = 16384;  // cell-hash slots (>= 2 x distinct cells of a tile)
+
+__device__ __forceinline__ void grid_barrier(unsigned* ctr, unsigned target) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(ctr, 1u);
+    unsigned v;
+    for (;;) {
+      asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+      if (v >= target) break;
+      __nanosleep(64);
+    }
+  }
+  __syncthreads();
+}
+
+__global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict__ upd, uint64_t n,
+                                                        uint32_t seq0, uint32_t tile, uint32_t ch,
+                                                        DevGraph g, DevState s) {
+  extern __shared__ __align__(16) uint32_t f_buf[];
+  uint32_t* h_cell = f_buf;          // [ch] cell id (REMOTE_CELL: other ranks' updates)
+  uint32_t* h_cnt = f_buf + ch;      // [ch] count; after the scan (tile offset << 16) | count
+  uint32_t* h_aux = f_buf + 2 * ch;  // [ch] newest t; after the claim, the cell's batch rank base
+  uint2* stg = reinterpret_cast<uint2*>(f_buf + 3 * ch);    // [tile] (src vertex, rank), cell order
+  uint16_t* stp = reinterpret_cast<uint16_t*>(stg + tile);  // [tile] index in the tile
+  uint32_t* w_sum = reinterpret_cast<uint32_t*>(stp + ((tile + 1) & ~1u));  // [FT / 32]
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const unsigned G = gridDim.x;
+  for (uint32_t i = tid; i < ch; i += FT) {
+    h_cell[i] = NONE;
+    h_cnt[i] = 0;
+    h_aux[i] = 0;
+  }
+  __syncthreads();
+  const uint64_t base = (uint64_t)blockIdx.x * tile;
+  const uint32_t nt = base >= n ? 0u : (uint32_t)min((uint64_t)tile, n - base);
+
+  // ---- classify: validate, cell via the inverted index, rank within the tile's cell group
+  uint32_t sr[FPT];  // (hash slot << 16) | rank in the slot's group, NONE: no record
+  uint32_t vs[FPT];
+  uint32_t tl = 0;
+  constexpr int HP = FPT / 2;
+#pragma unroll
+  for (int hf = 0; hf < 2; ++hf) {  // two halves: a half's loads and gathers in flight together
+    uint4 mm[HP];
+    uint2 ee[HP];
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      const uint32_t k = (uint32_t)((hf * HP + q) * FT + tid);
+      mm[q] = k < nt ? __ldg(upd + base + k) : make_uint4(0, 0xFFFFFFFFu, 0, 0);
+    }
+#pragma unroll
+    for (int q = 0; q < HP; ++q) ee[q] = mm[q].y < g.A ? __ldg(g.einfo + mm[q].y) : make_uint2(0, 1);
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      const int j = hf * HP + q;
+      const uint32_t k = (uint32_t)(j * FT + tid);
+      sr[j] = NONE;
+      vs[j] = 0;
+      if (k >= nt) continue;
+      const uint4 m = mm[q];
+      const uint2 e = ee[q];
+      unsigned bad = 0;
+      if (m.x >= s.max_objects) bad |= ERR_OBJ;
+      if (m.y >= g.A) {
+        bad |= ERR_EDGE;
+      } else if (m.z >= e.y) {
+        bad |= ERR_OFF;
+      }
+      if (bad) {
+        const uint64_t i = base + k;
+        atomicOr(&s.st->ingest_err, bad);
+        atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
+        continue;
+      }
+      const uint32_t c0 = cellof(g, e.x);
+      const bool remote = s.n_ranks > 1 && owner_of(c0, g.n_cells, s.n_ranks) != s.rank;
+      const uint32_t c = remote ? REMOTE_CELL : c0;
+      uint32_t h = __umulhi(c * 2654435761u, ch);
+      volatile uint32_t* vc = h_cell;
+      for (;;) {
+        const uint32_t cur = vc[h];
+        if (cur == c) break;
+        if (cur == NONE) {
+          const uint32_t old = atomicCAS(&h_cell[h], NONE, c);
+          if (old == NONE || old == c) break;
+        }
+        h = (h + 1) & (ch - 1);
+      }
+      sr[j] = (h << 16) | atomicAdd(&h_cnt[h], 1u);
+      vs[j] = e.x;
+      atomicMax(&h_aux[h], m.w);
+      tl = max(tl, m.w);
+    }
+  }
+  tl = __reduce_max_sync(0xffffffffu, tl);
+  if (lane == 0 && tl) atomicMax(&s.st->t_max, tl);
+  __syncthreads();
+  {  // exclusive scan of the slot counts = each group's offset in the tile's cell order
+    const uint32_t spc = ch / FT;
+    uint32_t sum = 0;
+    for (uint32_t q = 0; q < spc; ++q) sum += h_cnt[tid * spc + q];
+    uint32_t x = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) w_sum[wid] = x;
+    __syncthreads();
+    uint32_t run = x - sum;
+    for (int w = 0; w < wid; ++w) run += w_sum[w];
+    for (uint32_t q = 0; q < spc; ++q) {
+      const uint32_t c = h_cnt[tid * spc + q];
+      h_cnt[tid * spc + q] = c | (run << 16);  // (counts and offsets <= FUSED_TILE < 2^16)
+      run += c;
+    }
+  }
+  // one claim per distinct cell of the tile on the batch counters
+  for (uint32_t i = tid; i < ch; i += FT) {
+    const uint32_t c = h_cell[i];
+    if (c != NONE && c != REMOTE_CELL) {
+      atomicMax(&s.bcount[c * BCOUNT_STRIDE + 1], h_aux[i]);
+      h_aux[i] = atomicAdd(&s.bcount[c * BCOUNT_STRIDE], h_cnt[i] & 0xFFFFu);
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < FPT; ++j) {
+    if (sr[j] == NONE) continue;
+    const uint32_t slot = sr[j] >> 16, lr = sr[j] & 0xFFFFu;
+    const uint32_t si = (h_cnt[slot] >> 16) + lr;
+    stg[si] = make_uint2(vs[j], h_cell[slot] == REMOTE_CELL ? NONE : h_aux[slot] + lr);
+    stp[si] = (uint16_t)(j * FT + tid);
+  }
+
+  // ---- alloc: every tile's counts are in; one extent per (batch, cell)
+  grid_barrier(&s.st->ingest_bar, G);
+  {
+    const bool err = *((volatile unsigned*)&s.st->ingest_err) != 0;
+    const uint32_t nw = G * (FT / 32);
+    for (uint32_t c0 = (blockIdx.x * (FT / 32) + wid) * 32; c0 < g.n_cells; c0 += nw * 32)
+      alloc_cell_warp(g, s, c0 + lane, err);
+  }
+  grid_barrier(&s.st->ingest_bar, 2 * G);
+  if (*((volatile unsigned*)&s.st->ingest_err)) return;  // the batch is rejected as a whole
+
+  // ---- scatter in cell order (consecutive threads write consecutive extent positions)
+  for (uint32_t k0 = 0; k0 < nt; k0 += FT * HP) {
+    uint32_t pos[HP], il[HP];
+    uint32_t vx[HP];
+    uint4 m[HP];
+    unsigned long long cur[HP];
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      const uint32_t k = k0 + (uint32_t)(q * FT + tid);
+      if (k < nt) {
+        const uint2 vr = stg[k];
+        il[q] = stp[k];
+        vx[q] = vr.x;
+        m[q] = __ldcs(upd + base + il[q]);  // (an L2 hit: read by this CTA in the classify)
+        pos[q] = vr.y == NONE ? NONE : s.bbase[cellof(g, vr.x)] + vr.y;
+        cur[q] = __ldcg(s.ot_key + m[q].x);
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      const uint32_t k = k0 + (uint32_t)(q * FT + tid);
+      if (k >= nt) continue;
+      const unsigned long long key =
+          ((unsigned long long)m[q].w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + il[q]));
+      if (pos[q] != NONE) {
+        s.ar.obj[pos[q]] = m[q].x;
+        s.ar.key[pos[q]] = key;
+        s.ar.vsrc[pos[q]] = vx[q];
+        s.ar.off[pos[q]] = m[q].z;
+        s.ar.edge[pos[q]] = m[q].y;
+      }
+      if (cur[q] == 0ull) {
+        const unsigned long long old = atomicMax(&s.ot_key[m[q].x], key);
+        if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+      } else if (key > cur[q]) {
+        atomicMax(&s.ot_key[m[q].x], key);
+      }
+    }
+  }
+}
+
+static size_t fused_smem(uint32_t tile, uint32_t ch) {
+  return (size_t)ch * 12 + (size_t)tile * 8 + (size_t)((tile + 1) & ~1u) * 2 + (FT / 32) * 4;
+}
+
+bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p) {
+  if (n == 0 || sm_count <= 0) return false;
+  const uint64_t grid = std::min<uint64_t>((uint64_t)sm_count, std::max<uint64_t>(1, (n + 2047) / 2048));
+  const uint64_t tile = (n + grid - 1) / grid;
+  if (tile > FUSED_TILE) return false;
+  const uint64_t want = 2 * std::min<uint64_t>(tile, (uint64_t)n_cells + 1);
+  uint32_t ch = FT;
+  while (ch < want) ch <<= 1;
+  if (ch > FUSED_CH_MAX) return false;
+  const size_t smem = fused_smem((uint32_t)tile, ch);
+  if (smem > 227 * 1024) return false;
+  p->grid = (uint32_t)grid;
+  p->tile = (uint32_t)tile;
+  p->ch = ch;
+  p->smem = smem;
+  return true;
+}
+
+cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
+                                const DevState& s, const IngestPlan& p, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_ingest_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    attr = true;
+  }
+  uint32_t tile = p.tile, ch = p.ch;
+  DevGraph gg_ = g;
+  DevState ss = s;
+  void* args[] = {(void*)&upd, (void*)&n, (void*)&seq0, (void*)&tile, (void*)&ch, (void*)&gg_, (void*)&ss};
+  // cooperative: every CTA is resident at once (the grid barriers need it), or the launch fails
+  return cudaLaunchCooperativeKernel((const void*)k_ingest_fused, dim3(p.grid), dim3(FT), args, p.smem, st);
 }
 
 // ---------------------------------------------------------------------------------------

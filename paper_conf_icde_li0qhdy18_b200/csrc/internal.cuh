@@ -56,6 +56,7 @@ struct DevStatus {
   unsigned int n_chain;     // queries the starting level promoted into the chained level this round
   unsigned int l0_exited;   // CTAs of the starting level's launch that have exited this round
   unsigned int round_end;   // (marks the end of the per-round reset region)
+  unsigned int ingest_bar;  // grid-barrier arrivals of the fused ingest launch (reset per batch)
 };
 
 struct DevGraph {
@@ -183,7 +184,16 @@ void launch_query_owner(const uint2* q, uint32_t nq, const DevGraph& g, const De
 // k-way merge of n_lists ascending (dist, obj) lists per query, layout [n_lists][n_q][k]
 void launch_merge_topk(uint32_t n_lists, uint32_t n_q, uint32_t k, const uint32_t* lobj,
                        const uint32_t* ldist, uint32_t* out_obj, uint32_t* out_dist, cudaStream_t st);
-size_t ingest_tmp_bytes(uint64_t n);  // classify -> scatter scratch (tmp + perm)
+size_t ingest_tmp_bytes(uint64_t n);
+// single-launch ingest (classify + alloc + scatter with grid barriers) for batches that fit
+// one resident wave; ingest_fused_plan returns false when the batch does not
+struct IngestPlan {
+  uint32_t grid, tile, ch;
+  size_t smem;
+};
+bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p);
+cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
+                                const DevState& s, const IngestPlan& p, cudaStream_t st);  // classify -> scatter scratch (tmp + perm)
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st);

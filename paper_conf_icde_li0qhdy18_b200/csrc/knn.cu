@@ -930,6 +930,9 @@ static uint32_t blocks_per_sm(int level, bool cta) {
       cudaFuncSetAttribute(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32, smem);
     }
+#ifdef GG_L0_PER_SM
+    if (!cta && level == 0) b = std::min(b, GG_L0_PER_SM);  // experiment hook: occupancy cap
+#endif
     if (b <= 0) b = 1;
   }
   return (uint32_t)b;
