@@ -338,9 +338,13 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   extern __shared__ __align__(16) uint32_t f_buf[];
   uint32_t* h_cell = f_buf;          // [ch] cell id (REMOTE_CELL: other ranks' updates)
   uint32_t* h_cnt = f_buf + ch;      // [ch] count; after the scan (tile offset << 16) | count
-  uint32_t* h_aux = f_buf + 2 * ch;  // [ch] newest t; after the claim, the cell's batch rank base
-  uint2* stg = reinterpret_cast<uint2*>(f_buf + 3 * ch);    // [tile] (src vertex, rank), cell order
-  uint16_t* stp = reinterpret_cast<uint16_t*>(stg + tile);  // [tile] index in the tile
+  uint32_t* h_aux = f_buf + 2 * ch;  // [ch] newest t; then the cell's batch rank base; then the
+                                     //      arena position of the group's first record minus its
+                                     //      tile offset
+  uint4* srec = reinterpret_cast<uint4*>(f_buf + 3 * ch);   // [tile] the records, tile order
+  uint2* stg = reinterpret_cast<uint2*>(srec + tile);       // [tile] (src vertex, slot | flags),
+                                                            //        cell order
+  uint16_t* stp = reinterpret_cast<uint16_t*>(stg + tile);  // [tile] tile index, cell order
   uint32_t* w_sum = reinterpret_cast<uint32_t*>(stp + ((tile + 1) & ~1u));  // [FT / 32]
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const unsigned G = gridDim.x;
@@ -353,22 +357,30 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   const uint64_t base = (uint64_t)blockIdx.x * tile;
   const uint32_t nt = base >= n ? 0u : (uint32_t)min((uint64_t)tile, n - base);
 
-  // ---- classify: validate, cell via the inverted index, rank within the tile's cell group
+  // ---- classify: validate, cell via the inverted index, rank within the tile's cell group;
+  //      the object's current key is read here too (in the same memory round as the inverted
+  //      index): ot_key only grows, so "not newer than this value" still means no atomic is
+  //      needed at the scatter, and a value of 0 marks a possibly new object
   uint32_t sr[FPT];  // (hash slot << 16) | rank in the slot's group, NONE: no record
   uint32_t vs[FPT];
+  uint32_t fl = 0;   // 2 bits per update: 1 = newer than the key read, 2 = key read was 0
   uint32_t tl = 0;
   constexpr int HP = FPT / 2;
 #pragma unroll
   for (int hf = 0; hf < 2; ++hf) {  // two halves: a half's loads and gathers in flight together
     uint4 mm[HP];
     uint2 ee[HP];
+    unsigned long long ck[HP];
 #pragma unroll
     for (int q = 0; q < HP; ++q) {
       const uint32_t k = (uint32_t)((hf * HP + q) * FT + tid);
-      mm[q] = k < nt ? __ldg(upd + base + k) : make_uint4(0, 0xFFFFFFFFu, 0, 0);
+      mm[q] = k < nt ? __ldcs(upd + base + k) : make_uint4(0, 0xFFFFFFFFu, 0, 0);
     }
 #pragma unroll
-    for (int q = 0; q < HP; ++q) ee[q] = mm[q].y < g.A ? __ldg(g.einfo + mm[q].y) : make_uint2(0, 1);
+    for (int q = 0; q < HP; ++q) {
+      ee[q] = mm[q].y < g.A ? __ldg(g.einfo + mm[q].y) : make_uint2(0, 1);
+      ck[q] = mm[q].x < s.max_objects ? __ldcg(s.ot_key + mm[q].x) : 0ull;
+    }
 #pragma unroll
     for (int q = 0; q < HP; ++q) {
       const int j = hf * HP + q;
@@ -378,6 +390,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
       if (k >= nt) continue;
       const uint4 m = mm[q];
       const uint2 e = ee[q];
+      srec[k] = m;
       unsigned bad = 0;
       if (m.x >= s.max_objects) bad |= ERR_OBJ;
       if (m.y >= g.A) {
@@ -391,6 +404,9 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
         atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
         continue;
       }
+      const unsigned long long key =
+          ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + k));
+      fl |= ((key > ck[q] ? 1u : 0u) | (ck[q] == 0ull ? 2u : 0u)) << (2 * j);
       const uint32_t c0 = cellof(g, e.x);
       const bool remote = s.n_ranks > 1 && owner_of(c0, g.n_cells, s.n_ranks) != s.rank;
       const uint32_t c = remote ? REMOTE_CELL : c0;
@@ -446,9 +462,9 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
 #pragma unroll
   for (int j = 0; j < FPT; ++j) {
     if (sr[j] == NONE) continue;
-    const uint32_t slot = sr[j] >> 16, lr = sr[j] & 0xFFFFu;
-    const uint32_t si = (h_cnt[slot] >> 16) + lr;
-    stg[si] = make_uint2(vs[j], h_cell[slot] == REMOTE_CELL ? NONE : h_aux[slot] + lr);
+    const uint32_t slot = sr[j] >> 16;
+    const uint32_t si = (h_cnt[slot] >> 16) + (sr[j] & 0xFFFFu);
+    stg[si] = make_uint2(vs[j], slot | (((fl >> (2 * j)) & 3u) << 16));
     stp[si] = (uint16_t)(j * FT + tid);
   }
 
@@ -463,49 +479,43 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   grid_barrier(&s.st->ingest_bar, 2 * G);
   if (*((volatile unsigned*)&s.st->ingest_err)) return;  // the batch is rejected as a whole
 
-  // ---- scatter in cell order (consecutive threads write consecutive extent positions)
-  for (uint32_t k0 = 0; k0 < nt; k0 += FT * HP) {
-    uint32_t pos[HP], il[HP];
-    uint32_t vx[HP];
-    uint4 m[HP];
-    unsigned long long cur[HP];
-#pragma unroll
-    for (int q = 0; q < HP; ++q) {
-      const uint32_t k = k0 + (uint32_t)(q * FT + tid);
-      if (k < nt) {
-        const uint2 vr = stg[k];
-        il[q] = stp[k];
-        vx[q] = vr.x;
-        m[q] = __ldcs(upd + base + il[q]);  // (an L2 hit: read by this CTA in the classify)
-        pos[q] = vr.y == NONE ? NONE : s.bbase[cellof(g, vr.x)] + vr.y;
-        cur[q] = __ldcg(s.ot_key + m[q].x);
-      }
+  // ---- scatter in cell order (consecutive threads write consecutive extent positions);
+  //      everything it reads is in shared memory but the extents' bases (one per group)
+  for (uint32_t i = tid; i < ch; i += FT) {
+    const uint32_t c = h_cell[i];
+    if (c != NONE && c != REMOTE_CELL) h_aux[i] = s.bbase[c] + h_aux[i] - (h_cnt[i] >> 16);
+  }
+  __syncthreads();
+#pragma unroll 4
+  for (uint32_t si = tid; si < nt; si += FT) {
+    const uint2 x = stg[si];
+    const uint32_t k = stp[si];
+    const uint4 m = srec[k];
+    const uint32_t slot = x.y & 0xFFFFu, f = x.y >> 16;
+    const unsigned long long key =
+        ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + k));
+    if (h_cell[slot] != REMOTE_CELL) {  // (REMOTE_CELL: a cell another rank owns)
+      const uint32_t pos = h_aux[slot] + si;
+      s.ar.obj[pos] = m.x;
+      s.ar.key[pos] = key;
+      s.ar.vsrc[pos] = x.x;
+      s.ar.off[pos] = m.z;
+      s.ar.edge[pos] = m.y;
     }
-#pragma unroll
-    for (int q = 0; q < HP; ++q) {
-      const uint32_t k = k0 + (uint32_t)(q * FT + tid);
-      if (k >= nt) continue;
-      const unsigned long long key =
-          ((unsigned long long)m[q].w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + il[q]));
-      if (pos[q] != NONE) {
-        s.ar.obj[pos[q]] = m[q].x;
-        s.ar.key[pos[q]] = key;
-        s.ar.vsrc[pos[q]] = vx[q];
-        s.ar.off[pos[q]] = m[q].z;
-        s.ar.edge[pos[q]] = m[q].y;
-      }
-      if (cur[q] == 0ull) {
-        const unsigned long long old = atomicMax(&s.ot_key[m[q].x], key);
-        if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
-      } else if (key > cur[q]) {
-        atomicMax(&s.ot_key[m[q].x], key);
-      }
+    // ot_key only grows: a key not above the value read needs no atomic; a live object takes a
+    // fire-and-forget RED.MAX; only an object read as 0 needs the old value back, to count it
+    // live exactly once
+    if (f & 2u) {
+      const unsigned long long old = atomicMax(&s.ot_key[m.x], key);
+      if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+    } else if (f & 1u) {
+      atomicMax(&s.ot_key[m.x], key);
     }
   }
 }
 
 static size_t fused_smem(uint32_t tile, uint32_t ch) {
-  return (size_t)ch * 12 + (size_t)tile * 8 + (size_t)((tile + 1) & ~1u) * 2 + (FT / 32) * 4;
+  return (size_t)ch * 12 + (size_t)tile * 24 + (size_t)((tile + 1) & ~1u) * 2 + (FT / 32) * 4;
 }
 
 bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p) {

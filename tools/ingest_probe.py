@@ -19,7 +19,9 @@ g = synth.config_graph(cfg)
 walk = DeviceRandomWalk(g, n_obj)
 ticks = -(-batch // n_obj)
 u = walk.ticks(ticks)[:batch].contiguous()
-grid = gg.GGrid(g, 1024, max_objects=n_obj, profile=True, log_capacity=int(batch * (reps + 2) * 1.1))
+mode = int(os.environ.get("GG_INGEST_KERNELS", "0"))  # opts.ingest_kernels (3: three launches)
+grid = gg.GGrid(g, 1024, max_objects=n_obj, profile=True, log_capacity=int(batch * (reps + 2) * 1.1),
+                ingest_kernels=mode)
 grid.ingest(u)
 torch.cuda.synchronize()
 grid.stats_reset()
@@ -28,6 +30,6 @@ for _ in range(reps):
 st = grid.stats()
 km = st["kernel_ms"]
 tot = sum(km[k] for k in ("ingest_classify", "ingest_alloc", "ingest_scatter"))
-print(f"{cfg} |O|={n_obj} batch={batch}: classify {km['ingest_classify']/reps:.3f} alloc {km['ingest_alloc']/reps:.3f} "
+print(f"{cfg} mode={mode} |O|={n_obj} batch={batch}: classify {km['ingest_classify']/reps:.3f} alloc {km['ingest_alloc']/reps:.3f} "
       f"scatter {km['ingest_scatter']/reps:.3f} ms  -> {batch*reps/(tot/1e3)/1e9:.2f} G updates/s, "
       f"{48*batch*reps/(tot/1e3)/1e9:.0f} GB/s algorithmic")
