@@ -209,7 +209,8 @@ def run_ours(args, cfg_name):
         grid.shard(world, rank)
     out_o = torch.empty((Q, k), dtype=torch.int32, device="cuda")
     out_d = torch.empty((Q, k), dtype=torch.int32, device="cuda")
-    l2 = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")  # > 126 MB L2
+    # > 126 MB L2 (BENCH_L2_MB: diagnostics only, e.g. a longer flush lets the host run further ahead)
+    l2 = torch.empty(int(os.environ.get("BENCH_L2_MB", "256")) << 20, dtype=torch.uint8, device="cuda")
 
     def step_inputs(s):
         u = walk.ticks(cfg["updates_per_object"])

@@ -827,12 +827,23 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
   return DONE;
 }
 
-constexpr int CTA_W = 8;  // warps per query in the CTA variant
+// warps per query of the CTA variant: 2 at the starting level (the bench's balls of ~300
+// vertices: 16 vertices per window; measured 9% faster than one warp per query, 8% faster than
+// four), 8 at the larger levels (experiment hooks)
+#ifndef GG_CTA_W0
+#define GG_CTA_W0 2
+#endif
+#ifndef GG_CTA_W
+#define GG_CTA_W 8
+#endif
+constexpr int CTA_W0 = GG_CTA_W0, CTA_W = GG_CTA_W;
+__host__ __device__ constexpr int cta_warps(int level) { return level == 0 ? CTA_W0 : CTA_W; }
 #ifndef GG_CTA_LEVEL
-#define GG_CTA_LEVEL 1  // first level run CTA-per-query (experiment hook; level 0 stays per-warp)
+#define GG_CTA_LEVEL 0  // first level run CTA-per-query (experiment hook; 1: level 0 one warp per query)
 #endif
 
-__global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
+template <int W>
+__global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ CtaShared sh;
   __shared__ uint32_t qslot;
@@ -869,7 +880,7 @@ __global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
     const uint32_t qi = qslot;
     __syncthreads();
     if (qi == NONE) break;
-    const int r = run_query_cta<CTA_W>(P, m, sh, qi);
+    const int r = run_query_cta<W>(P, m, sh, qi);
     if (threadIdx.x == 0 && r != DONE) finish_undone(P, qi, r);
     __syncthreads();
   }
@@ -878,7 +889,8 @@ __global__ void __launch_bounds__(CTA_W * 32) k_expand_cta(QParams P) {
 
 // Capacity ladder.  Levels 0-4 keep the query's working set in shared memory (~10, 24, 45, 95
 // and 190 KB): level 0 one warp per query (as many single-warp CTAs per SM as fit), levels 1-4
-// one 8-warp CTA per query (k_expand_cta; measured faster from level 1 up, slower at level 0);
+// one CTA per query (k_expand_cta: 2 warps at level 0, 8 from level 1 up; one warp per query,
+// k_expand, measured slower at every level);
 // level 5 is global memory sized from |V| (a query that reaches fewer than k objects may need
 // to settle the whole graph).
 constexpr int NLEVELS = EXPAND_LEVELS;
@@ -924,8 +936,9 @@ static uint32_t blocks_per_sm(int level, bool cta) {
   if (!b) {
     const int smem = (int)expand_warp_bytes(level, 1);
     if (cta) {
-      cudaFuncSetAttribute(k_expand_cta, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand_cta, CTA_W * 32, smem);
+      auto kern = cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>;
+      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, cta_warps(level) * 32, smem);
     } else {
       cudaFuncSetAttribute(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32, smem);
@@ -983,7 +996,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   blocks_per_sm(level, cta);  // (sets the shared-memory attribute)
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
-  cfg.blockDim = dim3(cta ? CTA_W * 32 : 32);
+  cfg.blockDim = dim3(cta ? cta_warps(level) * 32 : 32);
   cfg.dynamicSmemBytes = (size_t)smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
@@ -992,7 +1005,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   cfg.attrs = attr;
   cfg.numAttrs = L.pdl ? 1 : 0;
   if (cta) {
-    cudaLaunchKernelEx(&cfg, k_expand_cta, P);
+    cudaLaunchKernelEx(&cfg, cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>, P);
   } else {
     cudaLaunchKernelEx(&cfg, k_expand<true>, P);
   }
