@@ -127,6 +127,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
 #pragma unroll
     for (int q = 0; q < SPC; ++q) h_cnt[tid * SPC + q] |= (excl + loc[q]) << 16;  // counts <= CU
   }
+  __syncthreads();  // (the claims below read other threads' slots)
   for (int i = tid; i < CH; i += CT) {
     const uint32_t c = h_cell[i];
     if (c != NONE && c != REMOTE_CELL) {
@@ -450,6 +451,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
       run += c;
     }
   }
+  __syncthreads();  // (the claims below read other threads' slots)
   // one claim per distinct cell of the tile on the batch counters
   for (uint32_t i = tid; i < ch; i += FT) {
     const uint32_t c = h_cell[i];

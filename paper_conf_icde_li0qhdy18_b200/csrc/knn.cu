@@ -539,34 +539,27 @@ __global__ void k_expand(QParams P) {
 // phases of a round).  Used where one warp is too narrow: balls of thousands of vertices (the
 // larger levels, whose per-query tables would otherwise leave one or a few warps per SM) and
 // small batches, where the single query's latency is the metric ("G-Grid (L)", P@61891).
+template <int W>
 struct CtaShared {
-  uint32_t nf, nn, na, nc;
-  uint32_t flags;  // 1: retry (dirty cell met), 2: overflow
-  uint32_t red[32];
-  unsigned long long redl[32];
+  uint32_t nn[2], na[2];  // next-frontier and bucket sizes, by round parity (a round's counters
+                          // are reset one round later, when every thread has read them)
+  uint32_t nc;            // candidates
+  uint32_t flags;         // FL_RETRY (a dirty cell met) | FL_OVF (a capacity exceeded)
+  uint32_t red[2][W];     // per-warp next-frontier minimum, by round parity
+  uint32_t sum[W];
+  unsigned long long redl[W];
 };
 constexpr uint32_t FL_RETRY = 1, FL_OVF = 2;
 
 template <int W>
-__device__ __forceinline__ uint32_t block_min(uint32_t v, CtaShared& sh) {
-  v = __reduce_min_sync(0xffffffffu, v);
-  __syncthreads();
-  if ((threadIdx.x & 31) == 0) sh.red[threadIdx.x >> 5] = v;
-  __syncthreads();
-  uint32_t r = sh.red[0];
-#pragma unroll
-  for (int w = 1; w < W; ++w) r = min(r, sh.red[w]);
-  return r;
-}
-template <int W>
-__device__ __forceinline__ uint32_t block_sum(uint32_t v, CtaShared& sh) {
+__device__ __forceinline__ uint32_t block_sum(uint32_t v, CtaShared<W>& sh) {
   v = __reduce_add_sync(0xffffffffu, v);
   __syncthreads();
-  if ((threadIdx.x & 31) == 0) sh.red[threadIdx.x >> 5] = v;
+  if ((threadIdx.x & 31) == 0) sh.sum[threadIdx.x >> 5] = v;
   __syncthreads();
   uint32_t r = 0;
 #pragma unroll
-  for (int w = 0; w < W; ++w) r += sh.red[w];
+  for (int w = 0; w < W; ++w) r += sh.sum[w];
   return r;
 }
 
@@ -597,9 +590,10 @@ __device__ void block_sort(unsigned long long* a, uint32_t n, uint32_t cap) {
 }
 
 template <int W>
-__device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, uint32_t qi) {
+__device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& sh, uint32_t qi) {
   constexpr uint32_t T = W * 32;
-  const uint32_t tid = threadIdx.x;
+  const unsigned FULL = 0xffffffffu;
+  const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const DevGraph& g = P.g;
   const DevState& s = P.s;
   const Caps& cp = P.caps;
@@ -613,7 +607,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
   for (uint32_t i = tid; i < (H + 31) / 32; i += T) m.fin[i] = 0;
   for (uint32_t i = tid; i < (H + 3) / 4; i += T) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
   if (tid == 0) {
-    sh.nf = 0;
+    sh.nn[0] = sh.nn[1] = sh.na[0] = sh.na[1] = 0;
     sh.nc = 0;
     sh.flags = 0;
   }
@@ -630,21 +624,19 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
     const uint32_t o = owner_of(cellof(g, ei.x), g.n_cells, s.n_ranks);
     if (o != s.rank) rmask |= 1ull << o;
   }
+  const uint32_t seed_d = q.y == 0 ? 0u : ei.y - q.y;
   if (tid == 0) {
     const uint32_t seed_v = q.y == 0 ? ei.x : g.edst[q.x];
-    const uint32_t seed_d = q.y == 0 ? 0u : ei.y - q.y;
     bool imp;
     const int sl = tab_relax(m, H, seed_v, seed_d, imp);
     m.front0[0] = (uint32_t)sl;
     m.fin[sl >> 5] |= 1u << (sl & 31);
-    sh.nf = 1;
   }
   // objects on q's own arc ahead of q (reading R2), stored at vertex src(q.e)
   if (q.y > 0) {
     const uint32_t c = cellof(g, ei.x);
     if (s.cell_head[c] != NONE) {
       if (tid == 0) request_flush(s, c, P.epoch);
-      __syncthreads();
       return RETRY;
     }
     const uint2 vo = vobj_valid(s.v_obj[ei.x], s.cell_comp[c]);
@@ -666,40 +658,46 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
 
   uint32_t* front = m.front0;
   uint32_t* nfront = m.front1;
+  // frontier size and minimum: the next frontier holds the re-queued entries (their D read at
+  // partition) and every vertex improved during the round (each improvement's new D is seen
+  // here), so the minimum over those is exact
+  uint32_t nf = 1, blo = seed_d;
   uint32_t c_iter = 0, c_vert = 0, c_arcs = 0, c_harv = 0, c_objs = 0;
-  for (;;) {
+  for (uint32_t rnd = 0;; ++rnd) {
+    const uint32_t par = rnd & 1;
     ++c_iter;
-    const uint32_t nf = sh.nf;
-    uint32_t ml = INF;
-    for (uint32_t i = tid; i < nf; i += T) ml = min(ml, m.dist[front[i]]);
-    const uint32_t blo = block_min<W>(ml, sh);
+    // ---- 1. termination (nf, blo and the candidates are the same for every thread)
     if (nf == 0 || blo > lim) break;
     const uint32_t nc0 = sh.nc;
-    if (nc0 >= k) {
+    if (nc0 >= k) {  // every warp counts every candidate: the same total, no block reduction
       uint32_t cl = 0;
-      for (uint32_t i = tid; i < nc0; i += T) cl += cand_dist(m, i) < blo;
-      if (block_sum<W>(cl, sh) >= k) break;
+      for (uint32_t i = lane; i < nc0; i += 32) cl += cand_dist(m, i) < blo;
+      if (__reduce_add_sync(FULL, cl) >= k) break;
     }
-    // partition the frontier: the bucket [m, m + delta) is expanded, the rest re-queued
+    // ---- 2. partition the frontier: the bucket [m, m + delta) is expanded, the rest re-queued
     const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
-    if (tid == 0) {
-      sh.na = 0;
-      sh.nn = 0;
-    }
-    __syncthreads();
+    uint32_t mn = INF;
     for (uint32_t i = tid; i < nf; i += T) {
       const uint32_t sl = front[i];
-      if (m.dist[sl] < bhi) {
-        m.act[atomicAdd(&sh.na, 1u)] = sl;  // (act has F entries: na <= nf <= F)
+      const uint32_t ent = m.dist[sl];
+      if (ent < bhi) {
+        m.act[atomicAdd(&sh.na[par], 1u)] = sl;  // (act has F entries: na <= nf <= F)
         atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
       } else {
-        nfront[atomicAdd(&sh.nn, 1u)] = sl;
+        nfront[atomicAdd(&sh.nn[par], 1u)] = sl;
+        mn = min(mn, ent);
       }
     }
-    __syncthreads();
-    const uint32_t na = sh.na;
-    if (tid == 0) c_vert += na;
-    // expand: lane = (vertex, arc slot), T/4 vertices per window
+    __syncthreads();  // the bucket is complete
+    const uint32_t na = sh.na[par];
+    if (tid == 0) {  // the next round's counters (their last readers are past the barrier)
+      sh.nn[par ^ 1] = 0;
+      sh.na[par ^ 1] = 0;
+      c_vert += na;
+    }
+    // ---- 3. expand: lane = (vertex, arc slot), T/4 vertices per window; no barrier between
+    //         windows (appends and candidates are reserved with shared atomics; the outcome
+    //         flags are read at the end of the round)
     for (uint32_t w0 = 0; w0 < na; w0 += T / 4) {
       const uint32_t vi = w0 + (tid >> 2), s4 = tid & 3;
       if (vi < na) {
@@ -726,9 +724,10 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
           if (rr < 0) {
             atomicOr(&sh.flags, FL_OVF);
           } else if (imp) {
+            mn = min(mn, (uint32_t)nd);
             const uint32_t bit = 1u << (rr & 31);
             if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
-              const uint32_t p = atomicAdd(&sh.nn, 1u);
+              const uint32_t p = atomicAdd(&sh.nn[par], 1u);
               if (p < cp.F) nfront[p] = (uint32_t)rr;
               else atomicOr(&sh.flags, FL_OVF);
             }
@@ -773,22 +772,29 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
           }
         }
       }
-      __syncthreads();
-      const uint32_t fl = sh.flags;
-      if (fl & FL_OVF) return OVERFLOW;
-      if (fl & FL_RETRY) {
-        for (uint32_t i = tid; i < nf; i += T)
-          request_flush(s, cellof(g, m.key[front[i]]), P.epoch);
-        return RETRY;
-      }
     }
+    // ---- 4. round complete: the next frontier's minimum, the outcome flags
+    mn = __reduce_min_sync(FULL, mn);
+    if (lane == 0) sh.red[par][wid] = mn;
+    __syncthreads();
+    const uint32_t fl = sh.flags;
+    if (fl & FL_OVF) return OVERFLOW;
+    if (fl & FL_RETRY) {  // ask for every dirty cell the frontier will need, then retry
+      for (uint32_t i = tid; i < nf; i += T) request_flush(s, cellof(g, m.key[front[i]]), P.epoch);
+      return RETRY;
+    }
+    blo = sh.red[par][0];
+#pragma unroll
+    for (int w = 1; w < W; ++w) blo = min(blo, sh.red[par][w]);
+    nf = sh.nn[par];
     uint32_t* tmp = front;
     front = nfront;
     nfront = tmp;
-    if (tid == 0) sh.nf = sh.nn;
-    __syncthreads();
   }
 
+  // every warp leaves the loop in the same round; the barrier keeps a warp from rewriting the
+  // candidates below while another is still counting them for the termination test
+  __syncthreads();
   // the k smallest (dist, obj)
   const uint32_t nc = sh.nc;
   for (uint32_t i = tid; i < nc; i += T) {
@@ -805,9 +811,9 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
   }
   if (P.remote) {
     unsigned long long x = rmask;
-    x = ((unsigned long long)__reduce_or_sync(0xffffffffu, (uint32_t)(x >> 32)) << 32) |
-        __reduce_or_sync(0xffffffffu, (uint32_t)x);
-    if ((tid & 31) == 0) sh.redl[tid >> 5] = x;
+    x = ((unsigned long long)__reduce_or_sync(FULL, (uint32_t)(x >> 32)) << 32) |
+        __reduce_or_sync(FULL, (uint32_t)x);
+    if (lane == 0) sh.redl[wid] = x;
     __syncthreads();
     if (tid == 0) {
       unsigned long long r = 0;
@@ -827,11 +833,11 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared& sh, 
   return DONE;
 }
 
-// warps per query of the CTA variant: 2 at the starting level (the bench's balls of ~300
-// vertices: 16 vertices per window; measured 9% faster than one warp per query, 8% faster than
-// four), 8 at the larger levels (experiment hooks)
+// warps per query of the CTA variant: 3 at the starting level (the bench's balls of ~300
+// vertices, ~17 per round: one window of 24 vertices per round; measured 3 > 2 > 4 > 1 warps
+// per query), 8 at the larger levels (experiment hooks)
 #ifndef GG_CTA_W0
-#define GG_CTA_W0 2
+#define GG_CTA_W0 3
 #endif
 #ifndef GG_CTA_W
 #define GG_CTA_W 8
@@ -845,7 +851,7 @@ __host__ __device__ constexpr int cta_warps(int level) { return level == 0 ? CTA
 template <int W>
 __global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  __shared__ CtaShared sh;
+  __shared__ CtaShared<W> sh;
   __shared__ uint32_t qslot;
   const WarpMem m = carve(smem_raw, P.caps);
   pdl_trigger(P);
@@ -889,7 +895,7 @@ __global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
 
 // Capacity ladder.  Levels 0-4 keep the query's working set in shared memory (~10, 24, 45, 95
 // and 190 KB): level 0 one warp per query (as many single-warp CTAs per SM as fit), levels 1-4
-// one CTA per query (k_expand_cta: 2 warps at level 0, 8 from level 1 up; one warp per query,
+// one CTA per query (k_expand_cta: 3 warps at level 0, 8 from level 1 up; one warp per query,
 // k_expand, measured slower at every level);
 // level 5 is global memory sized from |V| (a query that reaches fewer than k objects may need
 // to settle the whole graph).
@@ -936,7 +942,7 @@ static uint32_t blocks_per_sm(int level, bool cta) {
   if (!b) {
     const int smem = (int)expand_warp_bytes(level, 1);
     if (cta) {
-      auto kern = cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>;
+      auto kern = level == 0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>;
       cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, cta_warps(level) * 32, smem);
     } else {
@@ -1005,7 +1011,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   cfg.attrs = attr;
   cfg.numAttrs = L.pdl ? 1 : 0;
   if (cta) {
-    cudaLaunchKernelEx(&cfg, cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>, P);
+    cudaLaunchKernelEx(&cfg, level == 0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>, P);
   } else {
     cudaLaunchKernelEx(&cfg, k_expand<true>, P);
   }
