@@ -833,11 +833,12 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
   return DONE;
 }
 
-// warps per query of the CTA variant: 3 at the starting level (the bench's balls of ~300
-// vertices, ~17 per round: one window of 24 vertices per round; measured 3 > 2 > 4 > 1 warps
-// per query), 8 at the larger levels (experiment hooks)
+// warps per query of the CTA variant: 4 at the starting level (the bench's balls of ~300
+// vertices, ~17 per round: one window of 32 vertices per round; measured 4 > 3 > 5 > 2 > 6 > 8
+// warps per query, and one warp per query slower than all but 8), 8 at the larger levels
+// (experiment hooks)
 #ifndef GG_CTA_W0
-#define GG_CTA_W0 3
+#define GG_CTA_W0 4
 #endif
 #ifndef GG_CTA_W
 #define GG_CTA_W 8
@@ -895,7 +896,7 @@ __global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
 
 // Capacity ladder.  Levels 0-4 keep the query's working set in shared memory (~10, 24, 45, 95
 // and 190 KB): level 0 one warp per query (as many single-warp CTAs per SM as fit), levels 1-4
-// one CTA per query (k_expand_cta: 3 warps at level 0, 8 from level 1 up; one warp per query,
+// one CTA per query (k_expand_cta: 4 warps at level 0, 8 from level 1 up; one warp per query,
 // k_expand, measured slower at every level);
 // level 5 is global memory sized from |V| (a query that reaches fewer than k objects may need
 // to settle the whole graph).
