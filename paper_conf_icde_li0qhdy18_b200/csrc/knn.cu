@@ -836,7 +836,9 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
 // warps per query of the CTA variant: 4 at the starting level (the bench's balls of ~300
 // vertices, ~17 per round: one window of 32 vertices per round; measured 4 > 3 > 5 > 2 > 6 > 8
 // warps per query, and one warp per query slower than all but 8), 8 at the larger levels
-// (experiment hooks)
+// (experiment hooks).  ptxas fits the 4-warp kernel in 32 registers (a few bytes of spills),
+// i.e. 16 CTAs = 64 warps per SM; capping it at 40-56 registers (launch-bounds min blocks
+// 12-1) measured 8-23% slower.
 #ifndef GG_CTA_W0
 #define GG_CTA_W0 4
 #endif
