@@ -10,10 +10,12 @@ export BENCH_ALLOW_SHORT=1
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_C1.csv \
     python bench.py --steps 2 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $OUT/launches_C1.log 2>&1
 echo "launch list rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k "regex:k_expand(<true>)?$" -s 3 -c 1 \
+# the starting level's kernel (k_expand_cta<4>) alternates with the chained level's (<8>): the 5th match
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_expand_cta -s 4 -c 1 \
     -o $OUT/expand_C1 python bench.py --steps 1 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $OUT/expand_C1.log 2>&1
 echo "expand rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_ingest -s 6 -c 3 \
+# one fused ingest launch per step (batches that fit one resident wave)
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_ingest -s 3 -c 1 \
     -o $OUT/ingest_C1 python bench.py --steps 1 --warmup 3 --no-cpu-baseline --e2e-steps 1 > $OUT/ingest_C1.log 2>&1
 echo "ingest rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_flush -s 1 -c 1 \

@@ -102,6 +102,6 @@ if os.path.exists(ll):
 
 open(os.path.join(dst, f"{tag}_summary.md"), "w").write("\n".join(lines) + "\n")
 for cfg, d in traffic.items():
-    # ingest capture holds 3 launches (classify, alloc, scatter) of one step: per-step bytes
+    # per launch: expand (the starting level), ingest (one fused launch per step), flush (C3)
     json.dump({k: v for k, v in d.items()}, open(os.path.join(dst, f"traffic_{cfg}.json"), "w"), indent=1)
 print("\n".join(lines))
