@@ -766,6 +766,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   const double ball = (double)k * h->V / (double)std::max<uint64_t>(1, h->n_live_hi());
   while (lvl0 < L - 2 && (k > expand_max_k(lvl0) || GG_BALL_FACTOR * ball > expand_table_slots(lvl0))) lvl0++;
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
+  const uint32_t ball_hint = (uint32_t)std::min(ball, 4.0e9);
   std::vector<uint32_t> n_in(L, 0);
   n_in[lvl0] = n_q;
   // The level above the starting one runs in the same round BESIDE it (a programmatic
@@ -799,10 +800,10 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
       RC(h->set_words(ws));
     }
     const bool conc = chain >= 0 && n_in[lvl0] > 0;
-    const uint32_t grid_c = conc ? std::min<uint32_t>(expand_grid(chain, n_q, h->sm_count), n_in[chain] + 16) : 0;
+    const uint32_t grid_c = conc ? std::min<uint32_t>(expand_grid(chain, n_q, h->sm_count, ball_hint), n_in[chain] + 16) : 0;
     uint32_t grid0 = 0;
     if (conc) {  // leave room for the chained level's CTAs (so they are resident from the start)
-      const uint32_t full = expand_grid(lvl0, n_in[lvl0], h->sm_count);
+      const uint32_t full = expand_grid(lvl0, n_in[lvl0], h->sm_count, ball_hint);
       const size_t b0 = expand_warp_bytes(lvl0, h->V) + 1024, bc = expand_warp_bytes(chain, h->V) + 1024;
       const uint32_t reserve = (uint32_t)(grid_c * ((bc + b0 - 1) / b0));
       grid0 = full > reserve + h->sm_count ? full - reserve : full;
@@ -822,6 +823,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
       E.out_dist = d_od;
       E.bound = d_bound;
       E.remote = d_remote;
+      E.ball_hint = ball_hint;
       return E;
     };
     for (int lvl = 0; lvl < L; ++lvl) {

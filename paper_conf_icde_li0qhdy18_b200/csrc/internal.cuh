@@ -252,9 +252,10 @@ struct ExpandLaunch {
   uint32_t grid = 0;                // 0: the default (expand_grid)
   bool trigger = false;             // let the next kernel of the stream start now (PDL)
   bool pdl = false;                 // launched as a programmatic dependent of the previous kernel
+  uint32_t ball_hint = 0xFFFFFFFFu;  // expected ball (vertices): picks the starting level's variant
 };
-// CTAs launch_expand uses for n queries at `level`
-uint32_t expand_grid(int level, uint32_t n, int sm_count);
+// CTAs launch_expand uses for n queries at `level` (ball_hint: expected ball in vertices)
+uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint);
 void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st);
 // prior-art comparison path (csrc/prior_art.cu)
 int prior_art_mu(int eta);

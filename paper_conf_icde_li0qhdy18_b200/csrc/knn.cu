@@ -933,9 +933,16 @@ size_t expand_warp_bytes(int level, uint32_t V) {
   return (warpmem_bytes(c) + 15) & ~size_t(15);
 }
 
-// CTA-per-query for the big shared-memory levels, and for small batches at any of them
-static bool use_cta(int level, uint32_t n, int sm_count) {
-  return level < NLEVELS - 1 && (level >= GG_CTA_LEVEL || n <= (uint32_t)sm_count);
+// CTA-per-query for the shared-memory levels, and for small batches at any of them; the
+// starting level runs one warp per query when the caller expects small balls (ball_hint below
+// kCtaBall vertices: measured C2 k=10, ball ~110: one warp 0.179 ms vs 4 warps 0.194 ms; C3,
+// ~240: 36.9 vs 36.3M q/s; C1, ~260: 0.330 vs 0.273 ms; C2 k=30, ~320: 0.398 vs 0.345 ms)
+constexpr uint32_t kCtaBall = 256;
+static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
+  if (level >= NLEVELS - 1) return false;
+  if (n <= (uint32_t)sm_count) return true;
+  if (level == 0) return GG_CTA_LEVEL == 0 && ball_hint >= kCtaBall;
+  return true;
 }
 
 // resident CTAs per SM of a shared-memory level's kernel (occupancy calculator, cached)
@@ -960,9 +967,9 @@ static uint32_t blocks_per_sm(int level, bool cta) {
   return (uint32_t)b;
 }
 
-uint32_t expand_grid(int level, uint32_t n, int sm_count) {
+uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level == NLEVELS - 1) return 0;  // (global scratch: sized by the caller's scratch warps)
-  return std::min<uint32_t>(n, (uint32_t)sm_count * blocks_per_sm(level, use_cta(level, n, sm_count)));
+  return std::min<uint32_t>(n, (uint32_t)sm_count * blocks_per_sm(level, use_cta(level, n, sm_count, ball_hint)));
 }
 
 void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st) {
@@ -1000,8 +1007,8 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
     k_expand<false><<<std::min<uint32_t>(L.n, std::max<uint32_t>(1, L.scratch_warps)), 32, 0, st>>>(P);
     return;
   }
-  const bool cta = L.chain_in != nullptr || use_cta(level, L.n, sm_count);
-  const uint32_t grid = L.grid ? L.grid : std::max<uint32_t>(1, expand_grid(level, L.n, sm_count));
+  const bool cta = L.chain_in != nullptr || use_cta(level, L.n, sm_count, L.ball_hint);
+  const uint32_t grid = L.grid ? L.grid : std::max<uint32_t>(1, expand_grid(level, L.n, sm_count, L.ball_hint));
   blocks_per_sm(level, cta);  // (sets the shared-memory attribute)
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
