@@ -21,7 +21,7 @@ constexpr uint32_t NONE = 0xFFFFFFFFu;
 constexpr uint32_t INF = 0xFFFFFFFFu;  // u32 distance "unreachable" (reading R18)
 constexpr unsigned long long EMPTY64 = ~0ull;
 constexpr uint32_t BCOUNT_STRIDE = 32;
-constexpr int EXPAND_LEVELS = 6;  // capacity ladder of the expansion (csrc/knn.cu)
+constexpr int EXPAND_LEVELS = 7;  // capacity ladder of the expansion (csrc/knn.cu)
 
 enum ErrBits : unsigned {
   ERR_OBJ = 1u,      // update obj >= max_objects

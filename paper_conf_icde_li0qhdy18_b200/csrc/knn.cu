@@ -846,7 +846,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
 #define GG_CTA_W 8
 #endif
 constexpr int CTA_W0 = GG_CTA_W0, CTA_W = GG_CTA_W;
-__host__ __device__ constexpr int cta_warps(int level) { return level == 0 ? CTA_W0 : CTA_W; }
+__host__ __device__ constexpr int cta_warps(int level) { return level <= 1 ? CTA_W0 : CTA_W; }
 #ifndef GG_CTA_LEVEL
 #define GG_CTA_LEVEL 0  // first level run CTA-per-query (experiment hook; 1: level 0 one warp per query)
 #endif
@@ -896,12 +896,11 @@ __global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
   if (threadIdx.x == 0) count_exit(P);
 }
 
-// Capacity ladder.  Levels 0-4 keep the query's working set in shared memory (~10, 24, 45, 95
-// and 190 KB): level 0 one warp per query (as many single-warp CTAs per SM as fit), levels 1-4
-// one CTA per query (k_expand_cta: 4 warps at level 0, 8 from level 1 up; one warp per query,
-// k_expand, measured slower at every level);
-// level 5 is global memory sized from |V| (a query that reaches fewer than k objects may need
-// to settle the whole graph).
+// Capacity ladder.  Levels 0-5 keep the query's working set in shared memory (~11, 15, 28, 45,
+// 95 and 190 KB): level 0 one warp per query when small balls are expected (as many
+// single-warp CTAs per SM as fit), else, like levels 1-5, one CTA per query (k_expand_cta: 4
+// warps at levels 0-1, 8 above); level 6 is global memory sized from |V| (a query that reaches
+// fewer than k objects may need to settle the whole graph).
 constexpr int NLEVELS = EXPAND_LEVELS;
 #ifndef GG_H0
 #define GG_H0 1024  // level-0 vertex table (experiment hook: -DGG_H0=..., -DGG_F0=...)
@@ -909,8 +908,15 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 #ifndef GG_F0
 #define GG_F0 96
 #endif
-const Caps kCaps[NLEVELS - 1] = {
-    {GG_H0, GG_F0, 64}, {2048, 512, 256}, {4096, 1024, 256}, {8192, 2048, 512}, {16384, 4096, 2048}};
+#ifndef GG_C0
+#define GG_C0 64
+#endif
+// level 1 takes 32 < k <= 96 (measured C2 k=40: 0.47 ms there vs 0.68 ms at the 2048-slot level;
+// widening level 0's candidate list instead cost the k=10 configs 2-4%).  Candidate capacities
+// are powers of two: the bitonic sorts pad to one.
+const Caps kCaps[NLEVELS - 1] = {{GG_H0, GG_F0, GG_C0}, {1280, 128, 128}, {2048, 512, 256},
+                                 {4096, 1024, 256},     {8192, 2048, 512}, {16384, 4096, 2048}};
+static_assert((GG_C0 & (GG_C0 - 1)) == 0, "candidate capacity must be a power of two");
 
 Caps caps_for(int level, uint32_t V) {
   if (level < NLEVELS - 1) return kCaps[level];
@@ -952,7 +958,7 @@ static uint32_t blocks_per_sm(int level, bool cta) {
   if (!b) {
     const int smem = (int)expand_warp_bytes(level, 1);
     if (cta) {
-      auto kern = level == 0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>;
+      auto kern = cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>;
       cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, cta_warps(level) * 32, smem);
     } else {
@@ -1021,7 +1027,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   cfg.attrs = attr;
   cfg.numAttrs = L.pdl ? 1 : 0;
   if (cta) {
-    cudaLaunchKernelEx(&cfg, level == 0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>, P);
+    cudaLaunchKernelEx(&cfg, cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>, P);
   } else {
     cudaLaunchKernelEx(&cfg, k_expand<true>, P);
   }
