@@ -589,14 +589,26 @@ __device__ void block_sort(unsigned long long* a, uint32_t n, uint32_t cap) {
   }
 }
 
-template <int W>
+// Capacities of a level: compile-time (constant shared-memory offsets and bounds: no registers
+// hold the working-memory pointers), or from the launch parameters.
+struct DynCaps {
+  __device__ static Caps get(const QParams& P) { return P.caps; }
+};
+template <uint32_t H_, uint32_t F_, uint32_t C_>
+struct FixCaps {
+  static_assert((C_ & (C_ - 1)) == 0, "candidate capacity must be a power of two");
+  __host__ __device__ static constexpr Caps get(const QParams&) { return Caps{H_, F_, C_}; }
+  static constexpr Caps caps() { return Caps{H_, F_, C_}; }
+};
+
+template <int W, class CP>
 __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& sh, uint32_t qi) {
   constexpr uint32_t T = W * 32;
   const unsigned FULL = 0xffffffffu;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const DevGraph& g = P.g;
   const DevState& s = P.s;
-  const Caps& cp = P.caps;
+  const Caps cp = CP::get(P);
   const uint32_t H = cp.H;
   const uint32_t k = P.k;
 
@@ -851,12 +863,19 @@ __host__ __device__ constexpr int cta_warps(int level) { return level <= 1 ? CTA
 #define GG_CTA_LEVEL 0  // first level run CTA-per-query (experiment hook; 1: level 0 one warp per query)
 #endif
 
-template <int W>
-__global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
+// resident CTAs per SM asked of ptxas (a register cap: 40) for the fixed-capacity level (level
+// 1; measured at C2 k=50: 0.496 ms vs 0.575 at 32 registers and 0.545 with runtime capacities).
+// Level 0 keeps runtime capacities: ptxas's own choice there (32 registers, 16 CTAs) measured
+// 3% faster at C1 than either fixed-capacity build.
+#ifndef GG_MINB0
+#define GG_MINB0 12
+#endif
+template <int W, class CP>
+__device__ __forceinline__ void expand_cta_body(const QParams& P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ CtaShared<W> sh;
   __shared__ uint32_t qslot;
-  const WarpMem m = carve(smem_raw, P.caps);
+  const WarpMem m = carve(smem_raw, CP::get(P));
   pdl_trigger(P);
   for (;;) {  // persistent: queries fetched dynamically
     if (threadIdx.x == 0) {
@@ -889,11 +908,20 @@ __global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
     const uint32_t qi = qslot;
     __syncthreads();
     if (qi == NONE) break;
-    const int r = run_query_cta<W>(P, m, sh, qi);
+    const int r = run_query_cta<W, CP>(P, m, sh, qi);
     if (threadIdx.x == 0 && r != DONE) finish_undone(P, qi, r);
     __syncthreads();
   }
   if (threadIdx.x == 0) count_exit(P);
+}
+// (two kernels: an explicit min-blocks launch bound changes ptxas's register choice even at 1)
+template <int W, class CP>
+__global__ void __launch_bounds__(W * 32) k_expand_cta(QParams P) {
+  expand_cta_body<W, CP>(P);
+}
+template <int W, class CP>
+__global__ void __launch_bounds__(W * 32, GG_MINB0) k_expand_cta_capped(QParams P) {
+  expand_cta_body<W, CP>(P);
 }
 
 // Capacity ladder.  Levels 0-5 keep the query's working set in shared memory (~11, 15, 28, 45,
@@ -914,9 +942,18 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 // level 1 takes 32 < k <= 96 (measured C2 k=40: 0.47 ms there vs 0.68 ms at the 2048-slot level;
 // widening level 0's candidate list instead cost the k=10 configs 2-4%).  Candidate capacities
 // are powers of two: the bitonic sorts pad to one.
-const Caps kCaps[NLEVELS - 1] = {{GG_H0, GG_F0, GG_C0}, {1280, 128, 128}, {2048, 512, 256},
-                                 {4096, 1024, 256},     {8192, 2048, 512}, {16384, 4096, 2048}};
-static_assert((GG_C0 & (GG_C0 - 1)) == 0, "candidate capacity must be a power of two");
+using Caps0 = FixCaps<GG_H0, GG_F0, GG_C0>;
+using Caps1 = FixCaps<1280, 128, 128>;
+const Caps kCaps[NLEVELS - 1] = {Caps0::caps(),     Caps1::caps(),     {2048, 512, 256},
+                                 {4096, 1024, 256}, {8192, 2048, 512}, {16384, 4096, 2048}};
+
+// the CTA kernel of a shared-memory level
+using CtaKernel = void (*)(QParams);
+static CtaKernel cta_kernel(int level) {
+  if (level == 0) return k_expand_cta<CTA_W0, DynCaps>;
+  if (level == 1) return k_expand_cta_capped<CTA_W0, Caps1>;
+  return k_expand_cta<CTA_W, DynCaps>;
+}
 
 Caps caps_for(int level, uint32_t V) {
   if (level < NLEVELS - 1) return kCaps[level];
@@ -958,7 +995,7 @@ static uint32_t blocks_per_sm(int level, bool cta) {
   if (!b) {
     const int smem = (int)expand_warp_bytes(level, 1);
     if (cta) {
-      auto kern = cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>;
+      const CtaKernel kern = cta_kernel(level);
       cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, cta_warps(level) * 32, smem);
     } else {
@@ -1027,7 +1064,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   cfg.attrs = attr;
   cfg.numAttrs = L.pdl ? 1 : 0;
   if (cta) {
-    cudaLaunchKernelEx(&cfg, cta_warps(level) == CTA_W0 ? k_expand_cta<CTA_W0> : k_expand_cta<CTA_W>, P);
+    cudaLaunchKernelEx(&cfg, cta_kernel(level), P);
   } else {
     cudaLaunchKernelEx(&cfg, k_expand<true>, P);
   }
