@@ -543,6 +543,7 @@ template <int W>
 struct CtaShared {
   uint32_t nn[2], na[2];  // next-frontier and bucket sizes, by round parity (a round's counters
                           // are reset one round later, when every thread has read them)
+  uint32_t stop[2];       // termination verdict (k candidates closer than the frontier), by parity
   uint32_t nc;            // candidates
   uint32_t flags;         // FL_RETRY (a dirty cell met) | FL_OVF (a capacity exceeded)
   uint32_t red[2][W];     // per-warp next-frontier minimum, by round parity
@@ -620,6 +621,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
   for (uint32_t i = tid; i < (H + 3) / 4; i += T) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
   if (tid == 0) {
     sh.nn[0] = sh.nn[1] = sh.na[0] = sh.na[1] = 0;
+    sh.stop[0] = sh.stop[1] = 0;
     sh.nc = 0;
     sh.flags = 0;
   }
@@ -680,11 +682,13 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
     ++c_iter;
     // ---- 1. termination (nf, blo and the candidates are the same for every thread)
     if (nf == 0 || blo > lim) break;
+    // warp 0 counts the candidates; the others partition meanwhile and read the verdict
+    // after the bucket barrier (a stopping round's partition is simply dropped)
     const uint32_t nc0 = sh.nc;
-    if (nc0 >= k) {  // every warp counts every candidate: the same total, no block reduction
+    if (nc0 >= k && wid == 0) {
       uint32_t cl = 0;
       for (uint32_t i = lane; i < nc0; i += 32) cl += cand_dist(m, i) < blo;
-      if (__reduce_add_sync(FULL, cl) >= k) break;
+      if (__reduce_add_sync(FULL, cl) >= k && lane == 0) sh.stop[par] = 1;
     }
     // ---- 2. partition the frontier: the bucket [m, m + delta) is expanded, the rest re-queued
     const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
@@ -701,10 +705,12 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
       }
     }
     __syncthreads();  // the bucket is complete
+    if (sh.stop[par]) break;
     const uint32_t na = sh.na[par];
     if (tid == 0) {  // the next round's counters (their last readers are past the barrier)
       sh.nn[par ^ 1] = 0;
       sh.na[par ^ 1] = 0;
+      sh.stop[par ^ 1] = 0;
       c_vert += na;
     }
     // ---- 3. expand: lane = (vertex, arc slot), T/4 vertices per window; no barrier between
@@ -804,8 +810,8 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
     nfront = tmp;
   }
 
-  // every warp leaves the loop in the same round; the barrier keeps a warp from rewriting the
-  // candidates below while another is still counting them for the termination test
+  // every warp leaves the loop in the same round (the verdicts are read after barriers); this
+  // barrier keeps a warp from rewriting the candidates below before every warp has left
   __syncthreads();
   // the k smallest (dist, obj)
   const uint32_t nc = sh.nc;
