@@ -557,3 +557,21 @@ def test_pipelined_queries_stage_commit(gg):
     with pytest.raises(gg.GGridError):
         grid.knn_commit(k, o, d)  # nothing staged
     grid.close()
+
+
+def test_ladder_boundaries_and_promotions(gg):
+    """k at the capacity-ladder boundaries (32 | 33: level 0 | level 1's 128 candidates; 96 | 97:
+    level 1 | level 2) and a density where the starting level is the 4-warp CTA variant
+    (expected ball ~440 vertices) but the sparsest queries overflow its 1,024-slot table and are
+    promoted to the level running beside it: every row the oracle's."""
+    g = synth.table_ii_graph("NY", scale=0.2)
+    upd = synth.RandomWalk(g, 1200, inject=True).ticks(3)
+    q = synth.queries(g, 600)
+    grid = gg.GGrid(g, 256, max_objects=2048)
+    grid.ingest(upd)
+    _assert_same(grid.knn(q, 10), _oracle(g, upd, q, 10), "k=10")
+    promoted = grid.stats()["expand_promotions"]
+    for k in (32, 33, 96, 97):
+        _assert_same(grid.knn(q[:200], k), _oracle(g, upd, q[:200], k), f"k={k}")
+    assert promoted > 0  # (3 with these seeds: the promotion path ran)
+    grid.close()
