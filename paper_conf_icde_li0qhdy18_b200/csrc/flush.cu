@@ -36,7 +36,10 @@
 namespace gg {
 
 namespace {
-constexpr int SW = 4;               // streaming warps
+#ifndef GG_SW
+#define GG_SW 4
+#endif
+constexpr int SW = GG_SW;           // streaming warps
 constexpr int FT = (SW + 1) * 32;   // + one index warp
 constexpr int RPT = 4;              // records per lane per group (one 128-bit load of obj)
 constexpr uint32_t STRIDE = SW * 32 * RPT;
