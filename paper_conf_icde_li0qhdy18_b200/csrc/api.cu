@@ -755,7 +755,11 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   }
   const DevGraph& g = h->g;
   const DevState& s = h->s;
-  h->launch(GGRID_K_SEED, [&] { launch_seed(d_q, n_q, g, s, epoch, h->seed_neighbors, q_copy, st); });
+  // a batch whose c_q and neighbour cells cover (nearly) every cell requests every dirty cell
+  // once instead (flushing a cell no query needs changes no answer: lazy == eager)
+  const bool seed_all = h->seed_neighbors && (uint64_t)n_q * (h->max_cell_degree + 1) >= 3ull * h->n_cells;
+  const int seed_mode = seed_all ? SEED_ALL : h->seed_neighbors ? SEED_NEIGHBORS : SEED_DST;
+  h->launch(GGRID_K_SEED, [&] { launch_seed(d_q, n_q, g, s, epoch, seed_mode, q_copy, st); });
   if (q_copy) d_q = q_copy;
 
   // starting level: k must fit the candidate list, and the vertex table should hold the
@@ -788,7 +792,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
   for (int round = 0;; ++round) {
     if (round > 100000) return GGRID_ECUDA;
     // round 0 cleans what the seed requested: c_q and its neighbour cells per query
-    const uint64_t seeded = (uint64_t)n_q * (h->seed_neighbors ? h->max_cell_degree + 1 : 2);
+    const uint64_t seeded = seed_all ? h->n_cells : (uint64_t)n_q * (h->seed_neighbors ? h->max_cell_degree + 1 : 2);
     RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin, 0,
                          round == 0 ? (uint32_t)std::min<uint64_t>(seeded, 1u << 30) : 0));
     if (round > 0) {  // round 0 was reset with the rest at the start

@@ -555,10 +555,15 @@ cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, con
 
 // ---------------------------------------------------------------------------------------
 // Alg. 4 line 1 (P@45660): c_q = getCell(q.e) and getNeighbors({c_q}) are cleaned first.
+// mode SEED_NEIGHBORS: c_q and its neighbour cells per query; SEED_DST: c_q and the cell of the
+// query arc's head; SEED_ALL: every dirty cell, each requested once by thread c (a batch large
+// enough to touch nearly every cell: one uncontended request per cell instead of ~n_q x 9
+// racing on the same cells).  Every mode validates the queries and copies mapped ones.
 __global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint32_t nq, DevGraph g,
-                                              DevState s, uint32_t epoch, int neighbors,
+                                              DevState s, uint32_t epoch, int mode,
                                               uint2* __restrict__ q_copy) {
   uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (mode == SEED_ALL && i < g.n_cells) request_flush(s, i, epoch);
   if (i >= nq) return;
   uint2 qq = q[i];
   // queries in mapped host memory are read across PCIe once, here, and kept in HBM for the
@@ -573,9 +578,10 @@ __global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint3
     atomicOr(&s.st->err, (unsigned)ERR_QUERY);
     return;
   }
+  if (mode == SEED_ALL) return;
   uint32_t c = cellof(g, e.x);
   request_flush(s, c, epoch);
-  if (neighbors) {
+  if (mode == SEED_NEIGHBORS) {
     for (uint32_t j = g.cadj_ptr[c]; j < g.cadj_ptr[c + 1]; ++j) request_flush(s, g.cadj[j], epoch);
   } else {
     request_flush(s, cellof(g, g.edst[qq.x]), epoch);
@@ -583,9 +589,10 @@ __global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint3
 }
 
 void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s, uint32_t epoch,
-                 int neighbors, uint2* q_copy, cudaStream_t st) {
-  if (nq == 0) return;
-  k_seed<<<(nq + 255) / 256, 256, 0, st>>>(q, nq, g, s, epoch, neighbors, q_copy);
+                 int mode, uint2* q_copy, cudaStream_t st) {
+  const uint32_t n = mode == SEED_ALL ? std::max(nq, g.n_cells) : nq;
+  if (n == 0) return;
+  k_seed<<<(n + 255) / 256, 256, 0, st>>>(q, nq, g, s, epoch, mode, q_copy);
 }
 
 // Every dirty cell (eager cleaning; all_cells additionally queues clean cells for GC).

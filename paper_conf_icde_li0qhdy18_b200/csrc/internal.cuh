@@ -198,8 +198,9 @@ void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st);
 // q_copy (nullable): also store the queries there (q in mapped host memory)
+enum SeedMode { SEED_DST = 0, SEED_NEIGHBORS = 1, SEED_ALL = 2 };
 void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s, uint32_t epoch,
-                 int neighbors, uint2* q_copy, cudaStream_t st);
+                 int mode, uint2* q_copy, cudaStream_t st);
 void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int all_cells,
                        cudaStream_t st);
 // Flush the cells flush_list[begin .. st->n_flush) writing compacted lists into `out`
