@@ -327,6 +327,9 @@ def run_ours(args, cfg_name):
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": traffic, "kernel": dom, "peak_source": peak_kind,
                 "launch_ms": dms / max(1, dl), "timed_in": "timed steps" if dom == "expand" else "breakdown steps"}
+    lp = os.path.join(ROOT, "profiles", f"limiters_{cfg_name}.json")
+    if os.path.exists(lp):  # what bounds the kernel when it is not HBM (ncu, the last profiling pass)
+        roofline["ncu_limiters"] = json.load(open(lp)).get(dom)
     updates_per_s = n_upd * K / (ingest_ms / 1e3) if ingest_ms > 0 else None
 
     # ---- e2e through the public API with pinned host buffers -------------------------------

@@ -48,6 +48,7 @@ lines = [f"# Profiling summary — round tag `{tag}`", "",
          "Source: `tools/profile_round.sh` under gpurun on one B200 (ncu 2025, `--clock-control none`).",
          "Raw pages: `profiles/%s_<capture>_raw.csv`; launch list: `profiles/%s_launches_C1.csv`." % (tag, tag), ""]
 traffic = {}
+issue = {}
 for cap in ("expand_C1", "ingest_C1", "flush_C3"):
     p = os.path.join(src, f"{cap}_raw.csv")
     if not os.path.exists(p):
@@ -82,6 +83,11 @@ for cap in ("expand_C1", "ingest_C1", "flush_C3"):
         kind = {"expand_C1": "expand", "ingest_C1": "ingest", "flush_C3": "flush"}[cap]
         cfg = cap.split("_")[1]
         traffic.setdefault(cfg, collections.defaultdict(float))[kind] += rd + wr
+        if "smsp__issue_active.avg.pct_of_peak_sustained_active" in hdr:  # (non-HBM limiters)
+            issue.setdefault(cfg, {})[kind] = {
+                "issue_slots_busy_pct": float(r[hdr.index("smsp__issue_active.avg.pct_of_peak_sustained_active")]),
+                "dram_throughput_pct": float(r[hdr.index("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed")]),
+                "top_stalls": top, "capture": f"profiles/{tag}_summary.md"}
 
 ll = os.path.join(src, "launches_C1.csv")
 if os.path.exists(ll):
@@ -104,4 +110,6 @@ open(os.path.join(dst, f"{tag}_summary.md"), "w").write("\n".join(lines) + "\n")
 for cfg, d in traffic.items():
     # per launch: expand (the starting level), ingest (one fused launch per step), flush (C3)
     json.dump({k: v for k, v in d.items()}, open(os.path.join(dst, f"traffic_{cfg}.json"), "w"), indent=1)
+for cfg, d in issue.items():
+    json.dump(d, open(os.path.join(dst, f"limiters_{cfg}.json"), "w"), indent=1)
 print("\n".join(lines))
