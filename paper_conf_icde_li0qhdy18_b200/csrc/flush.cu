@@ -389,6 +389,8 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
   extern __shared__ __align__(16) unsigned char smem_raw[];
   using SM = FlushSmem<HCAP, WCAP>;
   SM& sm = *reinterpret_cast<SM*>(smem_raw);
+  pdl_wait();   // (a programmatic dependent of the seed / status reset)
+  pdl_allow();  // the expansion may launch now (it waits for this grid before reading)
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const unsigned lt = lanemask_lt();
   const uint32_t lend = *((volatile unsigned*)&s.st->n_flush);
@@ -475,8 +477,9 @@ void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned l
   const int blocks_per_sm = blocks_per_sm_t<HCAP, WCAP>();
   uint32_t grid = (uint32_t)(sm_count * blocks_per_sm);
   if (max_ctas && max_ctas < grid) grid = max_ctas;  // few cells to clean: fewer idle CTAs
-  k_flush<HCAP, WCAP><<<grid, FT, sizeof(FlushSmem<HCAP, WCAP>), st>>>(
-      g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
+  cudaLaunchAttribute attr[1];
+  const cudaLaunchConfig_t cfg = pdl_config(dim3(grid), dim3(FT), sizeof(FlushSmem<HCAP, WCAP>), st, attr);
+  cudaLaunchKernelEx(&cfg, k_flush<HCAP, WCAP>, g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
 }
 template <int HCAP, int WCAP>
 int blocks_per_sm_t() {

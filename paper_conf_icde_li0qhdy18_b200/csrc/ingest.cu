@@ -562,6 +562,8 @@ cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, con
 __global__ void __launch_bounds__(256) k_seed(const uint2* __restrict__ q, uint32_t nq, DevGraph g,
                                               DevState s, uint32_t epoch, int mode,
                                               uint2* __restrict__ q_copy) {
+  pdl_wait();   // (launched as a programmatic dependent of the round's status reset)
+  pdl_allow();  // the flush may launch now (it waits for this grid before reading)
   uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (mode == SEED_ALL && i < g.n_cells) request_flush(s, i, epoch);
   if (i >= nq) return;
@@ -592,7 +594,9 @@ void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState&
                  int mode, uint2* q_copy, cudaStream_t st) {
   const uint32_t n = mode == SEED_ALL ? std::max(nq, g.n_cells) : nq;
   if (n == 0) return;
-  k_seed<<<(n + 255) / 256, 256, 0, st>>>(q, nq, g, s, epoch, mode, q_copy);
+  cudaLaunchAttribute attr[1];
+  const cudaLaunchConfig_t cfg = pdl_config(dim3((n + 255) / 256), dim3(256), 0, st, attr);
+  cudaLaunchKernelEx(&cfg, k_seed, q, nq, g, s, epoch, mode, q_copy);
 }
 
 // Every dirty cell (eager cleaning; all_cells additionally queues clean cells for GC).
@@ -646,6 +650,7 @@ void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t
 
 namespace gg {
 __global__ void k_set_words(WordSet ws) {
+  pdl_allow();  // a programmatic dependent (the seed / flush of a knn round) may launch now
   if (ws.fold_dst && threadIdx.x == 0) *ws.fold_dst |= *ws.fold_src;
   __syncwarp();
   if ((int)threadIdx.x < ws.n) *ws.p[threadIdx.x] = ws.v[threadIdx.x];

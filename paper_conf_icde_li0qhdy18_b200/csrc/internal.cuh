@@ -133,6 +133,26 @@ __device__ __forceinline__ uint32_t cellof(const DevGraph& g, uint32_t v) {
   return (t + ((v - t) >> 1)) >> (g.cs_shift - 1);
 }
 
+// Programmatic dependent launch (the knn round's seed -> flush -> expansion chain): a kernel
+// launched with pdl_config() may start while the previous one runs; it waits for it (and its
+// memory) at pdl_wait() before touching anything, and lets its own dependent launch early with
+// pdl_allow().  Both are no-ops for a normally launched kernel.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_allow() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+inline cudaLaunchConfig_t pdl_config(dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                                     cudaLaunchAttribute* attr) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cfg;
+}
+
 __device__ inline unsigned lanemask_lt() {
   unsigned m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));

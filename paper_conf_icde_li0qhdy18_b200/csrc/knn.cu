@@ -163,11 +163,13 @@ struct QParams {
   const uint32_t* wait_exited;
   uint32_t wait_total;
   int trigger;
+  int wait_prior;  // launched as a programmatic dependent that must see the previous grid (flush)
 };
 
 // programmatic dependent launch: the next kernel of the stream may start right away (it
 // depends on this one only through the promotion ring and the exit counter)
 __device__ __forceinline__ void pdl_trigger(const QParams& P) {
+  if (P.wait_prior) pdl_wait();  // the round's flush has finished and its lists are visible
   if (P.trigger) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
@@ -1050,6 +1052,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.wait_exited = L.wait_exited;
   P.wait_total = L.wait_total;
   P.trigger = L.trigger ? 1 : 0;
+  P.wait_prior = L.chain_in ? 0 : 1;  // (a chained level runs beside the level below it)
   const int smem = (int)expand_warp_bytes(level, g.V);
   if (level == NLEVELS - 1) {
     P.scratch = static_cast<unsigned char*>(L.scratch);
@@ -1068,7 +1071,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = L.pdl ? 1 : 0;
+  cfg.numAttrs = 1;  // programmatic dependent of the flush (waits for it) or, chained, of the level below
   if (cta) {
     cudaLaunchKernelEx(&cfg, cta_kernel(level), P);
   } else {
