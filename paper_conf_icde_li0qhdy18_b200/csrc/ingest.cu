@@ -347,6 +347,8 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
                                                             //        cell order
   uint16_t* stp = reinterpret_cast<uint16_t*>(stg + tile);  // [tile] tile index, cell order
   uint32_t* w_sum = reinterpret_cast<uint32_t*>(stp + ((tile + 1) & ~1u));  // [FT / 32]
+  pdl_wait();   // (a programmatic dependent of the batch's status reset)
+  pdl_allow();  // the next kernel (a knn round's status reset) may launch; it waits for this grid
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const unsigned G = gridDim.x;
   for (uint32_t i = tid; i < ch; i += FT) {
@@ -540,17 +542,19 @@ bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p
 
 cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                                 const DevState& s, const IngestPlan& p, cudaStream_t st) {
-  static bool attr = false;
-  if (!attr) {
+  static bool smem_set = false;
+  if (!smem_set) {
     cudaFuncSetAttribute(k_ingest_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    attr = true;
+    smem_set = true;
   }
-  uint32_t tile = p.tile, ch = p.ch;
-  DevGraph gg_ = g;
-  DevState ss = s;
-  void* args[] = {(void*)&upd, (void*)&n, (void*)&seq0, (void*)&tile, (void*)&ch, (void*)&gg_, (void*)&ss};
-  // cooperative: every CTA is resident at once (the grid barriers need it), or the launch fails
-  return cudaLaunchCooperativeKernel((const void*)k_ingest_fused, dim3(p.grid), dim3(FT), args, p.smem, st);
+  // cooperative (every CTA resident at once, or the launch fails: the grid barriers need it) and
+  // a programmatic dependent of the batch's status reset
+  cudaLaunchAttribute attr[2];
+  cudaLaunchConfig_t cfg = pdl_config(dim3(p.grid), dim3(FT), p.smem, st, attr);
+  attr[1].id = cudaLaunchAttributeCooperative;
+  attr[1].val.cooperative = 1;
+  cfg.numAttrs = 2;
+  return cudaLaunchKernelEx(&cfg, k_ingest_fused, upd, n, seq0, p.tile, p.ch, g, s);
 }
 
 // ---------------------------------------------------------------------------------------
@@ -650,13 +654,17 @@ void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t
 
 namespace gg {
 __global__ void k_set_words(WordSet ws) {
-  pdl_allow();  // a programmatic dependent (the seed / flush of a knn round) may launch now
+  pdl_wait();   // (a programmatic dependent of the ingest before a knn round)
+  pdl_allow();  // a programmatic dependent (the seed / flush / ingest) may launch now
   if (ws.fold_dst && threadIdx.x == 0) *ws.fold_dst |= *ws.fold_src;
   __syncwarp();
   if ((int)threadIdx.x < ws.n) *ws.p[threadIdx.x] = ws.v[threadIdx.x];
 }
 void launch_set_words(const WordSet& ws, cudaStream_t st) {
-  if (ws.n || ws.fold_dst) k_set_words<<<1, 32, 0, st>>>(ws);
+  if (!ws.n && !ws.fold_dst) return;
+  cudaLaunchAttribute attr[1];
+  const cudaLaunchConfig_t cfg = pdl_config(dim3(1), dim3(32), 0, st, attr);
+  cudaLaunchKernelEx(&cfg, k_set_words, ws);
 }
 }  // namespace gg
 
