@@ -89,6 +89,13 @@ class ClockSampler:
         except Exception:
             self.p = None
 
+    def _rows(self):
+        return [r.split(",") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
+
+    def mark(self):
+        """Start of the timed region: samples before it (warm-up) are kept only as a fallback."""
+        self.mark_rows = len(self._rows()) if self.p is not None else 0
+
     def stop(self):
         if self.p is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
@@ -98,8 +105,15 @@ class ClockSampler:
         except Exception:
             self.p.kill()
         self.f.flush()
-        rows = [r.split(",") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
+        rows = self._rows()
         os.unlink(self.f.name)
+        window = "timed steps"
+        timed = rows[getattr(self, "mark_rows", 0):]
+        if timed:
+            rows = timed
+        else:  # a timed region shorter than the 100 ms sampling interval: the warm-up's last samples
+            rows = rows[-3:]
+            window = "last warm-up samples (timed region shorter than the sampling interval)"
         sm, mx, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for r in rows:
@@ -113,7 +127,7 @@ class ClockSampler:
                 if v.lower() == "active":
                     reasons.add(n)
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm), "window": window}
 
 
 def dist_setup():
@@ -239,10 +253,12 @@ def run_ours(args, cfg_name):
             du = torch.empty((n_upd_step, 4), dtype=torch.int32, device="cuda")
         dq = torch.from_numpy(q.view(np.int32)).to("cuda")
         barrier()
+        if s == 0:  # (started with the warm-up: nvidia-smi needs ~0.1-0.3 s to report)
+            clocks = ClockSampler(dev)
         if s == args.warmup:
             grid.stats_reset()
             st0 = grid.stats()
-            clocks = ClockSampler(dev)
+            clocks.mark()
         if s == args.warmup + args.steps:  # end of the timed steps
             clk = clocks.stop()
             grid.sync()  # (raises a deferred ingest error, if any)
