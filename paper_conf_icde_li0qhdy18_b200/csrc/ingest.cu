@@ -22,11 +22,17 @@ namespace gg {
 // It also orders its tile by cell (hash slot): tmp[] holds, in that order, each update's
 // (source vertex, rank in the cell's batch extent) and perm[] its index in the tile, so the
 // scatter's consecutive threads write consecutive arena positions (runs per cell).
-constexpr int CT = 256;            // threads
+#ifndef GG_INGEST_CT
+#define GG_INGEST_CT 1024
+#endif
+constexpr int CT = GG_INGEST_CT;   // threads
 constexpr int CPT = 8;             // updates per thread
 constexpr int CU = CT * CPT;       // updates per CTA (tile)
-constexpr int CH = 4096;           // hash slots (>= 2*CU)
+constexpr int CH = 2 * CU;         // hash slots (>= 2*CU)
+constexpr int CH_BITS = 31 - __builtin_clz(CH);
+static_assert((1 << CH_BITS) == CH, "hash slots: a power of two");
 constexpr int SPC = CH / CT;       // hash slots per thread in the scan
+constexpr int SCATTER_SMEM = CU * 16;
 static_assert(CU < 65536, "tile offsets and counts are packed in 16 bits");
 constexpr uint32_t REMOTE_CELL = 0xFFFFFFFEu;  // classify: pseudo-cell of other ranks' updates
 constexpr int CLASSIFY_SMEM = (3 * CH + CT / 32) * 4;
@@ -85,7 +91,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
     const uint32_t c0 = cellof(g, e.x);
     const bool remote = s.n_ranks > 1 && owner_of(c0, g.n_cells, s.n_ranks) != s.rank;
     const uint32_t c = remote ? REMOTE_CELL : c0;
-    uint32_t h = (c * 2654435761u) >> 20;  // 12 bits
+    uint32_t h = (c * 2654435761u) >> (32 - CH_BITS);
     volatile uint32_t* vc = h_cell;
     for (;;) {
       const uint32_t cur = vc[h];
@@ -221,7 +227,7 @@ __global__ void __launch_bounds__(CT) k_ingest_scatter(const uint4* __restrict__
                                                        uint32_t seq0, DevGraph g, DevState s,
                                                        const uint2* __restrict__ tmp,
                                                        const uint16_t* __restrict__ perm) {
-  __shared__ uint4 su[CU];
+  extern __shared__ uint4 su[];  // CU records (SCATTER_SMEM bytes)
   const int tid = threadIdx.x;
   const uint64_t base = (uint64_t)blockIdx.x * CU;
   const uint32_t nt = (n - base) < (uint64_t)CU ? (uint32_t)(n - base) : (uint32_t)CU;
@@ -302,8 +308,13 @@ void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st) 
 }
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_ingest_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, SCATTER_SMEM);
+    attr = true;
+  }
   unsigned blocks = (unsigned)((n + CU - 1) / CU);
-  k_ingest_scatter<<<blocks, CT, 0, st>>>(upd, n, seq0, g, s, tmp,
+  k_ingest_scatter<<<blocks, CT, SCATTER_SMEM, st>>>(upd, n, seq0, g, s, tmp,
                                           perm_of(const_cast<uint2*>(tmp), n));
 }
 
