@@ -26,7 +26,10 @@ namespace gg {
 #define GG_INGEST_CT 1024
 #endif
 constexpr int CT = GG_INGEST_CT;   // threads
-constexpr int CPT = 8;             // updates per thread
+#ifndef GG_INGEST_CPT
+#define GG_INGEST_CPT 8
+#endif
+constexpr int CPT = GG_INGEST_CPT; // updates per thread
 constexpr int CU = CT * CPT;       // updates per CTA (tile)
 constexpr int CH = 2 * CU;         // hash slots (>= 2*CU)
 constexpr int CH_BITS = 31 - __builtin_clz(CH);
