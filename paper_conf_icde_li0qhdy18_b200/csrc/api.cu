@@ -608,7 +608,20 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   }
   RC(h->sync());
   const unsigned err = h->h_status->ingest_err;
-  if (err & (ERR_OBJ | ERR_EDGE | ERR_OFF)) return GGRID_EINVAL;
+  if (err & (ERR_OBJ | ERR_EDGE | ERR_OFF)) {
+    if (getenv("GGRID_DEBUG")) {  // diagnosis of a rejected batch (item 0)
+      const uint32_t bi = h->h_status->bad_index;
+      fprintf(stderr, "ggrid_ingest: batch of %llu rejected, err=0x%x first bad index=%u (%s path)\n",
+              (unsigned long long)n, err, bi, fused ? "fused" : "three-launch");
+      if (bi < n) {
+        uint4 r;
+        if (cudaMemcpy(&r, d_u + bi, sizeof(r), cudaMemcpyDeviceToHost) == cudaSuccess)
+          fprintf(stderr, "ggrid_ingest: record %u = (obj %u, edge %u, offset %u, t %u)\n", bi, r.x,
+                  r.y, r.z, r.w);
+      }
+    }
+    return GGRID_EINVAL;
+  }
   if (err & ERR_ARENA) return GGRID_ENOMEM;
   h->seq_next += n;
   h->stats.n_updates = h->seq_next;
