@@ -8,7 +8,16 @@
  * Conventions (all calls):
  *  - Plain pointers and sizes; no torch / C++ types.  Every pointer argument named
  *    "host or device" may be either; the library detects which (cudaPointerGetAttributes)
- *    and never retains it after the call returns.
+ *    and never retains it after the call returns -- except under opts.async_ingest, where
+ *    a device `u` of ggrid_ingest is read by kernels still queued when the call returns:
+ *    it must stay valid and unmodified until the next synchronous call (ggrid_sync,
+ *    ggrid_knn, ggrid_flush_all, ggrid_stats, ...) or until a stream ordered after the
+ *    library by ggrid_signal_stream reaches it.
+ *  - Stream order of caller memory.  Device (and pinned host) memory a call reads or writes
+ *    may be produced or consumed by caller work that is still queued.  Each call orders its
+ *    device work after everything queued so far on the legacy default stream (which itself
+ *    follows every blocking stream) -- or, with opts.stream, after that stream.  Producers on
+ *    other non-blocking streams must be named with ggrid_wait_stream before the call.
  *  - Return value 0 = GGRID_OK, negative = error (see GGRID_E*); ggrid_strerror() names it.
  *    On an error no observable state changes (ingest rejects the whole batch).
  *  - All integers are unsigned 32-bit unless noted ("4-byte integers", P@59405).
@@ -269,6 +278,18 @@ int ggrid_prior_art_clean(ggrid_t h, uint32_t eta, uint32_t bucket_size, uint32_
  * lane holds afterwards. */
 int ggrid_prior_art_bundle(const uint32_t* obj, const uint64_t* key, uint32_t eta, uint32_t* out_obj,
                            uint64_t* out_key);
+
+/* Order the library after caller work: every device operation of later calls on h starts
+ * only after all work queued on `stream` (a cudaStream_t, or NULL = the legacy default
+ * stream) before this call has finished -- e.g. the kernel that produced a device update
+ * batch on a non-blocking stream.  Event record + stream wait; no host synchronisation.
+ * Errors: EINVAL (null h), ECUDA. */
+int ggrid_wait_stream(ggrid_t h, void* stream);
+
+/* The converse: work queued on `stream` after this call starts only after every device
+ * operation h has queued so far (e.g. the asynchronous ingest of a device buffer the caller
+ * wants to reuse or free).  Errors: EINVAL, ECUDA. */
+int ggrid_signal_stream(ggrid_t h, void* stream);
 
 /* Drain the handle's stream.  Returns the deferred error of an asynchronous ingest batch
  * (opts.async_ingest) that was rejected since the last report, else GGRID_OK; the error is

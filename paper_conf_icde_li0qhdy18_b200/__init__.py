@@ -26,7 +26,7 @@ KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "fl
 EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_query_stage", "ggrid_knn_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_sync", "ggrid_set_profile", "ggrid_flush_all",
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
            "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk",
-           "ggrid_prior_art_clean", "ggrid_prior_art_bundle"]
+           "ggrid_prior_art_clean", "ggrid_prior_art_bundle", "ggrid_wait_stream", "ggrid_signal_stream"]
 
 
 class GGridError(RuntimeError):
@@ -104,6 +104,8 @@ def lib():
             "ggrid_merge_topk": ([P, u32, u32, u32, P, P, P, P], i32),
             "ggrid_prior_art_clean": ([P, u32, u32, u32, P, P, ctypes.POINTER(ggrid_prior_art_result)], i32),
             "ggrid_prior_art_bundle": ([P, P, u32, P, P], i32),
+            "ggrid_wait_stream": ([P, P], i32),
+            "ggrid_signal_stream": ([P, P], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -141,6 +143,26 @@ def _u32(a):
     return a.contiguous()
 
 
+def _cuda_stream_of(*arrays):
+    """cudaStream_t of torch's current stream on the device of the first CUDA tensor among
+    `arrays` (None if there is none): the stream whose queued work produced / consumes them."""
+    for a in arrays:
+        if a is not None and not isinstance(a, np.ndarray) and getattr(a, "is_cuda", False):
+            import torch
+            return torch.cuda.current_stream(a.device).cuda_stream
+    return None
+
+
+def _order_inputs(h, *arrays):
+    """ggrid_wait_stream on torch's current stream when a CUDA tensor is passed: the library's
+    stream then starts after the kernels that produced the tensors (stream 0 is the legacy
+    default stream; the C ABI orders after it by itself unless opts.stream was given)."""
+    st = _cuda_stream_of(*arrays)
+    if st is not None:
+        _check(lib().ggrid_wait_stream(h, st), "ggrid_wait_stream")
+    return st
+
+
 # ------------------------------------------------------------------------ the C ABI names
 def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 256,
                 max_objects: int = 1 << 24, log_capacity: int = 0, delta: int = 0,
@@ -166,7 +188,10 @@ def ggrid_ingest(h, updates, n: int | None = None):
     """Append updates: (n, 4) u32 (obj, edge, offset, t) numpy array or torch tensor."""
     u = _u32(updates)
     cnt = int(u.shape[0]) if n is None else int(n)
+    st = _order_inputs(h, u)
     _check(lib().ggrid_ingest(h, _ptr(u), cnt), "ggrid_ingest")
+    if st is not None:  # (async ingest) the caller's later work on u waits for the kernels reading it
+        _check(lib().ggrid_signal_stream(h, st), "ggrid_signal_stream")
 
 
 def ggrid_sync(h):
@@ -182,6 +207,7 @@ def ggrid_set_profile(h, mask: int):
 def ggrid_ingest_stage(h, updates):
     """Start the asynchronous copy of a batch (keep `updates` alive until the commit)."""
     u = _u32(updates)
+    _order_inputs(h, u)
     _check(lib().ggrid_ingest_stage(h, _ptr(u), int(u.shape[0])), "ggrid_ingest_stage")
     return u
 
@@ -193,6 +219,7 @@ def ggrid_ingest_commit(h):
 def ggrid_query_stage(h, queries):
     """Start the asynchronous copy of a query batch (keep `queries` alive until knn_commit)."""
     q = _u32(queries)
+    _order_inputs(h, q)
     _check(lib().ggrid_query_stage(h, _ptr(q), int(q.shape[0])), "ggrid_query_stage")
     return q
 
@@ -200,6 +227,7 @@ def ggrid_query_stage(h, queries):
 def ggrid_knn_commit(h, k: int, out_obj, out_dist):
     """Answer the oldest staged query batch into out_obj / out_dist (preallocated, (n, k))."""
     n = ctypes.c_uint32(0)
+    _order_inputs(h, out_obj, out_dist)
     _check(lib().ggrid_knn_commit(h, int(k), _ptr(out_obj), _ptr(out_dist), ctypes.byref(n)),
            "ggrid_knn_commit")
     return out_obj, out_dist
@@ -216,6 +244,7 @@ def ggrid_knn(h, queries, k: int, out_obj=None, out_dist=None):
         out_obj = np.empty((nq, k), np.uint32)
     if out_dist is None:
         out_dist = np.empty((nq, k), np.uint32)
+    _order_inputs(h, q, out_obj, out_dist)
     _check(lib().ggrid_knn(h, _ptr(q), nq, int(k), _ptr(out_obj), _ptr(out_dist)), "ggrid_knn")
     return out_obj, out_dist
 
@@ -233,6 +262,7 @@ def ggrid_knn_ex(h, queries, k: int, bound=None, out_obj=None, out_dist=None, ou
     if out_remote is True:
         out_remote = np.empty(nq, np.uint64)
     b = None if bound is None else _u32(bound)
+    _order_inputs(h, q, b, out_obj, out_dist, None if out_remote is None or out_remote is True else out_remote)
     _check(lib().ggrid_knn_ex(h, _ptr(q), nq, int(k), _ptr(b), _ptr(out_obj), _ptr(out_dist), _ptr(out_remote)),
            "ggrid_knn_ex")
     return out_obj, out_dist, out_remote
@@ -247,6 +277,7 @@ def ggrid_query_owner(h, queries, out_rank=None):
     nq = int(q.shape[0])
     if out_rank is None:
         out_rank = np.empty(nq, np.uint32)
+    _order_inputs(h, q, out_rank)
     _check(lib().ggrid_query_owner(h, _ptr(q), nq, _ptr(out_rank)), "ggrid_query_owner")
     return out_rank
 
@@ -259,6 +290,7 @@ def ggrid_merge_topk(h, lists_obj, lists_dist, out_obj=None, out_dist=None):
         out_obj = np.empty((nq, k), np.uint32)
     if out_dist is None:
         out_dist = np.empty((nq, k), np.uint32)
+    _order_inputs(h, lo, ld, out_obj, out_dist)
     _check(lib().ggrid_merge_topk(h, L, nq, k, _ptr(lo), _ptr(ld), _ptr(out_obj), _ptr(out_dist)),
            "ggrid_merge_topk")
     return out_obj, out_dist
@@ -286,6 +318,24 @@ def ggrid_prior_art_bundle(obj, key, eta: int):
     ok = np.empty_like(ky)
     _check(lib().ggrid_prior_art_bundle(_ptr(ob), _ptr(ky), int(eta), _ptr(oo), _ptr(ok)), "ggrid_prior_art_bundle")
     return oo, ok
+
+
+def ggrid_wait_stream(h, stream=None):
+    """Later calls on h start after the work queued on `stream` (torch.cuda.Stream, raw
+    cudaStream_t int, or None = torch's current stream)."""
+    _check(lib().ggrid_wait_stream(h, _stream_handle(stream)), "ggrid_wait_stream")
+
+
+def ggrid_signal_stream(h, stream=None):
+    """Work queued on `stream` from now on starts after everything h has queued so far."""
+    _check(lib().ggrid_signal_stream(h, _stream_handle(stream)), "ggrid_signal_stream")
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return int(getattr(stream, "cuda_stream", stream))
 
 
 def ggrid_free(h):
@@ -348,6 +398,14 @@ class GGrid:
 
     def ingest(self, updates):
         ggrid_ingest(self.h, updates)
+        return self
+
+    def wait_stream(self, stream=None):
+        ggrid_wait_stream(self.h, stream)
+        return self
+
+    def signal_stream(self, stream=None):
+        ggrid_signal_stream(self.h, stream)
         return self
 
     def sync(self):

@@ -6,7 +6,10 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <new>
+#include <tuple>
 #include <utility>
 #include <vector>
 
@@ -95,6 +98,23 @@ void* device_view(const void* p) {
 
 }  // namespace
 
+namespace gg {
+cudaError_t func_attr_once(const void* kernel, cudaFuncAttribute attr, int value) {
+  static std::mutex mu;
+  static std::map<std::tuple<const void*, int, int, int>, cudaError_t> done;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return cudaGetLastError();
+  std::lock_guard<std::mutex> lock(mu);
+  const auto key = std::make_tuple(kernel, (int)attr, dev, value);
+  auto it = done.find(key);
+  if (it != done.end()) return it->second;
+  const cudaError_t e = cudaFuncSetAttribute(kernel, attr, value);
+  if (e != cudaSuccess) cudaGetLastError();
+  done[key] = e;
+  return e;
+}
+}  // namespace gg
+
 struct ggrid_s {
   int device = 0;
   cudaStream_t stream = nullptr;
@@ -135,6 +155,8 @@ struct ggrid_s {
   Staged qstaged[2];  // staged query batches (ggrid_query_stage / ggrid_knn_commit)
   int qstage_head = 0, n_qstaged = 0;
   cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_in = nullptr;   // caller's producer stream -> library streams (order_inputs)
+  cudaEvent_t ev_out = nullptr;  // library stream -> a caller's stream (ggrid_signal_stream)
   DBuf chain_ring;  // queries promoted into the chained level (NONE = not yet written)
   ggrid_stats_t stats{};
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending_ev;
@@ -163,6 +185,23 @@ struct ggrid_s {
     cudaEventCreate(&e);
     return e;
   }
+
+  // Order stream `on` after the work a caller queued on `producer` (cudaEventRecord +
+  // cudaStreamWaitEvent: no host wait).  Caller memory a call reads (device updates, queries,
+  // bounds) or writes (device / pinned outputs) may have been produced, or still be read, by
+  // that work; without this the library's non-blocking stream could read a buffer before its
+  // producer kernel wrote it (or overwrite it before the caller's reader ran).
+  int order_after(cudaStream_t producer, cudaStream_t on) {
+    if (producer == on) return GGRID_OK;
+    CK(cudaEventRecord(ev_in, producer));
+    CK(cudaStreamWaitEvent(on, ev_in, 0));
+    return GGRID_OK;
+  }
+  // The default producer: the legacy default stream (whose operations wait for every blocking
+  // stream) when the library runs on its own stream; the caller's own stream when opts.stream
+  // was given (then the library's work is already in the caller's order).  Work on other
+  // non-blocking streams is ordered with ggrid_wait_stream.
+  int order_inputs(cudaStream_t on) { return order_after(own_stream ? cudaStreamLegacy : stream, on); }
 
   // every kernel launch goes through here: counted, and timed in profile mode
   template <class F>
@@ -378,6 +417,9 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   if (cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking) != cudaSuccess) {
     return fail(GGRID_ECUDA);
   }
+  if (cudaEventCreateWithFlags(&h->ev_in, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&h->ev_out, cudaEventDisableTiming) != cudaSuccess)
+    return fail(GGRID_ECUDA);
   h->V = V;
   h->A = A;
   h->cs = cell_size;
@@ -549,6 +591,8 @@ int ggrid_free(ggrid_t h) {
     if (sb->consumed) cudaEventDestroy(sb->consumed);
   }
   if (h->copy_stream) cudaStreamDestroy(h->copy_stream);
+  if (h->ev_in) cudaEventDestroy(h->ev_in);
+  if (h->ev_out) cudaEventDestroy(h->ev_out);
 
   for (auto& pe : h->pending_ev) {
     cudaEventDestroy(pe.second.first);
@@ -580,6 +624,7 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
     }
     ws.add(&h->d_status->ingest_err, 0u);
     ws.add(&h->d_status->bad_index, 0xFFFFFFFFu);
+    ws.add(&h->d_status->batch_tmax, 0u);
     RC(h->set_words(ws));
   }
   const uint32_t seq0 = (uint32_t)h->seq_next;
@@ -635,6 +680,7 @@ int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
   if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
   CK(cudaSetDevice(h->device));
   const uint4* d_u = reinterpret_cast<const uint4*>(u);
+  RC(h->order_inputs(h->stream));  // u may be the output of a caller kernel still running
   if (!is_device_ptr(u)) {
     RC(h->upd_stage.ensure(n * sizeof(uint4)));
     CK(cudaMemcpyAsync(h->upd_stage.p, u, n * sizeof(uint4), cudaMemcpyHostToDevice, h->stream));
@@ -656,6 +702,7 @@ static int stage_into(ggrid_t h, ggrid_s::Staged* ring, int head, int count, con
   sb.n = n;
   // the kernels of this buffer's previous batch may still be reading it
   CK(cudaStreamWaitEvent(h->copy_stream, sb.consumed, 0));
+  RC(h->order_inputs(h->copy_stream));  // and src may still be being produced by the caller
   if (n) {
     // both buffers grow together: a cudaMalloc in the middle of a running pipeline stalls it
     RC(ring[0].buf.ensure(n * bytes_each));
@@ -703,6 +750,7 @@ static int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, u
                     uint64_t* out_remote = nullptr) {
   CK(cudaSetDevice(h->device));
   cudaStream_t st = h->stream;
+  RC(h->order_inputs(st));  // queries / bounds / outputs may be in use by caller work
   // optional per-query bound (host or device) and remote-rank masks (sharded mode)
   const uint32_t* d_bound = nullptr;
   if (bound) {
@@ -948,6 +996,7 @@ int ggrid_query_owner(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t* o
   if (!h || (n_q && (!q || !out_rank))) return GGRID_EINVAL;
   if (n_q == 0) return GGRID_OK;
   CK(cudaSetDevice(h->device));
+  RC(h->order_inputs(h->stream));
   const uint2* d_q = static_cast<const uint2*>(device_view(q));
   if (!d_q) {
     RC(h->q_stage.ensure((size_t)n_q * 8));
@@ -972,6 +1021,7 @@ int ggrid_merge_topk(ggrid_t h, uint32_t n_lists, uint32_t n_q, uint32_t k, cons
   if (!lists_obj || !lists_dist || !out_obj || !out_dist) return GGRID_EINVAL;
   CK(cudaSetDevice(h->device));
   cudaStream_t st = h->stream;
+  RC(h->order_inputs(st));
   const size_t in_n = (size_t)n_lists * n_q * k, out_n = (size_t)n_q * k;
   const uint32_t* d_lo = static_cast<const uint32_t*>(device_view(lists_obj));
   const uint32_t* d_ld = static_cast<const uint32_t*>(device_view(lists_dist));
@@ -1097,6 +1147,25 @@ int ggrid_set_profile(ggrid_t h, uint32_t mask) {
   if (!h) return GGRID_EINVAL;
   RC(h->sync());  // (collects the events of the previous mode)
   h->profile = mask;
+  return GGRID_OK;
+}
+
+int ggrid_wait_stream(ggrid_t h, void* stream) {
+  if (!h) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  cudaStream_t p = static_cast<cudaStream_t>(stream);
+  RC(h->order_after(p, h->stream));
+  RC(h->order_after(p, h->copy_stream));
+  return GGRID_OK;
+}
+
+int ggrid_signal_stream(ggrid_t h, void* stream) {
+  if (!h) return GGRID_EINVAL;
+  CK(cudaSetDevice(h->device));
+  cudaStream_t c = static_cast<cudaStream_t>(stream);
+  if (c == h->stream) return GGRID_OK;
+  CK(cudaEventRecord(h->ev_out, h->stream));
+  CK(cudaStreamWaitEvent(c, h->ev_out, 0));
   return GGRID_OK;
 }
 

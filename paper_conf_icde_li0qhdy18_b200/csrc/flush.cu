@@ -483,19 +483,18 @@ void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned l
 }
 template <int HCAP, int WCAP>
 int blocks_per_sm_t() {
-  static int blocks_per_sm = 0;
+  static int blocks_per_sm = 0;  // (occupancy: the same on every B200)
   const int smem = (int)sizeof(FlushSmem<HCAP, WCAP>);
+  func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (blocks_per_sm == 0) {
-    cudaFuncSetAttribute(k_flush<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     int b = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush<HCAP, WCAP>, FT, smem);
-    b = std::max(b, 1);
-    // ask for no more shared memory than the resident CTAs need: the rest stays L1, which
-    // holds the object-table lines the match phase gathers
-    const int carve = std::min(100, (b * (smem + 1024) * 100 + 228 * 1024 - 1) / (228 * 1024));
-    cudaFuncSetAttribute(k_flush<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-    blocks_per_sm = b;
+    blocks_per_sm = std::max(b, 1);
   }
+  // ask for no more shared memory than the resident CTAs need: the rest stays L1, which
+  // holds the object-table lines the match phase gathers (per device, like the size above)
+  const int carve = std::min(100, (blocks_per_sm * (smem + 1024) * 100 + 228 * 1024 - 1) / (228 * 1024));
+  func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
   return blocks_per_sm;
 }
 }  // namespace

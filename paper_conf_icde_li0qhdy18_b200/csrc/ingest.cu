@@ -37,8 +37,11 @@ static_assert((1 << CH_BITS) == CH, "hash slots: a power of two");
 constexpr int SPC = CH / CT;       // hash slots per thread in the scan
 constexpr int SCATTER_SMEM = CU * 16;
 static_assert(CU < 65536, "tile offsets and counts are packed in 16 bits");
+static_assert(CPT % 2 == 0, "the scatter works in two halves of CPT/2 updates per thread");
 constexpr uint32_t REMOTE_CELL = 0xFFFFFFFEu;  // classify: pseudo-cell of other ranks' updates
 constexpr int CLASSIFY_SMEM = (3 * CH + CT / 32) * 4;
+static_assert(CLASSIFY_SMEM <= 227 * 1024, "classify tile state exceeds shared memory");
+static_assert(SCATTER_SMEM <= 227 * 1024, "scatter tile exceeds shared memory");
 
 __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict__ upd, uint64_t n,
                                                         DevGraph g, DevState s,
@@ -112,7 +115,7 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
     tl = max(tl, m.w);
   }
   tl = __reduce_max_sync(0xffffffffu, tl);
-  if (lane == 0 && tl) atomicMax(&s.st->t_max, tl);
+  if (lane == 0 && tl) atomicMax(&s.st->batch_tmax, tl);  // (t_max: only if accepted, k_ingest_alloc)
   __syncthreads();
   // exclusive scan of the slot counts = each cell's group offset in the tile's sorted order
   {
@@ -219,8 +222,18 @@ __device__ __forceinline__ void alloc_cell_warp(const DevGraph& g, const DevStat
   s.bcount[c * BCOUNT_STRIDE] = 0;
 }
 
+// an accepted batch's newest t becomes t_now of the expiry rule (a rejected one changes nothing)
+__device__ __forceinline__ void commit_batch_tmax(const DevState& s, bool err) {
+  if (!err && blockIdx.x == 0 && threadIdx.x == 0) {
+    const unsigned bt = *((volatile unsigned*)&s.st->batch_tmax);
+    if (bt) atomicMax(&s.st->t_max, bt);
+  }
+}
+
 __global__ void __launch_bounds__(256) k_ingest_alloc(DevGraph g, DevState s) {
-  alloc_cell_warp(g, s, blockIdx.x * blockDim.x + threadIdx.x, s.st->ingest_err != 0);
+  const bool err = s.st->ingest_err != 0;
+  commit_batch_tmax(s, err);
+  alloc_cell_warp(g, s, blockIdx.x * blockDim.x + threadIdx.x, err);
 }
 
 // One CTA per classify tile.  The tile's updates are staged in shared memory (coalesced), then
@@ -298,11 +311,7 @@ static uint16_t* perm_of(uint2* tmp, uint64_t n) { return reinterpret_cast<uint1
 size_t ingest_tmp_bytes(uint64_t n) { return (size_t)n * (sizeof(uint2) + sizeof(uint16_t)); }
 void launch_ingest_classify(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
                             uint2* tmp, cudaStream_t st) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_ingest_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, CLASSIFY_SMEM);
-    attr = true;
-  }
+  func_attr_once(k_ingest_classify, cudaFuncAttributeMaxDynamicSharedMemorySize, CLASSIFY_SMEM);
   unsigned blocks = (unsigned)((n + CU - 1) / CU);
   k_ingest_classify<<<blocks, CT, CLASSIFY_SMEM, st>>>(upd, n, g, s, tmp, perm_of(tmp, n));
 }
@@ -311,11 +320,7 @@ void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st) 
 }
 void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                            const DevState& s, const uint2* tmp, cudaStream_t st) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_ingest_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, SCATTER_SMEM);
-    attr = true;
-  }
+  func_attr_once(k_ingest_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, SCATTER_SMEM);
   unsigned blocks = (unsigned)((n + CU - 1) / CU);
   k_ingest_scatter<<<blocks, CT, SCATTER_SMEM, st>>>(upd, n, seq0, g, s, tmp,
                                           perm_of(const_cast<uint2*>(tmp), n));
@@ -445,7 +450,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
     }
   }
   tl = __reduce_max_sync(0xffffffffu, tl);
-  if (lane == 0 && tl) atomicMax(&s.st->t_max, tl);
+  if (lane == 0 && tl) atomicMax(&s.st->batch_tmax, tl);  // (folded into t_max once accepted)
   __syncthreads();
   {  // exclusive scan of the slot counts = each group's offset in the tile's cell order
     const uint32_t spc = ch / FT;
@@ -490,6 +495,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   grid_barrier(&s.st->ingest_bar, G);
   {
     const bool err = *((volatile unsigned*)&s.st->ingest_err) != 0;
+    commit_batch_tmax(s, err);
     const uint32_t nw = G * (FT / 32);
     for (uint32_t c0 = (blockIdx.x * (FT / 32) + wid) * 32; c0 < g.n_cells; c0 += nw * 32)
       alloc_cell_warp(g, s, c0 + lane, err);
@@ -556,11 +562,8 @@ bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p
 
 cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                                 const DevState& s, const IngestPlan& p, cudaStream_t st) {
-  static bool smem_set = false;
-  if (!smem_set) {
-    cudaFuncSetAttribute(k_ingest_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    smem_set = true;
-  }
+  const cudaError_t ae = func_attr_once(k_ingest_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  if (ae != cudaSuccess) return ae;
   // cooperative (every CTA resident at once, or the launch fails: the grid barriers need it) and
   // a programmatic dependent of the batch's status reset
   cudaLaunchAttribute attr[2];

@@ -57,6 +57,8 @@ struct DevStatus {
   unsigned int l0_exited;   // CTAs of the starting level's launch that have exited this round
   unsigned int round_end;   // (marks the end of the per-round reset region)
   unsigned int ingest_bar;  // grid-barrier arrivals of the fused ingest launch (reset per batch)
+  unsigned int batch_tmax;  // newest t of the current ingest batch's valid updates (reset per
+                            // batch); folded into t_max only once the batch is accepted
 };
 
 struct DevGraph {
@@ -175,6 +177,14 @@ __device__ inline void request_flush(const DevState& s, uint32_t c, uint32_t epo
 
 // Launchers (defined in the .cu files; called by api.cu).
 namespace gg {
+// A kernel attribute set once per (kernel, attribute, device): the attribute is a property of
+// the kernel on the current device, so a process driving several devices needs it on each.
+// Thread-safe; returns the cudaFuncSetAttribute result of the first call.
+cudaError_t func_attr_once(const void* kernel, cudaFuncAttribute attr, int value);
+template <class K>
+inline cudaError_t func_attr_once(K* kernel, cudaFuncAttribute attr, int value) {
+  return func_attr_once(reinterpret_cast<const void*>(kernel), attr, value);
+}
 // Small device-side word stores (status counters).  A kernel, not cudaMemset/cudaMemcpy: those
 // can run on a copy engine and would queue behind a staged ingest transfer.
 struct WordSet {

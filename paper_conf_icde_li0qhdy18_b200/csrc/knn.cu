@@ -998,16 +998,16 @@ static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
 
 // resident CTAs per SM of a shared-memory level's kernel (occupancy calculator, cached)
 static uint32_t blocks_per_sm(int level, bool cta) {
-  static int bps[2][NLEVELS] = {};
+  static int bps[2][NLEVELS] = {};  // (occupancy: the same on every B200)
+  // the attribute is per device: set on every device this process launches on
+  if (cta) func_attr_once(cta_kernel(level), cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
+  else func_attr_once(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   int& b = bps[cta ? 1 : 0][level];
   if (!b) {
     const int smem = (int)expand_warp_bytes(level, 1);
     if (cta) {
-      const CtaKernel kern = cta_kernel(level);
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, cta_warps(level) * 32, smem);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, cta_kernel(level), cta_warps(level) * 32, smem);
     } else {
-      cudaFuncSetAttribute(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32, smem);
     }
 #ifdef GG_L0_PER_SM

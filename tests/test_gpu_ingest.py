@@ -110,3 +110,89 @@ def test_fused_many_small_batches(gg):
         _same(grid.knn(q, 4), oracle.knn_from_updates(g, np.concatenate(hist), q, 4), f"round {r}")
     assert grid.stats()["kernel_launches"]["ingest_alloc"] == 0
     grid.close()
+
+
+# ------------------------------------------------------------------ stream order of caller inputs
+def _poisoned_then_valid(torch, dst, src, stream, spin_cycles):
+    """dst is first filled with invalid records (edge = 2^32-1) synchronously; then, queued on
+    `stream` behind a spin kernel, overwritten with the valid batch src.  A library call that
+    read dst before the copy ran would see the invalid records (EINVAL) -- the race of the
+    round-1 C4 sweep (tools/c4_sweep.py)."""
+    dst.fill_(-1)
+    torch.cuda.synchronize()
+    with torch.cuda.stream(stream):
+        torch.cuda._sleep(spin_cycles)
+        dst.copy_(src)
+
+
+@pytest.mark.parametrize("producer", ["side_stream", "default_stream"])
+def test_device_input_ordered_after_producer(gg, producer):
+    """50 ingests of a 10^6-row device batch produced by still-running torch work, with no
+    host synchronisation between producing and ingesting: every batch is accepted and the
+    answers are the oracle's (ggrid_wait_stream / the legacy-stream ordering of the C ABI)."""
+    import torch
+
+    g = synth.table_ii_graph("NY", scale=0.2)
+    walk = synth.RandomWalk(g, 20_000)
+    grid = gg.GGrid(g, 256, max_objects=20_000, log_capacity=1 << 26)
+    side = torch.cuda.Stream() if producer == "side_stream" else torch.cuda.default_stream()
+    dev = torch.empty((1_000_000, 4), dtype=torch.int32, device="cuda")
+    hist = []
+    for it in range(50):
+        u = walk.ticks(50)  # 10^6 updates
+        hist.append(u)
+        src = torch.from_numpy(u.view(np.int32)).cuda()
+        _poisoned_then_valid(torch, dev, src, side, 2_000_000)
+        with torch.cuda.stream(side):
+            grid.ingest(dev)  # no synchronize: the library must wait for the copy
+    torch.cuda.synchronize()
+    q = synth.queries(g, 300)
+    _same(grid.knn(q, 10), oracle.knn_from_updates(g, np.concatenate(hist), q, 10), producer)
+    grid.close()
+
+
+def test_async_ingest_input_reuse_after_signal(gg):
+    """opts.async_ingest: the kernels of an ingest read the device batch after the call
+    returns.  The binding orders the caller's stream after them (ggrid_signal_stream), so the
+    caller may overwrite the buffer right away; answers stay the oracle's."""
+    import torch
+
+    g = synth.table_ii_graph("NY", scale=0.1)
+    walk = synth.RandomWalk(g, 5_000)
+    grid = gg.GGrid(g, 256, max_objects=5_000, async_ingest=True)
+    dev = torch.empty((200_000, 4), dtype=torch.int32, device="cuda")
+    hist = []
+    for it in range(20):
+        u = walk.ticks(40)
+        hist.append(u)
+        dev.copy_(torch.from_numpy(u.view(np.int32)))
+        grid.ingest(dev)
+        dev.fill_(-1)  # queued after the library's kernels on the caller's (current) stream
+    grid.sync()
+    q = synth.queries(g, 200)
+    _same(grid.knn(q, 8), oracle.knn_from_updates(g, np.concatenate(hist), q, 8), "async reuse")
+    grid.close()
+
+
+@pytest.mark.parametrize("mode", [0, 3])
+def test_rejected_batch_leaves_t_now(gg, mode):
+    """A rejected batch changes no observable state (ggrid.h): its valid records' far-future
+    t must not become t_now of the expiry rule (reading R21), which would expire every cached
+    extent of an index built with t_delta."""
+    g = synth.table_ii_graph("NY", scale=0.05)
+    walk = synth.RandomWalk(g, 2_000)
+    grid = gg.GGrid(g, 64, max_objects=2_000, t_delta=50_000, ingest_kernels=mode)
+    upd = walk.ticks(20)
+    grid.ingest(upd)
+    t_now = grid.stats()["t_now"]
+    bad = walk.ticks(2).copy()
+    bad[:, 3] = 4_000_000_000
+    bad[len(bad) // 3, 2] = 0xFFFFFFF0  # one offset out of range: the batch is rejected
+    with pytest.raises(gg.GGridError) as e:
+        grid.ingest(bad)
+    assert e.value.rc == gg.GGRID_EINVAL
+    assert grid.stats()["t_now"] == t_now
+    q = synth.queries(g, 200)
+    _same(grid.knn(q, 6), oracle.knn_from_updates(g, upd, q, 6), "after a rejected batch")
+    assert grid.stats()["records_expired"] == 0
+    grid.close()

@@ -38,7 +38,8 @@ def run_one(g, gname, n_obj, r, Q, k, cell_size, max_steps, l2):
     grid = gg.GGrid(g, cell_size, max_objects=n_obj, profile=True, log_capacity=cap)
     out_o = torch.empty((Q, k), dtype=torch.int32, device="cuda")
     out_d = torch.empty_like(out_o)
-    grid.ingest(walk.ticks(1))  # every object placed
+    grid.ingest(walk.ticks(1))  # every object placed (ordered after the walk kernels: the binding
+    # makes the library stream wait for torch's current stream, ggrid_wait_stream)
     rows = []
     gen_s = 0.0
     for s in range(1 + n_steps):  # step 0 = warm-up
