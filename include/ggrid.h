@@ -40,7 +40,7 @@ extern "C" {
 #define GGRID_ENOMEM (-2)    /* device or host allocation failed / log arena exhausted */
 #define GGRID_ECUDA (-3)     /* a CUDA runtime error (sticky errors included) */
 #define GGRID_ENCCL (-4)     /* reserved for the multi-GPU exchange */
-#define GGRID_EOVERFLOW (-5) /* the global arrival index seq would exceed 2^32-1 */
+#define GGRID_EOVERFLOW (-5) /* one ingest batch of more than 2^32-2 updates */
 #define GGRID_PAD 0xFFFFFFFFu
 
 /* Road network G = <V, E> (P@7808-8419): a directed graph, arc a = src[a] -> dst[a] with
@@ -127,7 +127,7 @@ enum {
 };
 
 typedef struct ggrid_stats_t {
-  uint64_t n_updates;        /* updates ingested (= next seq)                        */
+  uint64_t n_updates;        /* updates ingested                                     */
   uint64_t n_queries;        /* queries answered                                     */
   uint64_t knn_calls;
   uint64_t knn_rounds;       /* flush+expand rounds over all knn calls               */
@@ -156,6 +156,7 @@ typedef struct ggrid_stats_t {
   uint64_t records_expired;  /* cached records dropped unread by t_delta expiry       */
   uint64_t expand_promotions;/* query runs that overflowed a capacity level (rerun on the next) */
   uint64_t expand_retries;   /* query runs stopped by a cell with cached updates (rerun after its flush) */
+  uint64_t seq_rebases;      /* re-bases of the arrival index (every ~2^32 updates)  */
 } ggrid_stats_t;
 
 /* Build the index (graph grid, P@11423-15818; object table P@15869; message lists
@@ -166,12 +167,16 @@ typedef struct ggrid_stats_t {
  * Ownership: inputs are copied; *out is owned by the caller until ggrid_free. */
 int ggrid_build(const ggrid_graph* g, uint32_t cell_size, const ggrid_opts* opts, ggrid_t* out);
 
-/* Append n updates (Alg. 1, P@18177-19248, lazy: P@17773-17981).  The global arrival
- * index seq of u[i] is (updates ingested before this call) + i.  An object's location is
- * its update with the largest (t, seq) (readings R7/R8); t needs no order.
+/* Append n updates (Alg. 1, P@18177-19248, lazy: P@17773-17981).  Updates are ordered by
+ * arrival: u[i] arrives after every update of earlier calls and after u[0..i).  An object's
+ * location is its update with the largest (t, arrival) (readings R7/R8); t needs no
+ * order.  Internally the arrival index is a 32-bit seq that is re-based (one garbage
+ * collection plus a key rewrite, ggrid_stats.seq_rebases) whenever a batch would run past
+ * 2^32 - 1, so a handle accepts an unbounded stream.
  * u: host or device pointer to n records.  Errors: EINVAL (obj >= max_objects,
- * edge >= n_arcs, offset >= w[edge]: the whole batch is rejected), EOVERFLOW, ENOMEM
- * (log arena full even after garbage collection), ECUDA. */
+ * edge >= n_arcs, offset >= w[edge]: the whole batch is rejected), EOVERFLOW (a single batch
+ * of more than 2^32 - 2 updates), ENOMEM (log arena full even after garbage collection),
+ * ECUDA. */
 int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n);
 
 /* Pipelined ingest (the paper's pipelined transfer, P@45017-45625: the GPU works on one group

@@ -60,7 +60,8 @@ class ggrid_stats_t(ctypes.Structure):
         ("kernel_launches", ctypes.c_uint64 * NK), ("kernel_ms", ctypes.c_double * NK)] + [
         (n, ctypes.c_uint32) for n in ["n_cells", "cell_size", "delta", "n_vertices", "n_arcs", "max_objects",
                                        "t_delta", "t_now"]] + [("records_expired", ctypes.c_uint64),
-                                       ("expand_promotions", ctypes.c_uint64), ("expand_retries", ctypes.c_uint64)]
+                                       ("expand_promotions", ctypes.c_uint64), ("expand_retries", ctypes.c_uint64),
+                                       ("seq_rebases", ctypes.c_uint64)]
 
 
 class ggrid_prior_art_result(ctypes.Structure):

@@ -139,7 +139,12 @@ struct ggrid_s {
   DevStatus* d_status = nullptr;
   DevStatus* h_status = nullptr;  // pinned
   DevStatus* h_status_dev = nullptr;  // its mapped device alias (the kernels' store target)
-  uint64_t seq_next = 0;
+  // Arrival order (reading R7): the key of an update is (t << 32) | seq with seq = seq_next + i.
+  // seq starts at 1 (key 0 stays "no update"); when a batch would run past 2^32 - 1 the keys of
+  // the whole index are re-based (rebase()), so a handle takes any number of updates.
+  uint64_t seq_next = 1;
+  uint64_t n_ingested = 0;  // updates accepted (or queued, asynchronous) so far
+  uint64_t rebases = 0;
   uint32_t epoch = 0;
   DBuf upd_stage, tmp, q_stage, out_stage, lists, l2_scratch, dump_stage, gc_buf, misc, flush_spill,
       bound_stage, remote_stage, merge_stage;
@@ -272,6 +277,7 @@ struct ggrid_s {
   }
 
   int gc();
+  int rebase();
   int ensure_arena(uint64_t need_records, uint32_t need_ext);
   // upper bound of the objects live on the device (exact after a sync)
   uint64_t n_live_hi() const {
@@ -339,6 +345,22 @@ int ggrid_s::gc() {
   // gc_buf stays allocated (live-sized, small next to the arena): a cudaMalloc/cudaFree pair
   // per collection costs milliseconds and synchronises the device
   stats.gc_runs++;
+  return GGRID_OK;
+}
+
+// Re-basing of the arrival index (a sustained update stream, §8(f) N1: P@53218 "we can safely
+// delete the messages before t_now - t_Delta").  Only the ORDER of keys matters (the validity
+// test is key == ot_key[obj], and ot_key is a max).  After a garbage collection every live
+// object has at most one record left, the one whose key equals its ot_key (GC keeps exactly
+// the winners).  Rewriting every key k != 0 as (k & ~0xFFFFFFFF) | 1 in the arena AND in ot_key
+// therefore keeps every equality, and keeps every existing key below any later update's key
+// (t, seq >= 2) with the same t -- later arrivals still win ties (reading R7).
+int ggrid_s::rebase() {
+  RC(gc());  // (syncs: no ingest batch is in flight)
+  launch(GGRID_K_OTHER, [&] { launch_rebase_keys(s, h_status->arena_top, stream); });
+  RC(sync());
+  seq_next = 2;
+  rebases++;
   return GGRID_OK;
 }
 
@@ -607,9 +629,11 @@ int ggrid_free(ggrid_t h) {
 
 // ingest n updates already resident in device memory at d_u (the main stream must be
 // ordered after their arrival)
+static constexpr uint64_t kMaxBatch = 0xFFFFFFFEull;  // seq 2 .. 2^32-1 after a re-base
 static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
-  if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
+  if (n > kMaxBatch) return GGRID_EOVERFLOW;
   if (h->async_ingest) RC(h->take_deferred());  // an earlier batch was rejected
+  if (h->seq_next + n > 0x100000000ull) RC(h->rebase());
   const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
   RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
   IngestPlan fp;
@@ -648,7 +672,8 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
     h->pend_ext += ext_need;
     h->pend_updates += n;
     h->seq_next += n;
-    h->stats.n_updates = h->seq_next;
+    h->n_ingested += n;
+    h->stats.n_updates = h->n_ingested;
     return GGRID_OK;
   }
   RC(h->sync());
@@ -669,7 +694,8 @@ static int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   }
   if (err & ERR_ARENA) return GGRID_ENOMEM;
   h->seq_next += n;
-  h->stats.n_updates = h->seq_next;
+  h->n_ingested += n;
+  h->stats.n_updates = h->n_ingested;
   return GGRID_OK;
 }
 
@@ -677,7 +703,7 @@ int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
   if (!h) return GGRID_EINVAL;
   if (n == 0) return GGRID_OK;
   if (!u) return GGRID_EINVAL;
-  if (h->seq_next + n > 0x100000000ull) return GGRID_EOVERFLOW;
+  if (n > kMaxBatch) return GGRID_EOVERFLOW;
   CK(cudaSetDevice(h->device));
   const uint4* d_u = reinterpret_cast<const uint4*>(u);
   RC(h->order_inputs(h->stream));  // u may be the output of a caller kernel still running
@@ -986,7 +1012,7 @@ int ggrid_knn_ex(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, cons
 
 int ggrid_shard(ggrid_t h, uint32_t n_ranks, uint32_t rank) {
   if (!h || n_ranks == 0 || n_ranks > 64 || rank >= n_ranks || n_ranks > h->n_cells) return GGRID_EINVAL;
-  if (h->seq_next != 0) return GGRID_EINVAL;  // ownership is fixed before the first update
+  if (h->n_ingested != 0) return GGRID_EINVAL;  // ownership is fixed before the first update
   h->s.n_ranks = n_ranks;
   h->s.rank = rank;
   return GGRID_OK;
@@ -1242,6 +1268,7 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
   s.t_delta = h->t_delta;
   s.t_now = h->h_status->t_max;
   s.records_expired = h->h_status->records_expired;
+  s.seq_rebases = h->rebases;
   s.expand_promotions = h->h_status->ex_promoted;
   s.expand_retries = h->h_status->ex_retried;
   *out = s;

@@ -620,6 +620,19 @@ void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState&
   cudaLaunchKernelEx(&cfg, k_seed, q, nq, g, s, epoch, mode, q_copy);
 }
 
+// Arrival-index re-base (api.cu rebase(): right after a garbage collection)
+__global__ void __launch_bounds__(256) k_rebase_keys(DevState s, unsigned long long n_records) {
+  const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+  for (unsigned long long i = blockIdx.x * blockDim.x + threadIdx.x; i < n_records + s.max_objects; i += stride) {
+    unsigned long long* p = i < n_records ? s.ar.key + i : s.ot_key + (i - n_records);
+    const unsigned long long k = *p;
+    if (k) *p = (k & 0xFFFFFFFF00000000ull) | 1ull;
+  }
+}
+void launch_rebase_keys(const DevState& s, unsigned long long n_records, cudaStream_t st) {
+  k_rebase_keys<<<148 * 8, 256, 0, st>>>(s, n_records);
+}
+
 // Every dirty cell (eager cleaning; all_cells additionally queues clean cells for GC).
 __global__ void __launch_bounds__(256) k_mark_dirty(DevGraph g, DevState s, uint32_t epoch,
                                                     int all_cells) {

@@ -231,6 +231,8 @@ void launch_ingest_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const De
 enum SeedMode { SEED_DST = 0, SEED_NEIGHBORS = 1, SEED_ALL = 2 };
 void launch_seed(const uint2* q, uint32_t nq, const DevGraph& g, const DevState& s, uint32_t epoch,
                  int mode, uint2* q_copy, cudaStream_t st);
+// every nonzero key k of the arena's first n_records and of ot_key becomes (k & ~0xFFFFFFFF) | 1
+void launch_rebase_keys(const DevState& s, unsigned long long n_records, cudaStream_t st);
 void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int all_cells,
                        cudaStream_t st);
 // Flush the cells flush_list[begin .. st->n_flush) writing compacted lists into `out`

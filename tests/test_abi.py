@@ -34,11 +34,28 @@ def test_library_exports_every_declared_symbol(gg):
     assert sorted(gg.EXPORTS) == names
 
 
-def test_struct_layouts_match_header(gg):
-    # sizes the header implies on LP64
-    assert ctypes.sizeof(gg.ggrid_graph) == 8 + 5 * 8
-    assert ctypes.sizeof(gg.ggrid_opts) == 4 + 4 + 4 + 4 + 8 + 4 * 4 + 8 + 4 + 4  # async_ingest + tail padding
-    assert ctypes.sizeof(gg.ggrid_stats_t) == 16 * 8 + 8 * 8 + 8 * 8 + 8 * 4 + 8 + 2 * 8  # + promotions, retries
+def test_struct_layouts_match_header(gg, tmp_path):
+    """Every struct of include/ggrid.h: the C compiler's size and field offsets (gcc on the
+    header itself) equal the ctypes mirror of the binding."""
+    import subprocess
+
+    structs = {"ggrid_graph": gg.ggrid_graph, "ggrid_opts": gg.ggrid_opts, "ggrid_stats_t": gg.ggrid_stats_t,
+               "ggrid_prior_art_result": gg.ggrid_prior_art_result}
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "ggrid.h"', "int main(void) {"]
+    for name, cls in structs.items():
+        lines.append(f'  printf("{name} %zu\\n", sizeof({name}));')
+        for f, _ in cls._fields_:
+            lines.append(f'  printf("{name}.{f} %zu\\n", offsetof({name}, {f}));')
+    lines += ["  return 0;", "}"]
+    c = tmp_path / "layout.c"
+    c.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), str(c), "-o", str(exe)])
+    got = dict(l.split() for l in subprocess.check_output([str(exe)], text=True).splitlines())
+    for name, cls in structs.items():
+        assert int(got[name]) == ctypes.sizeof(cls), name
+        for f, _ in cls._fields_:
+            assert int(got[f"{name}.{f}"]) == getattr(cls, f).offset, f"{name}.{f}"
 
 
 def test_zvalue_worked_example(gg):

@@ -196,3 +196,49 @@ def test_rejected_batch_leaves_t_now(gg, mode):
     _same(grid.knn(q, 6), oracle.knn_from_updates(g, upd, q, 6), "after a rejected batch")
     assert grid.stats()["records_expired"] == 0
     grid.close()
+
+
+def test_sustained_stream_beyond_2_32_updates(gg):
+    """A handle takes more than 2^32 updates (a sustained stream): the 32-bit
+    arrival index is re-based at a garbage collection and the answers stay the oracle's.
+    Two device batches A, B (10^7 updates each) alternate 215 times (4.3e9 updates, ending
+    with B); by max-(t, arrival) the final snapshot equals the oracle's snapshot of [A, B]
+    (repeating a batch adds no t value, and the last copy of each holds every record's latest
+    arrival)."""
+    import torch
+
+    g = synth.table_ii_graph("NY")
+    walk = synth.RandomWalk(g, 100_000, inject=True)
+    a, b = walk.ticks(100), walk.ticks(100)
+    da = torch.from_numpy(a.view(np.int32)).cuda()
+    db = torch.from_numpy(b.view(np.int32)).cuda()
+    grid = gg.GGrid(g, 1024, max_objects=100_000, log_capacity=1 << 26)
+    q = synth.queries(g, 500)
+    for it in range(215):
+        grid.ingest(da)
+        grid.ingest(db)
+        if it == 3:  # before the re-base: answers of the stream so far
+            _same(grid.knn(q, 10), oracle.knn_from_updates(g, np.concatenate([a, b]), q, 10), "before")
+    st = grid.stats()
+    assert st["n_updates"] == 430 * len(a) > (1 << 32)
+    assert st["seq_rebases"] == 1
+    _same(grid.knn(q, 10), oracle.knn_from_updates(g, np.concatenate([a, b]), q, 10), "after the re-base")
+    # ties across the re-base: a batch re-sent after it still wins equal timestamps
+    grid.ingest(da)
+    _same(grid.knn(q, 10), oracle.knn_from_updates(g, np.concatenate([b, a]), q, 10), "A re-sent")
+    grid.close()
+
+
+def test_overflowing_batch_is_eoverflow(gg):
+    """A single batch of 2^32 - 1 updates cannot be ordered by a 32-bit arrival index (ggrid.h):
+    EOVERFLOW, checked before the buffer is read."""
+    import torch
+
+    g = synth.lattice_graph(8, 8, 1, 4)
+    grid = gg.GGrid(g, 16, max_objects=16)
+    tiny = torch.zeros((1, 4), dtype=torch.int32, device="cuda")
+    with pytest.raises(gg.GGridError) as e:
+        gg.ggrid_ingest(grid.h, tiny, (1 << 32) - 1)
+    assert e.value.rc == gg.GGRID_EOVERFLOW
+    assert grid.stats()["n_updates"] == 0
+    grid.close()
