@@ -112,6 +112,8 @@ def _group_by(dest, world):
 
 def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = False):
     """Exact kNN of this rank's queries ((n, 2) int32 CUDA tensor) on a sharded index.
+    Library calls are ordered after torch's current stream by the binding (ggrid_wait_stream),
+    so the torch ops and collectives that produce their inputs need no host synchronisation.
     routed=True: every query is already at the owner of its cell (skips route/return).
     Returns (obj, dist) int32 CUDA tensors (n, k), and the number of remote requests sent."""
     import torch
@@ -120,18 +122,11 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
     n = int(queries.shape[0])
     i32 = torch.int32
 
-    def ready():
-        # the library runs on its own stream: inputs made by torch ops (or collectives, which
-        # torch orders on its current stream) must be complete before a library call
-        if dev.type == "cuda":
-            torch.cuda.current_stream(dev).synchronize()
-
     idx = torch.arange(n, dtype=i32, device=dev)
     if routed:
         mine, src_counts = torch.cat([queries, idx[:, None]], 1), None
     else:
         owner = torch.empty(n, dtype=i32, device=dev)
-        ready()
         grid.query_owner(queries, owner)
         order, counts = _group_by(owner, world)
         mine, src_counts = _a2a(torch.cat([queries, idx[:, None]], 1)[order], counts, world)
@@ -140,7 +135,6 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
     own_o = torch.empty((m, k), dtype=i32, device=dev)
     own_d = torch.empty((m, k), dtype=i32, device=dev)
     mask = torch.empty(m, dtype=torch.int64, device=dev)
-    ready()
     grid.knn_ex(q_m, k, None, own_o, own_d, mask)
     # requests: (edge, offset, bound, local row) to every rank in the mask
     bits = ((mask[:, None] >> torch.arange(world, device=dev, dtype=torch.int64)[None, :]) & 1).bool()
@@ -151,7 +145,6 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
     rep_o = torch.empty((int(got.shape[0]), k), dtype=i32, device=dev)
     rep_d = torch.empty_like(rep_o)
     got_q, got_b = got[:, :2].contiguous(), got[:, 2].contiguous()
-    ready()
     grid.knn_ex(got_q, k, got_b, rep_o, rep_d)
     replies, _ = _a2a(torch.cat([rep_o, rep_d, got[:, 3:4], torch.full_like(got[:, 3:4], rank)], 1),
                       got_counts, world)
@@ -167,7 +160,6 @@ def sharded_knn(grid, queries, k: int, world: int, rank: int, routed: bool = Fal
         ld[r_t, r_q] = replies[:, k:2 * k]
     fo = torch.empty((m, k), dtype=i32, device=dev)
     fd = torch.empty((m, k), dtype=i32, device=dev)
-    ready()
     grid.merge_topk(lo, ld, fo, fd)
     if routed:
         return fo, fd, int(req.shape[0])

@@ -47,6 +47,15 @@ CONFIGS = {
     "C2": dict(graph="FLA", n_objects=100_000, updates_per_object=10, n_queries=10_000, k=50, cell_size=1024),
     "C3": dict(graph="USA", n_objects=1_000_000, updates_per_object=64, n_queries=1 << 16, k=10, cell_size=1024),
 }
+# The bench step of each config: `preload_ticks` ticks of the walk cached once before the timed
+# region (C3: 64 cached records per object = 64M records >> L2), then per step
+# `step_ticks` ticks (every object reports once per tick: f = 1, P@58136) and n_queries queries.
+BENCH_STEPS = {
+    "C0": dict(preload_ticks=0, step_ticks=10),
+    "C1": dict(preload_ticks=0, step_ticks=100),
+    "C2": dict(preload_ticks=0, step_ticks=10),
+    "C3": dict(preload_ticks=64, step_ticks=1),
+}
 
 
 def _twin_arrays(ea, eb):
