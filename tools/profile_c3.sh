@@ -1,0 +1,31 @@
+#!/bin/bash
+# Round profiling pass at the bench's default workload (C3, one GPU; run under gpurun):
+#   1. the launch list of the bench command (gpu__time_duration per launch: cold-cache, serialised)
+#   2. ncu --set full of the step's hot kernels: the expansion (first timed step), the flush (the
+#      second full flush of the 64M-record log), the three-launch ingest of the 64M bulk batch
+#      and of a 1M-update step batch
+# Usage: tools/profile_c3.sh <tag>; then python tools/summarize_profiles.py <tag>
+set -u
+TAG=${1:-r2}
+OUT=gpurun_out/prof_$TAG
+mkdir -p $OUT
+export BENCH_ALLOW_SHORT=1
+B="python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-parity --e2e-steps 1"
+ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_C3.csv \
+    python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-parity --e2e-steps 1 > $OUT/launches_C3.log 2>&1
+echo "launch list rc=$?"
+cap() {  # name regex skip
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:$2 -s $3 -c 1 -o $OUT/$1 $B \
+      > $OUT/$1.log 2>&1
+  echo "$1 rc=$?"
+}
+cap expand_C3 k_expand_cta 3
+cap flush_C3 k_flush 1
+cap ingestscatter_C3 k_ingest_scatter 1
+cap ingestclassify_C3 k_ingest_classify 1
+cap stepscatter_C3 k_ingest_scatter 5
+for f in $OUT/*.ncu-rep; do
+  ncu -i $f --page raw --csv > ${f%.ncu-rep}_raw.csv 2>/dev/null
+  ncu -i $f --page source --csv > ${f%.ncu-rep}_source.csv 2>/dev/null
+done
+ls -la $OUT

@@ -45,14 +45,13 @@ def raw_rows(path):
 
 
 lines = [f"# Profiling summary — round tag `{tag}`", "",
-         "Source: `tools/profile_round.sh` under gpurun on one B200 (ncu 2025, `--clock-control none`).",
+         "Source: `tools/profile_c3.sh` (earlier rounds: `tools/profile_round.sh`) under gpurun on one B200 (ncu 2025, `--clock-control none`).",
          "Raw pages: `profiles/%s_<capture>_raw.csv`; launch list: `profiles/%s_launches_C1.csv`." % (tag, tag), ""]
 traffic = {}
 issue = {}
-for cap in ("expand_C1", "ingest_C1", "flush_C3"):
+caps = sorted(f[:-len("_raw.csv")] for f in os.listdir(src) if f.endswith("_raw.csv"))
+for cap in caps:
     p = os.path.join(src, f"{cap}_raw.csv")
-    if not os.path.exists(p):
-        continue
     shutil.copy(p, os.path.join(dst, f"{tag}_{cap}_raw.csv"))
     for hdr, units, r in raw_rows(p):
         name = r[hdr.index("Kernel Name")].split("(")[0]
@@ -80,8 +79,9 @@ for cap in ("expand_C1", "ingest_C1", "flush_C3"):
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
         rd *= scale.get(units[hdr.index("dram__bytes_read.sum")], 1)
         wr *= scale.get(units[hdr.index("dram__bytes_write.sum")], 1)
-        kind = {"expand_C1": "expand", "ingest_C1": "ingest", "flush_C3": "flush"}[cap]
-        cfg = cap.split("_")[1]
+        kind, cfg = cap.rsplit("_", 1)
+        kind = {"ingestscatter": "ingest_bulk_scatter", "ingestclassify": "ingest_bulk_classify",
+                "stepscatter": "ingest_step_scatter"}.get(kind, kind)
         traffic.setdefault(cfg, collections.defaultdict(float))[kind] += rd + wr
         if "smsp__issue_active.avg.pct_of_peak_sustained_active" in hdr:  # (non-HBM limiters)
             issue.setdefault(cfg, {})[kind] = {
@@ -89,9 +89,9 @@ for cap in ("expand_C1", "ingest_C1", "flush_C3"):
                 "dram_throughput_pct": float(r[hdr.index("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed")]),
                 "top_stalls": top, "capture": f"profiles/{tag}_summary.md"}
 
-ll = os.path.join(src, "launches_C1.csv")
-if os.path.exists(ll):
-    shutil.copy(ll, os.path.join(dst, f"{tag}_launches_C1.csv"))
+for ll in [os.path.join(src, f) for f in sorted(os.listdir(src)) if f.startswith("launches_") and f.endswith(".csv")]:
+    lcfg = os.path.basename(ll)[len("launches_"):-4]
+    shutil.copy(ll, os.path.join(dst, f"{tag}_launches_{lcfg}.csv"))
     rows = list(csv.reader(open(ll)))
     hi = [i for i, r in enumerate(rows) if r and r[0] == "ID"][0]
     h = rows[hi]
@@ -99,7 +99,7 @@ if os.path.exists(ll):
     for r in rows[hi + 1:]:
         agg[r[h.index("Kernel Name")].split("(")[0]].append(float(r[h.index("Metric Value")].replace(",", "")))
     tot = sum(sum(v) for k, v in agg.items() if "gg::" in k)
-    lines += ["## Launch list, default bench (C1), cold-cache serialised (`gpu__time_duration.sum`)", "",
+    lines += [f"## Launch list, bench ({lcfg}), cold-cache serialised (`gpu__time_duration.sum`)", "",
               "| kernel | launches | mean µs | share of library time |", "|---|---|---|---|"]
     for k, v in sorted(agg.items(), key=lambda x: -sum(x[1])):
         share = f"{100 * sum(v) / tot:.1f}%" if "gg::" in k else "(torch L2 flush, untimed)"
