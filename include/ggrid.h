@@ -31,6 +31,9 @@
 
 #include <stdint.h>
 
+#if defined(__GNUC__)
+#pragma GCC visibility push(default) /* the library is built with -fvisibility=hidden */
+#endif
 #ifdef __cplusplus
 extern "C" {
 #endif
@@ -341,6 +344,9 @@ const char* ggrid_version(void);
 
 #ifdef __cplusplus
 }
+#endif
+#if defined(__GNUC__)
+#pragma GCC visibility pop
 #endif
 
 #endif /* GGRID_H */

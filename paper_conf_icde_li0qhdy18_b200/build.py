@@ -18,7 +18,8 @@ LIB = os.path.join(PKG, "libggrid.so")
 SOURCES = ["api.cu", "ingest.cu", "flush.cu", "knn.cu", "prior_art.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUDE]
+FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
+         "-I" + INCLUDE]
 # experiment hooks: extra nvcc flags and an alternative output path (default build unaffected)
 EXTRA = os.environ.get("GGRID_NVCC_FLAGS", "").split()
 if os.environ.get("GGRID_LIB_OUT"):
