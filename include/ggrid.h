@@ -42,7 +42,7 @@ extern "C" {
 #define GGRID_EINVAL (-1)    /* bad argument (range, null pointer, k, offsets, ...) */
 #define GGRID_ENOMEM (-2)    /* device or host allocation failed / log arena exhausted */
 #define GGRID_ECUDA (-3)     /* a CUDA runtime error (sticky errors included) */
-#define GGRID_ENCCL (-4)     /* reserved for the multi-GPU exchange */
+#define GGRID_ENCCL (-4)     /* the multi-GPU exchange failed (NCCL or the caller's all-to-all) */
 #define GGRID_EOVERFLOW (-5) /* one ingest batch of more than 2^32-2 updates */
 #define GGRID_PAD 0xFFFFFFFFu
 
@@ -60,6 +60,14 @@ typedef struct ggrid_graph {
   const int32_t* x;
   const int32_t* y;
 } ggrid_graph;
+
+/* A caller-supplied all-to-all of byte segments (multi-process use without NCCL, see
+ * "multi-GPU"): send[p] (send_bytes[p]) goes to rank p; recv[p] (recv_bytes[p]) receives
+ * rank p's segment for this rank.  Device pointers on this rank's device; `stream` (a
+ * cudaStream_t) has completed all prior work when the function is called, and the function
+ * must return only once recv is complete.  Returns 0 on success. */
+typedef int (*ggrid_alltoall_fn)(void* ctx, void* const* send, const uint64_t* send_bytes, void* const* recv,
+                                 const uint64_t* recv_bytes, uint32_t n_ranks, void* stream);
 
 /* Build options; pass NULL for defaults (each 0 field also means "default"). */
 typedef struct ggrid_opts {
@@ -97,7 +105,32 @@ typedef struct ggrid_opts {
                               scatter separated by grid barriers), larger batches by
                               three launches; 3 = always the three launches.  Both
                               produce the same index state.                        */
+  /* ---- multi-GPU (see "multi-GPU" below).  All 0 = one GPU.            */
+  uint32_t n_gpus;         /* > 1: ONE index over n_gpus shards driven by this process,
+                              shard r on devices[r] (cell ownership, one request/reply
+                              exchange per query batch)                            */
+  const int* devices;      /* n_gpus device ordinals (NULL = 0 .. n_gpus-1).  An ordinal
+                              may repeat (several shards on one device: the loopback
+                              exchange -- a test mode of the same protocol)         */
+  uint32_t exchange_kind;  /* GGRID_EXCHANGE_*: 0 = auto (NCCL when the devices are
+                              distinct and libnccl loads, else loopback)            */
+  uint32_t n_ranks, rank;  /* multi-process (one process per GPU): this handle is shard
+                              `rank` of `n_ranks`; every rank builds with the same graph
+                              and ingests the same update stream                    */
+  const void* nccl_id;     /* multi-process over NCCL: the 128-byte ncclUniqueId made by
+                              ggrid_nccl_unique_id on one rank and shared by the caller */
+  ggrid_alltoall_fn exchange;
+                           /* multi-process without NCCL: the caller's all-to-all of
+                              byte segments (device pointers on this rank's device;
+                              send[p] goes to rank p, recv[p] receives rank p's
+                              send[rank]; the stream's prior work is complete when it
+                              is called; return 0 on success)                      */
+  void* exchange_ctx;      /* passed to exchange                                    */
 } ggrid_opts;
+
+#define GGRID_EXCHANGE_AUTO 0u
+#define GGRID_EXCHANGE_LOOPBACK 1u
+#define GGRID_EXCHANGE_NCCL 2u
 
 typedef struct ggrid_s* ggrid_t;
 
@@ -160,6 +193,8 @@ typedef struct ggrid_stats_t {
   uint64_t expand_promotions;/* query runs that overflowed a capacity level (rerun on the next) */
   uint64_t expand_retries;   /* query runs stopped by a cell with cached updates (rerun after its flush) */
   uint64_t seq_rebases;      /* re-bases of the arrival index (every ~2^32 updates)  */
+  uint32_t n_shards;         /* shards of the index (1: one GPU)                      */
+  uint32_t exchange_kind;    /* GGRID_EXCHANGE_* in use (0: none; 3: the caller's all-to-all) */
 } ggrid_stats_t;
 
 /* Build the index (graph grid, P@11423-15818; object table P@15869; message lists
@@ -216,7 +251,31 @@ int ggrid_knn_commit(ggrid_t h, uint32_t k, uint32_t* out_obj, uint32_t* out_dis
 int ggrid_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
               uint32_t* out_dist);
 
-/* ---- cell-ownership sharding across ranks (one process per GPU) ------------
+/* ---- multi-GPU -------------------------------------------------------------
+ *
+ * An index over R shards answers exactly what one GPU answers (Def. 1).  Shard r owns the
+ * contiguous Z-order range of cells c with floor(c R / n_cells) == r (the graph is replicated;
+ * logs and cleaned lists live on the owner; the object table is replicated).  The library runs
+ * the whole exchange: ggrid_ingest feeds the batch to every shard; ggrid_knn splits the batch
+ * into R contiguous origin shares and answers them with one request/reply round (route to
+ * the owner of each query's cell, owner's k nearest own objects + the shards its search
+ * entered, bounded requests to those shards, replies, first-k merge, answers back), every step
+ * in kernels on the shards' devices, transfers over NCCL (ncclSend/ncclRecv groups over
+ * NVLink/NVSwitch), peer copies (loopback) or a caller all-to-all (opts.exchange).
+ *   - one process, several GPUs:  opts.n_gpus = R (opts.devices);
+ *   - one process per GPU:        opts.n_ranks = R, opts.rank, and opts.nccl_id (or
+ *                                 opts.exchange); ggrid_knn is then collective: every rank
+ *                                 calls it with its own query batch (sizes may differ) and
+ *                                 receives the answers to its own rows.
+ * On a multi-GPU handle the staged calls (ggrid_*_stage / _commit), ggrid_knn_ex,
+ * ggrid_shard, ggrid_query_owner, ggrid_merge_topk and ggrid_prior_art_clean return EINVAL.
+ * Errors: ENCCL (libnccl missing, communicator set-up or a transfer failed). */
+
+/* A fresh ncclUniqueId (128 bytes into out) for opts.nccl_id: made on one rank, shared with
+ * the others by the caller.  Errors: EINVAL (null), ENCCL (libnccl.so.2 not loadable). */
+int ggrid_nccl_unique_id(void* out);
+
+/* ---- cell-ownership sharding primitives (one shard per handle; the protocol's steps) ------
  *
  * ggrid_shard makes this handle rank `rank` of `n_ranks` (<= 64): it owns the contiguous
  * Z-order range of cells c with floor(c * n_ranks / n_cells) == rank.  Every rank ingests the

@@ -26,7 +26,8 @@ KERNEL_KINDS = ["ingest_classify", "ingest_alloc", "ingest_scatter", "seed", "fl
 EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_commit", "ggrid_query_stage", "ggrid_knn_commit", "ggrid_knn", "ggrid_free", "ggrid_strerror", "ggrid_sync", "ggrid_set_profile", "ggrid_flush_all",
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
            "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk",
-           "ggrid_prior_art_clean", "ggrid_prior_art_bundle", "ggrid_wait_stream", "ggrid_signal_stream"]
+           "ggrid_prior_art_clean", "ggrid_prior_art_bundle", "ggrid_wait_stream", "ggrid_signal_stream",
+           "ggrid_nccl_unique_id"]
 
 
 class GGridError(RuntimeError):
@@ -41,12 +42,21 @@ class ggrid_graph(ctypes.Structure):
                 ("x", ctypes.c_void_p), ("y", ctypes.c_void_p)]
 
 
+ALLTOALL_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(ctypes.c_void_p),
+                               ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_void_p),
+                               ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32, ctypes.c_void_p)
+GGRID_EXCHANGE_AUTO, GGRID_EXCHANGE_LOOPBACK, GGRID_EXCHANGE_NCCL = 0, 1, 2
+
+
 class ggrid_opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("max_k", ctypes.c_uint32), ("max_objects", ctypes.c_uint32),
                 ("log_capacity", ctypes.c_uint64), ("delta", ctypes.c_uint32),
                 ("seed_neighbors", ctypes.c_uint32), ("profile", ctypes.c_uint32),
                 ("t_delta", ctypes.c_uint32), ("stream", ctypes.c_void_p), ("async_ingest", ctypes.c_uint32),
-                ("ingest_kernels", ctypes.c_uint32)]
+                ("ingest_kernels", ctypes.c_uint32), ("n_gpus", ctypes.c_uint32),
+                ("devices", ctypes.POINTER(ctypes.c_int)), ("exchange_kind", ctypes.c_uint32),
+                ("n_ranks", ctypes.c_uint32), ("rank", ctypes.c_uint32), ("nccl_id", ctypes.c_void_p),
+                ("exchange", ALLTOALL_FN), ("exchange_ctx", ctypes.c_void_p)]
 
 
 NK = 8
@@ -61,7 +71,8 @@ class ggrid_stats_t(ctypes.Structure):
         (n, ctypes.c_uint32) for n in ["n_cells", "cell_size", "delta", "n_vertices", "n_arcs", "max_objects",
                                        "t_delta", "t_now"]] + [("records_expired", ctypes.c_uint64),
                                        ("expand_promotions", ctypes.c_uint64), ("expand_retries", ctypes.c_uint64),
-                                       ("seq_rebases", ctypes.c_uint64)]
+                                       ("seq_rebases", ctypes.c_uint64), ("n_shards", ctypes.c_uint32),
+                                       ("exchange_kind", ctypes.c_uint32)]
 
 
 class ggrid_prior_art_result(ctypes.Structure):
@@ -107,6 +118,7 @@ def lib():
             "ggrid_prior_art_bundle": ([P, P, u32, P, P], i32),
             "ggrid_wait_stream": ([P, P], i32),
             "ggrid_signal_stream": ([P, P], i32),
+            "ggrid_nccl_unique_id": ([P], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -165,11 +177,20 @@ def _order_inputs(h, *arrays):
 
 
 # ------------------------------------------------------------------------ the C ABI names
+_KEEP = {}  # ctypes objects (callbacks, device lists, ids) that must outlive their handle
+
+
 def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 256,
                 max_objects: int = 1 << 24, log_capacity: int = 0, delta: int = 0,
                 seed_neighbors: bool = True, profile: bool = False, t_delta: int = 0, stream=None,
-                async_ingest: bool = False, ingest_kernels: int = 0):
-    """ggrid_build(graph, cell_size) -> handle (c_void_p).  graph: dict(n_vertices, src, dst, w[, x, y])."""
+                async_ingest: bool = False, ingest_kernels: int = 0, n_gpus: int = 0, devices=None,
+                exchange_kind: int = 0, n_ranks: int = 0, rank: int = 0, nccl_id: bytes | None = None,
+                exchange=None):
+    """ggrid_build(graph, cell_size) -> handle (c_void_p).  graph: dict(n_vertices, src, dst, w[, x, y]).
+
+    Multi-GPU (ggrid.h "multi-GPU"): n_gpus/devices (one process, several shards; a repeated
+    device = loopback test mode), or n_ranks/rank with nccl_id (128 bytes,
+    ggrid_nccl_unique_id) or exchange (a Python all-to-all, see alltoall_callback)."""
     src, dst, w = (np.ascontiguousarray(graph[k], np.uint32) for k in ("src", "dst", "w"))
     x = graph.get("x")
     y = graph.get("y")
@@ -177,12 +198,84 @@ def ggrid_build(graph: dict, cell_size: int, *, device: int = 0, max_k: int = 25
     y = None if y is None else np.ascontiguousarray(y, np.int32)
     g = ggrid_graph(int(graph["n_vertices"]), len(src), src.ctypes.data, dst.ctypes.data, w.ctypes.data,
                     None if x is None else x.ctypes.data, None if y is None else y.ctypes.data)
+    keep = []
+    dev_arr = None
+    if devices is not None:
+        dev_arr = (ctypes.c_int * len(devices))(*[int(d) for d in devices])
+        keep.append(dev_arr)
+        n_gpus = n_gpus or len(devices)
+    idbuf = None
+    if nccl_id is not None:
+        idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128)
+        keep.append(idbuf)
+    cb = ALLTOALL_FN(0)
+    if exchange is not None:
+        cb = exchange if isinstance(exchange, ALLTOALL_FN) else ALLTOALL_FN(exchange)
+        keep.append(cb)
     o = ggrid_opts(int(device), int(max_k), int(max_objects), int(log_capacity), int(delta),
                    0 if seed_neighbors else 2, int(profile), int(t_delta), stream,
-                   1 if async_ingest else 0, int(ingest_kernels))
+                   1 if async_ingest else 0, int(ingest_kernels), int(n_gpus),
+                   ctypes.cast(dev_arr, ctypes.POINTER(ctypes.c_int)) if dev_arr is not None else None,
+                   int(exchange_kind), int(n_ranks), int(rank),
+                   ctypes.cast(idbuf, ctypes.c_void_p) if idbuf is not None else None, cb, None)
     h = ctypes.c_void_p()
     _check(lib().ggrid_build(ctypes.byref(g), int(cell_size), ctypes.byref(o), ctypes.byref(h)), "ggrid_build")
+    if keep:
+        _KEEP[h.value] = keep
     return h
+
+
+def ggrid_nccl_unique_id() -> bytes:
+    """A fresh 128-byte ncclUniqueId for ggrid_build(n_ranks=..., nccl_id=...)."""
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().ggrid_nccl_unique_id(buf), "ggrid_nccl_unique_id")
+    return buf.raw
+
+
+def alltoall_callback(torch_group=None):
+    """An opts.exchange all-to-all over torch.distributed (any backend; gloo exchanges through
+    host memory).  Device segments are viewed as uint8 CUDA tensors of this rank's device."""
+    import torch
+    import torch.distributed as dist
+
+    def fn(ctx, send, sbytes, recv, rbytes, n_ranks, stream):
+        try:
+            dev = torch.cuda.current_device()
+            ins, outs = [], []
+            for p in range(n_ranks):
+                ins.append(_u8_view(send[p], sbytes[p], dev))
+                outs.append(_u8_view(recv[p], rbytes[p], dev))
+            if dist.get_backend(torch_group) == "gloo":
+                hi = [t.cpu() for t in ins]
+                ho = [torch.empty(int(rbytes[p]), dtype=torch.uint8) for p in range(n_ranks)]
+                dist.all_to_all(ho, hi, group=torch_group)
+                for p in range(n_ranks):
+                    if rbytes[p]:
+                        outs[p].copy_(ho[p])
+            else:
+                dist.all_to_all(outs, ins, group=torch_group)
+            torch.cuda.synchronize(dev)
+            return 0
+        except Exception as e:  # (reported to the library as a failed exchange: ENCCL)
+            import sys
+            print("ggrid exchange callback failed:", repr(e), file=sys.stderr)
+            return 1
+
+    return ALLTOALL_FN(fn)
+
+
+def _u8_view(ptr, nbytes, dev):
+    """A uint8 CUDA tensor over nbytes of device memory at ptr (no copy)."""
+    import torch
+
+    n = int(nbytes)
+    if n == 0 or not ptr:
+        return torch.empty(0, dtype=torch.uint8, device=f"cuda:{dev}")
+
+    class _Arr:
+        __cuda_array_interface__ = {"shape": (n,), "typestr": "|u1", "data": (int(ptr), False), "version": 3}
+
+    return torch.as_tensor(_Arr(), device=f"cuda:{dev}")
 
 
 def ggrid_ingest(h, updates, n: int | None = None):
@@ -342,6 +435,7 @@ def _stream_handle(stream):
 def ggrid_free(h):
     if h:
         lib().ggrid_free(h)
+        _KEEP.pop(h.value if hasattr(h, "value") else h, None)
 
 
 def ggrid_flush_all(h):

@@ -106,6 +106,19 @@ int ggrid_s::ensure_arena(uint64_t need_records, uint32_t need_ext) {
 }
 
 // ------------------------------------------------------------------------------------------
+static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts& opts_in, ggrid_t* out);
+
+// a call on the front handle of an in-process multi-GPU index, applied to every shard in turn
+template <class F>
+static int each_shard(ggrid_t h, F&& f) {
+  for (uint32_t r = 0; r < multi_n(h->multi); ++r) RC(f(multi_shard(h->multi, (int)r)));
+  return GGRID_OK;
+}
+#define SINGLE_ONLY(h) \
+  do {                 \
+    if ((h) && (h)->multi) return GGRID_EINVAL; \
+  } while (0)
+
 extern "C" {
 
 const char* ggrid_version(void) { return "ggrid-b200 0.1 (sm_100a)"; }
@@ -133,6 +146,31 @@ uint64_t ggrid_zvalue(uint32_t x, uint32_t y) {
 
 int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opts, ggrid_t* out) {
   if (!gr || !out) return GGRID_EINVAL;
+  *out = nullptr;
+  ggrid_opts o{};
+  if (opts) o = *opts;
+  if (o.exchange_kind > GGRID_EXCHANGE_NCCL) return GGRID_EINVAL;
+  if (o.n_gpus > 1) {
+    if (o.n_ranks > 1) return GGRID_EINVAL;  // (one process drives all shards, or one each)
+    return multi_build(gr, cell_size, o, out, build_one);
+  }
+  ggrid_t h = nullptr;
+  RC(build_one(gr, cell_size, o, &h));
+  if (o.n_ranks > 1) {
+    const int rc = rank_attach(h, o);
+    if (rc != GGRID_OK) {
+      ggrid_free(h);
+      return rc;
+    }
+  }
+  *out = h;
+  return GGRID_OK;
+}
+
+}  // extern "C"
+
+static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts& opts_in, ggrid_t* out) {
+  const ggrid_opts* opts = &opts_in;
   *out = nullptr;
   const uint32_t V = gr->n_vertices, A = gr->n_arcs;
   if (V == 0 || V >= 0xFFFFFFFEu || A >= 0xFFFFFFFEu || cell_size == 0) return GGRID_EINVAL;
@@ -329,8 +367,17 @@ int ggrid_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts* opt
   return GGRID_OK;
 }
 
+extern "C" {
+
 int ggrid_free(ggrid_t h) {
   if (!h) return GGRID_OK;
+  if (h->multi) {
+    multi_free(h->multi);
+    delete h;
+    return GGRID_OK;
+  }
+  if (h->xchg) exchange_free(h->xchg);
+  for (DBuf& b : h->mx) b.release();
   if (h->stream) cudaStreamSynchronize(h->stream);
   if (h->copy_stream) cudaStreamSynchronize(h->copy_stream);
   for (void* p : h->allocs) cudaFree(p);
@@ -435,6 +482,7 @@ int ggrid_ingest(ggrid_t h, const ggrid_update* u, uint64_t n) {
   if (n == 0) return GGRID_OK;
   if (!u) return GGRID_EINVAL;
   if (n > kMaxBatch) return GGRID_EOVERFLOW;
+  if (h->multi) return multi_ingest(h->multi, u, n);
   CK(cudaSetDevice(h->device));
   const uint4* d_u = reinterpret_cast<const uint4*>(u);
   RC(h->order_inputs(h->stream));  // u may be the output of a caller kernel still running
@@ -471,6 +519,7 @@ static int stage_into(ggrid_t h, ggrid_s::Staged* ring, int head, int count, con
 }
 
 int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n) {
+  SINGLE_ONLY(h);
   if (!h || (n && !u) || h->n_staged == 2) return GGRID_EINVAL;
   CK(cudaSetDevice(h->device));
   RC(stage_into(h, h->staged, h->stage_head, h->n_staged, u, n, sizeof(uint4)));
@@ -479,6 +528,7 @@ int ggrid_ingest_stage(ggrid_t h, const ggrid_update* u, uint64_t n) {
 }
 
 int ggrid_query_stage(ggrid_t h, const ggrid_query* q, uint32_t n_q) {
+  SINGLE_ONLY(h);
   if (!h || (n_q && !q) || h->n_qstaged == 2) return GGRID_EINVAL;
   CK(cudaSetDevice(h->device));
   RC(stage_into(h, h->qstaged, h->qstage_head, h->n_qstaged, q, n_q, sizeof(uint2)));
@@ -487,6 +537,7 @@ int ggrid_query_stage(ggrid_t h, const ggrid_query* q, uint32_t n_q) {
 }
 
 int ggrid_ingest_commit(ggrid_t h) {
+  SINGLE_ONLY(h);
   if (!h || h->n_staged == 0) return GGRID_EINVAL;
   CK(cudaSetDevice(h->device));
   ggrid_s::Staged& sb = h->staged[h->stage_head];
@@ -710,6 +761,7 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
 }
 
 int ggrid_knn_commit(ggrid_t h, uint32_t k, uint32_t* out_obj, uint32_t* out_dist, uint32_t* n_q) {
+  SINGLE_ONLY(h);
   if (!h || h->n_qstaged == 0 || k == 0 || k > h->max_k) return GGRID_EINVAL;
   ggrid_s::Staged& sb = h->qstaged[h->qstage_head];
   if (n_q) *n_q = (uint32_t)sb.n;
@@ -727,13 +779,27 @@ int ggrid_knn_commit(ggrid_t h, uint32_t k, uint32_t* out_obj, uint32_t* out_dis
 int ggrid_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj,
               uint32_t* out_dist) {
   if (!h || k == 0 || k > h->max_k) return GGRID_EINVAL;
+  if (h->xchg) {  // one rank of a multi-process index: collective, even with no queries of its own
+    if (n_q && (!q || !out_obj || !out_dist)) return GGRID_EINVAL;
+    CK(cudaSetDevice(h->device));
+    RC(rank_knn(h, q, n_q, k, out_obj, out_dist));
+    h->stats.knn_calls++;
+    return GGRID_OK;
+  }
   if (n_q == 0) return GGRID_OK;
   if (!q || !out_obj || !out_dist) return GGRID_EINVAL;
+  if (h->multi) {
+    RC(multi_knn(h->multi, q, n_q, k, out_obj, out_dist));
+    h->stats.n_queries += n_q;
+    h->stats.knn_calls++;
+    return GGRID_OK;
+  }
   return knn_impl(h, q, n_q, k, out_obj, out_dist);
 }
 
 int ggrid_knn_ex(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, const uint32_t* bound,
                  uint32_t* out_obj, uint32_t* out_dist, uint64_t* out_remote) {
+  SINGLE_ONLY(h);
   if (!h || k == 0 || k > h->max_k) return GGRID_EINVAL;
   if (n_q == 0) return GGRID_OK;
   if (!q || !out_obj || !out_dist) return GGRID_EINVAL;
@@ -741,6 +807,7 @@ int ggrid_knn_ex(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, cons
 }
 
 int ggrid_shard(ggrid_t h, uint32_t n_ranks, uint32_t rank) {
+  SINGLE_ONLY(h);
   if (!h || n_ranks == 0 || n_ranks > 64 || rank >= n_ranks || n_ranks > h->n_cells) return GGRID_EINVAL;
   if (h->n_ingested != 0) return GGRID_EINVAL;  // ownership is fixed before the first update
   h->s.n_ranks = n_ranks;
@@ -749,6 +816,7 @@ int ggrid_shard(ggrid_t h, uint32_t n_ranks, uint32_t rank) {
 }
 
 int ggrid_query_owner(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t* out_rank) {
+  SINGLE_ONLY(h);
   if (!h || (n_q && (!q || !out_rank))) return GGRID_EINVAL;
   if (n_q == 0) return GGRID_OK;
   CK(cudaSetDevice(h->device));
@@ -772,6 +840,7 @@ int ggrid_query_owner(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t* o
 
 int ggrid_merge_topk(ggrid_t h, uint32_t n_lists, uint32_t n_q, uint32_t k, const uint32_t* lists_obj,
                      const uint32_t* lists_dist, uint32_t* out_obj, uint32_t* out_dist) {
+  SINGLE_ONLY(h);
   if (!h || n_lists == 0 || n_lists > 32 || k == 0) return GGRID_EINVAL;
   if (n_q == 0) return GGRID_OK;
   if (!lists_obj || !lists_dist || !out_obj || !out_dist) return GGRID_EINVAL;
@@ -805,6 +874,7 @@ int ggrid_merge_topk(ggrid_t h, uint32_t n_lists, uint32_t n_q, uint32_t k, cons
 
 int ggrid_prior_art_clean(ggrid_t h, uint32_t eta, uint32_t bucket_size, uint32_t write_mode,
                           uint32_t* out_edge, uint32_t* out_off, ggrid_prior_art_result* res) {
+  SINGLE_ONLY(h);
   if (!h || (eta != 4 && eta != 5) || bucket_size == 0 || bucket_size > 4096 || write_mode > 1)
     return GGRID_EINVAL;
   CK(cudaSetDevice(h->device));
@@ -901,6 +971,7 @@ int ggrid_prior_art_bundle(const uint32_t* obj, const uint64_t* key, uint32_t et
 
 int ggrid_set_profile(ggrid_t h, uint32_t mask) {
   if (!h) return GGRID_EINVAL;
+  if (h->multi) return each_shard(h, [&](ggrid_t x) { return ggrid_set_profile(x, mask); });
   RC(h->sync());  // (collects the events of the previous mode)
   h->profile = mask;
   return GGRID_OK;
@@ -908,6 +979,7 @@ int ggrid_set_profile(ggrid_t h, uint32_t mask) {
 
 int ggrid_wait_stream(ggrid_t h, void* stream) {
   if (!h) return GGRID_EINVAL;
+  if (h->multi) return each_shard(h, [&](ggrid_t x) { return ggrid_wait_stream(x, stream); });
   CK(cudaSetDevice(h->device));
   cudaStream_t p = static_cast<cudaStream_t>(stream);
   RC(h->order_after(p, h->stream));
@@ -917,6 +989,7 @@ int ggrid_wait_stream(ggrid_t h, void* stream) {
 
 int ggrid_signal_stream(ggrid_t h, void* stream) {
   if (!h) return GGRID_EINVAL;
+  if (h->multi) return each_shard(h, [&](ggrid_t x) { return ggrid_signal_stream(x, stream); });
   CK(cudaSetDevice(h->device));
   cudaStream_t c = static_cast<cudaStream_t>(stream);
   if (c == h->stream) return GGRID_OK;
@@ -927,6 +1000,7 @@ int ggrid_signal_stream(ggrid_t h, void* stream) {
 
 int ggrid_sync(ggrid_t h) {
   if (!h) return GGRID_EINVAL;
+  if (h->multi) return each_shard(h, [&](ggrid_t x) { return ggrid_sync(x); });
   CK(cudaSetDevice(h->device));
   RC(h->sync());
   return h->take_deferred();
@@ -934,6 +1008,7 @@ int ggrid_sync(ggrid_t h) {
 
 int ggrid_flush_all(ggrid_t h) {
   if (!h) return GGRID_EINVAL;
+  if (h->multi) return each_shard(h, [&](ggrid_t x) { return ggrid_flush_all(x); });
   CK(cudaSetDevice(h->device));
   RC(h->ensure_arena(h->flush_need(), 0));
   h->epoch++;
@@ -948,6 +1023,9 @@ int ggrid_flush_all(ggrid_t h) {
 int ggrid_cell_objects(ggrid_t h, uint32_t cell, uint32_t* obj, uint32_t* edge, uint32_t* off,
                        uint32_t cap, uint32_t* n) {
   if (!h || !n || cell >= h->n_cells) return GGRID_EINVAL;
+  if (h->multi)  // the shard owning the cell
+    return ggrid_cell_objects(multi_shard(h->multi, (int)owner_of(cell, h->n_cells, multi_n(h->multi))), cell, obj,
+                              edge, off, cap, n);
   if (cap && (!obj || !edge || !off)) return GGRID_EINVAL;
   CK(cudaSetDevice(h->device));
   RC(h->ensure_arena(h->flush_need(), 0));
@@ -977,6 +1055,40 @@ int ggrid_cell_objects(ggrid_t h, uint32_t cell, uint32_t* obj, uint32_t* edge, 
 
 int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
   if (!h || !out) return GGRID_EINVAL;
+  if (h->multi) {  // shard 0's header; work counters and timings summed over the shards
+    ggrid_stats_t t{};
+    RC(ggrid_stats(multi_shard(h->multi, 0), &t));
+    for (uint32_t r = 1; r < multi_n(h->multi); ++r) {
+      ggrid_stats_t x{};
+      RC(ggrid_stats(multi_shard(h->multi, (int)r), &x));
+      t.knn_rounds += x.knn_rounds;
+      t.cells_flushed += x.cells_flushed;
+      t.records_flushed += x.records_flushed;
+      t.objects_written += x.objects_written;
+      t.arena_used += x.arena_used;
+      t.arena_capacity += x.arena_capacity;
+      t.gc_runs += x.gc_runs;
+      t.launches += x.launches;
+      t.expand_iterations += x.expand_iterations;
+      t.expand_vertices += x.expand_vertices;
+      t.expand_arcs += x.expand_arcs;
+      t.expand_harvested += x.expand_harvested;
+      t.expand_objects += x.expand_objects;
+      for (int i = 0; i < GGRID_NK; ++i) {
+        t.kernel_launches[i] += x.kernel_launches[i];
+        t.kernel_ms[i] += x.kernel_ms[i];
+      }
+      t.records_expired += x.records_expired;
+      t.expand_promotions += x.expand_promotions;
+      t.expand_retries += x.expand_retries;
+    }
+    t.n_queries = h->stats.n_queries;
+    t.knn_calls = h->stats.knn_calls;
+    t.n_shards = multi_n(h->multi);
+    t.exchange_kind = strcmp(multi_exchange_name(h->multi), "nccl") == 0 ? GGRID_EXCHANGE_NCCL : GGRID_EXCHANGE_LOOPBACK;
+    *out = t;
+    return GGRID_OK;
+  }
   RC(h->sync());
   ggrid_stats_t s = h->stats;
   s.cells_flushed = h->h_status->cells_flushed;
@@ -999,6 +1111,8 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
   s.t_now = h->h_status->t_max;
   s.records_expired = h->h_status->records_expired;
   s.seq_rebases = h->rebases;
+  s.n_shards = h->s.n_ranks;
+  s.exchange_kind = h->xchg ? (strcmp(exchange_name(h->xchg), "nccl") == 0 ? GGRID_EXCHANGE_NCCL : 3u) : 0u;
   s.expand_promotions = h->h_status->ex_promoted;
   s.expand_retries = h->h_status->ex_retried;
   *out = s;
@@ -1007,6 +1121,7 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
 
 int ggrid_stats_reset(ggrid_t h) {
   if (!h) return GGRID_EINVAL;
+  if (h->multi) return each_shard(h, [&](ggrid_t x) { return ggrid_stats_reset(x); });
   RC(h->sync());
   h->stats.launches = 0;
   for (int i = 0; i < GGRID_NK; ++i) {
@@ -1018,6 +1133,7 @@ int ggrid_stats_reset(ggrid_t h) {
 
 int ggrid_vertex_cell(ggrid_t h, uint32_t* cell_of_vertex) {
   if (!h || !cell_of_vertex) return GGRID_EINVAL;
+  if (h->multi) return ggrid_vertex_cell(multi_shard(h->multi, 0), cell_of_vertex);
   memcpy(cell_of_vertex, h->user_cell.data(), (size_t)h->V * 4);
   return GGRID_OK;
 }

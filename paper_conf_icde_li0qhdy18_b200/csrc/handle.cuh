@@ -142,6 +142,11 @@ struct ggrid_s {
   int stage_head = 0, n_staged = 0;
   Staged qstaged[2];  // staged query batches (ggrid_query_stage / ggrid_knn_commit)
   int qstage_head = 0, n_qstaged = 0;
+  // multi-GPU (multi.cu): the front handle of an in-process index over several shards, or this
+  // shard's transport when it is one rank of a multi-process index
+  MultiIndex* multi = nullptr;
+  Exchange* xchg = nullptr;
+  DBuf mx[16];  // the exchange protocol's device buffers
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_in = nullptr;   // caller's producer stream -> library streams (order_inputs)
   cudaEvent_t ev_out = nullptr;  // library stream -> a caller's stream (ggrid_signal_stream)
@@ -293,3 +298,16 @@ __attribute__((visibility("hidden"))) int ingest_device(ggrid_t h, const uint4* 
 __attribute__((visibility("hidden"))) int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj, uint32_t* out_dist,
              const uint32_t* bound = nullptr, uint64_t* out_remote = nullptr);
 }
+// multi.cu
+int multi_build(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts& o, ggrid_t* out,
+                int (*build_one)(const ggrid_graph*, uint32_t, const ggrid_opts&, ggrid_t*));
+void multi_free(MultiIndex* mi);
+const char* multi_exchange_name(const MultiIndex* mi);
+uint32_t multi_n(const MultiIndex* mi);
+ggrid_t multi_shard(const MultiIndex* mi, int r);
+int multi_ingest(MultiIndex* mi, const ggrid_update* u, uint64_t n);
+int multi_knn(MultiIndex* mi, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj, uint32_t* out_dist);
+int rank_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t* out_obj, uint32_t* out_dist);
+int rank_attach(ggrid_t h, const ggrid_opts& o);
+void exchange_free(Exchange* e);
+const char* exchange_name(const Exchange* e);

@@ -85,6 +85,19 @@ __device__ __forceinline__ uint32_t vhash(uint32_t v, uint32_t H) { return __umu
 
 constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^32-1)
 
+// A vertex entering the frontier will be expanded in a later round: its inline adjacency record
+// and object index are fetched into L2 now, so the expansion's dependent load hits L2 instead of
+// DRAM (the USA-shaped graph's 0.9 GB of per-vertex records is far beyond L2).
+#ifndef GG_PREFETCH
+#define GG_PREFETCH 0
+#endif
+__device__ __forceinline__ void prefetch_vertex(const DevGraph& g, const DevState& s, uint32_t v) {
+  if (GG_PREFETCH) {
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(g.vadj + (size_t)v * 4));
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(s.v_obj + v));
+  }
+}
+
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
 __device__ __forceinline__ int tab_relax(const WarpMem& m, uint32_t H, uint32_t v, uint32_t d,
                                          bool& improved) {
@@ -402,6 +415,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
           if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
             has = true;
             nslot = (uint32_t)rr;
+            prefetch_vertex(g, s, dst);
           }
         }
       };
@@ -747,6 +761,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
             mn = min(mn, (uint32_t)nd);
             const uint32_t bit = 1u << (rr & 31);
             if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+              prefetch_vertex(g, s, dst);
               const uint32_t p = atomicAdd(&sh.nn[par], 1u);
               if (p < cp.F) nfront[p] = (uint32_t)rr;
               else atomicOr(&sh.flags, FL_OVF);

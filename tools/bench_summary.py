@@ -16,4 +16,5 @@ for path in sys.argv[1:]:
           f"roof={b.get('roofline', {}).get('kernel')}:{b.get('roofline', {}).get('frac', 0):.3f} "
           f"launch_ms={b.get('roofline', {}).get('launch_ms', 0):.4f} "
           f"L0={b['per_kernel']['expand'].get('level0_ms_per_step', 0):.4f} Lhi={b['per_kernel']['expand'].get('higher_levels_ms_per_step', 0):.4f} "
+          f"parity={(b.get('parity') or {}).get('rows_exact')}/{(b.get('parity') or {}).get('rows')} "
           f"rounds={b.get('knn_rounds_per_step')} promo={b.get('expand_promotions_per_step')} retry={b.get('expand_retries_per_step')} clocks={b.get('clocks', {}).get('sm_mhz')}")
