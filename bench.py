@@ -23,7 +23,8 @@ max over ranks).  The line also carries:
 Multi-GPU: --gpus N without a torchrun environment re-launches itself under torchrun with N
 ranks.  Ranks own contiguous Z-order ranges of cells (cell-ownership sharding, SURVEY §8(e));
 the global batch of Q queries is fixed and split across ranks (strong scaling); queries are
-answered with one request/reply exchange (dist.sharded_knn).
+answered with one request/reply exchange that the library runs itself (ggrid.h "multi-GPU":
+route, owner search, bounded requests, replies, merge, return -- kernels + NCCL send/recv).
 """
 from __future__ import annotations
 
@@ -251,12 +252,12 @@ def run_ours(args, cfg_name):
     from paper_conf_icde_li0qhdy18_b200 import dist as gdist
 
     world, rank, local = dist_setup()
+    backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")
     if world > 1:
         import torch.distributed as dist
 
         # one process per GPU over NCCL; BENCH_DIST_BACKEND=gloo lets the harness be exercised
         # with several ranks sharing one GPU (a test mode, not a measurement)
-        backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")
         dev_i = local % max(1, torch.cuda.device_count())
         torch.cuda.set_device(dev_i)
         if backend == "nccl":
@@ -291,13 +292,22 @@ def run_ours(args, cfg_name):
         step_q.append(synth.queries(g, Q, seed=synth.SEED_QUERIES + s)[lo:hi])
     t_gen = time.perf_counter() - t_setup
 
+    # cell-ownership sharding: this rank's handle is shard `rank` of `world` and
+    # the library runs the query exchange itself (ggrid.h "multi-GPU"): over NCCL between GPUs,
+    # over a gloo all-to-all callback in the one-GPU harness mode (BENCH_DIST_BACKEND=gloo)
+    shard_opts = {}
+    if shard:
+        if backend == "nccl":
+            uid = [gg.ggrid_nccl_unique_id() if rank == 0 else None]
+            torch.distributed.broadcast_object_list(uid, src=0)
+            shard_opts = dict(n_ranks=world, rank=rank, nccl_id=uid[0])
+        else:
+            shard_opts = dict(n_ranks=world, rank=rank, exchange=gg.alltoall_callback())
     stream = torch.cuda.Stream()
     t0 = time.perf_counter()
     grid = gg.GGrid(g, cell_size, max_objects=n_obj, profile=PROFILE_ALL, log_capacity=log_cap,
-                    delta=args.delta, stream=stream.cuda_stream, async_ingest=True)
+                    delta=args.delta, stream=stream.cuda_stream, async_ingest=True, **shard_opts)
     t_build = time.perf_counter() - t0
-    if shard:  # cell-ownership sharding: logs of own cells only
-        grid.shard(world, rank)
     out_o = torch.empty((Qr, k), dtype=torch.int32, device="cuda")
     out_d = torch.empty((Qr, k), dtype=torch.int32, device="cuda")
     # > 126 MB L2
@@ -353,7 +363,6 @@ def run_ours(args, cfg_name):
     times = []
     st0 = st1 = sb0 = None
     clk = None
-    remote_requests = 0
     last_out = None
     for s in range(n_steps_total):
         u = step_u[s]
@@ -386,13 +395,7 @@ def run_ours(args, cfg_name):
             if world > 1:
                 gdist.broadcast_updates(du, src=0)
             grid.ingest(du)
-            if shard:  # owner search + bounded requests/replies + merge, all ordered on `stream`
-                oo, od, n_req = gdist.sharded_knn(grid, dq, k, world, rank)
-                out_o.copy_(oo)
-                out_d.copy_(od)
-                remote_requests += n_req if args.warmup <= s < args.warmup + args.steps else 0
-            else:
-                grid.knn(dq, k, out_o, out_d)
+            grid.knn(dq, k, out_o, out_d)  # (sharded: collective over the ranks, inside the library)
             e1.record(stream)
         e1.synchronize()
         hist.append(u)
@@ -405,6 +408,11 @@ def run_ours(args, cfg_name):
     grid.sync()
     sb1 = grid.stats()
     total_ms = gdist.max_over_ranks(sum(times), device="cuda")
+    req_all = 0.0
+    if shard:  # bounded requests sent over the timed steps, summed over the ranks
+        t_req = torch.tensor([float(st1["remote_requests"] - st0["remote_requests"])], dtype=torch.float64, device="cuda")
+        torch.distributed.all_reduce(t_req)
+        req_all = float(t_req.item())
     K = args.steps
     value = Q * K / (total_ms / 1e3)  # the global batch Q per step, all ranks (max-over-ranks time)
 
@@ -516,30 +524,30 @@ def run_ours(args, cfg_name):
     # profile-mode events (an event queued behind a staged copy costs ~50 us), preloaded and
     # flushed like the first (untimed).
     grid.close()
-    grid = gg.GGrid(g, cell_size, max_objects=n_obj, log_capacity=log_cap, delta=args.delta, async_ingest=True)
-    if shard:
-        grid.shard(world, rank)
+    if shard and backend == "nccl":  # a fresh communicator for the fresh index
+        uid = [gg.ggrid_nccl_unique_id() if rank == 0 else None]
+        torch.distributed.broadcast_object_list(uid, src=0)
+        shard_opts["nccl_id"] = uid[0]
+    grid = gg.GGrid(g, cell_size, max_objects=n_obj, log_capacity=log_cap, delta=args.delta, async_ingest=True,
+                    **shard_opts)
     if len(preload):
         grid.ingest(torch.from_numpy(preload.view(np.int32)).to("cuda"))
         grid.flush_all()
-    dq_e = torch.empty((Qr, 2), dtype=torch.int32, device="cuda")
     h_o = torch.empty((Qr, k), dtype=torch.int32).pin_memory()
     h_d = torch.empty((Qr, k), dtype=torch.int32).pin_memory()
 
     def e2e_stage(hu, hq):
+        if shard:  # (the staged calls are single-shard; a sharded rank ingests directly)
+            grid.ingest(hu)
+            return
         grid.ingest_stage(hu)
-        if not shard:
-            grid.query_stage(hq)  # copied behind the update batch on the library's copy stream
+        grid.query_stage(hq)  # copied behind the update batch on the library's copy stream
 
     def e2e_knn(hq):
         if not shard:
             grid.knn_commit(k, h_o, h_d)  # the staged queries; answers written to pinned memory in place
             return
-        dq_e.copy_(hq, non_blocking=True)
-        o, d_, _ = gdist.sharded_knn(grid, dq_e, k, world, rank)
-        h_o.copy_(o, non_blocking=True)
-        h_d.copy_(d_, non_blocking=True)
-        torch.cuda.current_stream().synchronize()
+        grid.knn(hq, k, h_o, h_d)  # (collective; the library copies the pinned batch in and out)
 
     n_e2e = max(1, args.e2e_steps)
     w_e2e = 3
@@ -557,16 +565,20 @@ def run_ours(args, cfg_name):
         scratch_q.copy_(hq)
     torch.cuda.synchronize()
     del scratch_u, scratch_q
+    def e2e_commit():
+        if not shard:
+            grid.ingest_commit()
+
     for s in range(w_e2e):  # warm-up steps
         e2e_stage(hus[s], hqs[s])
-        grid.ingest_commit()
+        e2e_commit()
         e2e_knn(hqs[s])
     hus, hqs = [None] + hus[w_e2e:], [None] + hqs[w_e2e:]
     barrier()
     t0 = time.perf_counter()
     e2e_stage(hus[1], hqs[1])
     for s in range(1, n_e2e + 1):
-        grid.ingest_commit()
+        e2e_commit()
         if s + 1 <= n_e2e:
             e2e_stage(hus[s + 1], hqs[s + 1])  # overlaps the queries below
         e2e_knn(hqs[s])
@@ -597,7 +609,8 @@ def run_ours(args, cfg_name):
                 "parity": parity, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(st1["launches"]),
                 "clocks": clk,
                 "knn_rounds_per_step": (st1["knn_rounds"] - st0["knn_rounds"]) / K,
-                "remote_requests_per_step_rank0": remote_requests / K if shard else None,
+                "exchange": ({"kind": "nccl" if backend == "nccl" else "gloo all-to-all callback (harness mode)",
+                              "requests_per_step_all_ranks": req_all / K} if shard else None),
                 "expand_work_per_query": {n: v / (Qr * K) for n, v in dx.items()}, "delta": st1["delta"],
                 "expand_promotions_per_step": (st1["expand_promotions"] - st0["expand_promotions"]) / K,
                 "expand_retries_per_step": (st1["expand_retries"] - st0["expand_retries"]) / K,

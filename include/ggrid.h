@@ -195,6 +195,7 @@ typedef struct ggrid_stats_t {
   uint64_t seq_rebases;      /* re-bases of the arrival index (every ~2^32 updates)  */
   uint32_t n_shards;         /* shards of the index (1: one GPU)                      */
   uint32_t exchange_kind;    /* GGRID_EXCHANGE_* in use (0: none; 3: the caller's all-to-all) */
+  uint64_t remote_requests;  /* bounded requests this shard (all shards: summed) sent to others */
 } ggrid_stats_t;
 
 /* Build the index (graph grid, P@11423-15818; object table P@15869; message lists

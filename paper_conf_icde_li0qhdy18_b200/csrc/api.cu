@@ -1081,6 +1081,7 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
       t.records_expired += x.records_expired;
       t.expand_promotions += x.expand_promotions;
       t.expand_retries += x.expand_retries;
+      t.remote_requests += x.remote_requests;
     }
     t.n_queries = h->stats.n_queries;
     t.knn_calls = h->stats.knn_calls;

@@ -41,6 +41,9 @@ struct Exchange {
   virtual int alltoall(int r, void* const* send, const uint64_t* sbytes, void* const* recv,
                        const uint64_t* rbytes, cudaStream_t st) = 0;
   virtual const char* name() const = 0;
+  // An unexpected failure on one shard mid-protocol: release the peers (their pending and
+  // later transfers fail instead of waiting forever).  Sticky.
+  virtual void abort() {}
 };
 
 namespace {
@@ -50,16 +53,24 @@ struct Barrier {
   std::condition_variable cv;
   int n = 1, count = 0;
   uint64_t gen = 0;
-  void wait() {
+  bool aborted = false;
+  bool wait() {  // false: aborted
     std::unique_lock<std::mutex> lk(m);
+    if (aborted) return false;
     const uint64_t g = gen;
     if (++count == n) {
       count = 0;
       ++gen;
       cv.notify_all();
     } else {
-      cv.wait(lk, [&] { return gen != g; });
+      cv.wait(lk, [&] { return gen != g || aborted; });
     }
+    return !aborted;
+  }
+  void abort() {
+    std::lock_guard<std::mutex> lk(m);
+    aborted = true;
+    cv.notify_all();
   }
 };
 
@@ -76,16 +87,17 @@ struct LoopbackExchange : Exchange {
     int rc = cudaStreamSynchronize(st) == cudaSuccess ? GGRID_OK : GGRID_ECUDA;
     sends[r] = send;
     sb[r] = sbytes;
-    bar.wait();  // every shard's segments are posted
+    if (!bar.wait()) return GGRID_ECUDA;  // every shard's segments are posted (or a peer failed)
     for (int p = 0; p < n && rc == GGRID_OK; ++p) {
       if (sb[p][r] != rbytes[p]) rc = GGRID_ECUDA;  // (a protocol bug: sizes agree by construction)
       else if (rbytes[p] && cudaMemcpyAsync(recv[p], sends[p][r], rbytes[p], cudaMemcpyDefault, st) != cudaSuccess)
         rc = GGRID_ECUDA;
     }
     if (cudaStreamSynchronize(st) != cudaSuccess) rc = GGRID_ECUDA;
-    bar.wait();  // every copy out of the senders' buffers is done
+    if (!bar.wait()) return GGRID_ECUDA;  // every copy out of the senders' buffers is done
     return rc;
   }
+  void abort() override { bar.abort(); }
 };
 
 struct NcclApi {
@@ -97,6 +109,7 @@ struct NcclApi {
   ncclResult_t (*groupEnd)() = nullptr;
   ncclResult_t (*send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
   ncclResult_t (*recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*commAbort)(ncclComm_t) = nullptr;
   bool ok = false;
 };
 
@@ -116,6 +129,7 @@ const NcclApi& nccl() {
     api.groupEnd = reinterpret_cast<decltype(api.groupEnd)>(sym("ncclGroupEnd"));
     api.send = reinterpret_cast<decltype(api.send)>(sym("ncclSend"));
     api.recv = reinterpret_cast<decltype(api.recv)>(sym("ncclRecv"));
+    api.commAbort = reinterpret_cast<decltype(api.commAbort)>(sym("ncclCommAbort"));
     api.ok = api.getUniqueId && api.commInitAll && api.commInitRank && api.commDestroy && api.groupStart &&
              api.groupEnd && api.send && api.recv;
   });
@@ -143,6 +157,14 @@ struct NcclExchange : Exchange {
     if (a.groupEnd() != ncclSuccess) rc = GGRID_ENCCL;
     return rc;
   }
+  void abort() override {
+    if (!nccl().commAbort) return;
+    for (ncclComm_t& c : comms)
+      if (c) {
+        nccl().commAbort(c);
+        c = nullptr;
+      }
+  }
   int n_ranks = 1;
 };
 
@@ -164,14 +186,33 @@ struct CallbackExchange : Exchange {
 //   reply / answer   k obj, k dist, row               (2k + 1 words)
 
 // per-destination counts of the route phase (dest = owner of the query's cell)
+// (an invalid query -- edge >= n_arcs or offset >= w -- sets *err: every shard learns it from the
+// count exchange and the whole batch is rejected, EINVAL, on every shard alike)
 __global__ void k_route_count(const uint2* __restrict__ q, uint32_t n, DevGraph g, DevState s,
-                              uint32_t* __restrict__ dest, uint32_t* __restrict__ counts) {
+                              uint32_t* __restrict__ dest, uint32_t* __restrict__ counts, uint32_t* __restrict__ err) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
-  const uint32_t e = q[i].x;
-  const uint32_t o = e < g.A ? owner_of(cellof(g, g.einfo[e].x), g.n_cells, s.n_ranks) : s.rank;
+  const uint2 qq = q[i];
+  uint32_t o = s.rank;
+  if (qq.x < g.A) {
+    const uint2 ei = g.einfo[qq.x];
+    if (qq.y < ei.y) o = owner_of(cellof(g, ei.x), g.n_cells, s.n_ranks);
+    else *err = 1u;
+  } else {
+    *err = 1u;
+  }
   dest[i] = o;
   atomicAdd(&counts[o], 1u);
+}
+
+// count-exchange records: (count for peer p, this shard's error word)
+__global__ void k_count_pairs(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ err, uint32_t R,
+                              uint32_t* __restrict__ pairs) {
+  const uint32_t p = threadIdx.x;
+  if (p < R) {
+    pairs[2 * p] = counts[p];
+    pairs[2 * p + 1] = *err;
+  }
 }
 
 // scatter into destination segments (offsets = exclusive scan of counts, computed per CTA from
@@ -259,29 +300,64 @@ inline uint32_t blocks(uint64_t n, uint32_t per) { return (uint32_t)std::max<uin
 // (device, n*k each).  Every shard of the index calls this at the same time (collective).
 static int shard_knn(ggrid_t h, Exchange* ex, int r, int R, const uint2* d_q, uint32_t n, uint32_t k,
                      uint32_t* d_oo, uint32_t* d_od) {
+  // Any failure from here on leaves the peers inside the protocol: abort the exchange so they
+  // fail too instead of waiting (a rejected batch is decided collectively, see k_route_count).
+#undef RC
+#undef CK
+#define RC(x)                  \
+  do {                         \
+    const int r_ = (x);        \
+    if (r_ != GGRID_OK) {      \
+      ex->abort();             \
+      return r_;               \
+    }                          \
+  } while (0)
+#define CK(x)                                                                  \
+  do {                                                                         \
+    const cudaError_t e_ = (x);                                                \
+    if (e_ != cudaSuccess) {                                                   \
+      ex->abort();                                                             \
+      return e_ == cudaErrorMemoryAllocation ? GGRID_ENOMEM : GGRID_ECUDA;     \
+    }                                                                          \
+  } while (0)
   cudaStream_t st = h->stream;
   RC(h->order_inputs(st));
   DBuf* B = h->mx;
-  // counts + cursors: [0,R) counts, [R,2R) cursors, host copies below
+  // [0,64) counts, [64,128) cursors, [128,192) count pairs sent, [192,256) pairs received,
+  // [256] the error word
   RC(B[0].ensure(4096));
   uint32_t* counts = B[0].as<uint32_t>();
   uint32_t* cursors = counts + 64;
-  uint32_t* rcounts = counts + 128;  // counts received from each peer
+  uint32_t* spairs = counts + 128;
+  uint32_t* rpairs = counts + 192;
+  uint32_t* err = counts + 256;
   std::vector<uint32_t> sc(R), rcv(R), rq_s(R), rq_r(R);
-  auto zero_counts = [&] { CK(cudaMemsetAsync(counts, 0, 4 * 192, st)); return GGRID_OK; };
+  auto zero_counts = [&] {
+    CK(cudaMemsetAsync(counts, 0, 4 * 128, st));
+    return GGRID_OK;
+  };
+  CK(cudaMemsetAsync(err, 0, 4, st));
   std::vector<void*> sp(R), rp(R);
   std::vector<uint64_t> sbytes(R), rbytes(R);
-  // exchange R u32 counts (device) -> host copies of sent and received counts
+  std::vector<uint32_t> hp(2 * R), hr(2 * R);
+  bool rejected = false;
+  // exchange (count for p, error word) pairs -> host copies of sent and received counts
   auto count_exchange = [&](std::vector<uint32_t>& sent, std::vector<uint32_t>& got) {
+    k_count_pairs<<<1, 64, 0, st>>>(counts, err, (uint32_t)R, spairs);
     for (int p = 0; p < R; ++p) {
-      sp[p] = counts + p;
-      rp[p] = rcounts + p;
-      sbytes[p] = rbytes[p] = 4;
+      sp[p] = spairs + 2 * p;
+      rp[p] = rpairs + 2 * p;
+      sbytes[p] = rbytes[p] = 8;
     }
     RC(ex->alltoall(r, sp.data(), sbytes.data(), rp.data(), rbytes.data(), st));
-    CK(cudaMemcpyAsync(sent.data(), counts, 4 * R, cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(got.data(), rcounts, 4 * R, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(hp.data(), spairs, 8 * R, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(hr.data(), rpairs, 8 * R, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
+    for (int p = 0; p < R; ++p) {
+      sent[p] = hp[2 * p];
+      got[p] = hr[2 * p];
+      rejected |= hr[2 * p + 1] != 0 || hp[2 * p + 1] != 0;
+    }
     return GGRID_OK;
   };
   auto data_exchange = [&](void* sbase, const std::vector<uint32_t>& sn, void* rbase, const std::vector<uint32_t>& rn,
@@ -310,11 +386,12 @@ static int shard_knn(ggrid_t h, Exchange* ex, int r, int R, const uint2* d_q, ui
   RC(B[1].ensure((size_t)n * 4 + 16));
   RC(B[2].ensure((size_t)n * 16 + 16));
   if (n) {
-    k_route_count<<<blocks(n, 256), 256, 0, st>>>(d_q, n, g, s, B[1].as<uint32_t>(), counts);
+    k_route_count<<<blocks(n, 256), 256, 0, st>>>(d_q, n, g, s, B[1].as<uint32_t>(), counts, err);
     k_route_scatter<<<blocks(n, 256), 256, 0, st>>>(d_q, n, B[1].as<uint32_t>(), counts, R, cursors, B[2].as<uint4>());
   }
   h->stats.launches += 2;
   RC(count_exchange(sc, rcv));
+  if (rejected) return GGRID_EINVAL;  // (every shard saw the same error words)
   const uint64_t m = sum(rcv);
   RC(B[3].ensure(m * 16 + 16));
   RC(data_exchange(B[2].p, sc, B[3].p, rcv, 16));
@@ -338,6 +415,7 @@ static int shard_knn(ggrid_t h, Exchange* ex, int r, int R, const uint2* d_q, ui
   if (m) k_request_count<<<blocks(m, 256), 256, 0, st>>>(mask, (uint32_t)m, counts);
   RC(count_exchange(rq_s, rq_r));
   const uint64_t n_req = sum(rq_s), n_got = sum(rq_r);
+  h->stats.remote_requests += n_req;
   RC(B[7].ensure(n_req * 16 + 16));
   RC(B[8].ensure(n_got * 16 + 16));
   if (m && n_req)
@@ -388,6 +466,18 @@ static int shard_knn(ggrid_t h, Exchange* ex, int r, int R, const uint2* d_q, ui
   CK(cudaStreamSynchronize(st));
   CK(cudaGetLastError());
   return GGRID_OK;
+#undef RC
+#undef CK
+#define RC(x)                      \
+  do {                             \
+    int r_ = (x);                  \
+    if (r_ != GGRID_OK) return r_; \
+  } while (0)
+#define CK(x)                                                                             \
+  do {                                                                                    \
+    cudaError_t e_ = (x);                                                                 \
+    if (e_ != cudaSuccess) return e_ == cudaErrorMemoryAllocation ? GGRID_ENOMEM : GGRID_ECUDA; \
+  } while (0)
 }
 
 // ----------------------------------------------------------------------------- the index
@@ -507,12 +597,15 @@ int multi_knn(MultiIndex* mi, const ggrid_query* q, uint32_t n_q, uint32_t k, ui
     const uint32_t base = n_q / R, extra = n_q % R;
     const uint32_t lo = r * base + std::min<uint32_t>(r, extra), cnt = base + (r < (int)extra ? 1 : 0);
     DBuf& in = h->mx[14];
-    RC(in.ensure((size_t)cnt * 8 + (size_t)cnt * k * 8 + 16));
+    if (in.ensure((size_t)cnt * 8 + (size_t)cnt * k * 8 + 16) != GGRID_OK ||
+        h->order_inputs(h->stream) != GGRID_OK ||
+        (cnt && cudaMemcpyAsync(in.p, q + lo, (size_t)cnt * 8, cudaMemcpyDefault, h->stream) != cudaSuccess)) {
+      mi->ex->abort();  // (the peers are entering the protocol)
+      return GGRID_ENOMEM;
+    }
     uint2* d_q = in.as<uint2>();
     uint32_t* d_oo = reinterpret_cast<uint32_t*>(d_q + cnt);
     uint32_t* d_od = d_oo + (size_t)cnt * k;
-    RC(h->order_inputs(h->stream));
-    if (cnt) CK(cudaMemcpyAsync(d_q, q + lo, (size_t)cnt * 8, cudaMemcpyDefault, h->stream));
     RC(shard_knn(h, mi->ex.get(), r, R, d_q, cnt, k, d_oo, d_od));
     if (cnt) {
       CK(cudaMemcpyAsync(out_obj + (size_t)lo * k, d_oo, (size_t)cnt * k * 4, cudaMemcpyDefault, h->stream));
@@ -529,12 +622,15 @@ int rank_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
   Exchange* ex = h->xchg;
   const int R = (int)h->s.n_ranks, r = (int)h->s.rank;
   DBuf& in = h->mx[14];
-  RC(in.ensure((size_t)n_q * 8 + (size_t)n_q * k * 8 + 16));
+  if (in.ensure((size_t)n_q * 8 + (size_t)n_q * k * 8 + 16) != GGRID_OK ||
+      h->order_inputs(h->stream) != GGRID_OK ||
+      (n_q && cudaMemcpyAsync(in.p, q, (size_t)n_q * 8, cudaMemcpyDefault, h->stream) != cudaSuccess)) {
+    ex->abort();
+    return GGRID_ENOMEM;
+  }
   uint2* d_q = in.as<uint2>();
   uint32_t* d_oo = reinterpret_cast<uint32_t*>(d_q + n_q);
   uint32_t* d_od = d_oo + (size_t)n_q * k;
-  RC(h->order_inputs(h->stream));
-  if (n_q) CK(cudaMemcpyAsync(d_q, q, (size_t)n_q * 8, cudaMemcpyDefault, h->stream));
   RC(shard_knn(h, ex, r, R, d_q, n_q, k, d_oo, d_od));
   if (n_q) {
     CK(cudaMemcpyAsync(out_obj, d_oo, (size_t)n_q * k * 4, cudaMemcpyDefault, h->stream));
