@@ -58,16 +58,19 @@ struct WarpMem {
   uint32_t* act;             // F: the round's active slots (the bucket being expanded)
   uint8_t* listed;           // H: vertex expanded at least once (objects harvested); a vertex is
                              //    in one round's active list at most once, so plain stores
+  uint2* stage;              // STAGE: the chunk's arcs (dst, D + w), compacted (one-warp variant)
 };
+constexpr uint32_t STAGE = 128;  // arcs of a chunk of 32 bucket vertices (4 inline slots each)
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 12ull * c.C + 4ull * (3ull * c.F + (c.H + 31) / 32) + ((c.H + 3) & ~3u);
+  return 8ull * c.H + 12ull * c.C + 4ull * (3ull * c.F + (c.H + 31) / 32) + ((c.H + 3) & ~3u) + 8ull * STAGE;
 }
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   WarpMem m;
   m.cand = reinterpret_cast<unsigned long long*>(base);
-  uint32_t* p = reinterpret_cast<uint32_t*>(m.cand + c.C);
+  m.stage = reinterpret_cast<uint2*>(m.cand + c.C);
+  uint32_t* p = reinterpret_cast<uint32_t*>(m.stage + STAGE);
   m.key = p; p += c.H;
   m.dist = p; p += c.H;
   m.cobj = p; p += c.C;
@@ -90,6 +93,11 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 // DRAM (the USA-shaped graph's 0.9 GB of per-vertex records is far beyond L2).
 #ifndef GG_PREFETCH
 #define GG_PREFETCH 0
+#endif
+// one-warp variant: lane = vertex chunks with compacted arcs (1) or lane = (vertex, slot)
+// windows of 8 vertices (0, the round-1 design)
+#ifndef GG_WARP_ARCS
+#define GG_WARP_ARCS 1
 #endif
 __device__ __forceinline__ void prefetch_vertex(const DevGraph& g, const DevState& s, uint32_t v) {
   if (GG_PREFETCH) {
@@ -363,6 +371,153 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
     __syncwarp();
     c_vert += na;
 
+#if GG_WARP_ARCS
+    // ---- 3. expand the bucket in chunks of 32 vertices, lane = vertex: ONE dependent global
+    //         round trip per chunk loads each vertex's 32-byte inline arc record (two 16-byte
+    //         loads) and, at its first expansion, its cell state and object index; the chunk's
+    //         real arcs are then compacted into shared memory (warp prefix sum over the lanes'
+    //         arc counts) and relaxed 32 at a time, lane = arc -- no lane idles on an empty slot
+    for (uint32_t c0 = 0; c0 < na; c0 += 32) {
+      const uint32_t vi = c0 + lane;
+      const bool vv = vi < na;
+      uint32_t vslot = 0, u = 0, du = INF, hcell = 0, hd = NONE;
+      uint4 a01 = make_uint4(0, 0, 0, 0), a23 = make_uint4(0, 0, 0, 0);
+      uint2 cc = make_uint2(0, 0), v0 = make_uint2(0, 0);
+      bool harv = false;
+      if (vv) {
+        vslot = m.act[vi];
+        u = m.key[vslot];
+        du = m.dist[vslot];  // (an improvement after this read re-queues the vertex: fin bit cleared)
+        const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)u * 4);
+        a01 = rec[0];
+        a23 = rec[1];
+        harv = !m.listed[vslot];
+        if (harv) {
+          m.listed[vslot] = 1;
+          hcell = cellof(g, u);
+          hd = s.cell_head[hcell];
+          cc = s.cell_comp[hcell];
+          v0 = s.v_obj[u];
+        }
+      }
+      const bool overflow_arcs = a23.w == WMAX;  // more than 4 arcs: 3 inline, the rest in the CSR
+      // compact the real arcs (w != 0) of the chunk: (dst, du + w), skipping sums >= INF
+      auto real = [&](uint32_t w) { return w != 0 && w != WMAX && (unsigned long long)du + w < INF; };
+      const uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
+      const uint32_t cnt = r0 + r1 + r2 + r3;
+      uint32_t pre = cnt;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, pre, o);
+        if (lane >= (uint32_t)o) pre += y;
+      }
+      const uint32_t n_arc = __shfl_sync(FULL, pre, 31);
+      pre -= cnt;
+      if (r0) m.stage[pre++] = make_uint2(a01.x, du + a01.y);
+      if (r1) m.stage[pre++] = make_uint2(a01.z, du + a01.w);
+      if (r2) m.stage[pre++] = make_uint2(a23.x, du + a23.y);
+      if (r3) m.stage[pre++] = make_uint2(a23.z, du + a23.w);
+      c_arcs += cnt;
+      const bool dirty = harv && hd != NONE;
+      const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
+      const uint32_t ev = __reduce_or_sync(FULL, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
+      __syncwarp();
+      // relax: lane = arc of the staged list
+      for (uint32_t j0 = 0; j0 < n_arc; j0 += 32) {
+        bool has = false, ovf = false;
+        uint32_t nslot = 0;
+        if (j0 + lane < n_arc) {
+          const uint2 a = m.stage[j0 + lane];
+          bool imp;
+          const int rr = tab_relax(m, H, a.x, a.y, imp);
+          if (rr < 0) {
+            ovf = true;
+          } else if (imp) {
+            mn = min(mn, a.y);
+            const uint32_t bit = 1u << (rr & 31);
+            if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+              has = true;
+              nslot = (uint32_t)rr;
+              prefetch_vertex(g, s, a.x);
+            }
+          }
+        }
+        if (__any_sync(FULL, ovf)) return OVERFLOW;
+        const unsigned hm = __ballot_sync(FULL, has);
+        if (nn + __popc(hm) > cp.F) return OVERFLOW;
+        if (has) nfront[nn + __popc(hm & lt)] = nslot;
+        nn += __popc(hm);
+      }
+      __syncwarp();  // (the stage is rewritten by the next chunk)
+      // vertices with more than 4 arcs: arcs 3.. from the CSR, one per lane per step (rare)
+      if (ev & 2u) {
+        uint32_t b0 = 0, b1 = 0;
+        if (overflow_arcs) {
+          b0 = g.rowptr[u] + 3;
+          b1 = g.rowptr[u + 1];
+        }
+        const uint32_t most = __reduce_max_sync(FULL, b1 - b0);
+        for (uint32_t j = 0; j < most; ++j) {
+          bool has = false, ovf = false;
+          uint32_t nslot = 0;
+          if (b0 + j < b1) {
+            const uint2 av = g.adj[b0 + j];
+            ++c_arcs;
+            const unsigned long long nd = (unsigned long long)du + av.y;
+            if (nd < INF) {
+              bool imp;
+              const int rr = tab_relax(m, H, av.x, (uint32_t)nd, imp);
+              if (rr < 0) {
+                ovf = true;
+              } else if (imp) {
+                mn = min(mn, (uint32_t)nd);
+                const uint32_t bit = 1u << (rr & 31);
+                if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+                  has = true;
+                  nslot = (uint32_t)rr;
+                }
+              }
+            }
+          }
+          if (__any_sync(FULL, ovf)) return OVERFLOW;
+          const unsigned hm = __ballot_sync(FULL, has);
+          if (nn + __popc(hm) > cp.F) return OVERFLOW;
+          if (has) nfront[nn + __popc(hm & lt)] = nslot;
+          nn += __popc(hm);
+        }
+      }
+      if (ev & 4u) {  // a cell with cached updates: lazy flush, then retry (Alg. 4 l.2-4)
+        if (dirty) request_flush(s, hcell, P.epoch);
+        request_lookahead(P, m, front, nf, lane);
+        return RETRY;
+      }
+      c_harv += harv;
+      if (track) {
+        const uint32_t o = harv ? owner_of(hcell, g.n_cells, s.n_ranks) : s.rank;
+        const unsigned long long bm = o != s.rank ? 1ull << o : 0ull;
+        rmask |= ((unsigned long long)__reduce_or_sync(FULL, (uint32_t)(bm >> 32)) << 32) |
+                 __reduce_or_sync(FULL, (uint32_t)bm);
+      }
+      if (ev & 8u) {  // harvest the objects of the vertices expanded for the first time
+        const uint32_t most = __reduce_max_sync(FULL, vo.y);
+        c_objs += vo.y;
+        for (uint32_t j = 0; j < most; ++j) {
+          bool hc = false;
+          uint32_t ob = 0, oo = 0;
+          if (j < vo.y) {
+            const uint32_t p = vo.x + j;
+            ob = s.ar.obj[p];
+            const unsigned long long kk = s.ar.key[p];
+            const uint32_t oe = s.ar.edge[p];
+            oo = s.ar.off[p];
+            const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
+            hc = !same_ahead && kk == s.ot_key[ob];
+          }
+          if (!cand_push(m, nc, cp.C, hc, vslot, oo, ob, lt)) return OVERFLOW;
+        }
+      }
+    }
+#else
     // ---- 3. expand: 8 vertices per window, lane = (vertex, arc slot); the next window's
     //         global loads (inline arcs, object metadata) are issued before this window's
     //         relaxations
@@ -487,6 +642,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
       }
       cur = nxt;
     }
+#endif
     uint32_t* tmp = front;
     front = nfront;
     nfront = tmp;

@@ -425,7 +425,7 @@ static int shard_knn(ggrid_t h, Exchange* ex, int r, int R, const uint2* d_q, ui
   // ---- replies: own objects within the bound
   const size_t rw = 2 * (size_t)k + 1;  // answer record words
   RC(B[9].ensure(n_got * 12 + n_got * k * 8 + 16));
-  RC(B[10].ensure(std::max(n_got, n_req) * rw * 4 + 16));
+  RC(B[10].ensure(std::max(n_got, m) * rw * 4 + 16));  // replies sent, then the answers returned
   uint2* got_q = B[9].as<uint2>();
   uint32_t* got_b = reinterpret_cast<uint32_t*>(got_q + n_got);
   uint32_t* rep_o = got_b + n_got;
