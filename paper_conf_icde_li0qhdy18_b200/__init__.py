@@ -245,15 +245,18 @@ def alltoall_callback(torch_group=None):
             for p in range(n_ranks):
                 ins.append(_u8_view(send[p], sbytes[p], dev))
                 outs.append(_u8_view(recv[p], rbytes[p], dev))
-            if dist.get_backend(torch_group) == "gloo":
-                hi = [t.cpu() for t in ins]
-                ho = [torch.empty(int(rbytes[p]), dtype=torch.uint8) for p in range(n_ranks)]
-                dist.all_to_all(ho, hi, group=torch_group)
-                for p in range(n_ranks):
-                    if rbytes[p]:
-                        outs[p].copy_(ho[p])
-            else:
-                dist.all_to_all(outs, ins, group=torch_group)
+            ssz = [int(sbytes[p]) for p in range(n_ranks)]
+            rsz = [int(rbytes[p]) for p in range(n_ranks)]
+            host = dist.get_backend(torch_group) == "gloo"  # (gloo: CPU tensors, no list all_to_all)
+            cat_in = torch.cat(ins) if sum(ssz) else torch.empty(0, dtype=torch.uint8, device=f"cuda:{dev}")
+            cat_in = cat_in.cpu() if host else cat_in
+            cat_out = torch.empty(sum(rsz), dtype=torch.uint8, device="cpu" if host else f"cuda:{dev}")
+            dist.all_to_all_single(cat_out, cat_in, rsz, ssz, group=torch_group)
+            off = 0
+            for p in range(n_ranks):
+                if rsz[p]:
+                    outs[p].copy_(cat_out[off:off + rsz[p]])
+                off += rsz[p]
             torch.cuda.synchronize(dev)
             return 0
         except Exception as e:  # (reported to the library as a failed exchange: ENCCL)

@@ -347,6 +347,8 @@ static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts
   if ((rc = h->alloc(&s.cell_head, h->n_cells, false))) return fail(rc);
   if (cudaMemset(s.cell_head, 0xFF, (size_t)h->n_cells * 4)) return fail(GGRID_ECUDA);
   if ((rc = h->alloc(&s.cell_pending, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&s.listed_cell, o.max_objects, false))) return fail(rc);
+  if (cudaMemset(s.listed_cell, 0xFF, (size_t)o.max_objects * 4)) return fail(GGRID_ECUDA);
   if ((rc = h->alloc(&s.cell_req, h->n_cells))) return fail(rc);
   if ((rc = h->alloc(&s.v_obj, V))) return fail(rc);
   if ((rc = h->alloc(&s.cell_comp, h->n_cells))) return fail(rc);

@@ -85,7 +85,7 @@ template <class B>
 __device__ void walk_extents(B& bf, const DevState& s, uint32_t e, uint2 comp, uint32_t t_cut) {
   uint32_t n = 0, pre = 0;
   unsigned long long nrec = 0, nexp = 0;
-  while (e != NONE && n < XMAX) {
+  while (is_extent(e) && n < XMAX) {
     const uint32_t st = s.x_start[e], ln = s.x_len[e], nxt = s.x_next[e];
     if (t_cut && s.x_tmax[e] < t_cut) {
       nexp += ln;
@@ -101,7 +101,7 @@ __device__ void walk_extents(B& bf, const DevState& s, uint32_t e, uint2 comp, u
     e = nxt;
   }
   bf.comp_done = 0;
-  if (e == NONE && n < XMAX) {
+  if (!is_extent(e) && n < XMAX) {
     if (comp.y) {
       bf.xs[n] = comp.x;
       bf.xl[n] = comp.y;
@@ -255,6 +255,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
         first &= !((vj == vi) & (j < i));
       }
       const uint32_t q = ob0 + r;
+      s.listed_cell[sm.w_obj[i]] = c;
       out.obj[q] = sm.w_obj[i];
       out.key[q] = sm.w_key[i];
       out.vsrc[q] = vi;
@@ -272,7 +273,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
       bool last = false;
       while (!last) {
         uint32_t sst, sln;
-        if (e2 != NONE) {
+        if (is_extent(e2)) {
           sst = s.x_start[e2];
           sln = (t_cut && s.x_tmax[e2] < t_cut) ? 0u : s.x_len[e2];
           e2 = s.x_next[e2];
@@ -331,6 +332,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
         for (int u = 0; u < U; ++u) {
           if (i0 + u * 32 >= n_win) continue;
           const uint32_t q = ob0 + atomicAdd(&cnt[vs[u] - cbeg], 1u);
+          s.listed_cell[ob[u]] = c;
           out.obj[q] = ob[u];
           out.key[q] = kk[u];
           out.vsrc[q] = vs[u];
@@ -342,6 +344,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
       for (uint32_t i = lane; i < n_win; i += 32) {
         const uint32_t vs = sm.w_vs[i];
         const uint32_t q = ob0 + atomicAdd(&cnt[vs - cbeg], 1u);
+        s.listed_cell[sm.w_obj[i]] = c;
         out.obj[q] = sm.w_obj[i];
         out.key[q] = sm.w_key[i];
         out.vsrc[q] = vs;
@@ -355,6 +358,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
         if (kk == otk[ob]) {
           const uint32_t vs = s.ar.vsrc[p];
           const uint32_t q = ob0 + atomicAdd(&cnt[vs - cbeg], 1u);
+          s.listed_cell[ob] = c;
           out.obj[q] = ob;
           out.key[q] = kk;
           out.vsrc[q] = vs;

@@ -287,6 +287,7 @@ __global__ void __launch_bounds__(CT) k_ingest_scatter(const uint4* __restrict__
       if (k >= nt) continue;
       const unsigned long long key =
           ((unsigned long long)m[q].w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + il[j]));
+      mark_moved(s, m[q].x, cellof(g, vr[j].x));
       if (pos[q] != NONE) {  // (NONE: a cell another rank owns)
         s.ar.obj[pos[q]] = m[q].x;
         s.ar.key[pos[q]] = key;
@@ -518,6 +519,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
     const uint32_t slot = x.y & 0xFFFFu, f = x.y >> 16;
     const unsigned long long key =
         ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + k));
+    mark_moved(s, m.x, cellof(g, x.x));
     if (h_cell[slot] != REMOTE_CELL) {  // (REMOTE_CELL: a cell another rank owns)
       const uint32_t pos = h_aux[slot] + si;
       s.ar.obj[pos] = m.x;

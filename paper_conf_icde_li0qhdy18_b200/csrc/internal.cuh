@@ -18,6 +18,11 @@
 namespace gg {
 
 constexpr uint32_t NONE = 0xFFFFFFFFu;
+// cell_head[c] == STALE: no cached extents, but c's cleaned list holds a record of an object
+// that has since reported from another cell (ingest marks it, reading R8); like a cell with
+// cached updates it is re-cleaned before its list is read.  A chain ends at NONE or STALE.
+constexpr uint32_t STALE = 0xFFFFFFFEu;
+__host__ __device__ inline bool is_extent(uint32_t e) { return e < STALE; }
 constexpr uint32_t INF = 0xFFFFFFFFu;  // u32 distance "unreachable" (reading R18)
 constexpr unsigned long long EMPTY64 = ~0ull;
 constexpr uint32_t BCOUNT_STRIDE = 32;
@@ -92,7 +97,8 @@ struct DevState {
   uint32_t* x_next;
   uint32_t* x_tmax;   // newest t of the extent's messages (zeta.t, P@20743)
   uint32_t ext_cap;
-  uint32_t* cell_head;     // newest pending extent or NONE (NONE = clean)
+  uint32_t* cell_head;     // newest pending extent, or NONE (clean), or STALE (see above)
+  uint32_t* listed_cell;   // [max_objects] the cell whose cleaned list holds o's record, or NONE
   uint32_t* cell_pending;  // cached records not yet cleaned
   uint32_t* cell_req;      // request epoch stamp (dedup of flush requests)
   uint2* v_obj;            // [V] (arena start, count) of the objects at each vertex
@@ -162,8 +168,17 @@ __device__ inline unsigned lanemask_lt() {
 }
 
 // Request a flush of cell c in this knn epoch (deduplicated by the epoch stamp).
+// Ingest: an update of object o from cell c_new leaves o's record in the cleaned list of
+// listed_cell[o] outdated when that is another cell: mark it STALE (unless it has cached
+// extents already).  With this, a clean cell's list holds only latest records, so the query
+// side needs no per-object validity gather (reading R8).
+__device__ __forceinline__ void mark_moved(const DevState& s, uint32_t o, uint32_t c_new) {
+  const uint32_t lc = s.listed_cell[o];
+  if (lc != NONE && lc != c_new) atomicCAS(&s.cell_head[lc], NONE, STALE);
+}
+
 __device__ inline void request_flush(const DevState& s, uint32_t c, uint32_t epoch) {
-  if (s.cell_head[c] == NONE) return;
+  if (s.cell_head[c] == NONE) return;  // (clean; a STALE cell is re-cleaned too)
   // plain read first: most requests of a batch hit an already-requested cell, so the
   // contended atomic is only issued by the first few
   if (*((volatile uint32_t*)&s.cell_req[c]) == epoch) return;

@@ -92,7 +92,7 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 // and object index are fetched into L2 now, so the expansion's dependent load hits L2 instead of
 // DRAM (the USA-shaped graph's 0.9 GB of per-vertex records is far beyond L2).
 #ifndef GG_PREFETCH
-#define GG_PREFETCH 0
+#define GG_PREFETCH 1  // (C3: expansion 1.75 -> 1.66 ms per 65,536 queries, r2b variants)
 #endif
 // one-warp variant: lane = vertex chunks with compacted arcs (1) or lane = (vertex, slot)
 // windows of 8 vertices (0, the round-1 design)
@@ -104,6 +104,16 @@ __device__ __forceinline__ void prefetch_vertex(const DevGraph& g, const DevStat
     asm volatile("prefetch.global.L2 [%0];" ::"l"(g.vadj + (size_t)v * 4));
     asm volatile("prefetch.global.L2 [%0];" ::"l"(s.v_obj + v));
   }
+}
+
+// A record read from a clean cell's list is its object's latest (ingest marks a cell whose list
+// an object has left STALE, and the query re-cleans STALE cells like dirty ones: reading R8), so
+// the object-table gather key == ot_key[obj] is only a debug cross-check (GG_HARVEST_VALIDATE=1).
+#ifndef GG_HARVEST_VALIDATE
+#define GG_HARVEST_VALIDATE 0
+#endif
+__device__ __forceinline__ bool valid_rec(const DevState& s, uint32_t p, uint32_t ob) {
+  return !GG_HARVEST_VALIDATE || s.ar.key[p] == s.ot_key[ob];
 }
 
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
@@ -314,7 +324,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
         const uint32_t p = vo.x + j;
         ob = s.ar.obj[p];
         const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
-        if (oe == q.x && oo >= q.y && s.ar.key[p] == s.ot_key[ob]) {
+        if (oe == q.x && oo >= q.y && valid_rec(s, p, ob)) {
           has = true;
           dd = oo - q.y;
         }
@@ -511,7 +521,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
             const uint32_t oe = s.ar.edge[p];
             oo = s.ar.off[p];
             const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
-            hc = !same_ahead && kk == s.ot_key[ob];
+            hc = !same_ahead && (!GG_HARVEST_VALIDATE || kk == s.ot_key[ob]);
           }
           if (!cand_push(m, nc, cp.C, hc, vslot, oo, ob, lt)) return OVERFLOW;
         }
@@ -635,7 +645,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
             const uint32_t oe = s.ar.edge[p];
             oo = s.ar.off[p];
             const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
-            hc = !same_ahead && kk == s.ot_key[ob];
+            hc = !same_ahead && (!GG_HARVEST_VALIDATE || kk == s.ot_key[ob]);
           }
           if (!cand_push(m, nc, cp.C, hc, cur.vslot, oo, ob, lt)) return OVERFLOW;
         }
@@ -830,7 +840,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
       const uint32_t p = vo.x + j;
       const uint32_t ob = s.ar.obj[p];
       const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
-      if (oe == q.x && oo >= q.y && s.ar.key[p] == s.ot_key[ob]) {
+      if (oe == q.x && oo >= q.y && valid_rec(s, p, ob)) {
         const uint32_t i = atomicAdd(&sh.nc, 1u);
         if (i < cp.C) {
           m.cand[i] = ((unsigned long long)SPECIAL << 32) | (oo - q.y);
@@ -950,7 +960,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
               const unsigned long long kk = s.ar.key[p];
               const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
               const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
-              if (!same_ahead && kk == s.ot_key[ob]) {
+              if (!same_ahead && (!GG_HARVEST_VALIDATE || kk == s.ot_key[ob])) {
                 const uint32_t i = atomicAdd(&sh.nc, 1u);
                 if (i < cp.C) {
                   m.cand[i] = ((unsigned long long)vslot << 32) | oo;
@@ -1110,7 +1120,8 @@ __global__ void __launch_bounds__(W * 32, GG_MINB0) k_expand_cta_capped(QParams 
 // fewer than k objects may need to settle the whole graph).
 constexpr int NLEVELS = EXPAND_LEVELS;
 #ifndef GG_H0
-#define GG_H0 1024  // level-0 vertex table (experiment hook: -DGG_H0=..., -DGG_F0=...)
+#define GG_H0 896  // level-0 vertex table (C3 one-warp: 1,024 -> 896 slots = more warps per SM,
+                   // 1.66 -> 1.54 ms; 768: 1.53 ms but promotions; experiment hook -DGG_H0=...)
 #endif
 #ifndef GG_F0
 #define GG_F0 96

@@ -42,7 +42,7 @@ __global__ void k_pa_count(DevGraph g, DevState s, uint32_t bsize, uint32_t* __r
     return;
   }
   uint32_t n = 0;
-  for (uint32_t e = s.cell_head[c]; e != NONE; e = s.x_next[e]) n += (s.x_len[e] + bsize - 1) / bsize;
+  for (uint32_t e = s.cell_head[c]; is_extent(e); e = s.x_next[e]) n += (s.x_len[e] + bsize - 1) / bsize;
   n += (s.cell_comp[c].y + bsize - 1) / bsize;
   cnt[c] = n;
 }
@@ -55,7 +55,7 @@ __global__ void k_pa_fill(DevGraph g, DevState s, uint32_t bsize, const uint32_t
   auto emit = [&](uint32_t st, uint32_t ln) {
     for (uint32_t a = 0; a < ln; a += bsize) out[o++] = PaBucket{st + a, min(bsize, ln - a)};
   };
-  for (uint32_t e = s.cell_head[c]; e != NONE; e = s.x_next[e]) emit(s.x_start[e], s.x_len[e]);
+  for (uint32_t e = s.cell_head[c]; is_extent(e); e = s.x_next[e]) emit(s.x_start[e], s.x_len[e]);
   emit(s.cell_comp[c].x, s.cell_comp[c].y);
 }
 

@@ -122,6 +122,20 @@ def _rank_worker(rank, world, port, q_out):
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
+        _rank_body(rank, world, q_out)
+    except Exception as e:  # (reported, so the test fails instead of waiting for a result)
+        q_out.put((rank, -1, repr(e), 0))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+def _rank_body(rank, world, q_out):
+    import torch
+
+    import paper_conf_icde_li0qhdy18_b200 as gg
+
+    if True:
         torch.cuda.set_device(0)
         g = synth.table_ii_graph("NY", scale=0.05)
         walk = synth.RandomWalk(g, 3000, inject=True)
@@ -140,8 +154,6 @@ def _rank_worker(rank, world, port, q_out):
         st = grid.stats()
         q_out.put((rank, bad_total, int(st["n_shards"]), int(st["exchange_kind"])))
         grid.close()
-    finally:
-        dist.destroy_process_group()
 
 
 @pytest.mark.parametrize("world", [2, 3])
@@ -156,7 +168,7 @@ def test_multiprocess_ranks_callback_exchange(gg, world):
     procs = [ctx.Process(target=_rank_worker, args=(r, world, port, q_out)) for r in range(world)]
     for p in procs:
         p.start()
-    res = sorted(q_out.get(timeout=600) for _ in range(world))
+    res = sorted(q_out.get(timeout=300) for _ in range(world))
     for p in procs:
         p.join(timeout=120)
     assert all(bad == 0 for _, bad, _, _ in res), res

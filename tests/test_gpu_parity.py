@@ -575,3 +575,26 @@ def test_ladder_boundaries_and_promotions(gg):
         _assert_same(grid.knn(q[:200], k), _oracle(g, upd, q[:200], k), f"k={k}")
     assert promoted > 0  # (3 with these seeds: the promotion path ran)
     grid.close()
+
+
+def test_moved_objects_leave_clean_cells_stale(gg):
+    """Objects jumping between cells every round (uniform random relocation, 4-vertex cells):
+    the cell an object left is marked STALE at ingest and re-cleaned before its list is read,
+    so answers stay exact without the per-object validity gather (reading R8).  Queries are
+    interleaved with the jumps; some rounds re-send older timestamps (late arrivals)."""
+    g = synth.table_ii_graph("NY", scale=0.01)
+    rng = np.random.default_rng(5)
+    n_obj = 300
+    grid = gg.GGrid(g, 4, max_objects=n_obj)
+    hist = []
+    for r in range(12):
+        arc, off = synth.random_locations(g, n_obj, rng)
+        t = np.full(n_obj, 1000 * r, np.uint32) if r % 4 != 3 else np.full(n_obj, 1000 * (r - 2), np.uint32)
+        u = np.stack([np.arange(n_obj, dtype=np.uint32)[rng.permutation(n_obj)], arc, off, t], 1).astype(np.uint32)
+        u[:, 1] = arc[u[:, 0]]
+        u[:, 2] = off[u[:, 0]]
+        hist.append(u)
+        grid.ingest(u)
+        q = synth.queries(g, 150, seed=600 + r)
+        _assert_same(grid.knn(q, 7), _oracle(g, np.concatenate(hist), q, 7), f"round {r}")
+    grid.close()
