@@ -135,25 +135,24 @@ def _rank_body(rank, world, q_out):
 
     import paper_conf_icde_li0qhdy18_b200 as gg
 
-    if True:
-        torch.cuda.set_device(0)
-        g = synth.table_ii_graph("NY", scale=0.05)
-        walk = synth.RandomWalk(g, 3000, inject=True)
-        grid = gg.GGrid(g, 128, max_objects=3000, n_ranks=world, rank=rank, exchange=gg.alltoall_callback())
-        hist = []
-        bad_total = 0
-        for it in range(2):
-            u = walk.ticks(2)
-            hist.append(u)
-            grid.ingest(u)  # every rank ingests the whole stream
-            nq = 150 + 37 * rank  # different batch sizes per rank
-            q = synth.queries(g, nq, seed=1000 * rank + it)
-            go, gd = grid.knn(q, 8)  # collective
-            ro, rd = oracle.knn_from_updates(g, np.concatenate(hist), q, 8)
-            bad_total += int((~((go == ro).all(1) & (gd == rd).all(1))).sum())
-        st = grid.stats()
-        q_out.put((rank, bad_total, int(st["n_shards"]), int(st["exchange_kind"])))
-        grid.close()
+    torch.cuda.set_device(0)
+    g = synth.table_ii_graph("NY", scale=0.05)
+    walk = synth.RandomWalk(g, 3000, inject=True)
+    grid = gg.GGrid(g, 128, max_objects=3000, n_ranks=world, rank=rank, exchange=gg.alltoall_callback())
+    hist = []
+    bad_total = 0
+    for it in range(2):
+        u = walk.ticks(2)
+        hist.append(u)
+        grid.ingest(u)  # every rank ingests the whole stream
+        nq = 150 + 37 * rank  # different batch sizes per rank
+        q = synth.queries(g, nq, seed=1000 * rank + it)
+        go, gd = grid.knn(q, 8)  # collective
+        ro, rd = oracle.knn_from_updates(g, np.concatenate(hist), q, 8)
+        bad_total += int((~((go == ro).all(1) & (gd == rd).all(1))).sum())
+    st = grid.stats()
+    q_out.put((rank, bad_total, int(st["n_shards"]), int(st["exchange_kind"])))
+    grid.close()
 
 
 @pytest.mark.parametrize("world", [2, 3])
