@@ -472,6 +472,292 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
   }
 }
 
+// ---------------------------------------------------------------------------------------------
+// Bulk-copy (TMA engine) variant of the flush: the record stream of a CTA's cells never drains at
+// a cell boundary.  Warp roles (6 warps):
+//   producer (warp 0, one lane)  walks each cell's extent chain (+ its previous cleaned list) and
+//                                issues cp.async.bulk copies of CHUNK-record pieces of the obj and
+//                                key arrays into a ring of TS shared-memory stages, each stage's
+//                                landing signalled on its "full" mbarrier (transaction bytes);
+//   4 match warps                take the stages round-robin: ot_key[obj] gather (L1/L2), compare,
+//                                ballot-append the matching positions to the cell's winner list,
+//                                release the stage ("empty" mbarrier); the warp finishing a cell's
+//                                last piece queues the cell for indexing;
+//   index warp (warp 5)          builds R[c] of each matched cell (index_cell above) and frees its
+//                                slot for the producer.
+// Up to TSLOT cells are in flight per CTA.  The per-cell arithmetic is the one above.
+#ifndef GG_FLUSH_TMA
+#define GG_FLUSH_TMA 1
+#endif
+constexpr int TCHUNK = 256;  // records per stage (8 per match-warp lane)
+constexpr int TS = 8;        // stages
+constexpr int TSLOT = 4;     // cells in flight
+constexpr int TMW = 4;       // match warps
+constexpr int TFT = (TMW + 2) * 32;
+
+template <int WCAP>
+struct TSlot {
+  uint32_t c, head, has;
+  uint2 comp;
+  unsigned long long nrec, nexp;
+  uint32_t n_win;
+  unsigned long long state;  // (pieces of the cell << 32) + pieces matched: complete when equal
+  uint32_t spill_cap;
+  uint32_t* spill;
+  uint32_t w_pos[WCAP];
+};
+
+template <int HCAP, int WCAP>
+struct TFlushSmem {
+  uint32_t obj[TS][TCHUNK];
+  unsigned long long key[TS][TCHUNK];
+  unsigned long long full[TS], empty[TS];
+  uint32_t st_slot[TS], st_n[TS], st_pos[TS];
+  TSlot<WCAP> slot[TSLOT];
+  uint32_t slot_gen[TSLOT];  // cells indexed per slot (the producer reuses a slot when caught up)
+  uint32_t rq[TSLOT];        // matched cells for the index warp: entry i = slot | (i / TSLOT) << 4
+  uint32_t rq_n;             // entries pushed
+  // index warp only (index_cell)
+  unsigned long long w_key[WCAP];
+  uint32_t w_obj[WCAP];
+  uint32_t w_vs[WCAP];
+  uint32_t w_off[WCAP];
+  uint32_t w_edge[WCAP];
+  uint32_t hist[HCAP];
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned long long* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* b, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}" ::"r"(smem_u32(b)),
+      "r"(parity)
+      : "memory");
+}
+// global -> shared bulk copy (TMA engine; 16-byte aligned, multiple of 16 bytes), evict-first in
+// L2 (the log is read once)
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, unsigned long long* bar,
+                                          unsigned long long policy) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy)
+      : "memory");
+}
+
+// queue a matched cell for the index warp (at most TSLOT entries are pending: one per slot)
+__device__ __forceinline__ void rq_push(uint32_t* rq_n, uint32_t* rq, uint32_t b) {
+  __threadfence_block();  // (the cell's winners before its entry)
+  const uint32_t i = atomicAdd(rq_n, 1u);
+  ((volatile uint32_t*)rq)[i % TSLOT] = b | ((i / TSLOT) << 4);
+}
+
+template <int HCAP, int WCAP>
+__global__ void __launch_bounds__(TFT) k_flush_tma(DevGraph g, DevState s, Arena out, unsigned long long* out_top,
+                                                   uint32_t begin, int full_vobj, uint32_t* spill, uint32_t spill_cap,
+                                                   uint32_t t_cut) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  using SM = TFlushSmem<HCAP, WCAP>;
+  SM& sm = *reinterpret_cast<SM*>(smem_raw);
+  pdl_wait();
+  pdl_allow();
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const unsigned lt = lanemask_lt();
+  const uint32_t lend = *((volatile unsigned*)&s.st->n_flush);
+  if (blockIdx.x == 0 && tid == 0) s.st->flush_end = lend;
+  const uint32_t G = gridDim.x;
+  const uint32_t first_li = begin + blockIdx.x;
+  const uint32_t n_mine = first_li < lend ? (lend - first_li + G - 1) / G : 0;
+  if (tid == 0) {
+    for (int i = 0; i < TS; ++i) {
+      mbar_init(&sm.full[i], 1);
+      mbar_init(&sm.empty[i], 1);
+    }
+    for (int b = 0; b < TSLOT; ++b) {
+      sm.slot_gen[b] = 0;
+      sm.rq[b] = 0xFFFFFFF0u;  // (a lap tag no entry carries)
+    }
+    sm.rq_n = 0;
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (n_mine == 0) return;
+  volatile uint32_t* vgen = sm.slot_gen;
+  volatile uint32_t* vrq_n = &sm.rq_n;
+
+  if (wid == 0) {  // ---------------------------------------------------------------- producer
+    if (lane != 0) return;
+    unsigned long long policy;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(policy));
+    uint32_t seq = 0;  // stages issued
+    auto issue = [&](uint32_t b, uint32_t pos, uint32_t n) {  // one stage: records [pos, pos + n)
+      const uint32_t st = seq % TS, ph = (seq / TS) & 1u;
+      mbar_wait(&sm.empty[st], ph ^ 1u);
+      sm.st_slot[st] = b;
+      sm.st_n[st] = n;
+      sm.st_pos[st] = pos;
+      const uint32_t n4 = (n + 3u) & ~3u;  // (extents and lists are 4-record aligned and padded)
+      mbar_expect_tx(&sm.full[st], n4 * 12u);
+      bulk_load(sm.obj[st], s.ar.obj + pos, n4 * 4u, &sm.full[st], policy);
+      bulk_load(sm.key[st], s.ar.key + pos, n4 * 8u, &sm.full[st], policy);
+      ++seq;
+    };
+    uint32_t pc = s.flush_list[first_li];
+    for (uint32_t j = 0; j < n_mine; ++j) {
+      const uint32_t b = j % TSLOT;
+      while (vgen[b] != j / TSLOT) __nanosleep(32);  // the slot's previous cell is indexed
+      TSlot<WCAP>& sl = sm.slot[b];
+      const uint32_t c = pc;
+      const uint32_t head = s.cell_head[c];
+      const uint2 comp = s.cell_comp[c];
+      if (j + 1 < n_mine) pc = s.flush_list[first_li + (j + 1) * G];  // (one gather ahead)
+      sl.c = c;
+      sl.head = head;
+      sl.comp = comp;
+      sl.has = 1;
+      sl.n_win = 0;
+      sl.nrec = 0;
+      sl.nexp = 0;
+      sl.spill = spill + ((size_t)blockIdx.x * TSLOT + b) * spill_cap;
+      sl.spill_cap = spill_cap;
+      sl.state = 0;
+      __threadfence_block();
+      // walk the chain in segments of up to 16 extents: the pieces of every segment but the
+      // last are issued before the total is known; the total is added before the last segment's
+      uint32_t xs[16], xl[16];
+      uint32_t e = head;
+      unsigned long long issued = 0;
+      unsigned long long nrec = 0, nexp = 0;
+      bool done = false;
+      while (!done) {
+        uint32_t nx = 0;
+        while (is_extent(e) && nx < 16) {
+          const uint32_t a = s.x_start[e], l = s.x_len[e], nxt = s.x_next[e];
+          if (t_cut && s.x_tmax[e] < t_cut) {
+            nexp += l;
+          } else if (l) {
+            xs[nx] = a;
+            xl[nx] = l;
+            ++nx;
+            nrec += l;
+          }
+          e = nxt;
+        }
+        const bool last_seg = !is_extent(e);
+        if (last_seg && comp.y && nx < 16) {
+          xs[nx] = comp.x;
+          xl[nx] = comp.y;
+          ++nx;
+          nrec += comp.y;
+          done = true;
+        } else if (last_seg && !comp.y) {
+          done = true;
+        }
+        unsigned long long pieces = 0;
+        for (uint32_t x = 0; x < nx; ++x) pieces += (xl[x] + TCHUNK - 1) / TCHUNK;
+        if (done) {  // the total first: the cell completes when the match warps catch up with it
+          sl.nrec = nrec;
+          sl.nexp = nexp;
+          __threadfence_block();
+          const unsigned long long total = issued + pieces;
+          const unsigned long long old = atomicAdd(&sl.state, total << 32);
+          if ((old & 0xFFFFFFFFull) == total) rq_push(&sm.rq_n, sm.rq, b);  // (all matched, or none)
+        }
+        for (uint32_t x = 0; x < nx; ++x)
+          for (uint32_t o = 0; o < xl[x]; o += TCHUNK) issue(b, xs[x] + o, min((uint32_t)TCHUNK, xl[x] - o));
+        issued += pieces;
+      }
+    }
+    for (int w = 0; w < TMW; ++w) {  // one sentinel stage per match warp: no more pieces
+      const uint32_t st = seq % TS, ph = (seq / TS) & 1u;
+      mbar_wait(&sm.empty[st], ph ^ 1u);
+      sm.st_n[st] = 0xFFFFFFFFu;
+      mbar_expect_tx(&sm.full[st], 0);
+      ++seq;
+    }
+    return;
+  }
+
+  if (wid <= TMW) {  // ---------------------------------------------------------- match warps
+    const unsigned long long* __restrict__ otk = s.ot_key;
+    for (uint32_t seq = wid - 1;; seq += TMW) {
+      const uint32_t st = seq % TS, ph = (seq / TS) & 1u;
+      mbar_wait(&sm.full[st], ph);
+      const uint32_t n = sm.st_n[st];
+      if (n == 0xFFFFFFFFu) break;
+      const uint32_t b = sm.st_slot[st], pos = sm.st_pos[st];
+      TSlot<WCAP>& sl = sm.slot[b];
+      constexpr int R = TCHUNK / 32;
+      uint32_t o[R];
+      unsigned long long k[R], tg[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const uint32_t i = lane + 32 * r;
+        o[r] = sm.obj[st][i];
+        k[r] = sm.key[st][i];
+      }
+#pragma unroll
+      for (int r = 0; r < R; ++r) tg[r] = (lane + 32 * r) < n ? __ldg(otk + o[r]) : ~k[r];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sm.empty[st]);  // (the stage's words are in registers now)
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const bool hit = tg[r] == k[r];
+        const unsigned hm = __ballot_sync(0xffffffffu, hit);
+        if (hm) {
+          uint32_t base = 0;
+          if (lane == __ffs(hm) - 1) base = atomicAdd(&sl.n_win, (unsigned)__popc(hm));
+          base = __shfl_sync(0xffffffffu, base, __ffs(hm) - 1);
+          const uint32_t w = base + __popc(hm & lt);
+          if (hit) {
+            const uint32_t p = pos + lane + 32 * r;
+            if (w < (uint32_t)WCAP) sl.w_pos[w] = p;
+            else if (w - (uint32_t)WCAP < sl.spill_cap) sl.spill[w - WCAP] = p;
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) {
+        __threadfence_block();  // (the winners above before the piece counts as matched)
+        const unsigned long long now = atomicAdd(&sl.state, 1ull) + 1ull;
+        if ((now >> 32) != 0 && (now & 0xFFFFFFFFull) == (now >> 32)) rq_push(&sm.rq_n, sm.rq, b);
+      }
+    }
+    return;
+  }
+
+  // ------------------------------------------------------------------------------- index warp
+  (void)vrq_n;
+  for (uint32_t j = 0; j < n_mine; ++j) {  // entry j of the queue (its lap tag says when it is in)
+    uint32_t b = 0;
+    if (lane == 0) {
+      volatile uint32_t* vrq = sm.rq;
+      uint32_t v;
+      while (((v = vrq[j % TSLOT]) >> 4) != j / TSLOT) __nanosleep(32);
+      b = v & 15u;
+      __threadfence_block();
+    }
+    b = __shfl_sync(0xffffffffu, b, 0);
+    TSlot<WCAP>& sl = sm.slot[b];
+    index_cell<HCAP, WCAP>(sm, sl, g, s, out, out_top, full_vobj, lane, sl.spill, spill_cap, t_cut);
+    __syncwarp();
+    if (lane == 0) {
+      __threadfence_block();
+      vgen[b] = vgen[b] + 1;  // the producer may reuse the slot
+    }
+    __syncwarp();
+  }
+}
+
 template <int HCAP, int WCAP>
 int blocks_per_sm_t();
 template <int HCAP, int WCAP>
@@ -482,23 +768,34 @@ void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned l
   uint32_t grid = (uint32_t)(sm_count * blocks_per_sm);
   if (max_ctas && max_ctas < grid) grid = max_ctas;  // few cells to clean: fewer idle CTAs
   cudaLaunchAttribute attr[1];
+  if (GG_FLUSH_TMA) {
+    const cudaLaunchConfig_t cfg = pdl_config(dim3(grid), dim3(TFT), sizeof(TFlushSmem<HCAP, WCAP>), st, attr);
+    cudaLaunchKernelEx(&cfg, k_flush_tma<HCAP, WCAP>, g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
+    return;
+  }
   const cudaLaunchConfig_t cfg = pdl_config(dim3(grid), dim3(FT), sizeof(FlushSmem<HCAP, WCAP>), st, attr);
   cudaLaunchKernelEx(&cfg, k_flush<HCAP, WCAP>, g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
 }
 template <int HCAP, int WCAP>
 int blocks_per_sm_t() {
   static int blocks_per_sm = 0;  // (occupancy: the same on every B200)
-  const int smem = (int)sizeof(FlushSmem<HCAP, WCAP>);
-  func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  const int smem = GG_FLUSH_TMA ? (int)sizeof(TFlushSmem<HCAP, WCAP>) : (int)sizeof(FlushSmem<HCAP, WCAP>);
+  if (GG_FLUSH_TMA) func_attr_once(k_flush_tma<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  else func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (blocks_per_sm == 0) {
     int b = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush<HCAP, WCAP>, FT, smem);
+    if (GG_FLUSH_TMA) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush_tma<HCAP, WCAP>, TFT, smem);
+    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush<HCAP, WCAP>, FT, smem);
     blocks_per_sm = std::max(b, 1);
+#ifdef GG_FLUSH_TMA_CTAS
+    blocks_per_sm = std::min(blocks_per_sm, GG_FLUSH_TMA_CTAS);  // (experiment hook)
+#endif
   }
   // ask for no more shared memory than the resident CTAs need: the rest stays L1, which
   // holds the object-table lines the match phase gathers (per device, like the size above)
   const int carve = std::min(100, (blocks_per_sm * (smem + 1024) * 100 + 228 * 1024 - 1) / (228 * 1024));
-  func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+  if (GG_FLUSH_TMA) func_attr_once(k_flush_tma<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+  else func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
   return blocks_per_sm;
 }
 }  // namespace
@@ -532,7 +829,7 @@ size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, u
     case 4: bps = blocks_per_sm_t<1024, 2048>(); break;
     default: bps = blocks_per_sm_t<4096, 2048>(); break;
   }
-  return (size_t)sm_count * bps * NBUF * want * sizeof(uint32_t);
+  return (size_t)sm_count * bps * (NBUF > TSLOT ? NBUF : TSLOT) * want * sizeof(uint32_t);
 }
 
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
