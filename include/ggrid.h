@@ -359,6 +359,36 @@ int ggrid_wait_stream(ggrid_t h, void* stream);
  * wants to reuse or free).  Errors: EINVAL, ECUDA. */
 int ggrid_signal_stream(ggrid_t h, void* stream);
 
+/* The paper's query pipeline (Alg. 4-6, P@44429-52751) as a comparison path (
+ * not used by ggrid_knn): every dirty cell cleaned first (Alg. 4 l.2, eagerly); per query on
+ * the GPU, candidate cells = c_q, its neighbour cells and further rings until they hold
+ * >= rho k objects (rho = rho_x100 / 100, the paper's 1.8 is 180), Bellman-Ford over their
+ * vertices (Alg. 5), the k nearest of their objects (GPU_First_k) and the unresolved vertices
+ * (Def. 3, D <= l inclusive); then Refine_kNN (Alg. 6) on `threads` CPU threads (0 = all
+ * cores): a Dijkstra bounded by l - D[v] from every unresolved vertex, the union with the
+ * candidates, per-object minimum, first k.  Answers have ggrid_knn's format and must equal
+ * its rows (the method is exact under the readings of DESIGN.md).  q: host or device;
+ * out_obj / out_dist: HOST pointers (n_q*k).  res (nullable) receives the phase times and
+ * work counters.  Errors: EINVAL (k = 0 or > 4096, rho_x100 < 100, null pointers, a multi-GPU
+ * handle), ENOMEM (a query beyond the comparison path's caps: 64 candidate cells, 4,096
+ * candidate objects or 8,192 unresolved vertices), ECUDA. */
+typedef struct ggrid_prior_art_knn_result {
+  double ms_clean;           /* flush of every dirty cell                                 */
+  double ms_host_index;      /* host vertex -> objects index for the CPU refine          */
+  double ms_gpu;             /* Alg. 4 l.1-9 on the GPU (CUDA events)                    */
+  double ms_d2h;             /* candidates + unresolved vertices to the host             */
+  double ms_cpu_refine;      /* Alg. 6 on CPU threads                                    */
+  uint64_t cells;            /* candidate cells, summed over the queries                 */
+  uint64_t vertices;         /* vertices of those cells, summed                           */
+  uint64_t bf_iterations;    /* Bellman-Ford sweeps, summed                               */
+  uint64_t unresolved;       /* unresolved vertices, summed                               */
+  uint64_t refine_settled;   /* vertices settled by the refine Dijkstras                  */
+  uint32_t threads;          /* CPU threads used                                          */
+  uint32_t pad_;
+} ggrid_prior_art_knn_result;
+int ggrid_prior_art_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t rho_x100,
+                        uint32_t threads, uint32_t* out_obj, uint32_t* out_dist, ggrid_prior_art_knn_result* res);
+
 /* Drain the handle's stream.  Returns the deferred error of an asynchronous ingest batch
  * (opts.async_ingest) that was rejected since the last report, else GGRID_OK; the error is
  * reported once. */

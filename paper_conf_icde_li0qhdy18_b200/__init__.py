@@ -27,7 +27,7 @@ EXPORTS = ["ggrid_build", "ggrid_ingest", "ggrid_ingest_stage", "ggrid_ingest_co
            "ggrid_cell_objects", "ggrid_stats", "ggrid_stats_reset", "ggrid_vertex_cell", "ggrid_zvalue",
            "ggrid_version", "ggrid_shard", "ggrid_query_owner", "ggrid_knn_ex", "ggrid_merge_topk",
            "ggrid_prior_art_clean", "ggrid_prior_art_bundle", "ggrid_wait_stream", "ggrid_signal_stream",
-           "ggrid_nccl_unique_id"]
+           "ggrid_nccl_unique_id", "ggrid_prior_art_knn"]
 
 
 class GGridError(RuntimeError):
@@ -75,6 +75,12 @@ class ggrid_stats_t(ctypes.Structure):
                                        ("exchange_kind", ctypes.c_uint32), ("remote_requests", ctypes.c_uint64)]
 
 
+class ggrid_prior_art_knn_result(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_double) for n in ["ms_clean", "ms_host_index", "ms_gpu", "ms_d2h", "ms_cpu_refine"]] + [
+        (n, ctypes.c_uint64) for n in ["cells", "vertices", "bf_iterations", "unresolved", "refine_settled"]] + [
+        ("threads", ctypes.c_uint32), ("pad_", ctypes.c_uint32)]
+
+
 class ggrid_prior_art_result(ctypes.Structure):
     _fields_ = [(n, ctypes.c_double) for n in ["ms_prepare", "ms_shuffle", "ms_collect"]] + [
         (n, ctypes.c_uint64) for n in ["n_buckets", "n_bundles", "table_bytes", "objects_found", "objects_wrong"]]
@@ -119,6 +125,7 @@ def lib():
             "ggrid_wait_stream": ([P, P], i32),
             "ggrid_signal_stream": ([P, P], i32),
             "ggrid_nccl_unique_id": ([P], i32),
+            "ggrid_prior_art_knn": ([P, P, u32, u32, u32, u32, P, P, ctypes.POINTER(ggrid_prior_art_knn_result)], i32),
         }
         for name, (args, res) in sig.items():
             f = getattr(L, name)
@@ -407,6 +414,20 @@ def ggrid_prior_art_clean(h, eta: int = 5, bucket_size: int = 128, write_mode: i
     return {f: getattr(r, f) for f, _ in ggrid_prior_art_result._fields_}, e, o
 
 
+def ggrid_prior_art_knn(h, queries, k: int, rho: float = 1.8, threads: int = 0):
+    """The paper's query pipeline (Alg. 4-6: GPU candidates, CPU-thread Refine_kNN) as a
+    comparison path.  Returns (obj, dist, result dict); answers have ggrid_knn's format."""
+    q = _u32(queries)
+    nq = int(q.shape[0])
+    oo = np.empty((nq, k), np.uint32)
+    od = np.empty((nq, k), np.uint32)
+    r = ggrid_prior_art_knn_result()
+    _order_inputs(h, q)
+    _check(lib().ggrid_prior_art_knn(h, _ptr(q), nq, int(k), int(round(rho * 100)), int(threads), _ptr(oo), _ptr(od),
+                                     ctypes.byref(r)), "ggrid_prior_art_knn")
+    return oo, od, {f: getattr(r, f) for f, _ in ggrid_prior_art_knn_result._fields_ if f != "pad_"}
+
+
 def ggrid_prior_art_bundle(obj, key, eta: int):
     """Alg. 3 Step 1 (cache-and-shuffle) on one bundle; returns (obj, key) per lane after it."""
     ob = np.ascontiguousarray(obj, np.uint32)
@@ -553,6 +574,9 @@ class GGrid:
     def prior_art_clean(self, eta: int = 5, bucket_size: int = 128, write_mode: int = 0, locations: bool = False):
         return ggrid_prior_art_clean(self.h, eta, bucket_size, write_mode,
                                      self.stats()["max_objects"] if locations else None)
+
+    def prior_art_knn(self, queries, k: int, rho: float = 1.8, threads: int = 0):
+        return ggrid_prior_art_knn(self.h, queries, k, rho, threads)
 
     def flush_all(self):
         ggrid_flush_all(self.h)

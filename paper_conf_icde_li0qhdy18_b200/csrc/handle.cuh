@@ -147,6 +147,10 @@ struct ggrid_s {
   MultiIndex* multi = nullptr;
   Exchange* xchg = nullptr;
   DBuf mx[16];  // the exchange protocol's device buffers
+  // prior-art query comparison path (prior_art_knn.cu): host copy of the out-arc CSR, made on
+  // first use
+  std::vector<uint32_t> pa_rowptr;
+  std::vector<uint2> pa_adj;
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_in = nullptr;   // caller's producer stream -> library streams (order_inputs)
   cudaEvent_t ev_out = nullptr;  // library stream -> a caller's stream (ggrid_signal_stream)

@@ -40,7 +40,8 @@ def test_struct_layouts_match_header(gg, tmp_path):
     import subprocess
 
     structs = {"ggrid_graph": gg.ggrid_graph, "ggrid_opts": gg.ggrid_opts, "ggrid_stats_t": gg.ggrid_stats_t,
-               "ggrid_prior_art_result": gg.ggrid_prior_art_result}
+               "ggrid_prior_art_result": gg.ggrid_prior_art_result,
+               "ggrid_prior_art_knn_result": gg.ggrid_prior_art_knn_result}
     lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "ggrid.h"', "int main(void) {"]
     for name, cls in structs.items():
         lines.append(f'  printf("{name} %zu\\n", sizeof({name}));')

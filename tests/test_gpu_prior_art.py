@@ -86,3 +86,26 @@ def test_prior_art_rejects_bad_args(gg):
         with pytest.raises(gg.GGridError):
             grid.prior_art_clean(*args)
     grid.close()
+
+
+# --------------------------------------------------- the paper's query pipeline (Alg. 4-6)
+@pytest.mark.parametrize("graph,cs,n_obj,k,rho", [("lattice", 16, 100, 3, 1.8), ("lattice", 64, 100, 10, 1.4),
+                                                   ("ny", 256, 3000, 10, 1.8), ("ny", 64, 300, 20, 3.0)])
+def test_prior_art_query_pipeline_exact(gg, graph, cs, n_obj, k, rho):
+    """GPU candidate cells / Bellman-Ford / first-k / unresolved vertices (Alg. 4-5, Def. 3) and
+    Refine_kNN on CPU threads (Alg. 6) answer exactly what the oracle (and ggrid_knn) answers,
+    under the inclusive unresolved rule (reading R13) and the same-arc term (R2): sparse objects
+    (balls beyond the candidate cells) and ties (lattice weights 1..4) included."""
+    g = synth.lattice_graph(32, 32, 1, 4) if graph == "lattice" else synth.table_ii_graph("NY", scale=0.05)
+    upd = synth.RandomWalk(g, n_obj, inject=True).ticks(5)
+    q = synth.queries(g, 300)
+    grid = gg.GGrid(g, cs, max_objects=n_obj + 16)
+    grid.ingest(upd)
+    po, pd, res = grid.prior_art_knn(q, k, rho=rho, threads=4)
+    ro, rd = oracle.knn_from_updates(g, upd, q, k)
+    bad = np.flatnonzero(~((po == ro).all(1) & (pd == rd).all(1)))
+    assert len(bad) == 0, f"{len(bad)} rows differ; first {bad[0]}: got {list(zip(pd[bad[0]], po[bad[0]]))} ref {list(zip(rd[bad[0]], ro[bad[0]]))}"
+    go, gd = grid.knn(q, k)
+    assert np.array_equal(go, po) and np.array_equal(gd, pd)
+    assert res["cells"] >= len(q) and res["bf_iterations"] >= len(q) and res["threads"] == 4
+    grid.close()
