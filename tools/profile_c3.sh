@@ -14,16 +14,19 @@ B="python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-parity --e2e-step
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_C3.csv \
     python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-parity --e2e-steps 1 > $OUT/launches_C3.log 2>&1
 echo "launch list rc=$?"
-cap() {  # name regex skip
-  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:$2 -s $3 -c 1 -o $OUT/$1 $B \
-      > $OUT/$1.log 2>&1
+cap() {  # name function-name-regex skip
+  timeout 1200 ncu --set full --clock-control none --import-source on --kernel-name-base function \
+      -k "regex:$2" -s $3 -c 1 -o $OUT/$1 $B > $OUT/$1.log 2>&1
   echo "$1 rc=$?"
 }
-cap expand_C3 k_expand_cta 3
-cap flush_C3 k_flush 1
-cap ingestscatter_C3 k_ingest_scatter 1
-cap ingestclassify_C3 k_ingest_classify 1
-cap stepscatter_C3 k_ingest_scatter 5
+# the starting expansion level at C3 is the one-warp-per-query kernel (k_expand); the 4th launch
+# is the first timed step's
+cap expand_C3 '^k_expand$' 3
+# flush launches 0-2 are the three full flushes of the 64M-record log (no GC: 2^28-record arena)
+cap flush_C3 '^k_flush' 1
+cap ingestscatter_C3 '^k_ingest_scatter$' 1
+cap ingestclassify_C3 '^k_ingest_classify$' 1
+cap stepscatter_C3 '^k_ingest_scatter$' 5
 for f in $OUT/*.ncu-rep; do
   ncu -i $f --page raw --csv > ${f%.ncu-rep}_raw.csv 2>/dev/null
   ncu -i $f --page source --csv > ${f%.ncu-rep}_source.csv 2>/dev/null
