@@ -56,14 +56,13 @@ struct WarpMem {
   uint32_t* front1;          // F
   uint32_t* fin;             // H/32: slot is in the frontier
   uint32_t* act;             // F: the round's active slots (the bucket being expanded)
-  uint8_t* listed;           // H: vertex expanded at least once (objects harvested); a vertex is
-                             //    in one round's active list at most once, so plain stores
+  uint32_t* listed;          // H/32 bits: vertex expanded at least once (objects harvested)
   uint2* stage;              // STAGE: the chunk's arcs (dst, D + w), compacted (one-warp variant)
 };
 constexpr uint32_t STAGE = 128;  // arcs of a chunk of 32 bucket vertices (4 inline slots each)
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 12ull * c.C + 4ull * (3ull * c.F + (c.H + 31) / 32) + ((c.H + 3) & ~3u) + 8ull * STAGE;
+  return 8ull * c.H + 12ull * c.C + 4ull * (3ull * c.F + 2ull * ((c.H + 31) / 32)) + 8ull * STAGE;
 }
 
 __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
@@ -78,7 +77,7 @@ __device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
   m.front1 = p; p += c.F;
   m.fin = p; p += (c.H + 31) / 32;
   m.act = p; p += c.F;
-  m.listed = reinterpret_cast<uint8_t*>(p);
+  m.listed = p;
   return m;
 }
 
@@ -273,7 +272,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
     m.dist[i] = INF;
   }
   for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) m.fin[i] = 0;
-  for (uint32_t i = lane; i < (cp.H + 3) / 4; i += 32) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
+  for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) m.listed[i] = 0;
   __syncwarp();
 
   const uint2 q = P.q[qi];
@@ -401,9 +400,8 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
         const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)u * 4);
         a01 = rec[0];
         a23 = rec[1];
-        harv = !m.listed[vslot];
+        harv = !(atomicOr(&m.listed[vslot >> 5], 1u << (vslot & 31)) & (1u << (vslot & 31)));
         if (harv) {
-          m.listed[vslot] = 1;
           hcell = cellof(g, u);
           hd = s.cell_head[hcell];
           cc = s.cell_comp[hcell];
@@ -552,8 +550,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
           w.hd = s.cell_head[w.hcell];
           w.cc = s.cell_comp[w.hcell];
           w.v0 = s.v_obj[w.u];
-          w.harv = !m.listed[w.vslot];
-          if (w.harv) m.listed[w.vslot] = 1;
+          w.harv = !(atomicOr(&m.listed[w.vslot >> 5], 1u << (w.vslot & 31)) & (1u << (w.vslot & 31)));
         }
       }
       return w;
@@ -800,7 +797,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
     m.dist[i] = INF;
   }
   for (uint32_t i = tid; i < (H + 31) / 32; i += T) m.fin[i] = 0;
-  for (uint32_t i = tid; i < (H + 3) / 4; i += T) reinterpret_cast<uint32_t*>(m.listed)[i] = 0;
+  for (uint32_t i = tid; i < (H + 31) / 32; i += T) m.listed[i] = 0;
   if (tid == 0) {
     sh.nn[0] = sh.nn[1] = sh.na[0] = sh.na[1] = 0;
     sh.stop[0] = sh.stop[1] = 0;
@@ -912,8 +909,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
           hd = s.cell_head[hcell];
           cc = s.cell_comp[hcell];
           v0 = s.v_obj[u];
-          harv = !m.listed[vslot];  // (one thread per active vertex per round)
-          if (harv) m.listed[vslot] = 1;
+          harv = !(atomicOr(&m.listed[vslot >> 5], 1u << (vslot & 31)) & (1u << (vslot & 31)));
         }
         auto relax = [&](uint32_t dst, uint32_t w) {
           ++c_arcs;
