@@ -611,15 +611,38 @@ __global__ void __launch_bounds__(TFT) k_flush_tma(DevGraph g, DevState s, Arena
       bulk_load(sm.key[st], s.ar.key + pos, n4 * 8u, &sm.full[st], policy);
       ++seq;
     };
-    uint32_t pc = s.flush_list[first_li];
+    // Software pipeline over the CTA's cells: while cell j's pieces are issued, cell j+1's chain
+    // head, cleaned list and first extent are already being loaded (each a dependent global round
+    // trip: without this the ring drains at every cell boundary)
+    struct Ext {
+      uint32_t a, l, nxt, tm;
+    };
+    auto load_ext = [&](uint32_t e) {
+      Ext x{0, 0, NONE, 0};
+      if (is_extent(e)) x = Ext{s.x_start[e], s.x_len[e], s.x_next[e], s.x_tmax[e]};
+      return x;
+    };
+    uint32_t c_cur = s.flush_list[first_li];
+    uint32_t h_cur = s.cell_head[c_cur];
+    uint2 comp_cur = s.cell_comp[c_cur];
+    Ext x_cur = load_ext(h_cur);
+    uint32_t c_nxt = n_mine > 1 ? s.flush_list[first_li + G] : 0;
     for (uint32_t j = 0; j < n_mine; ++j) {
       const uint32_t b = j % TSLOT;
+      const uint32_t c = c_cur, head = h_cur;
+      const uint2 comp = comp_cur;
+      const Ext x0 = x_cur;
+      // next cell's head and list, and the cell after's id
+      uint32_t h_nxt = NONE;
+      uint2 comp_nxt = make_uint2(0, 0);
+      uint32_t c_nn = 0;
+      if (j + 1 < n_mine) {
+        h_nxt = s.cell_head[c_nxt];
+        comp_nxt = s.cell_comp[c_nxt];
+        if (j + 2 < n_mine) c_nn = s.flush_list[first_li + (j + 2) * G];
+      }
       while (vgen[b] != j / TSLOT) __nanosleep(32);  // the slot's previous cell is indexed
       TSlot<WCAP>& sl = sm.slot[b];
-      const uint32_t c = pc;
-      const uint32_t head = s.cell_head[c];
-      const uint2 comp = s.cell_comp[c];
-      if (j + 1 < n_mine) pc = s.flush_list[first_li + (j + 1) * G];  // (one gather ahead)
       sl.c = c;
       sl.head = head;
       sl.comp = comp;
@@ -635,22 +658,25 @@ __global__ void __launch_bounds__(TFT) k_flush_tma(DevGraph g, DevState s, Arena
       // last are issued before the total is known; the total is added before the last segment's
       uint32_t xs[16], xl[16];
       uint32_t e = head;
+      bool first = true;
       unsigned long long issued = 0;
       unsigned long long nrec = 0, nexp = 0;
-      bool done = false;
+      bool done = false, prefetched = j + 1 >= n_mine;
+      Ext x_nxt{0, 0, NONE, 0};
       while (!done) {
         uint32_t nx = 0;
         while (is_extent(e) && nx < 16) {
-          const uint32_t a = s.x_start[e], l = s.x_len[e], nxt = s.x_next[e];
-          if (t_cut && s.x_tmax[e] < t_cut) {
-            nexp += l;
-          } else if (l) {
-            xs[nx] = a;
-            xl[nx] = l;
+          const Ext x = first ? x0 : load_ext(e);
+          first = false;
+          if (t_cut && x.tm < t_cut) {
+            nexp += x.l;
+          } else if (x.l) {
+            xs[nx] = x.a;
+            xl[nx] = x.l;
             ++nx;
-            nrec += l;
+            nrec += x.l;
           }
-          e = nxt;
+          e = x.nxt;
         }
         const bool last_seg = !is_extent(e);
         if (last_seg && comp.y && nx < 16) {
@@ -673,9 +699,21 @@ __global__ void __launch_bounds__(TFT) k_flush_tma(DevGraph g, DevState s, Arena
           if ((old & 0xFFFFFFFFull) == total) rq_push(&sm.rq_n, sm.rq, b);  // (all matched, or none)
         }
         for (uint32_t x = 0; x < nx; ++x)
-          for (uint32_t o = 0; o < xl[x]; o += TCHUNK) issue(b, xs[x] + o, min((uint32_t)TCHUNK, xl[x] - o));
+          for (uint32_t o = 0; o < xl[x]; o += TCHUNK) {
+            issue(b, xs[x] + o, min((uint32_t)TCHUNK, xl[x] - o));
+            if (!prefetched) {  // (after the first piece: the next head has had a round trip)
+              x_nxt = load_ext(h_nxt);
+              prefetched = true;
+            }
+          }
         issued += pieces;
       }
+      if (!prefetched) x_nxt = load_ext(h_nxt);  // (a cell with no pieces)
+      c_cur = c_nxt;
+      h_cur = h_nxt;
+      comp_cur = comp_nxt;
+      x_cur = x_nxt;
+      c_nxt = c_nn;
     }
     for (int w = 0; w < TMW; ++w) {  // one sentinel stage per match warp: no more pieces
       const uint32_t st = seq % TS, ph = (seq / TS) & 1u;

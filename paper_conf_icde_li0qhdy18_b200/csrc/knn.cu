@@ -709,7 +709,8 @@ __global__ void k_expand(QParams P) {
     if (lane == 0 && r != DONE) finish_undone(P, qi, r);
     __syncwarp();
   }
-  if (lane == 0) count_exit(P);
+  __syncthreads();  // (the chained level waits for every CTA -- all of its warps -- to exit)
+  if (threadIdx.x == 0) count_exit(P);
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -1174,6 +1175,13 @@ static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   return true;
 }
 
+// one-warp-per-query kernel: warps (independent queries) per CTA.  Each CTA costs 1 KB of reserved
+// shared memory beside its warps' tables, so several warps per CTA fit more queries per SM
+#ifndef GG_WARP_WPC
+#define GG_WARP_WPC 4
+#endif
+constexpr uint32_t WPC = GG_WARP_WPC;
+
 // resident CTAs per SM of a shared-memory level's kernel (occupancy calculator, cached)
 static uint32_t blocks_per_sm(int level, bool cta) {
   static int bps[2][NLEVELS] = {};  // (occupancy: the same on every B200)
@@ -1186,7 +1194,7 @@ static uint32_t blocks_per_sm(int level, bool cta) {
     if (cta) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, cta_kernel(level), cta_warps(level) * 32, smem);
     } else {
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32, smem);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32 * WPC, smem * WPC);
     }
 #ifdef GG_L0_PER_SM
     if (!cta && level == 0) b = std::min(b, GG_L0_PER_SM);  // experiment hook: occupancy cap
@@ -1198,7 +1206,9 @@ static uint32_t blocks_per_sm(int level, bool cta) {
 
 uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level == NLEVELS - 1) return 0;  // (global scratch: sized by the caller's scratch warps)
-  return std::min<uint32_t>(n, (uint32_t)sm_count * blocks_per_sm(level, use_cta(level, n, sm_count, ball_hint)));
+  const bool cta = use_cta(level, n, sm_count, ball_hint);
+  const uint32_t per = cta ? 1u : WPC;  // queries a CTA runs at once
+  return std::min<uint32_t>((n + per - 1) / per, (uint32_t)sm_count * blocks_per_sm(level, cta));
 }
 
 void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st) {
@@ -1222,7 +1232,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.bound = L.bound;
   P.remote = L.remote;
   P.caps = caps_for(level, g.V);
-  P.warps_per_cta = 1;
+  P.warps_per_cta = 1;  // (the one-warp shared-memory kernel: WPC, set below)
   P.scratch = nullptr;
   P.exited = L.exited;
   P.chain_in = const_cast<uint32_t*>(L.chain_in);
@@ -1242,8 +1252,9 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   blocks_per_sm(level, cta);  // (sets the shared-memory attribute)
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
-  cfg.blockDim = dim3(cta ? cta_warps(level) * 32 : 32);
-  cfg.dynamicSmemBytes = (size_t)smem;
+  if (!cta) P.warps_per_cta = WPC;
+  cfg.blockDim = dim3(cta ? cta_warps(level) * 32 : 32 * WPC);
+  cfg.dynamicSmemBytes = (size_t)smem * (cta ? 1 : WPC);
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;

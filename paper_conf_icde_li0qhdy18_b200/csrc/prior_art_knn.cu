@@ -21,6 +21,7 @@
 #include <chrono>
 #include <queue>
 #include <thread>
+#include <unordered_map>
 
 #include "handle.cuh"
 
@@ -210,6 +211,14 @@ __global__ void k_pa_lists(DevGraph g, DevState s, const uint32_t* __restrict__ 
     out[o++] = make_uint4(s.ar.obj[p], s.ar.vsrc[p], s.ar.off[p], 0);
   }
 }
+// the unresolved vertices of every query, compacted (offsets from the host)
+__global__ void k_pa_compact_unres(const uint2* __restrict__ unres, const PaQueryOut* __restrict__ qo,
+                                   const unsigned long long* __restrict__ off, uint32_t nq, uint2* __restrict__ out) {
+  const uint32_t i = blockIdx.x;
+  if (i >= nq) return;
+  const uint32_t n = qo[i].n_unres;
+  for (uint32_t j = threadIdx.x; j < n; j += blockDim.x) out[off[i] + j] = unres[(size_t)i * PA_UCAP + j];
+}
 __global__ void k_pa_list_counts(DevGraph g, DevState s, uint32_t* __restrict__ cnt) {
   const uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
   if (c <= g.n_cells) cnt[c] = c < g.n_cells ? s.cell_comp[c].y : 0;
@@ -309,13 +318,21 @@ extern "C" int ggrid_prior_art_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q
     r.bf_iterations += x.iters;
     if (x.flags) return fail(GGRID_ENOMEM);  // (a candidate or unresolved cap: not this tool's range)
   }
-  std::vector<uint2> hun((size_t)n_q * PA_UCAP);
-  // (only the used part of each query's segment)
-  for (uint32_t i = 0; i < n_q; ++i)
-    if (hq[i].n_unres)
-      CK(cudaMemcpyAsync(hun.data() + (size_t)i * PA_UCAP, dunres.as<uint2>() + (size_t)i * PA_UCAP,
-                         (size_t)hq[i].n_unres * 8, cudaMemcpyDeviceToHost, st));
-  CK(cudaStreamSynchronize(st));
+  // the unresolved lists, compacted on the device and copied once
+  std::vector<unsigned long long> uoff(n_q + 1, 0);
+  for (uint32_t i = 0; i < n_q; ++i) uoff[i + 1] = uoff[i] + hq[i].n_unres;
+  std::vector<uint2> hun(std::max<unsigned long long>(1, uoff[n_q]));
+  {
+    DBuf doff, dcomp;
+    if (doff.ensure((size_t)(n_q + 1) * 8) || dcomp.ensure(hun.size() * 8)) return fail(GGRID_ENOMEM);
+    CK(cudaMemcpyAsync(doff.p, uoff.data(), (size_t)(n_q + 1) * 8, cudaMemcpyHostToDevice, st));
+    k_pa_compact_unres<<<n_q, 128, 0, st>>>(dunres.as<uint2>(), dqout.as<PaQueryOut>(),
+                                            doff.as<unsigned long long>(), n_q, dcomp.as<uint2>());
+    if (uoff[n_q]) CK(cudaMemcpyAsync(hun.data(), dcomp.p, uoff[n_q] * 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    doff.release();
+    dcomp.release();
+  }
   auto t4 = clk::now();
   r.ms_d2h = ms(t3, t4);
   r.unresolved = n_unres;
@@ -324,8 +341,7 @@ extern "C" int ggrid_prior_art_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q
   std::atomic<uint32_t> next{0};
   std::atomic<uint64_t> settled{0};
   auto worker = [&] {
-    std::vector<uint64_t> dist((size_t)h->V, ~0ull);
-    std::vector<uint32_t> touched;
+    std::unordered_map<uint32_t, uint64_t> dist;  // (a bounded search touches a small ball)
     std::vector<std::pair<uint64_t, uint32_t>> best;
     uint64_t n_settled = 0;
     for (;;) {
@@ -338,12 +354,12 @@ extern "C" int ggrid_prior_art_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q
         if (c != ~0ull) best.push_back({c >> 32, (uint32_t)c});
       }
       for (uint32_t u = 0; u < hq[i].n_unres; ++u) {
-        const uint2 uv = hun[(size_t)i * PA_UCAP + u];
+        const uint2 uv = hun[uoff[i] + u];
         const uint64_t radius = l - uv.y;  // dist(v, .) <= l - dist(q, v)
         using Item = std::pair<uint64_t, uint32_t>;
         std::priority_queue<Item, std::vector<Item>, std::greater<Item>> pq;
+        dist.clear();
         dist[uv.x] = 0;
-        touched.push_back(uv.x);
         pq.push({0, uv.x});
         while (!pq.empty()) {
           const Item it = pq.top();
@@ -358,15 +374,14 @@ extern "C" int ggrid_prior_art_knn(ggrid_t h, const ggrid_query* q, uint32_t n_q
           for (uint32_t a = h->pa_rowptr[x]; a < h->pa_rowptr[x + 1]; ++a) {
             const uint2 arc = h->pa_adj[a];
             const uint64_t nd = it.first + arc.y;
-            if (nd <= radius && nd < dist[arc.x]) {
-              if (dist[arc.x] == ~0ull) touched.push_back(arc.x);
+            if (nd > radius) continue;
+            auto f = dist.find(arc.x);
+            if (f == dist.end() || nd < f->second) {
               dist[arc.x] = nd;
               pq.push({nd, arc.x});
             }
           }
         }
-        for (uint32_t t : touched) dist[t] = ~0ull;
-        touched.clear();
       }
       // per-object minimum (reading R14), then the first k by (dist, obj)
       std::sort(best.begin(), best.end(), [](const std::pair<uint64_t, uint32_t>& a, const std::pair<uint64_t, uint32_t>& b) {
