@@ -223,6 +223,7 @@ static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts
   // the expiry cut reads t_now on the host, so expiry keeps ingest synchronous
   h->async_ingest = (o.async_ingest && !o.t_delta) ? 1 : 0;
   h->fused_ingest = o.ingest_kernels == 3 ? 0 : 1;
+  if (const char* fk = getenv("GGRID_FLUSH_KERNEL")) h->flush_kernel = atoi(fk);  // (experiment hook)
   h->s.n_ranks = 1;
   h->s.rank = 0;
 
@@ -453,6 +454,7 @@ int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
     h->pend_updates += n;
     h->seq_next += n;
     h->n_ingested += n;
+    h->recs_since_flush += n;
     h->stats.n_updates = h->n_ingested;
     return GGRID_OK;
   }
@@ -475,6 +477,7 @@ int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   if (err & ERR_ARENA) return GGRID_ENOMEM;
   h->seq_next += n;
   h->n_ingested += n;
+  h->recs_since_flush += n;
   h->stats.n_updates = h->n_ingested;
   return GGRID_OK;
 }

@@ -486,9 +486,6 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
 //   index warp (warp 5)          builds R[c] of each matched cell (index_cell above) and frees its
 //                                slot for the producer.
 // Up to TSLOT cells are in flight per CTA.  The per-cell arithmetic is the one above.
-#ifndef GG_FLUSH_TMA
-#define GG_FLUSH_TMA 1
-#endif
 constexpr int TCHUNK = 256;  // records per stage (8 per match-warp lane)
 constexpr int TS = 8;        // stages
 constexpr int TSLOT = 4;     // cells in flight
@@ -797,16 +794,16 @@ __global__ void __launch_bounds__(TFT) k_flush_tma(DevGraph g, DevState s, Arena
 }
 
 template <int HCAP, int WCAP>
-int blocks_per_sm_t();
+int blocks_per_sm_t(bool tma);
 template <int HCAP, int WCAP>
 void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned long long* out_top,
               uint32_t begin, int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap,
-              uint32_t t_cut, uint32_t max_ctas, cudaStream_t st) {
-  const int blocks_per_sm = blocks_per_sm_t<HCAP, WCAP>();
+              uint32_t t_cut, uint32_t max_ctas, bool tma, cudaStream_t st) {
+  const int blocks_per_sm = blocks_per_sm_t<HCAP, WCAP>(tma);
   uint32_t grid = (uint32_t)(sm_count * blocks_per_sm);
   if (max_ctas && max_ctas < grid) grid = max_ctas;  // few cells to clean: fewer idle CTAs
   cudaLaunchAttribute attr[1];
-  if (GG_FLUSH_TMA) {
+  if (tma) {
     const cudaLaunchConfig_t cfg = pdl_config(dim3(grid), dim3(TFT), sizeof(TFlushSmem<HCAP, WCAP>), st, attr);
     cudaLaunchKernelEx(&cfg, k_flush_tma<HCAP, WCAP>, g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
     return;
@@ -815,24 +812,22 @@ void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned l
   cudaLaunchKernelEx(&cfg, k_flush<HCAP, WCAP>, g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
 }
 template <int HCAP, int WCAP>
-int blocks_per_sm_t() {
-  static int blocks_per_sm = 0;  // (occupancy: the same on every B200)
-  const int smem = GG_FLUSH_TMA ? (int)sizeof(TFlushSmem<HCAP, WCAP>) : (int)sizeof(FlushSmem<HCAP, WCAP>);
-  if (GG_FLUSH_TMA) func_attr_once(k_flush_tma<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+int blocks_per_sm_t(bool tma) {
+  static int bps[2] = {0, 0};  // (occupancy: the same on every B200)
+  int& blocks_per_sm = bps[tma ? 1 : 0];
+  const int smem = tma ? (int)sizeof(TFlushSmem<HCAP, WCAP>) : (int)sizeof(FlushSmem<HCAP, WCAP>);
+  if (tma) func_attr_once(k_flush_tma<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   else func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (blocks_per_sm == 0) {
     int b = 0;
-    if (GG_FLUSH_TMA) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush_tma<HCAP, WCAP>, TFT, smem);
+    if (tma) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush_tma<HCAP, WCAP>, TFT, smem);
     else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush<HCAP, WCAP>, FT, smem);
     blocks_per_sm = std::max(b, 1);
-#ifdef GG_FLUSH_TMA_CTAS
-    blocks_per_sm = std::min(blocks_per_sm, GG_FLUSH_TMA_CTAS);  // (experiment hook)
-#endif
   }
   // ask for no more shared memory than the resident CTAs need: the rest stays L1, which
   // holds the object-table lines the match phase gathers (per device, like the size above)
   const int carve = std::min(100, (blocks_per_sm * (smem + 1024) * 100 + 228 * 1024 - 1) / (228 * 1024));
-  if (GG_FLUSH_TMA) func_attr_once(k_flush_tma<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+  if (tma) func_attr_once(k_flush_tma<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
   else func_attr_once(k_flush<HCAP, WCAP>, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
   return blocks_per_sm;
 }
@@ -858,29 +853,35 @@ size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, u
   }
   *cap = want;
   if (!want) return 0;
-  int bps = 0;
-  switch (v) {
-    case 0: bps = blocks_per_sm_t<1024, 128>(); break;
-    case 1: bps = blocks_per_sm_t<4096, 128>(); break;
-    case 2: bps = blocks_per_sm_t<1024, 512>(); break;
-    case 3: bps = blocks_per_sm_t<4096, 512>(); break;
-    case 4: bps = blocks_per_sm_t<1024, 2048>(); break;
-    default: bps = blocks_per_sm_t<4096, 2048>(); break;
+  // (either kernel may run: room for the larger of their per-CTA spill areas)
+  size_t per_sm = 0;
+  for (int t = 0; t < 2; ++t) {
+    int bps = 0;
+    switch (v) {
+      case 0: bps = blocks_per_sm_t<1024, 128>(t); break;
+      case 1: bps = blocks_per_sm_t<4096, 128>(t); break;
+      case 2: bps = blocks_per_sm_t<1024, 512>(t); break;
+      case 3: bps = blocks_per_sm_t<4096, 512>(t); break;
+      case 4: bps = blocks_per_sm_t<1024, 2048>(t); break;
+      default: bps = blocks_per_sm_t<4096, 2048>(t); break;
+    }
+    per_sm = std::max(per_sm, (size_t)bps * (t ? TSLOT : NBUF));
   }
-  return (size_t)sm_count * bps * (NBUF > TSLOT ? NBUF : TSLOT) * want * sizeof(uint32_t);
+  return (size_t)sm_count * per_sm * want * sizeof(uint32_t);
 }
 
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
                   int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap, uint32_t t_cut,
-                  uint32_t max_ctas, cudaStream_t st) {
+                  uint32_t max_ctas, int tma, cudaStream_t st) {
+  const bool t = tma != 0;
   switch (flush_variant(g.cs, objects_per_cell)) {
-    case 0: launch_t<1024, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
-    case 1: launch_t<4096, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
-    case 2: launch_t<1024, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
-    case 3: launch_t<4096, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
-    case 4: launch_t<1024, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
-    default: launch_t<4096, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, st); break;
+    case 0: launch_t<1024, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;
+    case 1: launch_t<4096, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;
+    case 2: launch_t<1024, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;
+    case 3: launch_t<4096, 512>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;
+    case 4: launch_t<1024, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;
+    default: launch_t<4096, 2048>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;
   }
 }
 

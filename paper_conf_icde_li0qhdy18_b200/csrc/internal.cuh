@@ -257,10 +257,11 @@ void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int
 size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, uint32_t* cap);
 // t_cut: extents whose newest t is below it are expired (dropped unread); 0 = none.
 // max_ctas: an upper bound on the cells listed (0 = unknown): caps the persistent grid
+// tma: the bulk-copy ring kernel (k_flush_tma; long cell logs) instead of the streaming one
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
                   int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap, uint32_t t_cut,
-                  uint32_t max_ctas, cudaStream_t st);
+                  uint32_t max_ctas, int tma, cudaStream_t st);
 
 // v_obj[v] = (start, n) is valid only if start lies inside the cell's current cleaned list
 // (lists only move up the arena between garbage collections, which rewrite every entry).

@@ -1117,8 +1117,13 @@ __global__ void __launch_bounds__(W * 32, GG_MINB0) k_expand_cta_capped(QParams 
 // fewer than k objects may need to settle the whole graph).
 constexpr int NLEVELS = EXPAND_LEVELS;
 #ifndef GG_H0
-#define GG_H0 896  // level-0 vertex table (C3 one-warp: 1,024 -> 896 slots = more warps per SM,
-                   // 1.66 -> 1.54 ms; 768: 1.53 ms but promotions; experiment hook -DGG_H0=...)
+#define GG_H0 1024  // level-0 vertex table of the CTA-per-query kernel (experiment hook: -DGG_H0=...)
+#endif
+// ... and of the one-warp-per-query kernel (small expected balls, C3): fewer slots = more queries
+// resident per SM (with 4 warps per CTA: 1,024 -> 896 -> 768 slots = 18 -> 20 -> 24 warps per SM;
+// C3 expansion 1.66 -> 1.46 -> 1.37 ms, 7 promotions per 65,536 queries at 768)
+#ifndef GG_H0W
+#define GG_H0W 768
 #endif
 #ifndef GG_F0
 #define GG_F0 96
@@ -1143,7 +1148,7 @@ static CtaKernel cta_kernel(int level) {
 }
 
 Caps caps_for(int level, uint32_t V) {
-  if (level < NLEVELS - 1) return kCaps[level];
+  if (level < NLEVELS - 1) return kCaps[level];  // (level 0 one-warp mode: caps_mode below)
   uint32_t H = 1u << 15;
   while (H < 2ull * V && H < (1u << 27)) H <<= 1;
   const uint32_t F = std::min<uint32_t>(H / 2, 1u << 22);
@@ -1157,6 +1162,16 @@ int expand_levels() { return NLEVELS; }
 uint32_t expand_table_slots(int level) { return caps_for(level, 1).H; }
 
 uint32_t expand_max_k(int level) { return caps_for(level, 1).C - 32; }
+
+// the caps a level runs with in a given mode (the one-warp kernel's level 0 has its own table)
+static Caps caps_mode(int level, uint32_t V, bool cta) {
+  Caps c = caps_for(level, V);
+  if (level == 0 && !cta) c.H = GG_H0W;
+  return c;
+}
+static size_t warp_bytes_mode(int level, uint32_t V, bool cta) {
+  return (warpmem_bytes(caps_mode(level, V, cta)) + 15) & ~size_t(15);
+}
 
 size_t expand_warp_bytes(int level, uint32_t V) {
   const Caps c = caps_for(level, V);
@@ -1190,7 +1205,7 @@ static uint32_t blocks_per_sm(int level, bool cta) {
   else func_attr_once(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   int& b = bps[cta ? 1 : 0][level];
   if (!b) {
-    const int smem = (int)expand_warp_bytes(level, 1);
+    const int smem = (int)warp_bytes_mode(level, 1, cta);
     if (cta) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, cta_kernel(level), cta_warps(level) * 32, smem);
     } else {
@@ -1231,7 +1246,8 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.out_dist = L.out_dist;
   P.bound = L.bound;
   P.remote = L.remote;
-  P.caps = caps_for(level, g.V);
+  const bool cta_mode = level < NLEVELS - 1 && (L.chain_in != nullptr || use_cta(level, L.n, sm_count, L.ball_hint));
+  P.caps = caps_mode(level, g.V, cta_mode);
   P.warps_per_cta = 1;  // (the one-warp shared-memory kernel: WPC, set below)
   P.scratch = nullptr;
   P.exited = L.exited;
@@ -1241,7 +1257,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.wait_total = L.wait_total;
   P.trigger = L.trigger ? 1 : 0;
   P.wait_prior = L.chain_in ? 0 : 1;  // (a chained level runs beside the level below it)
-  const int smem = (int)expand_warp_bytes(level, g.V);
+  const int smem = (int)warp_bytes_mode(level, g.V, cta_mode);
   if (level == NLEVELS - 1) {
     P.scratch = static_cast<unsigned char*>(L.scratch);
     k_expand<false><<<std::min<uint32_t>(L.n, std::max<uint32_t>(1, L.scratch_warps)), 32, 0, st>>>(P);

@@ -79,10 +79,13 @@ def test_c0_interleaved_rounds_lazy_equals_eager(gg):
     eager.close()
 
 
-def test_flush_parity_and_cells(gg):
+@pytest.mark.parametrize("kernel", ["auto", "ring", "streaming"])
+def test_flush_parity_and_cells(gg, kernel, monkeypatch):
     """After ggrid_flush_all the cells' object lists are exactly the oracle's latest-per-object
     snapshot, each object once, in the cell of its arc's source vertex; flushing twice is a
-    no-op (idempotent)."""
+    no-op (idempotent).  Both flush kernels (the bulk-copy ring and the streaming one; GGRID_FLUSH_KERNEL
+    forces one, `auto` picks by log length per cell)."""
+    monkeypatch.setenv("GGRID_FLUSH_KERNEL", {"auto": "0", "ring": "1", "streaming": "2"}[kernel])
     g = synth.table_ii_graph("NY", scale=0.05)
     upd = synth.RandomWalk(g, 2000, inject=True).ticks(12)
     grid = gg.GGrid(g, 256, max_objects=4096)
@@ -597,4 +600,23 @@ def test_moved_objects_leave_clean_cells_stale(gg):
         grid.ingest(u)
         q = synth.queries(g, 150, seed=600 + r)
         _assert_same(grid.knn(q, 7), _oracle(g, np.concatenate(hist), q, 7), f"round {r}")
+    grid.close()
+
+
+@pytest.mark.parametrize("kernel", ["1", "2"])
+def test_flush_kernels_interleaved_rounds(gg, kernel, monkeypatch):
+    """Interleaved ingest / query rounds with either flush kernel forced (long chains of small
+    extents, STALE cells, cleaned lists re-read): every round the oracle's answer."""
+    monkeypatch.setenv("GGRID_FLUSH_KERNEL", kernel)
+    g = synth.table_ii_graph("NY", scale=0.05)
+    walk = synth.RandomWalk(g, 3000, inject=True)
+    grid = gg.GGrid(g, 64, max_objects=3000)
+    hist = []
+    for r in range(6):
+        for _ in range(3):
+            u = walk.ticks(2)
+            hist.append(u)
+            grid.ingest(u)
+        q = synth.queries(g, 200, seed=900 + r)
+        _assert_same(grid.knn(q, 8), _oracle(g, np.concatenate(hist), q, 8), f"kernel {kernel} round {r}")
     grid.close()
