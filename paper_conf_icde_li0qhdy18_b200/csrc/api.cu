@@ -352,6 +352,7 @@ static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts
   if (cudaMemset(s.listed_cell, 0xFF, (size_t)o.max_objects * 4)) return fail(GGRID_ECUDA);
   if ((rc = h->alloc(&s.cell_req, h->n_cells))) return fail(rc);
   if ((rc = h->alloc(&s.v_obj, V))) return fail(rc);
+  if ((rc = h->alloc(&s.vhas, (size_t)V / 32 + 2))) return fail(rc);
   if ((rc = h->alloc(&s.cell_comp, h->n_cells))) return fail(rc);
   s.vcnt = nullptr;
   if (cell_size > 4096 && (rc = h->alloc(&s.vcnt, V))) return fail(rc);

@@ -362,8 +362,9 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   uint32_t* h_aux = f_buf + 2 * ch;  // [ch] newest t; then the cell's batch rank base; then the
                                      //      arena position of the group's first record minus its
                                      //      tile offset
-  uint4* srec = reinterpret_cast<uint4*>(f_buf + 3 * ch);   // [tile] the records, tile order
-  uint2* stg = reinterpret_cast<uint2*>(srec + tile);       // [tile] (src vertex, slot | flags),
+  // (the tile's records are not staged: the scatter re-reads them from L2 -- the batch was just
+  // read -- which leaves shared memory to a hash of >= one slot per update of the tile)
+  uint2* stg = reinterpret_cast<uint2*>(f_buf + 3 * ch);    // [tile] (src vertex, slot | flags),
                                                             //        cell order
   uint16_t* stp = reinterpret_cast<uint16_t*>(stg + tile);  // [tile] tile index, cell order
   uint32_t* w_sum = reinterpret_cast<uint32_t*>(stp + ((tile + 1) & ~1u));  // [FT / 32]
@@ -397,7 +398,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
 #pragma unroll
     for (int q = 0; q < HP; ++q) {
       const uint32_t k = (uint32_t)((hf * HP + q) * FT + tid);
-      mm[q] = k < nt ? __ldcs(upd + base + k) : make_uint4(0, 0xFFFFFFFFu, 0, 0);
+      mm[q] = k < nt ? __ldg(upd + base + k) : make_uint4(0, 0xFFFFFFFFu, 0, 0);  // (kept in L2: re-read)
     }
 #pragma unroll
     for (int q = 0; q < HP; ++q) {
@@ -413,7 +414,6 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
       if (k >= nt) continue;
       const uint4 m = mm[q];
       const uint2 e = ee[q];
-      srec[k] = m;
       unsigned bad = 0;
       if (m.x >= s.max_objects) bad |= ERR_OBJ;
       if (m.y >= g.A) {
@@ -515,7 +515,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   for (uint32_t si = tid; si < nt; si += FT) {
     const uint2 x = stg[si];
     const uint32_t k = stp[si];
-    const uint4 m = srec[k];
+    const uint4 m = __ldg(upd + base + k);
     const uint32_t slot = x.y & 0xFFFFu, f = x.y >> 16;
     const unsigned long long key =
         ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)(base + k));
@@ -541,7 +541,7 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
 }
 
 static size_t fused_smem(uint32_t tile, uint32_t ch) {
-  return (size_t)ch * 12 + (size_t)tile * 24 + (size_t)((tile + 1) & ~1u) * 2 + (FT / 32) * 4;
+  return (size_t)ch * 12 + (size_t)tile * 8 + (size_t)((tile + 1) & ~1u) * 2 + (FT / 32) * 4;
 }
 
 bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p) {
@@ -549,9 +549,16 @@ bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p
   const uint64_t grid = std::min<uint64_t>((uint64_t)sm_count, std::max<uint64_t>(1, (n + 2047) / 2048));
   const uint64_t tile = (n + grid - 1) / grid;
   if (tile > FUSED_TILE) return false;
-  const uint64_t want = 2 * std::min<uint64_t>(tile, (uint64_t)n_cells + 1);
+  // cell-hash slots: >= 2 per distinct cell of a tile when that fits, else >= one more than the
+  // tile's updates (never full: at most one distinct cell per update; C3's 1M-update step, 6,757
+  // updates per tile over 23k cells, takes 8,192 slots)
+  const uint64_t m = std::min<uint64_t>(tile, (uint64_t)n_cells + 1);
   uint32_t ch = FT;
-  while (ch < want) ch <<= 1;
+  while (ch < 2 * m) ch <<= 1;
+  if (ch > FUSED_CH_MAX || fused_smem((uint32_t)tile, ch) > 227 * 1024) {
+    ch = FT;
+    while (ch < m + 1) ch <<= 1;
+  }
   if (ch > FUSED_CH_MAX) return false;
   const size_t smem = fused_smem((uint32_t)tile, ch);
   if (smem > 227 * 1024) return false;

@@ -102,6 +102,9 @@ struct DevState {
   uint32_t* cell_pending;  // cached records not yet cleaned
   uint32_t* cell_req;      // request epoch stamp (dedup of flush requests)
   uint2* v_obj;            // [V] (arena start, count) of the objects at each vertex
+  uint32_t* vhas;          // [V/32 + 1] bit v: v may hold objects in its cell's cleaned list (a
+                           // superset, rebuilt per cell by the flush): the query reads v_obj only
+                           // for these (L2-resident: 3 MB at USA scale)
   uint2* cell_comp;        // [n_cells] (arena start, count) of the cell's compacted list
   uint32_t* vcnt;          // [V] flush scratch, only when cell_size > 4096 (else null)
   uint32_t* bcount;        // [n_cells * BCOUNT_STRIDE] per-batch count ([0]) and newest t ([1]),
@@ -265,6 +268,7 @@ void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
 
 // v_obj[v] = (start, n) is valid only if start lies inside the cell's current cleaned list
 // (lists only move up the arena between garbage collections, which rewrite every entry).
+__device__ __forceinline__ bool vhas_bit(const DevState& s, uint32_t v) { return (s.vhas[v >> 5] >> (v & 31)) & 1u; }
 __device__ __forceinline__ uint2 vobj_valid(uint2 vo, uint2 comp) {
   return (vo.x >= comp.x && vo.x < comp.x + comp.y) ? vo : make_uint2(0, 0);
 }
