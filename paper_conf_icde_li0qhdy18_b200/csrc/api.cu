@@ -388,7 +388,7 @@ int ggrid_free(ggrid_t h) {
   for (DBuf* b : {&h->upd_stage, &h->tmp, &h->q_stage, &h->out_stage, &h->lists, &h->l2_scratch,
                   &h->dump_stage, &h->gc_buf, &h->misc, &h->flush_spill, &h->bound_stage,
                   &h->remote_stage, &h->merge_stage, &h->staged[0].buf,
-                  &h->staged[1].buf, &h->qstaged[0].buf, &h->qstaged[1].buf, &h->chain_ring})
+                  &h->staged[1].buf, &h->qstaged[0].buf, &h->qstaged[1].buf, &h->chain_ring, &h->qsort_buf})
     b->release();
   for (ggrid_s::Staged* sb : {&h->staged[0], &h->staged[1], &h->qstaged[0], &h->qstaged[1]}) {
     if (sb->done) cudaEventDestroy(sb->done);
@@ -661,6 +661,16 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
     }
   }
   std::vector<const uint32_t*> in_list(L, nullptr);
+  // (experiment hook) the starting level takes the queries in the order of their arcs' source
+  // vertices (Z-order ids): spatially close queries run close in time and share L2 lines
+  if (getenv("GGRID_SORT_QUERIES") && n_q >= 4096) {
+    const size_t tb = sort_queries_tmp_bytes(n_q);
+    RC(h->qsort_buf.ensure(tb + (size_t)n_q * 16 + 64));
+    unsigned char* base = h->qsort_buf.as<unsigned char>();
+    uint32_t* perm = reinterpret_cast<uint32_t*>(base + tb);
+    if (launch_sort_queries(d_q, n_q, g, base, tb, perm, st) != 0) return GGRID_ECUDA;
+    in_list[lvl0] = perm;
+  }
   int cur = 0;
   uint32_t flush_begin = 0;
   for (int round = 0;; ++round) {

@@ -240,9 +240,9 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
     return;  // the cell stays dirty
   }
   const uint32_t ob0 = (uint32_t)o0;
-  // the cell's "may hold objects" bits: cleared, then set below for the vertices of the new list
+  // (GG_VHAS) the cell's "may hold objects" bits: cleared, then set below for the new list
   // (boundary words shared with a neighbouring cell: masked atomics)
-  for (uint32_t wd = (cbeg >> 5) + lane; wd <= ((cbeg + nvert - 1) >> 5); wd += 32) {
+  for (uint32_t wd = (cbeg >> 5) + lane; GG_VHAS && wd <= ((cbeg + nvert - 1) >> 5); wd += 32) {
     const uint32_t lo = max(cbeg, wd << 5), hi = min(cbeg + nvert, (wd << 5) + 32);
     const uint32_t span = hi - lo;
     const uint32_t mask = (span == 32 ? 0xFFFFFFFFu : ((1u << span) - 1u)) << (lo & 31);
@@ -272,7 +272,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
       out.edge[q] = sm.w_edge[i];
       if (first) {
         s.v_obj[vi] = make_uint2(q, cv);
-        atomicOr(&s.vhas[vi >> 5], 1u << (vi & 31));
+        if (GG_VHAS) atomicOr(&s.vhas[vi >> 5], 1u << (vi & 31));
       }
     }
   } else {
@@ -323,7 +323,7 @@ __device__ void index_cell(SM& sm, B& bf, const DevGraph& g, const DevState& s, 
       const uint32_t b = cnt[i];
       const uint32_t en = (i + 1 < nvert) ? cnt[i + 1] : n_win;
       if (full_vobj || en != b) s.v_obj[cbeg + i] = make_uint2(ob0 + b, en - b);
-      if (en != b) atomicOr(&s.vhas[(cbeg + i) >> 5], 1u << ((cbeg + i) & 31));
+      if (GG_VHAS && en != b) atomicOr(&s.vhas[(cbeg + i) >> 5], 1u << ((cbeg + i) & 31));
     }
     __syncwarp();
     if (spilled) {

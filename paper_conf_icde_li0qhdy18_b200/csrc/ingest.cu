@@ -540,6 +540,12 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   }
 }
 
+// a tile whose 2-slots-per-cell hash does not fit shared memory: fused with a hash of one slot
+// per update (1) or the three-launch path (0; measured faster at C3's 1M-update step, r2i: 0.144
+// vs 0.170 ms -- probe chains at 82% load)
+#ifndef GG_FUSED_TIGHT
+#define GG_FUSED_TIGHT 0
+#endif
 static size_t fused_smem(uint32_t tile, uint32_t ch) {
   return (size_t)ch * 12 + (size_t)tile * 8 + (size_t)((tile + 1) & ~1u) * 2 + (FT / 32) * 4;
 }
@@ -555,7 +561,7 @@ bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p
   const uint64_t m = std::min<uint64_t>(tile, (uint64_t)n_cells + 1);
   uint32_t ch = FT;
   while (ch < 2 * m) ch <<= 1;
-  if (ch > FUSED_CH_MAX || fused_smem((uint32_t)tile, ch) > 227 * 1024) {
+  if (GG_FUSED_TIGHT && (ch > FUSED_CH_MAX || fused_smem((uint32_t)tile, ch) > 227 * 1024)) {
     ch = FT;
     while (ch < m + 1) ch <<= 1;
   }

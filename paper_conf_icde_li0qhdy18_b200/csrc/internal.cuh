@@ -268,6 +268,14 @@ void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
 
 // v_obj[v] = (start, n) is valid only if start lies inside the cell's current cleaned list
 // (lists only move up the arena between garbage collections, which rewrite every entry).
+// (experiment hook) GG_VHAS=1: the flush maintains the may-hold-objects bitmap and the query reads a
+// vertex's object index only when its bit is set.  Measured slower at C3 (r2i: expansion 1.367 ->
+// 1.424 ms -- the index read becomes a second dependent trip for the vertices that hold objects --
+// and the step's flush 0.127 -> 0.154 ms for the bitmap upkeep), so off: the index is read in the
+// same round trip as the vertex's arcs.
+#ifndef GG_VHAS
+#define GG_VHAS 0
+#endif
 __device__ __forceinline__ bool vhas_bit(const DevState& s, uint32_t v) { return (s.vhas[v >> 5] >> (v & 31)) & 1u; }
 __device__ __forceinline__ uint2 vobj_valid(uint2 vo, uint2 comp) {
   return (vo.x >= comp.x && vo.x < comp.x + comp.y) ? vo : make_uint2(0, 0);
@@ -324,6 +332,10 @@ void launch_pa_collect(const DevState& s, uint32_t max_objects, uint32_t n_bundl
                        uint32_t* out_edge, uint32_t* out_off, unsigned long long* counts, cudaStream_t st);
 void launch_pa_bundle(const uint32_t* obj, const unsigned long long* key, int eta, uint32_t* out_obj,
                       unsigned long long* out_key, cudaStream_t st);
+// queries ordered by their arcs' internal source vertex (cub radix sort): perm[i] = query index
+size_t sort_queries_tmp_bytes(uint32_t n);
+int launch_sort_queries(const uint2* q, uint32_t n, const DevGraph& g, void* tmp, size_t tmp_bytes, uint32_t* perm,
+                        cudaStream_t st);
 int expand_levels();
 uint32_t expand_table_slots(int level);  // vertex-table capacity H of a level
 uint32_t expand_max_k(int level);

@@ -101,6 +101,7 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 __device__ __forceinline__ void prefetch_vertex(const DevGraph& g, const DevState& s, uint32_t v) {
   if (GG_PREFETCH) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(g.vadj + (size_t)v * 4));
+    if (!GG_VHAS) asm volatile("prefetch.global.L2 [%0];" ::"l"(s.v_obj + v));
   }
 }
 
@@ -404,7 +405,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
           hcell = cellof(g, u);
           hd = s.cell_head[hcell];
           cc = s.cell_comp[hcell];
-          if (vhas_bit(s, u)) v0 = s.v_obj[u];  // (most vertices hold no object: no index read)
+          if (!GG_VHAS || vhas_bit(s, u)) v0 = s.v_obj[u];  // (GG_VHAS: most vertices hold no object)
         }
       }
       const bool overflow_arcs = a23.w == WMAX;  // more than 4 arcs: 3 inline, the rest in the CSR
@@ -548,7 +549,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
           w.hcell = cellof(g, w.u);
           w.hd = s.cell_head[w.hcell];
           w.cc = s.cell_comp[w.hcell];
-          if (vhas_bit(s, w.u)) w.v0 = s.v_obj[w.u];
+          if (!GG_VHAS || vhas_bit(s, w.u)) w.v0 = s.v_obj[w.u];
           w.harv = !(atomicOr(&m.listed[w.vslot >> 5], 1u << (w.vslot & 31)) & (1u << (w.vslot & 31)));
         }
       }
@@ -908,7 +909,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
           hcell = cellof(g, u);
           hd = s.cell_head[hcell];
           cc = s.cell_comp[hcell];
-          if (vhas_bit(s, u)) v0 = s.v_obj[u];
+          if (!GG_VHAS || vhas_bit(s, u)) v0 = s.v_obj[u];
           harv = !(atomicOr(&m.listed[vslot >> 5], 1u << (vslot & 31)) & (1u << (vslot & 31)));
         }
         auto relax = [&](uint32_t dst, uint32_t w) {

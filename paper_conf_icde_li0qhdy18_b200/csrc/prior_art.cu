@@ -20,6 +20,7 @@
 //     counts those objects (objects_wrong) against the object table.
 // T has one entry per (object, bundle): max_objects x bundles x 16 B — the reason this design
 // cannot be run at USA scale (the comparison tool reports it).
+#include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 
 #include "internal.cuh"
@@ -234,4 +235,39 @@ void launch_pa_bundle(const uint32_t* obj, const unsigned long long* key, int et
   k_pa_bundle<<<1, 32, 0, st>>>(obj, key, eta, out_obj, out_key);
 }
 
+}  // namespace gg
+
+namespace gg {
+namespace {
+__global__ void k_query_keys(const uint2* __restrict__ q, uint32_t n, DevGraph g, uint32_t* __restrict__ key,
+                             uint32_t* __restrict__ idx) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t e = q[i].x;
+  key[i] = e < g.A ? g.einfo[e].x : 0u;
+  idx[i] = i;
+}
+}  // namespace
+// layout of tmp: [cub temp | keys in | keys out | idx in] ; perm = idx out
+size_t sort_queries_tmp_bytes(uint32_t n) {
+  size_t t = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, t, (const uint32_t*)nullptr, (uint32_t*)nullptr, (const uint32_t*)nullptr,
+                                  (uint32_t*)nullptr, (int)n);
+  return ((t + 255) & ~size_t(255)) + 3 * (((size_t)n * 4 + 255) & ~size_t(255));
+}
+int launch_sort_queries(const uint2* q, uint32_t n, const DevGraph& g, void* tmp, size_t tmp_bytes, uint32_t* perm,
+                        cudaStream_t st) {
+  size_t t = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, t, (const uint32_t*)nullptr, (uint32_t*)nullptr, (const uint32_t*)nullptr,
+                                  (uint32_t*)nullptr, (int)n);
+  const size_t ta = (t + 255) & ~size_t(255), na = ((size_t)n * 4 + 255) & ~size_t(255);
+  unsigned char* b = static_cast<unsigned char*>(tmp);
+  uint32_t* kin = reinterpret_cast<uint32_t*>(b + ta);
+  uint32_t* kout = reinterpret_cast<uint32_t*>(b + ta + na);
+  uint32_t* iin = reinterpret_cast<uint32_t*>(b + ta + 2 * na);
+  k_query_keys<<<(n + 255) / 256, 256, 0, st>>>(q, n, g, kin, iin);
+  int bits = 1;
+  while (bits < 32 && (1ull << bits) < g.V) ++bits;
+  return cub::DeviceRadixSort::SortPairs(b, t, kin, kout, iin, perm, (int)n, 0, bits, st) == cudaSuccess ? 0 : 1;
+}
 }  // namespace gg
