@@ -499,10 +499,19 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
 //   index warp (warp 5)          builds R[c] of each matched cell (index_cell above) and frees its
 //                                slot for the producer.
 // Up to TSLOT cells are in flight per CTA.  The per-cell arithmetic is the one above.
-constexpr int TCHUNK = 256;  // records per stage (8 per match-warp lane)
-constexpr int TS = 8;        // stages
-constexpr int TSLOT = 4;     // cells in flight
-constexpr int TMW = 4;       // match warps
+#ifndef GG_TCHUNK
+#define GG_TCHUNK 256
+#endif
+#ifndef GG_TS
+#define GG_TS 8
+#endif
+#ifndef GG_TMW
+#define GG_TMW 4
+#endif
+constexpr int TCHUNK = GG_TCHUNK;  // records per stage (8 per match-warp lane)
+constexpr int TS = GG_TS;          // stages
+constexpr int TSLOT = 4;           // cells in flight
+constexpr int TMW = GG_TMW;        // match warps
 constexpr int TFT = (TMW + 2) * 32;
 
 template <int WCAP>
