@@ -581,7 +581,10 @@ __device__ __forceinline__ void rq_push(uint32_t* rq_n, uint32_t* rq, uint32_t b
 }
 
 template <int HCAP, int WCAP>
-__global__ void __launch_bounds__(TFT) k_flush_tma(DevGraph g, DevState s, Arena out, unsigned long long* out_top,
+#ifndef GG_TMA_MINB
+#define GG_TMA_MINB 1
+#endif
+__global__ void __launch_bounds__(TFT, GG_TMA_MINB) k_flush_tma(DevGraph g, DevState s, Arena out, unsigned long long* out_top,
                                                    uint32_t begin, int full_vobj, uint32_t* spill, uint32_t spill_cap,
                                                    uint32_t t_cut) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
