@@ -512,6 +512,10 @@ constexpr int TCHUNK = GG_TCHUNK;  // records per stage (8 per match-warp lane)
 constexpr int TS = GG_TS;          // stages
 constexpr int TSLOT = 4;           // cells in flight
 constexpr int TMW = GG_TMW;        // match warps
+// each stage must always be consumed by the same match warp (stage s: sequence numbers s, s + TS,
+// ... go to warp s % TMW): a warp waiting on a phase two ahead of its stage's barrier would read
+// the parity of an older phase as complete
+static_assert(TS % TMW == 0, "stages must be a multiple of the match warps");
 constexpr int TFT = (TMW + 2) * 32;
 
 template <int WCAP>
