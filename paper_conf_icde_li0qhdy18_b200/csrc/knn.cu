@@ -90,6 +90,9 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 // A vertex entering the frontier will be expanded in a later round: its inline adjacency record
 // and object index are fetched into L2 now, so the expansion's dependent load hits L2 instead of
 // DRAM (the USA-shaped graph's 0.9 GB of per-vertex records is far beyond L2).
+#ifndef GG_PREFETCH_VOBJ
+#define GG_PREFETCH_VOBJ 1
+#endif
 #ifndef GG_PREFETCH
 #define GG_PREFETCH 1  // (C3: expansion 1.75 -> 1.66 ms per 65,536 queries, r2b variants)
 #endif
@@ -101,7 +104,7 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 __device__ __forceinline__ void prefetch_vertex(const DevGraph& g, const DevState& s, uint32_t v) {
   if (GG_PREFETCH) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(g.vadj + (size_t)v * 4));
-    if (!GG_VHAS) asm volatile("prefetch.global.L2 [%0];" ::"l"(s.v_obj + v));
+    if (!GG_VHAS && GG_PREFETCH_VOBJ) asm volatile("prefetch.global.L2 [%0];" ::"l"(s.v_obj + v));
   }
 }
 
@@ -410,7 +413,9 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
       }
       const bool overflow_arcs = a23.w == WMAX;  // more than 4 arcs: 3 inline, the rest in the CSR
       // compact the real arcs (w != 0) of the chunk: (dst, du + w), skipping sums >= INF
-      auto real = [&](uint32_t w) { return w != 0 && w != WMAX && (unsigned long long)du + w < INF; };
+      // a real arc (1 <= w < WMAX) whose sum stays below INF (du < INF: a bucket vertex); 32-bit
+      const uint32_t room = INF - du;
+      auto real = [&](uint32_t w) { return (w - 1u < WMAX - 1u) & (w < room); };
       const uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
       const uint32_t cnt = r0 + r1 + r2 + r3;
       uint32_t pre = cnt;
@@ -710,6 +715,433 @@ __global__ void k_expand(QParams P) {
     __syncwarp();
   }
   __syncthreads();  // (the chained level waits for every CTA -- all of its warps -- to exit)
+  if (threadIdx.x == 0) count_exit(P);
+}
+
+// ---------------------------------------------------------------------------------------------
+// Paired variant of the one-warp kernel (GG_PAIR): each half-warp (16 lanes) runs its own query
+// with its own shared-memory table, and the two halves execute every phase of a round -- the
+// termination test, the frontier partition, the chunk load + arc compaction, the relax passes and
+// the harvest -- in the same instructions, each on its own data (loop bounds are the larger of
+// the two halves'; half-warp ballots, shuffles and reductions).  A round's bucket (~14 vertices at
+// C3) and its arcs (~34) fill 16-lane passes far better than 32-lane ones, so a query costs fewer
+// warp instructions; the queries resident per SM are the same (shared memory per query).  A half
+// whose query ends fetches the next one while the other continues.  Same arithmetic and outcome
+// rules as run_query (DONE / RETRY / OVERFLOW).
+#ifndef GG_PAIR
+#define GG_PAIR 0
+#endif
+
+struct HalfWarp {
+  uint32_t h, hl, base;
+  unsigned mask, lt;
+};
+__device__ __forceinline__ uint32_t hsum(const HalfWarp& W, uint32_t x) {
+#pragma unroll
+  for (int o = 8; o > 0; o >>= 1) x += __shfl_xor_sync(W.mask, x, o);
+  return x;
+}
+__device__ __forceinline__ uint32_t hmin(const HalfWarp& W, uint32_t x) {
+#pragma unroll
+  for (int o = 8; o > 0; o >>= 1) x = min(x, __shfl_xor_sync(W.mask, x, o));
+  return x;
+}
+__device__ __forceinline__ uint32_t hmax(const HalfWarp& W, uint32_t x) {
+#pragma unroll
+  for (int o = 8; o > 0; o >>= 1) x = max(x, __shfl_xor_sync(W.mask, x, o));
+  return x;
+}
+__device__ __forceinline__ uint32_t hor(const HalfWarp& W, uint32_t x) {
+#pragma unroll
+  for (int o = 8; o > 0; o >>= 1) x |= __shfl_xor_sync(W.mask, x, o);
+  return x;
+}
+// the larger of the two halves' (half-uniform) values: the shared loop bound of a phase
+__device__ __forceinline__ uint32_t both_max(uint32_t v) { return max(v, __shfl_xor_sync(0xffffffffu, v, 16)); }
+
+__device__ __forceinline__ bool cand_push16(const WarpMem& m, const HalfWarp& W, uint32_t& nc, uint32_t C, bool has,
+                                            uint32_t slot, uint32_t off, uint32_t obj) {
+  const unsigned hm = __ballot_sync(W.mask, has) & W.mask;
+  if (!hm) return true;
+  if (nc + __popc(hm) > C) return false;
+  if (has) {
+    const uint32_t i = nc + __popc(hm & W.lt);
+    m.cand[i] = ((unsigned long long)slot << 32) | off;
+    m.cobj[i] = obj;
+  }
+  nc += __popc(hm);
+  return true;
+}
+
+__device__ void half_sort(unsigned long long* a, uint32_t n, uint32_t cap, const HalfWarp& W) {
+  uint32_t n2 = 1;
+  while (n2 < n) n2 <<= 1;
+  if (n2 > cap) n2 = cap;
+  for (uint32_t i = n + W.hl; i < n2; i += 16) a[i] = EMPTY64;
+  __syncwarp(W.mask);
+  for (uint32_t size = 2; size <= n2; size <<= 1) {
+    for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+      for (uint32_t i = W.hl; i < n2 / 2; i += 16) {
+        const uint32_t lo = 2 * i - (i & (stride - 1));
+        const uint32_t hi = lo + stride;
+        const bool asc = (lo & size) == 0;
+        const unsigned long long x = a[lo], y = a[hi];
+        if ((x > y) == asc) {
+          a[lo] = y;
+          a[hi] = x;
+        }
+      }
+      __syncwarp(W.mask);
+    }
+  }
+}
+
+__global__ void k_expand_pair(QParams P) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const DevGraph& g = P.g;
+  const DevState& s = P.s;
+  const Caps cp = P.caps;
+  const uint32_t H = cp.H, k = P.k;
+  const int lane = threadIdx.x & 31;
+  const uint32_t warp = threadIdx.x >> 5;
+  HalfWarp W;
+  W.h = (uint32_t)lane >> 4;
+  W.hl = (uint32_t)lane & 15u;
+  W.base = W.h * 16;
+  W.mask = 0xFFFFu << W.base;
+  W.lt = lanemask_lt() & W.mask;
+  const size_t wbytes = (warpmem_bytes(cp) + 15) & ~size_t(15);
+  const WarpMem m = carve(smem_raw + (size_t)(2 * warp + W.h) * wbytes, cp);
+  pdl_trigger(P);
+  const bool track = P.remote != nullptr && s.n_ranks > 1;
+
+  // per-half (half-uniform) query state
+  uint32_t qi = NONE;
+  bool need = true, exhausted = false;
+  uint2 q = make_uint2(0, 0), ei = make_uint2(0, 0);
+  uint32_t lim = INF, nf = 0, nc = 0, blo = 0, fb = 0;
+  unsigned long long rmask = 0;
+  uint32_t c_iter = 0, c_vert = 0, c_arcs = 0, c_harv = 0, c_objs = 0;
+  int outcome = -1;  // set when the query ends (DONE / RETRY / OVERFLOW)
+
+  auto finish = [&](int r) {  // (half-divergent) write the answer or queue the query; fetch next
+    if (r == DONE && qi != NONE) {
+      for (uint32_t i = W.hl; i < nc; i += 16) {
+        const unsigned long long d = cand_dist(m, i);
+        m.cand[i] = d < INF ? ((d << 32) | m.cobj[i]) : EMPTY64;
+      }
+      __syncwarp(W.mask);
+      half_sort(m.cand, nc, cp.C, W);
+      for (uint32_t r2 = W.hl; r2 < k; r2 += 16) {
+        const unsigned long long dk = r2 < nc ? m.cand[r2] : EMPTY64;
+        const bool ok = dk != EMPTY64 && (uint32_t)(dk >> 32) <= lim;
+        P.out_obj[(size_t)qi * k + r2] = ok ? (uint32_t)dk : GGRID_PAD;
+        P.out_dist[(size_t)qi * k + r2] = ok ? (uint32_t)(dk >> 32) : GGRID_PAD;
+      }
+      const unsigned long long rm = ((unsigned long long)hor(W, (uint32_t)(rmask >> 32)) << 32) | hor(W, (uint32_t)rmask);
+      const uint32_t sa = hsum(W, c_arcs), sh = hsum(W, c_harv), so = hsum(W, c_objs);
+      if (W.hl == 0) {
+        if (P.remote) P.remote[qi] = rm;
+        atomicAdd(&s.st->ex_iters, (unsigned long long)c_iter);
+        atomicAdd(&s.st->ex_vertices, (unsigned long long)c_vert);
+        atomicAdd(&s.st->ex_arcs, (unsigned long long)sa);
+        atomicAdd(&s.st->ex_harvested, (unsigned long long)sh);
+        atomicAdd(&s.st->ex_objects, (unsigned long long)so);
+      }
+    } else if (qi != NONE && W.hl == 0) {
+      finish_undone(P, qi, r);
+    }
+    __syncwarp(W.mask);
+    need = true;
+  };
+
+  for (;;) {
+    // ---- A. a half without a query fetches and starts the next one
+    while (need && !exhausted) {
+      uint32_t li = 0;
+      if (W.hl == 0) li = atomicAdd(&s.st->expand_work[P.level], 1u);
+      li = __shfl_sync(W.mask, li, W.base);
+      if (li >= P.n) {
+        exhausted = true;
+        qi = NONE;
+        break;
+      }
+      qi = P.qlist ? P.qlist[li] : li;
+      need = false;
+      outcome = -1;
+      for (uint32_t i = W.hl; i < H; i += 16) {
+        m.key[i] = EMPTY32;
+        m.dist[i] = INF;
+      }
+      for (uint32_t i = W.hl; i < (H + 31) / 32; i += 16) {
+        m.fin[i] = 0;
+        m.listed[i] = 0;
+      }
+      __syncwarp(W.mask);
+      c_iter = c_vert = c_arcs = c_harv = c_objs = 0;
+      nc = 0;
+      rmask = 0;
+      fb = 0;
+      q = P.q[qi];
+      if (q.x >= g.A) {  // invalid query: reported by the seed kernel (EINVAL)
+        need = true;
+        continue;
+      }
+      ei = g.einfo[q.x];
+      if (q.y >= ei.y) {
+        need = true;
+        continue;
+      }
+      lim = P.bound ? P.bound[qi] : INF;
+      if (track) {
+        const uint32_t o = owner_of(cellof(g, ei.x), g.n_cells, s.n_ranks);
+        if (o != s.rank) rmask |= 1ull << o;
+      }
+      const uint32_t seed_v = q.y == 0 ? ei.x : g.edst[q.x];
+      const uint32_t seed_d = q.y == 0 ? 0u : ei.y - q.y;
+      if (W.hl == 0) {
+        bool imp;
+        const int sl = tab_relax(m, H, seed_v, seed_d, imp);
+        m.front0[0] = (uint32_t)sl;
+        m.fin[sl >> 5] |= 1u << (sl & 31);
+      }
+      __syncwarp(W.mask);
+      nf = 1;
+      blo = seed_d;
+      if (q.y > 0) {  // objects on q's own arc ahead of q (reading R2), stored at src(q.e)
+        const uint32_t c = cellof(g, ei.x);
+        if (s.cell_head[c] != NONE) {
+          if (W.hl == 0) request_flush(s, c, P.epoch);
+          finish(RETRY);
+          continue;
+        }
+        const uint2 vo = vobj_valid(s.v_obj[ei.x], s.cell_comp[c]);
+        bool ovf = false;
+        for (uint32_t j0 = 0; j0 < vo.y && !ovf; j0 += 16) {
+          const uint32_t j = j0 + W.hl;
+          bool has = false;
+          uint32_t ob = 0, dd = 0;
+          if (j < vo.y) {
+            const uint32_t pp = vo.x + j;
+            ob = s.ar.obj[pp];
+            const uint32_t oe = s.ar.edge[pp], oo = s.ar.off[pp];
+            if (oe == q.x && oo >= q.y && valid_rec(s, pp, ob)) {
+              has = true;
+              dd = oo - q.y;
+            }
+          }
+          ovf = !cand_push16(m, W, nc, cp.C, has, SPECIAL, dd, ob);
+        }
+        if (ovf) {
+          finish(OVERFLOW);
+          continue;
+        }
+      }
+    }
+    if (__all_sync(0xffffffffu, exhausted)) break;
+    bool act = !exhausted;
+
+    // ---- B. termination: k candidates strictly closer than anything not yet final
+    if (act) {
+      ++c_iter;
+      bool stop = nf == 0 || blo > lim;
+      if (!stop && nc >= k) {
+        uint32_t cl = 0;
+        for (uint32_t i = W.hl; i < nc; i += 16) cl += cand_dist(m, i) < blo;
+        stop = hsum(W, cl) >= k;
+      }
+      if (stop) {
+        finish(DONE);
+        act = false;
+      }
+    }
+    uint32_t* front = fb ? m.front1 : m.front0;
+    uint32_t* nfront = fb ? m.front0 : m.front1;
+
+    // ---- C. partition: the bucket [blo, blo + delta) into act, the rest re-queued
+    const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
+    uint32_t nn = 0, na = 0, mn = INF;
+    const uint32_t nf_b = both_max(act ? nf : 0u);
+    for (uint32_t b0 = 0; b0 < nf_b; b0 += 16) {
+      const uint32_t i = b0 + W.hl;
+      const uint32_t sl = (act && i < nf) ? front[i] : NONE;
+      const uint32_t ent = sl != NONE ? m.dist[sl] : INF;
+      const bool a = sl != NONE && ent < bhi;
+      const bool r = sl != NONE && !a;
+      const unsigned rm = __ballot_sync(W.mask, r) & W.mask;
+      if (r) {
+        nfront[nn + __popc(rm & W.lt)] = sl;
+        mn = min(mn, ent);
+      }
+      nn += __popc(rm);
+      const unsigned am = __ballot_sync(W.mask, a) & W.mask;
+      if (a) {
+        m.act[na + __popc(am & W.lt)] = sl;
+        atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
+      }
+      na += __popc(am);
+    }
+    __syncwarp();
+    if (act) c_vert += na;
+
+    // ---- D. expand the bucket in chunks of 16 vertices, lane = vertex; arcs compacted
+    int oc = -1;  // this half's outcome met in the round (RETRY / OVERFLOW)
+    const uint32_t na_b = both_max(na);
+    for (uint32_t c0 = 0; c0 < na_b; c0 += 16) {
+      const uint32_t vi = c0 + W.hl;
+      const bool vv = oc < 0 && vi < na;
+      uint32_t vslot = 0, u = 0, du = INF, hcell = 0, hd = NONE;
+      uint4 a01 = make_uint4(0, 0, 0, 0), a23 = make_uint4(0, 0, 0, 0);
+      uint2 cc = make_uint2(0, 0), v0 = make_uint2(0, 0);
+      bool harv = false;
+      if (vv) {
+        vslot = m.act[vi];
+        u = m.key[vslot];
+        du = m.dist[vslot];
+        const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)u * 4);
+        a01 = rec[0];
+        a23 = rec[1];
+        harv = !(atomicOr(&m.listed[vslot >> 5], 1u << (vslot & 31)) & (1u << (vslot & 31)));
+        if (harv) {
+          hcell = cellof(g, u);
+          hd = s.cell_head[hcell];
+          cc = s.cell_comp[hcell];
+          if (!GG_VHAS || vhas_bit(s, u)) v0 = s.v_obj[u];
+        }
+      }
+      const bool overflow_arcs = a23.w == WMAX;
+      const uint32_t room = INF - du;
+      auto real = [&](uint32_t w) { return (w - 1u < WMAX - 1u) & (w < room); };
+      const uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
+      const uint32_t cnt = r0 + r1 + r2 + r3;
+      uint32_t pre = cnt;
+#pragma unroll
+      for (int o = 1; o < 16; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(W.mask, pre, o, 16);
+        if (W.hl >= (uint32_t)o) pre += y;
+      }
+      const uint32_t n_arc = __shfl_sync(W.mask, pre, W.base + 15);
+      pre -= cnt;
+      if (r0) m.stage[pre++] = make_uint2(a01.x, du + a01.y);
+      if (r1) m.stage[pre++] = make_uint2(a01.z, du + a01.w);
+      if (r2) m.stage[pre++] = make_uint2(a23.x, du + a23.y);
+      if (r3) m.stage[pre++] = make_uint2(a23.z, du + a23.w);
+      c_arcs += cnt;
+      const bool dirty = harv && hd != NONE;
+      const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
+      const uint32_t ev = hor(W, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
+      __syncwarp();
+      // relax: lane = arc of this half's staged list
+      const uint32_t narc_b = both_max(n_arc);
+      for (uint32_t j0 = 0; j0 < narc_b; j0 += 16) {
+        bool has = false, ovf = false;
+        uint32_t nslot = 0;
+        if (j0 + W.hl < n_arc) {
+          const uint2 a = m.stage[j0 + W.hl];
+          bool imp;
+          const int rr = tab_relax(m, H, a.x, a.y, imp);
+          if (rr < 0) {
+            ovf = true;
+          } else if (imp) {
+            mn = min(mn, a.y);
+            const uint32_t bit = 1u << (rr & 31);
+            if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+              has = true;
+              nslot = (uint32_t)rr;
+              prefetch_vertex(g, s, a.x);
+            }
+          }
+        }
+        const unsigned ob_ = __ballot_sync(W.mask, ovf) & W.mask;
+        const unsigned hm = __ballot_sync(W.mask, has) & W.mask;
+        if (oc < 0 && (ob_ || nn + __popc(hm) > cp.F)) oc = OVERFLOW;
+        if (oc < 0) {
+          if (has) nfront[nn + __popc(hm & W.lt)] = nslot;
+          nn += __popc(hm);
+        }
+      }
+      __syncwarp();  // (the stage is rewritten by the next chunk)
+      // vertices with more than 4 arcs: arcs 3.. from the CSR, one per lane per step (rare)
+      if (both_max(ev & 2u)) {
+        uint32_t b0 = 0, b1 = 0;
+        if (overflow_arcs && oc < 0) {
+          b0 = g.rowptr[u] + 3;
+          b1 = g.rowptr[u + 1];
+        }
+        const uint32_t most = both_max(hmax(W, b1 - b0));
+        for (uint32_t j = 0; j < most; ++j) {
+          bool has = false, ovf = false;
+          uint32_t nslot = 0;
+          if (b0 + j < b1) {
+            const uint2 av = g.adj[b0 + j];
+            ++c_arcs;
+            const unsigned long long nd = (unsigned long long)du + av.y;
+            if (nd < INF) {
+              bool imp;
+              const int rr = tab_relax(m, H, av.x, (uint32_t)nd, imp);
+              if (rr < 0) {
+                ovf = true;
+              } else if (imp) {
+                mn = min(mn, (uint32_t)nd);
+                const uint32_t bit = 1u << (rr & 31);
+                if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+                  has = true;
+                  nslot = (uint32_t)rr;
+                }
+              }
+            }
+          }
+          const unsigned ob_ = __ballot_sync(W.mask, ovf) & W.mask;
+          const unsigned hm = __ballot_sync(W.mask, has) & W.mask;
+          if (oc < 0 && (ob_ || nn + __popc(hm) > cp.F)) oc = OVERFLOW;
+          if (oc < 0) {
+            if (has) nfront[nn + __popc(hm & W.lt)] = nslot;
+            nn += __popc(hm);
+          }
+        }
+      }
+      if (oc < 0 && (ev & 4u)) {  // a cell with cached updates: lazy flush, then retry
+        if (dirty) request_flush(s, hcell, P.epoch);
+        for (uint32_t i = W.hl; i < nf; i += 16) request_flush(s, cellof(g, m.key[front[i]]), P.epoch);
+        oc = RETRY;
+      }
+      if (oc < 0) {
+        c_harv += harv;
+        if (track) {
+          const uint32_t o = harv ? owner_of(hcell, g.n_cells, s.n_ranks) : s.rank;
+          if (o != s.rank) rmask |= 1ull << o;
+        }
+      }
+      if (both_max(oc < 0 ? (ev & 8u) : 0u)) {  // harvest the objects of first-expanded vertices
+        const uint32_t most = both_max(oc < 0 ? hmax(W, vo.y) : 0u);
+        if (oc < 0) c_objs += vo.y;
+        for (uint32_t j = 0; j < most; ++j) {
+          bool hc = false;
+          uint32_t ob = 0, oo = 0;
+          if (oc < 0 && j < vo.y) {
+            const uint32_t pp = vo.x + j;
+            ob = s.ar.obj[pp];
+            const uint32_t oe = s.ar.edge[pp];
+            oo = s.ar.off[pp];
+            const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
+            hc = !same_ahead && valid_rec(s, pp, ob);
+          }
+          const bool okp = cand_push16(m, W, nc, cp.C, hc, vslot, oo, ob);
+          if (!okp && oc < 0) oc = OVERFLOW;
+        }
+      }
+    }
+    // ---- E. round end
+    if (oc >= 0) {
+      finish(oc);
+    } else if (act) {
+      nf = nn;
+      blo = hmin(W, mn);
+      fb ^= 1u;
+    }
+    __syncwarp();
+  }
+  __syncthreads();  // (the chained level waits for every CTA to exit)
   if (threadIdx.x == 0) count_exit(P);
 }
 
@@ -1202,6 +1634,7 @@ static uint32_t blocks_per_sm(int level, bool cta) {
   static int bps[2][NLEVELS] = {};  // (occupancy: the same on every B200)
   // the attribute is per device: set on every device this process launches on
   if (cta) func_attr_once(cta_kernel(level), cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
+  else if (GG_PAIR && level == 0) func_attr_once(k_expand_pair, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   else func_attr_once(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   int& b = bps[cta ? 1 : 0][level];
   if (!b) {
@@ -1209,7 +1642,10 @@ static uint32_t blocks_per_sm(int level, bool cta) {
     if (cta) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, cta_kernel(level), cta_warps(level) * 32, smem);
     } else {
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32 * WPC, smem * WPC);
+      if (GG_PAIR && level == 0)  // (two queries per warp: two tables per warp)
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand_pair, 32 * WPC, 2 * smem * WPC);
+      else
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<true>, 32 * WPC, smem * WPC);
     }
 #ifdef GG_L0_PER_SM
     if (!cta && level == 0) b = std::min(b, GG_L0_PER_SM);  // experiment hook: occupancy cap
@@ -1222,7 +1658,7 @@ static uint32_t blocks_per_sm(int level, bool cta) {
 uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level == NLEVELS - 1) return 0;  // (global scratch: sized by the caller's scratch warps)
   const bool cta = use_cta(level, n, sm_count, ball_hint);
-  const uint32_t per = cta ? 1u : WPC;  // queries a CTA runs at once
+  const uint32_t per = cta ? 1u : (GG_PAIR && level == 0 ? 2 * WPC : WPC);  // queries a CTA runs at once
   return std::min<uint32_t>((n + per - 1) / per, (uint32_t)sm_count * blocks_per_sm(level, cta));
 }
 
@@ -1268,9 +1704,10 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   blocks_per_sm(level, cta);  // (sets the shared-memory attribute)
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
+  const bool pair = !cta && GG_PAIR && level == 0;
   if (!cta) P.warps_per_cta = WPC;
   cfg.blockDim = dim3(cta ? cta_warps(level) * 32 : 32 * WPC);
-  cfg.dynamicSmemBytes = (size_t)smem * (cta ? 1 : WPC);
+  cfg.dynamicSmemBytes = (size_t)smem * (cta ? 1 : (pair ? 2 * WPC : WPC));
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -1279,6 +1716,8 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   cfg.numAttrs = 1;  // programmatic dependent of the flush (waits for it) or, chained, of the level below
   if (cta) {
     cudaLaunchKernelEx(&cfg, cta_kernel(level), P);
+  } else if (pair) {
+    cudaLaunchKernelEx(&cfg, k_expand_pair, P);
   } else {
     cudaLaunchKernelEx(&cfg, k_expand<true>, P);
   }
