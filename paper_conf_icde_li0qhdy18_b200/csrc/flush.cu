@@ -585,10 +585,14 @@ __device__ __forceinline__ void rq_push(uint32_t* rq_n, uint32_t* rq, uint32_t b
 }
 
 template <int HCAP, int WCAP>
-#ifndef GG_TMA_MINB
-#define GG_TMA_MINB 1
+// (an explicit min-blocks bound -- even 1 -- changes ptxas's register choice: 72 registers, 4 CTAs
+// per SM, 0.233 ms at C3 vs 56 registers, 5 CTAs, 0.223 ms without one; r2 profiling pass)
+#ifdef GG_TMA_MINB
+#define TMA_BOUNDS __launch_bounds__(TFT, GG_TMA_MINB)
+#else
+#define TMA_BOUNDS __launch_bounds__(TFT)
 #endif
-__global__ void __launch_bounds__(TFT, GG_TMA_MINB) k_flush_tma(DevGraph g, DevState s, Arena out, unsigned long long* out_top,
+__global__ void TMA_BOUNDS k_flush_tma(DevGraph g, DevState s, Arena out, unsigned long long* out_top,
                                                    uint32_t begin, int full_vobj, uint32_t* spill, uint32_t spill_cap,
                                                    uint32_t t_cut) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
