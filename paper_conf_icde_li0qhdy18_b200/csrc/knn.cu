@@ -756,6 +756,17 @@ __device__ __forceinline__ uint32_t hor(const HalfWarp& W, uint32_t x) {
   for (int o = 8; o > 0; o >>= 1) x |= __shfl_xor_sync(W.mask, x, o);
   return x;
 }
+// full-warp forms for the phases both halves run in the same instructions
+__device__ __forceinline__ uint32_t horF(const HalfWarp&, uint32_t x) {
+#pragma unroll
+  for (int o = 8; o > 0; o >>= 1) x |= __shfl_xor_sync(0xffffffffu, x, o);
+  return x;
+}
+__device__ __forceinline__ uint32_t hmaxF(const HalfWarp&, uint32_t x) {
+#pragma unroll
+  for (int o = 8; o > 0; o >>= 1) x = max(x, __shfl_xor_sync(0xffffffffu, x, o));
+  return x;
+}
 // the larger of the two halves' (half-uniform) values: the shared loop bound of a phase
 __device__ __forceinline__ uint32_t both_max(uint32_t v) { return max(v, __shfl_xor_sync(0xffffffffu, v, 16)); }
 
@@ -764,6 +775,19 @@ __device__ __forceinline__ bool cand_push16(const WarpMem& m, const HalfWarp& W,
   const unsigned hm = __ballot_sync(W.mask, has) & W.mask;
   if (!hm) return true;
   if (nc + __popc(hm) > C) return false;
+  if (has) {
+    const uint32_t i = nc + __popc(hm & W.lt);
+    m.cand[i] = ((unsigned long long)slot << 32) | off;
+    m.cobj[i] = obj;
+  }
+  nc += __popc(hm);
+  return true;
+}
+
+__device__ __forceinline__ bool cand_push16F(const WarpMem& m, const HalfWarp& W, uint32_t& nc, uint32_t C, bool has,
+                                             uint32_t slot, uint32_t off, uint32_t obj) {
+  const unsigned hm = __ballot_sync(0xffffffffu, has) & W.mask;
+  if (hm && nc + __popc(hm) > C) return false;
   if (has) {
     const uint32_t i = nc + __popc(hm & W.lt);
     m.cand[i] = ((unsigned long long)slot << 32) | off;
@@ -941,16 +965,19 @@ __global__ void k_expand_pair(QParams P) {
     if (__all_sync(0xffffffffu, exhausted)) break;
     bool act = !exhausted;
 
-    // ---- B. termination: k candidates strictly closer than anything not yet final
-    if (act) {
-      ++c_iter;
-      bool stop = nf == 0 || blo > lim;
-      if (!stop && nc >= k) {
-        uint32_t cl = 0;
-        for (uint32_t i = W.hl; i < nc; i += 16) cl += cand_dist(m, i) < blo;
-        stop = hsum(W, cl) >= k;
-      }
-      if (stop) {
+    // ---- B. termination: k candidates strictly closer than anything not yet final (both
+    //         halves count in the same instructions; only the finish is per half)
+    {
+      if (act) ++c_iter;
+      const bool early = act && (nf == 0 || blo > lim);
+      const bool chk = act && !early && nc >= k;
+      const uint32_t nc_b = both_max(chk ? nc : 0u);
+      uint32_t cl = 0;
+      for (uint32_t i = W.hl; i < nc_b; i += 16)
+        if (chk && i < nc) cl += cand_dist(m, i) < blo;
+#pragma unroll
+      for (int o = 8; o > 0; o >>= 1) cl += __shfl_xor_sync(0xffffffffu, cl, o);
+      if (early || (chk && cl >= k)) {
         finish(DONE);
         act = false;
       }
@@ -968,13 +995,13 @@ __global__ void k_expand_pair(QParams P) {
       const uint32_t ent = sl != NONE ? m.dist[sl] : INF;
       const bool a = sl != NONE && ent < bhi;
       const bool r = sl != NONE && !a;
-      const unsigned rm = __ballot_sync(W.mask, r) & W.mask;
+      const unsigned rm = __ballot_sync(0xffffffffu, r) & W.mask;
       if (r) {
         nfront[nn + __popc(rm & W.lt)] = sl;
         mn = min(mn, ent);
       }
       nn += __popc(rm);
-      const unsigned am = __ballot_sync(W.mask, a) & W.mask;
+      const unsigned am = __ballot_sync(0xffffffffu, a) & W.mask;
       if (a) {
         m.act[na + __popc(am & W.lt)] = sl;
         atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
@@ -1017,10 +1044,10 @@ __global__ void k_expand_pair(QParams P) {
       uint32_t pre = cnt;
 #pragma unroll
       for (int o = 1; o < 16; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(W.mask, pre, o, 16);
+        const uint32_t y = __shfl_up_sync(0xffffffffu, pre, o, 16);
         if (W.hl >= (uint32_t)o) pre += y;
       }
-      const uint32_t n_arc = __shfl_sync(W.mask, pre, W.base + 15);
+      const uint32_t n_arc = __shfl_sync(0xffffffffu, pre, W.base + 15);
       pre -= cnt;
       if (r0) m.stage[pre++] = make_uint2(a01.x, du + a01.y);
       if (r1) m.stage[pre++] = make_uint2(a01.z, du + a01.w);
@@ -1029,7 +1056,7 @@ __global__ void k_expand_pair(QParams P) {
       c_arcs += cnt;
       const bool dirty = harv && hd != NONE;
       const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
-      const uint32_t ev = hor(W, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
+      const uint32_t ev = horF(W, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
       __syncwarp();
       // relax: lane = arc of this half's staged list
       const uint32_t narc_b = both_max(n_arc);
@@ -1052,8 +1079,8 @@ __global__ void k_expand_pair(QParams P) {
             }
           }
         }
-        const unsigned ob_ = __ballot_sync(W.mask, ovf) & W.mask;
-        const unsigned hm = __ballot_sync(W.mask, has) & W.mask;
+        const unsigned ob_ = __ballot_sync(0xffffffffu, ovf) & W.mask;
+        const unsigned hm = __ballot_sync(0xffffffffu, has) & W.mask;
         if (oc < 0 && (ob_ || nn + __popc(hm) > cp.F)) oc = OVERFLOW;
         if (oc < 0) {
           if (has) nfront[nn + __popc(hm & W.lt)] = nslot;
@@ -1068,7 +1095,7 @@ __global__ void k_expand_pair(QParams P) {
           b0 = g.rowptr[u] + 3;
           b1 = g.rowptr[u + 1];
         }
-        const uint32_t most = both_max(hmax(W, b1 - b0));
+        const uint32_t most = both_max(hmaxF(W, b1 - b0));
         for (uint32_t j = 0; j < most; ++j) {
           bool has = false, ovf = false;
           uint32_t nslot = 0;
@@ -1091,8 +1118,8 @@ __global__ void k_expand_pair(QParams P) {
               }
             }
           }
-          const unsigned ob_ = __ballot_sync(W.mask, ovf) & W.mask;
-          const unsigned hm = __ballot_sync(W.mask, has) & W.mask;
+          const unsigned ob_ = __ballot_sync(0xffffffffu, ovf) & W.mask;
+          const unsigned hm = __ballot_sync(0xffffffffu, has) & W.mask;
           if (oc < 0 && (ob_ || nn + __popc(hm) > cp.F)) oc = OVERFLOW;
           if (oc < 0) {
             if (has) nfront[nn + __popc(hm & W.lt)] = nslot;
@@ -1113,7 +1140,7 @@ __global__ void k_expand_pair(QParams P) {
         }
       }
       if (both_max(oc < 0 ? (ev & 8u) : 0u)) {  // harvest the objects of first-expanded vertices
-        const uint32_t most = both_max(oc < 0 ? hmax(W, vo.y) : 0u);
+        const uint32_t most = both_max(oc < 0 ? hmaxF(W, vo.y) : 0u);
         if (oc < 0) c_objs += vo.y;
         for (uint32_t j = 0; j < most; ++j) {
           bool hc = false;
@@ -1126,17 +1153,20 @@ __global__ void k_expand_pair(QParams P) {
             const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
             hc = !same_ahead && valid_rec(s, pp, ob);
           }
-          const bool okp = cand_push16(m, W, nc, cp.C, hc, vslot, oo, ob);
+          const bool okp = cand_push16F(m, W, nc, cp.C, hc, vslot, oo, ob);
           if (!okp && oc < 0) oc = OVERFLOW;
         }
       }
     }
     // ---- E. round end
+    uint32_t mnh = mn;
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) mnh = min(mnh, __shfl_xor_sync(0xffffffffu, mnh, o));
     if (oc >= 0) {
       finish(oc);
     } else if (act) {
       nf = nn;
-      blo = hmin(W, mn);
+      blo = mnh;
       fb ^= 1u;
     }
     __syncwarp();
