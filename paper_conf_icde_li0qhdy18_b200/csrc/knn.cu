@@ -1140,7 +1140,8 @@ __global__ void k_expand_pair(QParams P) {
         }
       }
       if (both_max(oc < 0 ? (ev & 8u) : 0u)) {  // harvest the objects of first-expanded vertices
-        const uint32_t most = both_max(oc < 0 ? hmaxF(W, vo.y) : 0u);
+        const uint32_t vmx = hmaxF(W, vo.y);  // (every lane of both halves runs the full-warp shuffles)
+        const uint32_t most = both_max(oc < 0 ? vmx : 0u);
         if (oc < 0) c_objs += vo.y;
         for (uint32_t j = 0; j < most; ++j) {
           bool hc = false;
