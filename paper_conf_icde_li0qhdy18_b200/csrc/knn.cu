@@ -96,6 +96,9 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 #ifndef GG_PREFETCH
 #define GG_PREFETCH 1  // (C3: expansion 1.75 -> 1.66 ms per 65,536 queries, r2b variants)
 #endif
+#ifndef GG_EARLY_LOADS
+#define GG_EARLY_LOADS 1
+#endif
 // one-warp variant: lane = vertex chunks with compacted arcs (1) or lane = (vertex, slot)
 // windows of 8 vertices (0, the round-1 design)
 #ifndef GG_WARP_ARCS
@@ -352,11 +355,13 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
     // ---- 1. termination: k candidates strictly closer than anything not yet final ---------
     if (nf == 0) break;
     if (blo > lim) break;  // every object not yet harvested is beyond the caller's bound
-    if (nc >= k) {
+    auto terminated = [&]() {
+      if (nc < k) return false;
       uint32_t cl = 0;
       for (uint32_t i = lane; i < nc; i += 32) cl += cand_dist(m, i) < blo;
-      if (__reduce_add_sync(FULL, cl) >= k) break;
-    }
+      return __reduce_add_sync(FULL, cl) >= k;
+    };
+    if ((!GG_EARLY_LOADS || !GG_WARP_ARCS) && terminated()) break;
 
     // ---- 2. partition the frontier: the bucket [m, m + delta) into act, the rest re-queued --
     const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
@@ -389,28 +394,53 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
     //         loads) and, at its first expansion, its cell state and object index; the chunk's
     //         real arcs are then compacted into shared memory (warp prefix sum over the lanes'
     //         arc counts) and relaxed 32 at a time, lane = arc -- no lane idles on an empty slot
-    for (uint32_t c0 = 0; c0 < na; c0 += 32) {
+    struct ChunkLd {
+      uint32_t vslot, u, du, hcell, hd;
+      uint4 a01, a23;
+      uint2 cc, v0;
+      bool vv, harv;
+    };
+    auto load_chunk = [&](uint32_t c0) {
+      ChunkLd x;
       const uint32_t vi = c0 + lane;
-      const bool vv = vi < na;
-      uint32_t vslot = 0, u = 0, du = INF, hcell = 0, hd = NONE;
-      uint4 a01 = make_uint4(0, 0, 0, 0), a23 = make_uint4(0, 0, 0, 0);
-      uint2 cc = make_uint2(0, 0), v0 = make_uint2(0, 0);
-      bool harv = false;
-      if (vv) {
-        vslot = m.act[vi];
-        u = m.key[vslot];
-        du = m.dist[vslot];  // (an improvement after this read re-queues the vertex: fin bit cleared)
-        const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)u * 4);
-        a01 = rec[0];
-        a23 = rec[1];
-        harv = !(atomicOr(&m.listed[vslot >> 5], 1u << (vslot & 31)) & (1u << (vslot & 31)));
-        if (harv) {
-          hcell = cellof(g, u);
-          hd = s.cell_head[hcell];
-          cc = s.cell_comp[hcell];
-          if (!GG_VHAS || vhas_bit(s, u)) v0 = s.v_obj[u];  // (GG_VHAS: most vertices hold no object)
+      x.vv = vi < na;
+      x.vslot = 0;
+      x.u = 0;
+      x.du = INF;
+      x.hcell = 0;
+      x.hd = NONE;
+      x.a01 = make_uint4(0, 0, 0, 0);
+      x.a23 = make_uint4(0, 0, 0, 0);
+      x.cc = make_uint2(0, 0);
+      x.v0 = make_uint2(0, 0);
+      x.harv = false;
+      if (x.vv) {
+        x.vslot = m.act[vi];
+        x.u = m.key[x.vslot];
+        x.du = m.dist[x.vslot];  // (an improvement after this read re-queues the vertex: fin cleared)
+        const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)x.u * 4);
+        x.a01 = rec[0];
+        x.a23 = rec[1];
+        x.harv = !(atomicOr(&m.listed[x.vslot >> 5], 1u << (x.vslot & 31)) & (1u << (x.vslot & 31)));
+        if (x.harv) {
+          x.hcell = cellof(g, x.u);
+          x.hd = s.cell_head[x.hcell];
+          x.cc = s.cell_comp[x.hcell];
+          if (!GG_VHAS || vhas_bit(s, x.u)) x.v0 = s.v_obj[x.u];  // (GG_VHAS: most hold no object)
         }
       }
+      return x;
+    };
+    // (GG_EARLY_LOADS) the first chunk's global loads go out before the termination count, whose
+    // shared-memory work then overlaps their latency; a stopping round just drops them
+    ChunkLd first = load_chunk(0);
+    if (GG_EARLY_LOADS && terminated()) break;
+    for (uint32_t c0 = 0; c0 < na; c0 += 32) {
+      const ChunkLd x = c0 == 0 ? first : load_chunk(c0);
+      const uint32_t vslot = x.vslot, u = x.u, du = x.du, hcell = x.hcell, hd = x.hd;
+      const uint4 a01 = x.a01, a23 = x.a23;
+      const uint2 cc = x.cc, v0 = x.v0;
+      const bool harv = x.harv;
       const bool overflow_arcs = a23.w == WMAX;  // more than 4 arcs: 3 inline, the rest in the CSR
       // compact the real arcs (w != 0) of the chunk: (dst, du + w), skipping sums >= INF
       // a real arc (1 <= w < WMAX) whose sum stays below INF (du < INF: a bucket vertex); 32-bit
