@@ -692,8 +692,10 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
     uint32_t grid0 = 0;
     if (conc) {  // leave room for the chained level's CTAs (so they are resident from the start)
       const uint32_t full = expand_grid(lvl0, n_in[lvl0], h->sm_count, ball_hint);
-      const size_t b0 = expand_warp_bytes(lvl0, h->V) + 1024, bc = expand_warp_bytes(chain, h->V) + 1024;
-      const uint32_t reserve = (uint32_t)(grid_c * ((bc + b0 - 1) / b0));
+      // (in shared memory: a starting-level CTA may hold several queries -- one-warp mode)
+      const size_t b0 = expand_block_bytes(lvl0, h->V, n_in[lvl0], h->sm_count, ball_hint, false);
+      const size_t bc = expand_block_bytes(chain, h->V, n_q, h->sm_count, ball_hint, true);
+      const uint32_t reserve = (uint32_t)((grid_c * bc + b0 - 1) / b0);
       grid0 = full > reserve + h->sm_count ? full - reserve : full;
     }
     auto base = [&](int lvl) {

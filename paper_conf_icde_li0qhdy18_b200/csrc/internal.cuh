@@ -336,6 +336,9 @@ void launch_pa_bundle(const uint32_t* obj, const unsigned long long* key, int et
 size_t sort_queries_tmp_bytes(uint32_t n);
 int launch_sort_queries(const uint2* q, uint32_t n, const DevGraph& g, void* tmp, size_t tmp_bytes, uint32_t* perm,
                         cudaStream_t st);
+// shared memory of one CTA of a level's kernel in the mode a launch of n queries takes (chained:
+// the level runs beside the one below it, CTA mode)
+size_t expand_block_bytes(int level, uint32_t V, uint32_t n, int sm_count, uint32_t ball_hint, bool chained);
 int expand_levels();
 uint32_t expand_table_slots(int level);  // vertex-table capacity H of a level
 uint32_t expand_max_k(int level);

@@ -96,8 +96,10 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 #ifndef GG_PREFETCH
 #define GG_PREFETCH 1  // (C3: expansion 1.75 -> 1.66 ms per 65,536 queries, r2b variants)
 #endif
+// (experiment hook) issue the first chunk's loads before the termination count: measured no
+// different at C3 (1.277 vs 1.280 ms, r2p) at 72 instead of 56 registers -- off
 #ifndef GG_EARLY_LOADS
-#define GG_EARLY_LOADS 1
+#define GG_EARLY_LOADS 0
 #endif
 // one-warp variant: lane = vertex chunks with compacted arcs (1) or lane = (vertex, slot)
 // windows of 8 vertices (0, the round-1 design)
@@ -386,7 +388,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
       na += __popc(am);
     }
     __syncwarp();
-    c_vert += na;
+    if (!GG_EARLY_LOADS || !GG_WARP_ARCS) c_vert += na;
 
 #if GG_WARP_ARCS
     // ---- 3. expand the bucket in chunks of 32 vertices, lane = vertex: ONE dependent global
@@ -433,10 +435,14 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
     };
     // (GG_EARLY_LOADS) the first chunk's global loads go out before the termination count, whose
     // shared-memory work then overlaps their latency; a stopping round just drops them
-    ChunkLd first = load_chunk(0);
-    if (GG_EARLY_LOADS && terminated()) break;
+    ChunkLd first;
+    if (GG_EARLY_LOADS) {
+      first = load_chunk(0);
+      if (terminated()) break;
+      c_vert += na;  // (counted for expanded rounds only)
+    }
     for (uint32_t c0 = 0; c0 < na; c0 += 32) {
-      const ChunkLd x = c0 == 0 ? first : load_chunk(c0);
+      const ChunkLd x = (GG_EARLY_LOADS && c0 == 0) ? first : load_chunk(c0);
       const uint32_t vslot = x.vslot, u = x.u, du = x.du, hcell = x.hcell, hd = x.hd;
       const uint4 a01 = x.a01, a23 = x.a23;
       const uint2 cc = x.cc, v0 = x.v0;
@@ -1721,6 +1727,13 @@ uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   const bool cta = use_cta(level, n, sm_count, ball_hint);
   const uint32_t per = cta ? 1u : (GG_PAIR && level == 0 ? 2 * WPC : WPC);  // queries a CTA runs at once
   return std::min<uint32_t>((n + per - 1) / per, (uint32_t)sm_count * blocks_per_sm(level, cta));
+}
+
+size_t expand_block_bytes(int level, uint32_t V, uint32_t n, int sm_count, uint32_t ball_hint, bool chained) {
+  if (level == NLEVELS - 1) return 0;
+  const bool cta = chained || use_cta(level, n, sm_count, ball_hint);
+  const uint32_t per = cta ? 1u : (GG_PAIR && level == 0 ? 2 * WPC : WPC);
+  return warp_bytes_mode(level, V, cta) * per + 1024;  // (+ the per-CTA reservation)
 }
 
 void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st) {
