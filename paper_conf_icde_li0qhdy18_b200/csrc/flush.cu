@@ -764,32 +764,42 @@ __global__ void TMA_BOUNDS k_flush_tma(DevGraph g, DevState s, Arena out, unsign
       if (n == 0xFFFFFFFFu) break;
       const uint32_t b = sm.st_slot[st], pos = sm.st_pos[st];
       TSlot<WCAP>& sl = sm.slot[b];
-      constexpr int R = TCHUNK / 32;
-      uint32_t o[R];
-      unsigned long long k[R], tg[R];
+      // the stage in sub-pieces of 256 records (8 per lane in registers); the stage is released
+      // once its last sub-piece is in registers
+      constexpr int R = 8;
+      constexpr int NSUB = TCHUNK / (32 * R);
+      static_assert(TCHUNK % (32 * R) == 0, "pieces are whole sub-pieces of 256 records");
+#pragma unroll 1
+      for (int sub = 0; sub < NSUB; ++sub) {
+        const uint32_t sb0 = (uint32_t)sub * 32 * R;
+        uint32_t o[R];
+        unsigned long long k[R], tg[R];
 #pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const uint32_t i = lane + 32 * r;
-        o[r] = sm.obj[st][i];
-        k[r] = sm.key[st][i];
-      }
+        for (int r = 0; r < R; ++r) {
+          const uint32_t i = sb0 + lane + 32 * r;
+          o[r] = sm.obj[st][i];
+          k[r] = sm.key[st][i];
+        }
 #pragma unroll
-      for (int r = 0; r < R; ++r) tg[r] = (lane + 32 * r) < n ? __ldg(otk + o[r]) : ~k[r];
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&sm.empty[st]);  // (the stage's words are in registers now)
+        for (int r = 0; r < R; ++r) tg[r] = (sb0 + lane + 32 * r) < n ? __ldg(otk + o[r]) : ~k[r];
+        if (sub == NSUB - 1) {
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&sm.empty[st]);  // (the stage's words are in registers now)
+        }
 #pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const bool hit = tg[r] == k[r];
-        const unsigned hm = __ballot_sync(0xffffffffu, hit);
-        if (hm) {
-          uint32_t base = 0;
-          if (lane == __ffs(hm) - 1) base = atomicAdd(&sl.n_win, (unsigned)__popc(hm));
-          base = __shfl_sync(0xffffffffu, base, __ffs(hm) - 1);
-          const uint32_t w = base + __popc(hm & lt);
-          if (hit) {
-            const uint32_t p = pos + lane + 32 * r;
-            if (w < (uint32_t)WCAP) sl.w_pos[w] = p;
-            else if (w - (uint32_t)WCAP < sl.spill_cap) sl.spill[w - WCAP] = p;
+        for (int r = 0; r < R; ++r) {
+          const bool hit = tg[r] == k[r];
+          const unsigned hm = __ballot_sync(0xffffffffu, hit);
+          if (hm) {
+            uint32_t base = 0;
+            if (lane == __ffs(hm) - 1) base = atomicAdd(&sl.n_win, (unsigned)__popc(hm));
+            base = __shfl_sync(0xffffffffu, base, __ffs(hm) - 1);
+            const uint32_t w = base + __popc(hm & lt);
+            if (hit) {
+              const uint32_t p = pos + sb0 + lane + 32 * r;
+              if (w < (uint32_t)WCAP) sl.w_pos[w] = p;
+              else if (w - (uint32_t)WCAP < sl.spill_cap) sl.spill[w - WCAP] = p;
+            }
           }
         }
       }
