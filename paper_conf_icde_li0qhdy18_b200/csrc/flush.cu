@@ -502,11 +502,15 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
 #ifndef GG_TCHUNK
 #define GG_TCHUNK 256
 #endif
+// 4 stages x 2 match warps: a small ring and 128 threads per CTA = 8 CTAs (cell pipelines) per SM
+// at 64 registers; C3 full flush 0.223 ms (8 x 4) -> 0.214-0.217 ms, 58.7% of measured HBM.
+// Larger rings or more match warps cost CTAs per SM and lose; register caps spill and lose
+// (profiles/flush_tma_*_r2*.log)
 #ifndef GG_TS
-#define GG_TS 8
+#define GG_TS 4
 #endif
 #ifndef GG_TMW
-#define GG_TMW 4
+#define GG_TMW 2
 #endif
 constexpr int TCHUNK = GG_TCHUNK;  // records per stage (8 per match-warp lane)
 constexpr int TS = GG_TS;          // stages
