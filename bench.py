@@ -469,7 +469,17 @@ def run_ours(args, cfg_name):
             "frac": t_model_ms / dms if dms > 0 else None}
     lp = os.path.join(ROOT, "profiles", f"limiters_{cfg_name}.json")
     if os.path.exists(lp):  # what bounds the kernel when it is not HBM (ncu, the last profiling pass)
-        roofline["ncu_limiters"] = json.load(open(lp)).get(dom)
+        lim = json.load(open(lp)).get(dom)
+        roofline["ncu_limiters"] = lim
+        if lim and lim.get("warp_instructions") and dom == "expand":
+            # issue roofline: the capture's warp instructions per query, issued at one per
+            # scheduler per cycle (148 SMs x 4 schedulers at the max clock), for this run's queries
+            inst_q = lim["warp_instructions"] / max(1, cfg["n_queries"] // world)
+            t_issue_ms = inst_q * Qr * K / (148 * 4 * sm_mhz_max * 1e6) * 1e3
+            roofline["issue_model"] = {"warp_instructions_per_query": inst_q, "schedulers": 148 * 4,
+                                       "clock_mhz": sm_mhz_max, "model_ms": t_issue_ms, "measured_ms": dms,
+                                       "frac": t_issue_ms / dms if dms > 0 else None,
+                                       "source": "ncu smsp__inst_executed.sum of one launch (profiles/limiters_C3.json)"}
     updates_per_s = n_step_upd * K / (ingest_ms / 1e3) if ingest_ms > 0 else None
 
     # ---- parity of the last timed step (rank 0's share) against the oracle -------------------

@@ -86,6 +86,10 @@ for cap in caps:
         if "smsp__issue_active.avg.pct_of_peak_sustained_active" in hdr:  # (non-HBM limiters)
             issue.setdefault(cfg, {})[kind] = {
                 "issue_slots_busy_pct": float(r[hdr.index("smsp__issue_active.avg.pct_of_peak_sustained_active")]),
+                "warp_instructions": float(r[hdr.index("smsp__inst_executed.sum")].replace(",", "")),
+                "duration_ns": float(r[hdr.index("gpu__time_duration.sum")].replace(",", "")) * (
+                    1e3 if units[hdr.index("gpu__time_duration.sum")] == "us" else
+                    1e6 if units[hdr.index("gpu__time_duration.sum")] == "ms" else 1.0),
                 "dram_throughput_pct": float(r[hdr.index("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed")]),
                 "top_stalls": top, "capture": f"profiles/{tag}_summary.md"}
 
