@@ -30,6 +30,7 @@
 //     smallest (dist<<32 | obj) (readings R5, R6).
 // Capacities are per variant ("level"); a query that overflows one is retried on the next.
 #include <algorithm>
+#include <type_traits>
 
 #include "internal.cuh"
 
@@ -46,38 +47,50 @@ struct Caps {
   uint32_t H, F, C;  // table slots, frontier, candidates
 };
 
-// byte layout of one warp's working memory
-struct WarpMem {
+// byte layout of one query's working memory; S = the frontier's slot index type (u16 in shared
+// memory, where tables have <= 16,384 slots; u32 for the global-memory level)
+template <class S>
+struct WarpMemT {
   uint32_t* key;             // H: vertex of the slot (EMPTY32 = free)
   uint32_t* dist;            // H: its tentative distance D
   unsigned long long* cand;  // C: (slot<<32 | offset); at the end (dist<<32 | obj)
   uint32_t* cobj;            // C: object ids
-  uint32_t* front0;          // F
-  uint32_t* front1;          // F
+  S* front0;                 // F
+  S* front1;                 // F
   uint32_t* fin;             // H/32: slot is in the frontier
-  uint32_t* act;             // F: the round's active slots (the bucket being expanded)
+  S* act;                    // F: the round's active slots (the bucket being expanded)
   uint32_t* listed;          // H/32 bits: vertex expanded at least once (objects harvested)
   uint2* stage;              // STAGE: the chunk's arcs (dst, D + w), compacted (one-warp variant)
 };
-constexpr uint32_t STAGE = 128;  // arcs of a chunk of 32 bucket vertices (4 inline slots each)
+using WarpMem = WarpMemT<uint32_t>;   // global-memory level
+using WarpMemS = WarpMemT<uint16_t>;  // shared-memory levels
+// arcs staged per chunk of 32 bucket vertices (at most 4 inline each = 128; a chunk with more real
+// arcs than STAGE promotes its query -- rare: ~2.5 arcs per road vertex)
+#ifndef GG_STAGE
+#define GG_STAGE 112
+#endif
+constexpr uint32_t STAGE = GG_STAGE;
 
-__host__ __device__ inline size_t warpmem_bytes(const Caps& c) {
-  return 8ull * c.H + 12ull * c.C + 4ull * (3ull * c.F + 2ull * ((c.H + 31) / 32)) + 8ull * STAGE;
+__host__ __device__ inline size_t warpmem_bytes(const Caps& c, size_t slot_bytes) {
+  const size_t fr = (3ull * c.F * slot_bytes + 15) & ~size_t(15);
+  return 8ull * c.C + 8ull * STAGE + 8ull * c.H + 4ull * c.C + 8ull * ((c.H + 31) / 32) + fr;
 }
 
-__device__ inline WarpMem carve(unsigned char* base, const Caps& c) {
-  WarpMem m;
+template <class S>
+__device__ inline WarpMemT<S> carve(unsigned char* base, const Caps& c) {
+  WarpMemT<S> m;
   m.cand = reinterpret_cast<unsigned long long*>(base);
   m.stage = reinterpret_cast<uint2*>(m.cand + c.C);
   uint32_t* p = reinterpret_cast<uint32_t*>(m.stage + STAGE);
   m.key = p; p += c.H;
   m.dist = p; p += c.H;
   m.cobj = p; p += c.C;
-  m.front0 = p; p += c.F;
-  m.front1 = p; p += c.F;
   m.fin = p; p += (c.H + 31) / 32;
-  m.act = p; p += c.F;
-  m.listed = p;
+  m.listed = p; p += (c.H + 31) / 32;
+  S* f = reinterpret_cast<S*>(p);
+  m.front0 = f; f += c.F;
+  m.front1 = f; f += c.F;
+  m.act = f;
   return m;
 }
 
@@ -124,7 +137,8 @@ __device__ __forceinline__ bool valid_rec(const DevState& s, uint32_t p, uint32_
 }
 
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
-__device__ __forceinline__ int tab_relax(const WarpMem& m, uint32_t H, uint32_t v, uint32_t d,
+template <class M>
+__device__ __forceinline__ int tab_relax(const M& m, uint32_t H, uint32_t v, uint32_t d,
                                          bool& improved) {
   uint32_t sl = vhash(v, H);
   volatile uint32_t* vk = m.key;
@@ -220,7 +234,8 @@ __device__ __forceinline__ void count_exit(const QParams& P) {
 }
 
 // current distance of candidate i (exact once its source vertex is settled)
-__device__ __forceinline__ unsigned long long cand_dist(const WarpMem& m, uint32_t i) {
+template <class M>
+__device__ __forceinline__ unsigned long long cand_dist(const M& m, uint32_t i) {
   const unsigned long long a = m.cand[i];
   const uint32_t slot = (uint32_t)(a >> 32), off = (uint32_t)a;
   if (slot == SPECIAL) return off;
@@ -228,7 +243,8 @@ __device__ __forceinline__ unsigned long long cand_dist(const WarpMem& m, uint32
 }
 
 // Append one ballot's worth of candidates (false: capacity exceeded)
-__device__ __forceinline__ bool cand_push(const WarpMem& m, uint32_t& nc, uint32_t C, bool has,
+template <class M>
+__device__ __forceinline__ bool cand_push(const M& m, uint32_t& nc, uint32_t C, bool has,
                                           uint32_t slot, uint32_t off, uint32_t obj, unsigned lt) {
   const unsigned hm = __ballot_sync(0xffffffffu, has);
   if (!hm) return true;
@@ -244,8 +260,8 @@ __device__ __forceinline__ bool cand_push(const WarpMem& m, uint32_t& nc, uint32
 
 // Ask for the flush of every dirty cell the frontier will need, so a retried query is
 // unlikely to stop again for the same reason.
-__device__ void request_lookahead(const QParams& P, const WarpMem& m, const uint32_t* front,
-                                  uint32_t nf, int lane) {
+template <class M, class S>
+__device__ void request_lookahead(const QParams& P, const M& m, const S* front, uint32_t nf, int lane) {
   for (uint32_t i = lane; i < nf; i += 32) {
     const uint32_t v = m.key[front[i]];
     request_flush(P.s, cellof(P.g, v), P.epoch);
@@ -266,7 +282,8 @@ __device__ void finish_undone(const QParams& P, uint32_t qi, int r) {
   }
 }
 
-__device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uint32_t qi, int lane) {
+template <class M>
+__device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t qi, int lane) {
   const unsigned FULL = 0xffffffffu;
   const DevGraph& g = P.g;
   const DevState& s = P.s;
@@ -304,8 +321,8 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
     seed_v = g.edst[q.x];
     seed_d = ei.y - q.y;
   }
-  uint32_t* front = m.front0;
-  uint32_t* nfront = m.front1;
+  auto* front = m.front0;
+  auto* nfront = m.front1;
   uint32_t nf = 1, nc = 0;
   if (lane == 0) {
     bool imp;
@@ -461,6 +478,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
         if (lane >= (uint32_t)o) pre += y;
       }
       const uint32_t n_arc = __shfl_sync(FULL, pre, 31);
+      if (n_arc > STAGE) return OVERFLOW;  // (the next level's table takes it)
       pre -= cnt;
       if (r0) m.stage[pre++] = make_uint2(a01.x, du + a01.y);
       if (r1) m.stage[pre++] = make_uint2(a01.z, du + a01.w);
@@ -691,7 +709,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const WarpMem& m, uin
       cur = nxt;
     }
 #endif
-    uint32_t* tmp = front;
+    auto* tmp = front;
     front = nfront;
     nfront = tmp;
     nf = nn;
@@ -735,10 +753,11 @@ __global__ void k_expand(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
   const uint32_t warp = threadIdx.x >> 5;
-  const size_t wbytes = (warpmem_bytes(P.caps) + 15) & ~size_t(15);
+  using S = typename std::conditional<SMEM, uint16_t, uint32_t>::type;
+  const size_t wbytes = (warpmem_bytes(P.caps, sizeof(S)) + 15) & ~size_t(15);
   const uint32_t gw = blockIdx.x * P.warps_per_cta + warp;
   unsigned char* base = SMEM ? smem_raw + (size_t)warp * wbytes : P.scratch + (size_t)gw * wbytes;
-  const WarpMem m = carve(base, P.caps);
+  const WarpMemT<S> m = carve<S>(base, P.caps);
   pdl_trigger(P);
   for (;;) {  // persistent: queries fetched dynamically
     uint32_t li = 0;
@@ -806,7 +825,7 @@ __device__ __forceinline__ uint32_t hmaxF(const HalfWarp&, uint32_t x) {
 // the larger of the two halves' (half-uniform) values: the shared loop bound of a phase
 __device__ __forceinline__ uint32_t both_max(uint32_t v) { return max(v, __shfl_xor_sync(0xffffffffu, v, 16)); }
 
-__device__ __forceinline__ bool cand_push16(const WarpMem& m, const HalfWarp& W, uint32_t& nc, uint32_t C, bool has,
+__device__ __forceinline__ bool cand_push16(const WarpMemS& m, const HalfWarp& W, uint32_t& nc, uint32_t C, bool has,
                                             uint32_t slot, uint32_t off, uint32_t obj) {
   const unsigned hm = __ballot_sync(W.mask, has) & W.mask;
   if (!hm) return true;
@@ -820,7 +839,7 @@ __device__ __forceinline__ bool cand_push16(const WarpMem& m, const HalfWarp& W,
   return true;
 }
 
-__device__ __forceinline__ bool cand_push16F(const WarpMem& m, const HalfWarp& W, uint32_t& nc, uint32_t C, bool has,
+__device__ __forceinline__ bool cand_push16F(const WarpMemS& m, const HalfWarp& W, uint32_t& nc, uint32_t C, bool has,
                                              uint32_t slot, uint32_t off, uint32_t obj) {
   const unsigned hm = __ballot_sync(0xffffffffu, has) & W.mask;
   if (hm && nc + __popc(hm) > C) return false;
@@ -870,8 +889,8 @@ __global__ void k_expand_pair(QParams P) {
   W.base = W.h * 16;
   W.mask = 0xFFFFu << W.base;
   W.lt = lanemask_lt() & W.mask;
-  const size_t wbytes = (warpmem_bytes(cp) + 15) & ~size_t(15);
-  const WarpMem m = carve(smem_raw + (size_t)(2 * warp + W.h) * wbytes, cp);
+  const size_t wbytes = (warpmem_bytes(cp, 2) + 15) & ~size_t(15);
+  const WarpMemS m = carve<uint16_t>(smem_raw + (size_t)(2 * warp + W.h) * wbytes, cp);
   pdl_trigger(P);
   const bool track = P.remote != nullptr && s.n_ranks > 1;
 
@@ -1018,8 +1037,8 @@ __global__ void k_expand_pair(QParams P) {
         act = false;
       }
     }
-    uint32_t* front = fb ? m.front1 : m.front0;
-    uint32_t* nfront = fb ? m.front0 : m.front1;
+    auto* front = fb ? m.front1 : m.front0;
+    auto* nfront = fb ? m.front0 : m.front1;
 
     // ---- C. partition: the bucket [blo, blo + delta) into act, the rest re-queued
     const uint32_t bhi = (blo > INF - g.delta) ? INF : blo + g.delta;
@@ -1282,7 +1301,7 @@ struct FixCaps {
 };
 
 template <int W, class CP>
-__device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& sh, uint32_t qi) {
+__device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& sh, uint32_t qi) {
   constexpr uint32_t T = W * 32;
   const unsigned FULL = 0xffffffffu;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -1349,8 +1368,8 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
   __syncthreads();
   if (sh.nc > cp.C) return OVERFLOW;
 
-  uint32_t* front = m.front0;
-  uint32_t* nfront = m.front1;
+  auto* front = m.front0;
+  auto* nfront = m.front1;
   // frontier size and minimum: the next frontier holds the re-queued entries (their D read at
   // partition) and every vertex improved during the round (each improvement's new D is seen
   // here), so the minimum over those is exact
@@ -1484,7 +1503,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMem& m, CtaShared<W>& s
 #pragma unroll
     for (int w = 1; w < W; ++w) blo = min(blo, sh.red[par][w]);
     nf = sh.nn[par];
-    uint32_t* tmp = front;
+    auto* tmp = front;
     front = nfront;
     nfront = tmp;
   }
@@ -1560,7 +1579,7 @@ __device__ __forceinline__ void expand_cta_body(const QParams& P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ CtaShared<W> sh;
   __shared__ uint32_t qslot;
-  const WarpMem m = carve(smem_raw, CP::get(P));
+  const WarpMemS m = carve<uint16_t>(smem_raw, CP::get(P));
   pdl_trigger(P);
   for (;;) {  // persistent: queries fetched dynamically
     if (threadIdx.x == 0) {
@@ -1622,7 +1641,7 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 // resident per SM (with 4 warps per CTA: 1,024 -> 896 -> 768 slots = 18 -> 20 -> 24 warps per SM;
 // C3 expansion 1.66 -> 1.46 -> 1.37 ms, 7 promotions per 65,536 queries at 768)
 #ifndef GG_H0W
-#define GG_H0W 768
+#define GG_H0W 704
 #endif
 #ifndef GG_F0
 #define GG_F0 96
@@ -1669,12 +1688,12 @@ static Caps caps_mode(int level, uint32_t V, bool cta) {
   return c;
 }
 static size_t warp_bytes_mode(int level, uint32_t V, bool cta) {
-  return (warpmem_bytes(caps_mode(level, V, cta)) + 15) & ~size_t(15);
+  return (warpmem_bytes(caps_mode(level, V, cta), level == NLEVELS - 1 ? 4 : 2) + 15) & ~size_t(15);
 }
 
 size_t expand_warp_bytes(int level, uint32_t V) {
   const Caps c = caps_for(level, V);
-  return (warpmem_bytes(c) + 15) & ~size_t(15);
+  return (warpmem_bytes(c, level == NLEVELS - 1 ? 4 : 2) + 15) & ~size_t(15);
 }
 
 // CTA-per-query for the shared-memory levels, and for small batches at any of them; the
