@@ -553,6 +553,9 @@ struct TFlushSmem {
   uint32_t hist[HCAP];
 };
 
+#ifndef GG_MBAR_SUSPEND_NS
+#define GG_MBAR_SUSPEND_NS 1000000
+#endif
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(unsigned long long* b, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
@@ -563,11 +566,13 @@ __device__ __forceinline__ void mbar_expect_tx(unsigned long long* b, uint32_t b
 __device__ __forceinline__ void mbar_arrive(unsigned long long* b) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
+// (a suspend-time hint: the waiting warp sleeps until the phase completes instead of spinning
+// through try_wait, which took ~16% of the kernel's issue slots at C3)
 __device__ __forceinline__ void mbar_wait(unsigned long long* b, uint32_t parity) {
   asm volatile(
       "{\n .reg .pred p;\n"
-      "W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W_%=;\n}" ::"r"(smem_u32(b)),
-      "r"(parity)
+      "W_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n @!p bra W_%=;\n}" ::"r"(smem_u32(b)),
+      "r"(parity), "r"(GG_MBAR_SUSPEND_NS)
       : "memory");
 }
 // global -> shared bulk copy (TMA engine; 16-byte aligned, multiple of 16 bytes), evict-first in
