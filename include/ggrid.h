@@ -196,6 +196,8 @@ typedef struct ggrid_stats_t {
   uint32_t n_shards;         /* shards of the index (1: one GPU)                      */
   uint32_t exchange_kind;    /* GGRID_EXCHANGE_* in use (0: none; 3: the caller's all-to-all) */
   uint64_t remote_requests;  /* bounded requests this shard (all shards: summed) sent to others */
+  uint64_t expand_resumes;   /* promoted query runs the next level continued from their exported
+                                state instead of restarting (a subset of expand_promotions) */
 } ggrid_stats_t;
 
 /* Build the index (graph grid, P@11423-15818; object table P@15869; message lists

@@ -72,7 +72,8 @@ class ggrid_stats_t(ctypes.Structure):
                                        "t_delta", "t_now"]] + [("records_expired", ctypes.c_uint64),
                                        ("expand_promotions", ctypes.c_uint64), ("expand_retries", ctypes.c_uint64),
                                        ("seq_rebases", ctypes.c_uint64), ("n_shards", ctypes.c_uint32),
-                                       ("exchange_kind", ctypes.c_uint32), ("remote_requests", ctypes.c_uint64)]
+                                       ("exchange_kind", ctypes.c_uint32), ("remote_requests", ctypes.c_uint64),
+                                       ("expand_resumes", ctypes.c_uint64)]
 
 
 class ggrid_prior_art_knn_result(ctypes.Structure):

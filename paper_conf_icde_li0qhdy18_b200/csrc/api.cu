@@ -388,7 +388,7 @@ int ggrid_free(ggrid_t h) {
   for (DBuf* b : {&h->upd_stage, &h->tmp, &h->q_stage, &h->out_stage, &h->lists, &h->l2_scratch,
                   &h->dump_stage, &h->gc_buf, &h->misc, &h->flush_spill, &h->bound_stage,
                   &h->remote_stage, &h->merge_stage, &h->staged[0].buf,
-                  &h->staged[1].buf, &h->qstaged[0].buf, &h->qstaged[1].buf, &h->chain_ring, &h->qsort_buf})
+                  &h->staged[1].buf, &h->qstaged[0].buf, &h->qstaged[1].buf, &h->chain_ring, &h->qsort_buf, &h->resume_buf})
     b->release();
   for (ggrid_s::Staged* sb : {&h->staged[0], &h->staged[1], &h->qstaged[0], &h->qstaged[1]}) {
     if (sb->done) cudaEventDestroy(sb->done);
@@ -556,6 +556,11 @@ int ggrid_ingest_commit(ggrid_t h) {
   return rc;
 }
 
+// resumable promotions (knn.cu promote_export): on by default; 0 restarts promoted queries
+#ifndef GG_RESUME
+#define GG_RESUME 1
+#endif
+constexpr uint32_t kResumeCap = 4096;  // records per round (~7 KB each at the one-warp level)
 #ifndef GG_BALL_FACTOR
 #define GG_BALL_FACTOR 2.0  // vertex-table slots per expected ball vertex (experiment hook)
 #endif
@@ -688,6 +693,16 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
       RC(h->set_words(ws));
     }
     const bool conc = chain >= 0 && n_in[lvl0] > 0;
+    // the chained level resumes the starting level's promotions from their exported state
+    // (one-warp starting level only; records beyond kResumeCap promote without state)
+    uint32_t resume_cap = 0;
+    if (conc && GG_RESUME) {
+      const size_t rb = expand_resume_bytes(lvl0, n_in[lvl0], h->sm_count, ball_hint);
+      if (rb) {
+        resume_cap = std::min<uint32_t>(n_in[lvl0], kResumeCap);
+        RC(h->resume_buf.ensure(rb * resume_cap));
+      }
+    }
     const uint32_t grid_c = conc ? std::min<uint32_t>(expand_grid(chain, n_q, h->sm_count, ball_hint), n_in[chain] + 16) : 0;
     uint32_t grid0 = 0;
     if (conc) {  // leave room for the chained level's CTAs (so they are resident from the start)
@@ -714,6 +729,10 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
       E.bound = d_bound;
       E.remote = d_remote;
       E.ball_hint = ball_hint;
+      if (resume_cap && (lvl == lvl0 || lvl == chain)) {
+        E.resume = h->resume_buf.p;
+        E.resume_cap = resume_cap;
+      }
       return E;
     };
     for (int lvl = 0; lvl < L; ++lvl) {
@@ -1100,6 +1119,7 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
       t.expand_promotions += x.expand_promotions;
       t.expand_retries += x.expand_retries;
       t.remote_requests += x.remote_requests;
+      t.expand_resumes += x.expand_resumes;
     }
     t.n_queries = h->stats.n_queries;
     t.knn_calls = h->stats.knn_calls;
@@ -1134,6 +1154,7 @@ int ggrid_stats(ggrid_t h, ggrid_stats_t* out) {
   s.exchange_kind = h->xchg ? (strcmp(exchange_name(h->xchg), "nccl") == 0 ? GGRID_EXCHANGE_NCCL : 3u) : 0u;
   s.expand_promotions = h->h_status->ex_promoted;
   s.expand_retries = h->h_status->ex_retried;
+  s.expand_resumes = h->h_status->ex_resumed;
   *out = s;
   return GGRID_OK;
 }

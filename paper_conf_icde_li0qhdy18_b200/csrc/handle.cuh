@@ -157,6 +157,7 @@ struct ggrid_s {
   cudaEvent_t ev_in = nullptr;   // caller's producer stream -> library streams (order_inputs)
   cudaEvent_t ev_out = nullptr;  // library stream -> a caller's stream (ggrid_signal_stream)
   DBuf chain_ring;
+  DBuf resume_buf;  // resumable-promotion records (one per chain-ring slot, up to kResumeCap)
   DBuf qsort_buf;  // (GGRID_SORT_QUERIES experiment)  // queries promoted into the chained level (NONE = not yet written)
   ggrid_stats_t stats{};
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> pending_ev;

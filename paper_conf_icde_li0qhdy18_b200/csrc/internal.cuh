@@ -46,6 +46,7 @@ struct DevStatus {
   unsigned long long ex_iters, ex_vertices, ex_arcs, ex_harvested, ex_objects;  // expansion work
   unsigned long long records_expired;  // dropped unread by t_delta expiry
   unsigned long long ex_promoted, ex_retried;  // expansion outcomes: capacity overflow / dirty cell
+  unsigned long long ex_resumed;  // promoted runs continued from their exported state
   unsigned int ext_top;     // next free extent
   unsigned int err;         // ErrBits of the current knn / flush / gc call
   unsigned int ingest_err;  // ErrBits of the current ingest batch (classify / alloc / scatter)
@@ -314,6 +315,10 @@ struct ExpandLaunch {
   bool trigger = false;             // let the next kernel of the stream start now (PDL)
   bool pdl = false;                 // launched as a programmatic dependent of the previous kernel
   uint32_t ball_hint = 0xFFFFFFFFu;  // expected ball (vertices): picks the starting level's variant
+  // resumable promotions: records (expand_resume_bytes each) indexed by promotion-ring slot,
+  // written by the one-warp starting level and read by the chained level (both get the buffer)
+  void* resume = nullptr;
+  uint32_t resume_cap = 0;
 };
 // CTAs launch_expand uses for n queries at `level` (ball_hint: expected ball in vertices)
 uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint);
@@ -343,6 +348,8 @@ int expand_levels();
 uint32_t expand_table_slots(int level);  // vertex-table capacity H of a level
 uint32_t expand_max_k(int level);
 size_t expand_warp_bytes(int level, uint32_t V);
+// bytes per resumable-promotion record if `level` runs n queries one warp per query, else 0
+size_t expand_resume_bytes(int level, uint32_t n, int sm_count, uint32_t ball_hint);
 void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t* obj,
                       uint32_t* edge, uint32_t* off, uint32_t cap, uint32_t* n_out, cudaStream_t st);
 }  // namespace gg

@@ -29,6 +29,7 @@
 //     (reading R13) and Alg. 6's refinement fused into the same expansion.  Output: the k
 //     smallest (dist<<32 | obj) (readings R5, R6).
 // Capacities are per variant ("level"); a query that overflows one is retried on the next.
+#include <cstdio>
 #include <algorithm>
 #include <type_traits>
 
@@ -39,6 +40,36 @@ namespace gg {
 namespace {
 
 enum { DONE = 0, RETRY = 1, OVERFLOW = 2 };
+// (experiment hook) GG_TAIL_DEBUG=1: printf each level-0 promotion (reason, rounds, time) and each
+// chained-level query's start/end times, to measure the promoted queries' tail
+#ifndef GG_TAIL_DEBUG
+#define GG_TAIL_DEBUG 0
+#endif
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#if GG_TAIL_DEBUG
+#define OVF_AT(why) do { if (lane == 0) printf("P %u %d %u %u %llu\n", qi, (why), c_iter, nn, gtime()); return OVERFLOW; } while (0)
+#else
+#define OVF_AT(why) return OVERFLOW
+#endif
+// An overflow of the one-warp kernel inside a chunk (arc stage, table or frontier full) leaves a
+// state the next level can resume from instead of restarting (see promote_export): the chunk's
+// vertices harvested at this load lose their listed bits (their objects were not read yet) and
+// the chunk and the rest of the bucket act[c0..na) stay to be expanded.
+#define OVF_RES(why)                                                              \
+  do {                                                                            \
+    if (harv) atomicAnd(&m.listed[vslot >> 5], ~(1u << (vslot & 31)));             \
+    rs.ok = true;                                                                 \
+    rs.c0 = c0;                                                                   \
+    rs.na = na;                                                                   \
+    rs.nc = nc;                                                                   \
+    rs.rmask = rmask;                                                             \
+    __syncwarp();                                                                 \
+    OVF_AT(why);                                                                  \
+  } while (0)
 constexpr int MAXP = 128;                  // probe limit of the vertex table
 constexpr uint32_t SPECIAL = 0xFFFFFFFFu;  // candidate slot of a same-arc object
 constexpr uint32_t WMAX = 0xFFFFFFFFu;     // inline-adjacency overflow marker
@@ -189,6 +220,59 @@ __device__ void warp_sort(unsigned long long* a, uint32_t n, uint32_t cap, int l
   }
 }
 
+// State of a query promoted out of the one-warp kernel mid-search (OVF_RES), resumed by the
+// chained level instead of restarted: at C3 the promoted queries (~28 of 65,536, all on a full
+// 704-slot table) overflow after ~90% of their rounds, and a restart at the next level put
+// ~100 us of serial search after the starting level's end.
+struct Resume {
+  bool ok;
+  uint32_t c0, na, nc;
+  unsigned long long rmask;
+};
+// record layout (global memory, one per promotion-ring slot; caps = the exporting level's):
+// header {qi, n_act, nc, valid, rmask}, key[H], dist[H], listed[W], fin[W], act[F], cand[C],
+// cobj[C]  (W = H/32 words; the slots of act/cand refer to the exported table)
+struct RecHdr {
+  uint32_t qi, n_act, nc, valid;
+  unsigned long long rmask;
+  uint32_t pad[2];
+};
+static_assert(sizeof(RecHdr) == 32, "resume record header");
+struct RecView {
+  RecHdr* hdr;
+  uint32_t *key, *dist, *listed, *fin, *act;
+  unsigned long long* cand;
+  uint32_t* cobj;
+};
+__host__ __device__ inline size_t resume_bytes(const Caps& c) {
+  const size_t w = (c.H + 31) / 32;
+  return (sizeof(RecHdr) + 8ull * c.H + 8ull * w + 4ull * (c.F + (c.F & 1u)) + 12ull * c.C + 15) & ~size_t(15);
+}
+__device__ inline RecView rec_view(unsigned char* base, const Caps& c) {
+  RecView r;
+  const uint32_t w = (c.H + 31) / 32;
+  r.hdr = reinterpret_cast<RecHdr*>(base);
+  r.key = reinterpret_cast<uint32_t*>(base + sizeof(RecHdr));
+  r.dist = r.key + c.H;
+  r.listed = r.dist + c.H;
+  r.fin = r.listed + w;
+  r.act = r.fin + w;
+  r.cand = reinterpret_cast<unsigned long long*>(r.act + c.F + (c.F & 1u));  // (8-byte aligned)
+  r.cobj = reinterpret_cast<uint32_t*>(r.cand + c.C);
+  return r;
+}
+
+// slot of a vertex known to be in the table (-1: not found)
+template <class M>
+__device__ __forceinline__ int tab_find(const M& m, uint32_t H, uint32_t v) {
+  uint32_t sl = vhash(v, H);
+  for (int p = 0; p < MAXP; ++p) {
+    if (m.key[sl] == v) return (int)sl;
+    sl = sl + 1 == H ? 0 : sl + 1;
+  }
+  return -1;
+}
+
 struct QParams {
   DevGraph g;
   DevState s;
@@ -216,6 +300,11 @@ struct QParams {
   uint32_t wait_total;
   int trigger;
   int wait_prior;  // launched as a programmatic dependent that must see the previous grid (flush)
+  // resumable promotions (one-warp starting level -> chained level): one record per ring slot
+  unsigned char* resume;
+  uint32_t resume_cap;    // records (ring slots at or past it promote without state)
+  uint32_t resume_bytes;  // bytes per record
+  Caps rcaps;             // the exporting level's capacities (record layout)
 };
 
 // programmatic dependent launch: the next kernel of the stream may start right away (it
@@ -229,7 +318,12 @@ __device__ __forceinline__ void pdl_trigger(const QParams& P) {
 __device__ __forceinline__ void count_exit(const QParams& P) {
   if (P.exited) {
     __threadfence();
-    atomicAdd(P.exited, 1u);
+    const uint32_t o = atomicAdd(P.exited, 1u);
+#if GG_TAIL_DEBUG
+    if (o + 1 == gridDim.x) printf("E %llu\n", gtime());
+#else
+    (void)o;
+#endif
   }
 }
 
@@ -277,13 +371,66 @@ __device__ void finish_undone(const QParams& P, uint32_t qi, int r) {
   } else if (P.level < P.last_level) {
     atomicAdd(&P.s.st->ex_promoted, 1ull);
     P.promote_list[atomicAdd(P.promote_count, 1u)] = qi;
+#if GG_TAIL_DEBUG
+    printf("Q %u %llu\n", qi, gtime());
+#endif
   } else {
     atomicOr(&P.s.st->err, (unsigned)ERR_FAIL);
   }
 }
 
+// Promotion of a query that overflowed the one-warp kernel, to the chained level: the ring slot
+// is taken first, the working state (OVF_RES) is written to that slot's record, then the ring
+// entry is published (fence: a reader that sees the entry sees the record).  A state that cannot
+// be resumed (rs.ok false) is published with valid = 0 and the next level restarts the query.
 template <class M>
-__device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t qi, int lane) {
+__device__ void promote_export(const QParams& P, const M& m, uint32_t qi, int lane, const Resume& rs) {
+  uint32_t t = 0;
+  if (lane == 0) {
+    atomicAdd(&P.s.st->ex_promoted, 1ull);
+    t = atomicAdd(P.promote_count, 1u);
+  }
+  t = __shfl_sync(0xffffffffu, t, 0);
+  if (t < P.resume_cap) {
+    const Caps& c = P.caps;
+    const RecView r = rec_view(P.resume + (size_t)t * P.resume_bytes, c);
+    const uint32_t n_act = rs.ok ? rs.na - rs.c0 : 0;
+    if (rs.ok) {
+      for (uint32_t i = lane; i < c.H; i += 32) {
+        r.key[i] = m.key[i];
+        r.dist[i] = m.dist[i];
+      }
+      for (uint32_t i = lane; i < (c.H + 31) / 32; i += 32) {
+        r.listed[i] = m.listed[i];
+        r.fin[i] = m.fin[i];
+      }
+      for (uint32_t i = lane; i < n_act; i += 32) r.act[i] = m.act[rs.c0 + i];
+      for (uint32_t i = lane; i < rs.nc; i += 32) {
+        r.cand[i] = m.cand[i];
+        r.cobj[i] = m.cobj[i];
+      }
+    }
+    if (lane == 0) {
+      RecHdr h;
+      h.qi = qi;
+      h.n_act = n_act;
+      h.nc = rs.ok ? rs.nc : 0;
+      h.valid = rs.ok ? 1u : 0u;
+      h.rmask = rs.rmask;
+      h.pad[0] = h.pad[1] = 0;
+      *r.hdr = h;
+    }
+    __threadfence();
+  }
+  __syncwarp();
+#if GG_TAIL_DEBUG
+  if (lane == 0) printf("Q %u %llu\n", qi, gtime());
+#endif
+  if (lane == 0) P.promote_list[t] = qi;
+}
+
+template <class M>
+__device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t qi, int lane, Resume& rs) {
   const unsigned FULL = 0xffffffffu;
   const DevGraph& g = P.g;
   const DevState& s = P.s;
@@ -478,7 +625,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
         if (lane >= (uint32_t)o) pre += y;
       }
       const uint32_t n_arc = __shfl_sync(FULL, pre, 31);
-      if (n_arc > STAGE) return OVERFLOW;  // (the next level's table takes it)
+      if (n_arc > STAGE) OVF_RES(1);  // (the next level's table takes it)
       pre -= cnt;
       if (r0) m.stage[pre++] = make_uint2(a01.x, du + a01.y);
       if (r1) m.stage[pre++] = make_uint2(a01.z, du + a01.w);
@@ -509,9 +656,9 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
             }
           }
         }
-        if (__any_sync(FULL, ovf)) return OVERFLOW;
+        if (__any_sync(FULL, ovf)) OVF_RES(2);
         const unsigned hm = __ballot_sync(FULL, has);
-        if (nn + __popc(hm) > cp.F) return OVERFLOW;
+        if (nn + __popc(hm) > cp.F) OVF_RES(3);
         if (has) nfront[nn + __popc(hm & lt)] = nslot;
         nn += __popc(hm);
       }
@@ -546,9 +693,9 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
               }
             }
           }
-          if (__any_sync(FULL, ovf)) return OVERFLOW;
+          if (__any_sync(FULL, ovf)) OVF_RES(2);
           const unsigned hm = __ballot_sync(FULL, has);
-          if (nn + __popc(hm) > cp.F) return OVERFLOW;
+          if (nn + __popc(hm) > cp.F) OVF_RES(3);
           if (has) nfront[nn + __popc(hm & lt)] = nslot;
           nn += __popc(hm);
         }
@@ -580,7 +727,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
             const bool same_ahead = q.y > 0 && oe == q.x && oo >= q.y;  // already a candidate
             hc = !same_ahead && (!GG_HARVEST_VALIDATE || kk == s.ot_key[ob]);
           }
-          if (!cand_push(m, nc, cp.C, hc, vslot, oo, ob, lt)) return OVERFLOW;
+          if (!cand_push(m, nc, cp.C, hc, vslot, oo, ob, lt)) OVF_AT(4);
         }
       }
     }
@@ -765,8 +912,15 @@ __global__ void k_expand(QParams P) {
     li = __shfl_sync(0xffffffffu, li, 0);
     if (li >= P.n) break;
     const uint32_t qi = P.qlist ? P.qlist[li] : li;
-    const int r = run_query(P, m, qi, lane);
-    if (lane == 0 && r != DONE) finish_undone(P, qi, r);
+    Resume rs;
+    rs.ok = false;
+    rs.rmask = 0;
+    const int r = run_query(P, m, qi, lane, rs);
+    if (SMEM && r == OVERFLOW && P.resume) {
+      promote_export(P, m, qi, lane, rs);
+    } else if (lane == 0 && r != DONE) {
+      finish_undone(P, qi, r);
+    }
     __syncwarp();
   }
   __syncthreads();  // (the chained level waits for every CTA -- all of its warps -- to exit)
@@ -1301,7 +1455,8 @@ struct FixCaps {
 };
 
 template <int W, class CP>
-__device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& sh, uint32_t qi) {
+__device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& sh, uint32_t qi,
+                             uint32_t rslot) {
   constexpr uint32_t T = W * 32;
   const unsigned FULL = 0xffffffffu;
   const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -1337,43 +1492,111 @@ __device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& 
     if (o != s.rank) rmask |= 1ull << o;
   }
   const uint32_t seed_d = q.y == 0 ? 0u : ei.y - q.y;
-  if (tid == 0) {
-    const uint32_t seed_v = q.y == 0 ? ei.x : g.edst[q.x];
-    bool imp;
-    const int sl = tab_relax(m, H, seed_v, seed_d, imp);
-    m.front0[0] = (uint32_t)sl;
-    m.fin[sl >> 5] |= 1u << (sl & 31);
-  }
-  // objects on q's own arc ahead of q (reading R2), stored at vertex src(q.e)
-  if (q.y > 0) {
-    const uint32_t c = cellof(g, ei.x);
-    if (s.cell_head[c] != NONE) {
-      if (tid == 0) request_flush(s, c, P.epoch);
-      return RETRY;
+  uint32_t nf = 1, blo = seed_d;
+  // a query promoted with its state (promote_export): the record's table, frontier (its fin
+  // bits plus the unexpanded rest of its bucket), listed bits and candidates are re-hashed into
+  // this level's table, and the search continues from there
+  const RecView rv = rslot != NONE ? rec_view(P.resume + (size_t)rslot * P.resume_bytes, P.rcaps) : RecView{};
+  const bool resumed = rslot != NONE && __ldcg(&rv.hdr->valid) == 1u && __ldcg(&rv.hdr->qi) == qi;
+  if (resumed) {
+    const uint32_t H0 = P.rcaps.H;
+    for (uint32_t i = tid; i < H0; i += T) {
+      const uint32_t v = __ldcg(rv.key + i);
+      if (v == EMPTY32) continue;
+      bool imp;
+      const int sl = tab_relax(m, H, v, __ldcg(rv.dist + i), imp);
+      if (sl < 0) {
+        atomicOr(&sh.flags, FL_OVF);
+        continue;
+      }
+      const uint32_t bit = 1u << (sl & 31);
+      if (__ldcg(rv.listed + (i >> 5)) & (1u << (i & 31))) atomicOr(&m.listed[sl >> 5], bit);
+      if ((__ldcg(rv.fin + (i >> 5)) & (1u << (i & 31))) && !(atomicOr(&m.fin[sl >> 5], bit) & bit)) {
+        const uint32_t p = atomicAdd(&sh.nn[1], 1u);
+        if (p < cp.F) m.front0[p] = (uint16_t)sl;
+      }
     }
-    const uint2 vo = vobj_valid(s.v_obj[ei.x], s.cell_comp[c]);
-    for (uint32_t j = tid; j < vo.y; j += T) {
-      const uint32_t p = vo.x + j;
-      const uint32_t ob = s.ar.obj[p];
-      const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
-      if (oe == q.x && oo >= q.y && valid_rec(s, p, ob)) {
-        const uint32_t i = atomicAdd(&sh.nc, 1u);
-        if (i < cp.C) {
-          m.cand[i] = ((unsigned long long)SPECIAL << 32) | (oo - q.y);
-          m.cobj[i] = ob;
+    __syncthreads();
+    const uint32_t n_act = __ldcg(&rv.hdr->n_act), nc0 = __ldcg(&rv.hdr->nc);
+    for (uint32_t j = tid; j < n_act; j += T) {
+      const int sl = tab_find(m, H, __ldcg(rv.key + __ldcg(rv.act + j)));
+      if (sl < 0) {
+        atomicOr(&sh.flags, FL_OVF);
+        continue;
+      }
+      const uint32_t bit = 1u << (sl & 31);
+      if (!(atomicOr(&m.fin[sl >> 5], bit) & bit)) {
+        const uint32_t p = atomicAdd(&sh.nn[1], 1u);
+        if (p < cp.F) m.front0[p] = (uint16_t)sl;
+      }
+    }
+    for (uint32_t j = tid; j < nc0 && j < cp.C; j += T) {
+      const unsigned long long a = __ldcg(rv.cand + j);
+      const uint32_t s0 = (uint32_t)(a >> 32);
+      int ns = (int)SPECIAL;
+      if (s0 != SPECIAL) {
+        ns = tab_find(m, H, __ldcg(rv.key + s0));
+        if (ns < 0) atomicOr(&sh.flags, FL_OVF);
+      }
+      m.cand[j] = ((unsigned long long)(uint32_t)ns << 32) | (uint32_t)a;
+      m.cobj[j] = __ldcg(rv.cobj + j);
+    }
+    if (tid == 0) {
+      sh.nc = nc0;
+      rmask |= __ldcg(&rv.hdr->rmask);
+      atomicAdd(&s.st->ex_resumed, 1ull);
+    }
+    __syncthreads();
+    nf = sh.nn[1];
+    if (nf > cp.F || nc0 > cp.C || (sh.flags & FL_OVF)) return OVERFLOW;
+    uint32_t mn = INF;
+    for (uint32_t i = tid; i < nf; i += T) mn = min(mn, m.dist[m.front0[i]]);
+    mn = __reduce_min_sync(FULL, mn);
+    if (lane == 0) sh.red[1][wid] = mn;
+    __syncthreads();
+    blo = sh.red[1][0];
+#pragma unroll
+    for (int w = 1; w < W; ++w) blo = min(blo, sh.red[1][w]);
+    // (sh.nn[1] and sh.red[1] are round 1's: round 0 resets nn[1] after its bucket barrier,
+    // which every thread passes after reading nf above)
+  } else {
+    if (tid == 0) {
+      const uint32_t seed_v = q.y == 0 ? ei.x : g.edst[q.x];
+      bool imp;
+      const int sl = tab_relax(m, H, seed_v, seed_d, imp);
+      m.front0[0] = (uint32_t)sl;
+      m.fin[sl >> 5] |= 1u << (sl & 31);
+    }
+    // objects on q's own arc ahead of q (reading R2), stored at vertex src(q.e)
+    if (q.y > 0) {
+      const uint32_t c = cellof(g, ei.x);
+      if (s.cell_head[c] != NONE) {
+        if (tid == 0) request_flush(s, c, P.epoch);
+        return RETRY;
+      }
+      const uint2 vo = vobj_valid(s.v_obj[ei.x], s.cell_comp[c]);
+      for (uint32_t j = tid; j < vo.y; j += T) {
+        const uint32_t p = vo.x + j;
+        const uint32_t ob = s.ar.obj[p];
+        const uint32_t oe = s.ar.edge[p], oo = s.ar.off[p];
+        if (oe == q.x && oo >= q.y && valid_rec(s, p, ob)) {
+          const uint32_t i = atomicAdd(&sh.nc, 1u);
+          if (i < cp.C) {
+            m.cand[i] = ((unsigned long long)SPECIAL << 32) | (oo - q.y);
+            m.cobj[i] = ob;
+          }
         }
       }
     }
+    __syncthreads();
+    if (sh.nc > cp.C) return OVERFLOW;
   }
-  __syncthreads();
-  if (sh.nc > cp.C) return OVERFLOW;
 
   auto* front = m.front0;
   auto* nfront = m.front1;
   // frontier size and minimum: the next frontier holds the re-queued entries (their D read at
   // partition) and every vertex improved during the round (each improvement's new D is seen
   // here), so the minimum over those is exact
-  uint32_t nf = 1, blo = seed_d;
   uint32_t c_iter = 0, c_vert = 0, c_arcs = 0, c_harv = 0, c_objs = 0;
   for (uint32_t rnd = 0;; ++rnd) {
     const uint32_t par = rnd & 1;
@@ -1538,6 +1761,9 @@ __device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& 
     }
   }
   const uint32_t sa = block_sum<W>(c_arcs, sh), sh_ = block_sum<W>(c_harv, sh), so = block_sum<W>(c_objs, sh);
+#if GG_TAIL_DEBUG
+  if (tid == 0 && P.level > 0) printf("W %u %u %u %u\n", qi, c_iter, c_vert, sa);
+#endif
   if (tid == 0) {
     atomicAdd(&s.st->ex_iters, (unsigned long long)c_iter);
     atomicAdd(&s.st->ex_vertices, (unsigned long long)c_vert);
@@ -1578,13 +1804,14 @@ template <int W, class CP>
 __device__ __forceinline__ void expand_cta_body(const QParams& P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ CtaShared<W> sh;
-  __shared__ uint32_t qslot;
+  __shared__ uint32_t qslot, rslot;
   const WarpMemS m = carve<uint16_t>(smem_raw, CP::get(P));
   pdl_trigger(P);
   for (;;) {  // persistent: queries fetched dynamically
     if (threadIdx.x == 0) {
       const uint32_t li = atomicAdd(&P.s.st->expand_work[P.level], 1u);
       uint32_t qi = NONE;
+      rslot = NONE;
       if (li < P.n) {
         qi = P.qlist ? P.qlist[li] : li;
       } else if (P.chain_in && li - P.n < P.chain_cap) {
@@ -1601,6 +1828,10 @@ __device__ __forceinline__ void expand_cta_body(const QParams& P) {
           if (v != NONE) {
             qi = v;
             *slot = NONE;  // (the ring is all-NONE again when the level has drained it)
+            if (P.resume && li - P.n < P.resume_cap) {
+              __threadfence();  // (the record was written before the entry)
+              rslot = li - P.n;
+            }
             break;
           }
           __nanosleep(1000);
@@ -1609,11 +1840,17 @@ __device__ __forceinline__ void expand_cta_body(const QParams& P) {
       qslot = qi;
     }
     __syncthreads();
-    const uint32_t qi = qslot;
+    const uint32_t qi = qslot, rs = rslot;
     __syncthreads();
     if (qi == NONE) break;
-    const int r = run_query_cta<W, CP>(P, m, sh, qi);
+#if GG_TAIL_DEBUG
+    const unsigned long long t0 = gtime();
+#endif
+    const int r = run_query_cta<W, CP>(P, m, sh, qi, rs);
     if (threadIdx.x == 0 && r != DONE) finish_undone(P, qi, r);
+#if GG_TAIL_DEBUG
+    if (threadIdx.x == 0 && P.level > 0) printf("L %u %d %llu %llu\n", qi, r, t0, gtime());
+#endif
     __syncthreads();
   }
   if (threadIdx.x == 0) count_exit(P);
@@ -1708,6 +1945,13 @@ static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   return true;
 }
 
+// bytes of one resumable-promotion record when `level` starts a batch of n queries with the
+// one-warp kernel (which exports the state of the queries it promotes), else 0
+size_t expand_resume_bytes(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
+  if (level >= NLEVELS - 2 || use_cta(level, n, sm_count, ball_hint) || (GG_PAIR && level == 0)) return 0;
+  return resume_bytes(caps_mode(level, 1, false));
+}
+
 // one-warp-per-query kernel: warps (independent queries) per CTA.  Each CTA costs 1 KB of reserved
 // shared memory beside its warps' tables, so several warps per CTA fit more queries per SM
 #ifndef GG_WARP_WPC
@@ -1786,6 +2030,16 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.wait_total = L.wait_total;
   P.trigger = L.trigger ? 1 : 0;
   P.wait_prior = L.chain_in ? 0 : 1;  // (a chained level runs beside the level below it)
+  P.resume = nullptr;
+  P.resume_cap = 0;
+  P.resume_bytes = 0;
+  P.rcaps = Caps{0, 0, 0};
+  if (L.resume && L.resume_cap) {  // (the exporting level: this one, or the one below a chained level)
+    P.rcaps = caps_mode(L.chain_in ? level - 1 : level, g.V, false);
+    P.resume = static_cast<unsigned char*>(L.resume);
+    P.resume_cap = L.resume_cap;
+    P.resume_bytes = (uint32_t)resume_bytes(P.rcaps);
+  }
   const int smem = (int)warp_bytes_mode(level, g.V, cta_mode);
   if (level == NLEVELS - 1) {
     P.scratch = static_cast<unsigned char*>(L.scratch);

@@ -580,6 +580,30 @@ def test_ladder_boundaries_and_promotions(gg):
     grid.close()
 
 
+def test_resumed_promotions_one_warp_level(gg):
+    """The one-warp starting level (dense objects: expected ball ~90 vertices) with every object in
+    the western half of the graph: eastern queries overflow the 704-slot table mid-search and are
+    promoted WITH their state (knn.cu promote_export) to the chained level, which re-hashes it and
+    continues; those that overflow there too restart at the levels above.  Every row the
+    oracle's, and the resume path ran."""
+    g = synth.table_ii_graph("NY", scale=0.2)
+    rng = np.random.default_rng(11)
+    west = np.nonzero(g["x"][g["src"]] < np.quantile(g["x"], 0.5))[0]
+    n = 6000
+    arc = rng.choice(west, n).astype(np.int64)
+    off = np.minimum((rng.random(n) * g["w"][arc]).astype(np.int64), g["w"][arc].astype(np.int64) - 1)
+    upd = np.stack([np.arange(n), arc, off, np.ones(n, np.int64)], 1).astype(np.uint32)
+    q = synth.queries(g, 1500, seed=77)
+    grid = gg.GGrid(g, 256, max_objects=n)
+    grid.ingest(upd)
+    for k in (10, 20):
+        _assert_same(grid.knn(q, k), _oracle(g, upd, q, k), f"k={k}")
+    st = grid.stats()
+    assert st["expand_promotions"] > 0
+    assert st["expand_resumes"] > 0
+    grid.close()
+
+
 def test_moved_objects_leave_clean_cells_stale(gg):
     """Objects jumping between cells every round (uniform random relocation, 4-vertex cells):
     the cell an object left is marked STALE at ingest and re-cleaned before its list is read,
