@@ -99,12 +99,17 @@ typedef struct ggrid_opts {
                               leaves its seq range unused.  Ignored (synchronous)
                               when t_delta != 0.  0 = default, synchronous.         */
   uint32_t ingest_kernels; /* 0 = default: a batch that fits one resident wave
-                              (<= 8,192 updates per SM and few enough distinct cells
-                              per SM tile for shared memory) is ingested by ONE
+                              (<= 8,192 updates per SM) is ingested by ONE
                               cooperative launch (classify, extent allocation and
-                              scatter separated by grid barriers), larger batches by
-                              three launches; 3 = always the three launches.  Both
-                              produce the same index state.                        */
+                              scatter separated by grid barriers) -- the direct
+                              variant (one rank atomic per update, no shared
+                              memory) when an SM tile would average under two
+                              updates per distinct cell, else the shared-memory
+                              cell-hash variant when its hash fits -- and larger
+                              batches by three launches.  1 = the cell-hash
+                              launch whenever it fits; 2 = the direct launch
+                              whenever it fits; 3 = always the three launches.
+                              All produce the same index state.                    */
   /* ---- multi-GPU (see "multi-GPU" below).  All 0 = one GPU.            */
   uint32_t n_gpus;         /* > 1: ONE index over n_gpus shards driven by this process,
                               shard r on devices[r] (cell ownership, one request/reply

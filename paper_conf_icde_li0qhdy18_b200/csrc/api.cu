@@ -222,7 +222,7 @@ static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts
   h->t_delta = o.t_delta;
   // the expiry cut reads t_now on the host, so expiry keeps ingest synchronous
   h->async_ingest = (o.async_ingest && !o.t_delta) ? 1 : 0;
-  h->fused_ingest = o.ingest_kernels == 3 ? 0 : 1;
+  h->ingest_mode = o.ingest_kernels <= 3 ? (int)o.ingest_kernels : 0;
   if (const char* fk = getenv("GGRID_FLUSH_KERNEL")) h->flush_kernel = atoi(fk);  // (experiment hook)
   h->s.n_ranks = 1;
   h->s.rank = 0;
@@ -359,6 +359,7 @@ static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts
   if ((rc = h->alloc(&s.bcount, (size_t)h->n_cells * BCOUNT_STRIDE))) return fail(rc);
   if ((rc = h->alloc(&s.bbase, h->n_cells))) return fail(rc);
   if ((rc = h->alloc(&s.flush_list, h->n_cells))) return fail(rc);
+  if ((rc = h->alloc(&s.ovf_list, h->n_cells))) return fail(rc);
   if ((rc = h->alloc(&h->d_status, 1))) return fail(rc);
   s.st = h->d_status;
   if (cudaMallocHost((void**)&h->h_status, sizeof(DevStatus)) != cudaSuccess) return fail(GGRID_ENOMEM);
@@ -419,7 +420,7 @@ int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
   RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
   IngestPlan fp;
-  const bool fused = h->fused_ingest && ingest_fused_plan(n, h->n_cells, h->sm_count, &fp);
+  const bool fused = h->ingest_mode != 3 && ingest_fused_plan(n, h->n_cells, h->sm_count, h->ingest_mode, &fp);
   if (!fused) RC(h->tmp.ensure(ingest_tmp_bytes(n)));
   {
     WordSet ws;
@@ -683,7 +684,7 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
     // round 0 cleans what the seed requested: c_q and its neighbour cells per query
     const uint64_t seeded = seed_all ? h->n_cells : (uint64_t)n_q * (h->seed_neighbors ? h->max_cell_degree + 1 : 2);
     RC(h->flush_list_run(s.ar, &h->d_status->arena_top, flush_begin, 0,
-                         round == 0 ? (uint32_t)std::min<uint64_t>(seeded, 1u << 30) : 0));
+                         round == 0 ? (uint32_t)std::min<uint64_t>(seeded, 1u << 30) : 0, round == 0));
     if (round > 0) {  // round 0 was reset with the rest at the start
       WordSet ws;
       ws.zero_range(h->d_status->n_next, EXPAND_LEVELS);

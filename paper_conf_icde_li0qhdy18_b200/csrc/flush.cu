@@ -410,8 +410,12 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
   pdl_allow();  // the expansion may launch now (it waits for this grid before reading)
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const unsigned lt = lanemask_lt();
-  const uint32_t lend = *((volatile unsigned*)&s.st->n_flush);
-  if (blockIdx.x == 0 && tid == 0) s.st->flush_end = lend;
+  // begin == OVF_PASS: the cells k_flush_warp left (s.ovf_list), not the request list
+  const bool ovf_pass = begin == OVF_PASS;
+  const uint32_t* __restrict__ flist = ovf_pass ? s.ovf_list : s.flush_list;
+  const uint32_t lend = *((volatile unsigned*)(ovf_pass ? &s.st->n_ovf : &s.st->n_flush));
+  if (ovf_pass) begin = 0;
+  else if (blockIdx.x == 0 && tid == 0) s.st->flush_end = lend;
   const uint32_t G = gridDim.x;
   const uint32_t first_li = begin + blockIdx.x;
   const uint32_t n_mine = first_li < lend ? (lend - first_li + G - 1) / G : 0;
@@ -442,7 +446,7 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
     const uint32_t c = pc, head = ph;
     const uint2 comp = pcomp;
     if (k + 1 < n_mine) {
-      pc = s.flush_list[first_li + (k + 1) * G];
+      pc = flist[first_li + (k + 1) * G];
       ph = s.cell_head[pc];
       pcomp = s.cell_comp[pc];
     }
@@ -453,7 +457,7 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
   };
 
   if (is_index && lane == 0 && n_mine) {
-    pc = s.flush_list[first_li];
+    pc = flist[first_li];
     ph = s.cell_head[pc];
     pcomp = s.cell_comp[pc];
     gather(0);
@@ -482,6 +486,186 @@ __global__ void __launch_bounds__(FT, GG_FLUSH_MINB) k_flush(DevGraph g, DevStat
       __syncwarp();
     }
     __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Warp-per-cell variant for short logs (a step's few dozen new records per cell, C3: ~43 new + ~43
+// listed): the CTA-per-cell pipelines above run a CTA's cells one after another through one index
+// warp, so a flush of every cell costs ~23 cells x the index warp's dependent chain per CTA.
+// Here each warp takes whole cells from a dynamic counter and runs every phase of one cell
+// itself -- chain walk, match (records in flight 4 per lane), winner payload gather, rank by
+// source vertex, scatter of R[c] -- with no CTA barrier: ~8k cells are in flight on the GPU at
+// once instead of ~1k.  Same arithmetic as index_cell (the staged, rank path).  A cell with more
+// than XW extents or more than WW winners is left to the CTA kernel: queued on ovf_list, which
+// the launcher hands to k_flush right after.
+constexpr int XW = 32;    // extents (including the cleaned list) per cell
+constexpr int WW = 128;   // winners per cell
+constexpr int FW = 8;     // warps per CTA
+struct WarpFlushSmem {
+  uint32_t xs[XW], xp[XW + 1];
+  uint32_t w_pos[WW], w_obj[WW], w_vs[WW], w_off[WW], w_edge[WW];
+  unsigned long long w_key[WW];
+};
+
+__global__ void __launch_bounds__(FW * 32, 5) k_flush_warp(DevGraph g, DevState s, Arena out,
+                                                          unsigned long long* out_top, uint32_t begin,
+                                                          uint32_t* ovf_list, uint32_t t_cut) {
+  __shared__ WarpFlushSmem wsm[FW];
+  pdl_wait();   // (a programmatic dependent of the seed / status reset)
+  pdl_allow();  // the overflow pass / expansion may launch now (they wait for this grid)
+  const int lane = threadIdx.x & 31;
+  WarpFlushSmem& m = wsm[threadIdx.x >> 5];
+  const unsigned lt = lanemask_lt();
+  const unsigned long long* __restrict__ otk = s.ot_key;
+  const uint32_t lend = *((volatile unsigned*)&s.st->n_flush);
+  if (blockIdx.x == 0 && threadIdx.x == 0) s.st->flush_end = lend;
+  unsigned long long n_written = 0, n_cells = 0, n_rec = 0, n_exp = 0;
+  for (;;) {
+    uint32_t li = 0;
+    if (lane == 0) li = atomicAdd(&s.st->flush_work, 1u);
+    li = begin + __shfl_sync(0xffffffffu, li, 0);
+    if (li >= lend) break;
+    const uint32_t c = s.flush_list[li];
+    const uint32_t head = s.cell_head[c];
+    const uint2 comp = s.cell_comp[c];
+    // ---- the cell's record sequence: its extents newest first (unexpired), then its cleaned list
+    uint32_t nx = 0, tot = 0, nexp = 0;
+    bool ovf = false;
+    if (lane == 0) {
+      uint32_t e = head;
+      while (is_extent(e)) {
+        const uint32_t st = s.x_start[e], ln = s.x_len[e], nxt = s.x_next[e];
+        if (t_cut && s.x_tmax[e] < t_cut) {
+          nexp += ln;
+        } else if (nx + 1 >= (uint32_t)XW) {
+          ovf = true;
+          break;
+        } else if (ln) {
+          m.xs[nx] = st;
+          m.xp[nx] = tot;
+          tot += ln;
+          ++nx;
+        }
+        e = nxt;
+      }
+      if (comp.y) {
+        m.xs[nx] = comp.x;
+        m.xp[nx] = tot;
+        tot += comp.y;
+        ++nx;
+      }
+      m.xp[nx] = tot;
+    }
+    nx = __shfl_sync(0xffffffffu, nx, 0);
+    tot = __shfl_sync(0xffffffffu, tot, 0);
+    ovf = __shfl_sync(0xffffffffu, ovf, 0);
+    __syncwarp();
+    // ---- match: the record whose key equals ot_key[obj] is its object's latest (R8)
+    uint32_t n_win = 0;
+    for (uint32_t b0 = 0; b0 < tot && !ovf; b0 += 128) {
+      uint32_t p[4], o[4];
+      unsigned long long k[4], tg[4];
+      int xj = 0;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t L = b0 + u * 32 + lane;
+        p[u] = NONE;
+        if (L < tot) {
+          while (m.xp[xj + 1] <= L) ++xj;
+          p[u] = m.xs[xj] + (L - m.xp[xj]);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        o[u] = p[u] != NONE ? __ldcs(s.ar.obj + p[u]) : 0u;
+        k[u] = p[u] != NONE ? __ldcs(s.ar.key + p[u]) : 0ull;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) tg[u] = p[u] != NONE ? __ldg(otk + o[u]) : ~k[u];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const bool hit = tg[u] == k[u];
+        const unsigned hm = __ballot_sync(0xffffffffu, hit);
+        const uint32_t w = n_win + __popc(hm & lt);
+        if (hit && w < (uint32_t)WW) {
+          m.w_pos[w] = p[u];
+          m.w_obj[w] = o[u];
+          m.w_key[w] = k[u];
+        }
+        n_win += __popc(hm);
+      }
+      if (n_win > (uint32_t)WW) ovf = true;
+    }
+    if (ovf) {  // the CTA kernel's spill / re-stream paths take it (right after this launch)
+      if (lane == 0) ovf_list[atomicAdd(&s.st->n_ovf, 1u)] = c;
+      continue;
+    }
+    __syncwarp();
+    // ---- R[c]: payload gather, then each winner's slot = its rank by (source vertex, index)
+    unsigned long long o0 = 0;
+    if (lane == 0) o0 = atomicAdd(out_top, (n_win + 3u) & ~3ull);
+    for (uint32_t i = lane; i < n_win; i += 32) {
+      const uint32_t pp = m.w_pos[i];
+      m.w_vs[i] = s.ar.vsrc[pp];
+      m.w_off[i] = s.ar.off[pp];
+      m.w_edge[i] = s.ar.edge[pp];
+    }
+    o0 = __shfl_sync(0xffffffffu, o0, 0);
+    __syncwarp();
+    if (o0 + ((n_win + 3u) & ~3ull) > out.cap) {
+      if (lane == 0) atomicOr(&s.st->err, (unsigned)ERR_ARENA);
+      continue;  // the cell stays dirty
+    }
+    const uint32_t cbeg = c * g.cs;
+    if (GG_VHAS) {  // the cell's "may hold objects" bits: cleared, then set for the new list
+      const uint32_t nvert = min(g.cs, g.V - cbeg);
+      for (uint32_t wd = (cbeg >> 5) + lane; wd <= ((cbeg + nvert - 1) >> 5); wd += 32) {
+        const uint32_t lo = max(cbeg, wd << 5), hi = min(cbeg + nvert, (wd << 5) + 32);
+        const uint32_t span = hi - lo;
+        const uint32_t mask = (span == 32 ? 0xFFFFFFFFu : ((1u << span) - 1u)) << (lo & 31);
+        atomicAnd(&s.vhas[wd], ~mask);
+      }
+      __syncwarp();
+    }
+    for (uint32_t i = lane; i < n_win; i += 32) {
+      const uint32_t vi = m.w_vs[i];
+      uint32_t r = 0, cv = 0;
+      bool first = true;
+      for (uint32_t j = 0; j < n_win; ++j) {
+        const uint32_t vj = m.w_vs[j];
+        r += (vj < vi) | ((vj == vi) & (j < i));
+        cv += vj == vi;
+        first &= !((vj == vi) & (j < i));
+      }
+      const uint32_t q = (uint32_t)o0 + r;
+      s.listed_cell[m.w_obj[i]] = c;
+      out.obj[q] = m.w_obj[i];
+      out.key[q] = m.w_key[i];
+      out.vsrc[q] = vi;
+      out.off[q] = m.w_off[i];
+      out.edge[q] = m.w_edge[i];
+      if (first) {
+        s.v_obj[vi] = make_uint2(q, cv);
+        if (GG_VHAS) atomicOr(&s.vhas[vi >> 5], 1u << (vi & 31));
+      }
+    }
+    if (lane == 0) {
+      s.cell_comp[c] = make_uint2((uint32_t)o0, n_win);
+      s.cell_head[c] = NONE;
+      s.cell_pending[c] = 0;
+    }
+    n_written += n_win;
+    n_cells += 1;
+    n_rec += tot;
+    n_exp += nexp;
+    __syncwarp();  // (the staging is rewritten by the next cell)
+  }
+  if (lane == 0 && n_cells) {
+    atomicAdd(&s.st->objects_written, n_written);
+    atomicAdd(&s.st->cells_flushed, n_cells);
+    atomicAdd(&s.st->records_flushed, n_rec);
+    if (n_exp) atomicAdd(&s.st->records_expired, n_exp);
   }
 }
 
@@ -850,11 +1034,28 @@ int blocks_per_sm_t(bool tma);
 template <int HCAP, int WCAP>
 void launch_t(const DevGraph& g, const DevState& s, const Arena& out, unsigned long long* out_top,
               uint32_t begin, int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap,
-              uint32_t t_cut, uint32_t max_ctas, bool tma, cudaStream_t st) {
+              uint32_t t_cut, uint32_t max_ctas, int mode, cudaStream_t st) {
+  const bool tma = mode == FLUSH_TMA;
+  cudaLaunchAttribute attr[1];
+  if (mode == FLUSH_WARP) {  // warp-per-cell pass (the caller then runs k_flush over OVF_PASS)
+    static int wbps[64] = {0};  // occupancy per device ordinal (set on first use)
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int& wb = wbps[dev & 63];
+    if (!wb) {
+      int b = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_flush_warp, FW * 32, 0);
+      wb = std::max(b, 1);
+    }
+    uint32_t wgrid = (uint32_t)(sm_count * wb);
+    if (max_ctas && max_ctas < wgrid) wgrid = max_ctas;
+    const cudaLaunchConfig_t wcfg = pdl_config(dim3(wgrid), dim3(FW * 32), 0, st, attr);
+    cudaLaunchKernelEx(&wcfg, k_flush_warp, g, s, out, out_top, begin, s.ovf_list, t_cut);
+    return;
+  }
   const int blocks_per_sm = blocks_per_sm_t<HCAP, WCAP>(tma);
   uint32_t grid = (uint32_t)(sm_count * blocks_per_sm);
   if (max_ctas && max_ctas < grid) grid = max_ctas;  // few cells to clean: fewer idle CTAs
-  cudaLaunchAttribute attr[1];
   if (tma) {
     const cudaLaunchConfig_t cfg = pdl_config(dim3(grid), dim3(TFT), sizeof(TFlushSmem<HCAP, WCAP>), st, attr);
     cudaLaunchKernelEx(&cfg, k_flush_tma<HCAP, WCAP>, g, s, out, out_top, begin, full_vobj, spill, spill_cap, t_cut);
@@ -925,8 +1126,8 @@ size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, u
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
                   int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap, uint32_t t_cut,
-                  uint32_t max_ctas, int tma, cudaStream_t st) {
-  const bool t = tma != 0;
+                  uint32_t max_ctas, int mode, cudaStream_t st) {
+  const int t = mode;
   switch (flush_variant(g.cs, objects_per_cell)) {
     case 0: launch_t<1024, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;
     case 1: launch_t<4096, 128>(g, s, out, out_top, begin, full_vobj, sm_count, spill, spill_cap, t_cut, max_ctas, t, st); break;

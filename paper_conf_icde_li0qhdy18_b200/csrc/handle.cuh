@@ -111,7 +111,7 @@ struct ggrid_s {
   // Until the next sync the status mirror is stale by the batches queued since; these bound
   // what they can have added (records incl. extent padding, extents, newly live objects).
   int async_ingest = 0;
-  int fused_ingest = 1;  // opts.ingest_kernels: one cooperative launch when the batch fits
+  int ingest_mode = 0;  // opts.ingest_kernels: 0 plan, 1 cell-hash launch, 2 direct launch, 3 three launches
   uint64_t pend_records = 0, pend_updates = 0;
   uint32_t pend_ext = 0;
   uint32_t max_cell_degree = 0;  // most neighbour cells of any cell
@@ -127,7 +127,7 @@ struct ggrid_s {
   // the whole index are re-based (rebase()), so a handle takes any number of updates.
   uint64_t seq_next = 1;
   uint64_t recs_since_flush = 0;  // records ingested since the last flush launch (kernel choice)
-  int flush_kernel = 0;           // GGRID_FLUSH_KERNEL: 0 = by log length, 1 = ring, 2 = streaming
+  int flush_kernel = 0;           // GGRID_FLUSH_KERNEL: 0 = by log length, 1 = ring, 2 = streaming, 3 = warp per cell
   uint64_t n_ingested = 0;  // updates accepted (or queued, asynchronous) so far
   uint64_t rebases = 0;
   uint32_t epoch = 0;
@@ -255,8 +255,9 @@ struct ggrid_s {
     return set_words(ws);
   }
 
+  // fresh: st->flush_work and st->n_ovf were zeroed since the last flush (a knn's round 0)
   int flush_list_run(const Arena& out, unsigned long long* out_top, uint32_t begin, int full_vobj = 0,
-                     uint32_t max_cells = 0) {
+                     uint32_t max_cells = 0, bool fresh = false) {
     const uint32_t opc = (uint32_t)((n_live_hi() + n_cells - 1) / std::max(1u, n_cells));
     uint32_t spill_cap = 0;
     const size_t sb = flush_spill_bytes(g.cs, opc, sm_count, &spill_cap);
@@ -269,12 +270,27 @@ struct ggrid_s {
     // bulk-copy ring; short ones (a few dozen records per cell per step) through the streaming
     // kernel, whose per-cell fixed cost is lower (C3 r2f: full flush 0.244 -> 0.224 ms with the
     // ring; the 1M-update step's flush 0.126 -> 0.155 ms with it)
+    // (the warp-per-cell kernel for a step's short logs: one warp runs every phase of a cell, with
+    // no CTA barrier; C3's 1M-update step flush 0.126 -> see DESIGN.md section 12)
     const uint64_t per_cell = recs_since_flush / std::max(1u, n_cells);
-    const int tma = flush_kernel == 1 || (flush_kernel == 0 && per_cell >= 512);
+    int mode = FLUSH_STREAM;
+    if (flush_kernel == 1 || (flush_kernel == 0 && per_cell >= 512)) mode = FLUSH_TMA;
+    else if (!full_vobj && (flush_kernel == 3 || (flush_kernel == 0 && per_cell <= 128))) mode = FLUSH_WARP;
+    if (mode == FLUSH_WARP && !fresh) {  // the warp kernel's cell counter and overflow list
+      WordSet ws;
+      ws.add(&d_status->flush_work, 0u);
+      ws.add(&d_status->n_ovf, 0u);
+      RC(set_words(ws));
+    }
     launch(GGRID_K_FLUSH, [&] {
-      launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, spill, spill_cap, t_cut, max_cells, tma,
+      launch_flush(g, s, out, out_top, begin, opc, full_vobj, sm_count, spill, spill_cap, t_cut, max_cells, mode,
                    stream);
     });
+    if (mode == FLUSH_WARP)  // the cells with more extents or winners than a warp stages
+      launch(GGRID_K_FLUSH, [&] {
+        launch_flush(g, s, out, out_top, OVF_PASS, opc, 0, sm_count, spill, spill_cap, t_cut,
+                     max_cells ? max_cells : (uint32_t)sm_count, FLUSH_STREAM, stream);
+      });
     if (begin == 0) recs_since_flush = 0;
     return GGRID_OK;
   }

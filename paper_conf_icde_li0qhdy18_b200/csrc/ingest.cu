@@ -8,6 +8,10 @@
 //   alloc    : one thread per cell carves this batch's extent for the cell out of the
 //              bump arena (warp-aggregated) and links it at the head of the cell's chain;
 //   scatter  : writes the SoA record and RED.MAX-es (t<<32|seq) into ot_key[o].
+// A batch that fits one resident wave runs the same three phases as ONE cooperative launch
+// with grid barriers between them: k_ingest_fused (per-tile cell hash in shared memory, for
+// batches with many updates per distinct cell) or k_ingest_direct (one rank atomic per
+// update, state in registers, for batches spread over many more cells than a tile holds).
 // No tombstones: a record is valid iff its key equals ot_key[obj] (reading R8/R9), which
 // also makes out-of-order arrivals harmless.
 #include <algorithm>
@@ -540,6 +544,122 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
   }
 }
 
+// ---------------------------------------------------------------------------------------
+// Direct single-launch ingest for a batch of at most one resident wave x DPT updates whose
+// tiles hit nearly as many distinct cells as they hold updates (C3's step: 1M updates over
+// 23k cells, ~0.3 updates per (tile, cell)), where a per-tile cell hash aggregates nothing and
+// only adds its shared-memory passes: every update takes its rank in its cell's batch extent
+// with one returning atomic on the cell's counter line, keeps (cell, rank, source vertex) in
+// registers across the two grid barriers (no shared memory, no tmp/perm round trip), and the
+// scatter re-reads its record from L2.  Same arithmetic and rejection rules as the paths above.
+constexpr int DT = 512;   // threads per CTA (2 CTAs per SM)
+constexpr int DPT = 8;    // updates per thread at most
+constexpr uint32_t RK_NEW = 1u << 30, RK_ZERO = 1u << 31;  // rank flags: key newer / key read 0
+constexpr uint32_t RK_MASK = RK_NEW - 1;
+
+__global__ void __launch_bounds__(DT, 2) k_ingest_direct(const uint4* __restrict__ upd, uint64_t n,
+                                                         uint32_t seq0, DevGraph g, DevState s) {
+  pdl_wait();   // (a programmatic dependent of the batch's status reset)
+  pdl_allow();  // the next kernel may launch; it waits for this grid
+  const uint32_t T = gridDim.x * DT;
+  const uint32_t tid = blockIdx.x * DT + threadIdx.x;
+  const int lane = threadIdx.x & 31;
+  uint32_t cl[DPT], rk[DPT], vs[DPT];  // cell (NONE: no update, REMOTE_CELL), rank | flags, src
+  uint32_t tl = 0;
+  constexpr int HP = 2;  // (quarters: registers)
+#pragma unroll
+  for (int hf = 0; hf < DPT / HP; ++hf) {  // a part's loads and gathers in flight together
+    uint4 mm[HP];
+    uint2 ee[HP];
+    unsigned long long ck[HP];
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      const uint64_t i = (uint64_t)(hf * HP + q) * T + tid;
+      mm[q] = i < n ? __ldg(upd + i) : make_uint4(0, 0xFFFFFFFFu, 0, 0);  // (re-read from L2)
+    }
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      ee[q] = mm[q].y < g.A ? __ldg(g.einfo + mm[q].y) : make_uint2(0, 1);
+      ck[q] = mm[q].x < s.max_objects ? __ldcg(s.ot_key + mm[q].x) : 0ull;
+    }
+#pragma unroll
+    for (int q = 0; q < HP; ++q) {
+      const int j = hf * HP + q;
+      const uint64_t i = (uint64_t)j * T + tid;
+      cl[j] = NONE;
+      rk[j] = 0;
+      vs[j] = 0;
+      if (i >= n) continue;
+      const uint4 m = mm[q];
+      const uint2 e = ee[q];
+      unsigned bad = 0;
+      if (m.x >= s.max_objects) bad |= ERR_OBJ;
+      if (m.y >= g.A) {
+        bad |= ERR_EDGE;
+      } else if (m.z >= e.y) {
+        bad |= ERR_OFF;
+      }
+      if (bad) {
+        atomicOr(&s.st->ingest_err, bad);
+        atomicMin(&s.st->bad_index, i < 0xFFFFFFFFull ? (unsigned)i : 0xFFFFFFFFu);
+        continue;
+      }
+      const unsigned long long key = ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
+      const uint32_t c0 = cellof(g, e.x);
+      const bool remote = s.n_ranks > 1 && owner_of(c0, g.n_cells, s.n_ranks) != s.rank;
+      cl[j] = remote ? REMOTE_CELL : c0;
+      vs[j] = e.x;
+      rk[j] = (key > ck[q] ? RK_NEW : 0u) | (ck[q] == 0ull ? RK_ZERO : 0u);
+      if (!remote) atomicMax(&s.bcount[c0 * BCOUNT_STRIDE + 1], m.w);  // the extent's zeta.t
+      tl = max(tl, m.w);
+    }
+  }
+  // ranks: one returning atomic per update, all of a thread's in flight together
+#pragma unroll
+  for (int j = 0; j < DPT; ++j) {
+    if (cl[j] < REMOTE_CELL) rk[j] |= atomicAdd(&s.bcount[cl[j] * BCOUNT_STRIDE], 1u);
+  }
+  tl = __reduce_max_sync(0xffffffffu, tl);
+  if (lane == 0 && tl) atomicMax(&s.st->batch_tmax, tl);  // (folded into t_max once accepted)
+
+  // ---- alloc: every rank is taken; one extent per (batch, cell)
+  const unsigned G = gridDim.x;
+  grid_barrier(&s.st->ingest_bar, G);
+  {
+    const bool err = *((volatile unsigned*)&s.st->ingest_err) != 0;
+    commit_batch_tmax(s, err);
+    const uint32_t nw = G * (DT / 32);
+    for (uint32_t c0 = (blockIdx.x * (DT / 32) + (threadIdx.x >> 5)) * 32; c0 < g.n_cells; c0 += nw * 32)
+      alloc_cell_warp(g, s, c0 + lane, err);
+  }
+  grid_barrier(&s.st->ingest_bar, 2 * G);
+  if (*((volatile unsigned*)&s.st->ingest_err)) return;  // the batch is rejected as a whole
+
+  // ---- scatter: record j of this thread to its cell's extent at bbase + rank
+#pragma unroll
+  for (int j = 0; j < DPT; ++j) {
+    if (cl[j] == NONE) continue;
+    const uint64_t i = (uint64_t)j * T + tid;
+    const uint4 m = __ldg(upd + i);
+    const uint32_t pos = cl[j] < REMOTE_CELL ? s.bbase[cl[j]] + (rk[j] & RK_MASK) : NONE;
+    const unsigned long long key = ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
+    mark_moved(s, m.x, cellof(g, vs[j]));
+    if (pos != NONE) {  // (NONE: a cell another rank owns)
+      s.ar.obj[pos] = m.x;
+      s.ar.key[pos] = key;
+      s.ar.vsrc[pos] = vs[j];
+      s.ar.off[pos] = m.z;
+      s.ar.edge[pos] = m.y;
+    }
+    if (rk[j] & RK_ZERO) {
+      const unsigned long long old = atomicMax(&s.ot_key[m.x], key);
+      if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+    } else if (rk[j] & RK_NEW) {
+      atomicMax(&s.ot_key[m.x], key);
+    }
+  }
+}
+
 // a tile whose 2-slots-per-cell hash does not fit shared memory: fused with a hash of one slot
 // per update (1) or the three-launch path (0; measured faster at C3's 1M-update step, r2i: 0.144
 // vs 0.170 ms -- probe chains at 82% load)
@@ -550,8 +670,24 @@ static size_t fused_smem(uint32_t tile, uint32_t ch) {
   return (size_t)ch * 12 + (size_t)tile * 8 + (size_t)((tile + 1) & ~1u) * 2 + (FT / 32) * 4;
 }
 
-bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p) {
+// mode: 0 = choose (direct when an SM tile would average under two updates per distinct cell),
+// 1 = the cell-hash launch only, 2 = the direct launch whenever it fits
+bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, int mode, IngestPlan* p) {
   if (n == 0 || sm_count <= 0) return false;
+  p->direct = false;
+  const uint64_t dgrid = (uint64_t)sm_count * 2;  // (2 CTAs of DT threads per SM)
+  if (mode != 1 && n <= dgrid * DT * DPT) {
+    const uint64_t tile = (n + sm_count - 1) / sm_count;  // a cell-hash tile: one CTA per SM
+    if (mode == 2 || tile <= 2ull * n_cells) {
+      p->direct = true;
+      // >= 2 updates per thread (all SMs once the batch is large); dgrid x DT x DPT >= n
+      p->grid = (uint32_t)std::min<uint64_t>(dgrid, (n + 2ull * DT - 1) / (2ull * DT));
+      p->tile = 0;
+      p->ch = 0;
+      p->smem = 0;
+      return true;
+    }
+  }
   const uint64_t grid = std::min<uint64_t>((uint64_t)sm_count, std::max<uint64_t>(1, (n + 2047) / 2048));
   const uint64_t tile = (n + grid - 1) / grid;
   if (tile > FUSED_TILE) return false;
@@ -577,6 +713,14 @@ bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p
 
 cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                                 const DevState& s, const IngestPlan& p, cudaStream_t st) {
+  if (p.direct) {
+    cudaLaunchAttribute attr[2];
+    cudaLaunchConfig_t cfg = pdl_config(dim3(p.grid), dim3(DT), 0, st, attr);
+    attr[1].id = cudaLaunchAttributeCooperative;
+    attr[1].val.cooperative = 1;
+    cfg.numAttrs = 2;
+    return cudaLaunchKernelEx(&cfg, k_ingest_direct, upd, n, seq0, g, s);
+  }
   const cudaError_t ae = func_attr_once(k_ingest_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   if (ae != cudaSuccess) return ae;
   // cooperative (every CTA resident at once, or the launch fails: the grid barriers need it) and

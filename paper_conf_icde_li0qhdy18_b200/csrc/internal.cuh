@@ -61,6 +61,7 @@ struct DevStatus {
   unsigned int expand_work[EXPAND_LEVELS];  // per-level dynamic work counters of the expand launches
   unsigned int n_chain;     // queries the starting level promoted into the chained level this round
   unsigned int l0_exited;   // CTAs of the starting level's launch that have exited this round
+  unsigned int n_ovf;       // entries in ovf_list (this round's warp-per-cell flush)
   unsigned int round_end;   // (marks the end of the per-round reset region)
   unsigned int ingest_bar;  // grid-barrier arrivals of the fused ingest launch (reset per batch)
   unsigned int batch_tmax;  // newest t of the current ingest batch's valid updates (reset per
@@ -113,6 +114,7 @@ struct DevState {
                            // CTA serialise in L2)
   uint32_t* bbase;         // [n_cells] per-batch arena base
   uint32_t* flush_list;    // [n_cells]
+  uint32_t* ovf_list;      // [n_cells] cells k_flush_warp left to the CTA kernel (st->n_ovf)
   DevStatus* st;
   // cell ownership across ranks: rank r owns the contiguous Z-order range of
   // cells c with floor(c * n_ranks / n_cells) == r; only owned cells keep logs and lists
@@ -239,8 +241,9 @@ size_t ingest_tmp_bytes(uint64_t n);
 struct IngestPlan {
   uint32_t grid, tile, ch;
   size_t smem;
+  bool direct;  // k_ingest_direct (per-update rank atomics, registers across the barriers)
 };
-bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, IngestPlan* p);
+bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, int mode, IngestPlan* p);
 cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                                 const DevState& s, const IngestPlan& p, cudaStream_t st);  // classify -> scatter scratch (tmp + perm)
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);
@@ -261,11 +264,15 @@ void launch_mark_dirty(const DevGraph& g, const DevState& s, uint32_t epoch, int
 size_t flush_spill_bytes(uint32_t cs, uint32_t objects_per_cell, int sm_count, uint32_t* cap);
 // t_cut: extents whose newest t is below it are expired (dropped unread); 0 = none.
 // max_ctas: an upper bound on the cells listed (0 = unknown): caps the persistent grid
-// tma: the bulk-copy ring kernel (k_flush_tma; long cell logs) instead of the streaming one
+// mode: FLUSH_STREAM the CTA-per-cell streaming kernel (k_flush), FLUSH_TMA its bulk-copy ring
+// variant (k_flush_tma; long cell logs), FLUSH_WARP one warp per cell (k_flush_warp; short logs)
+// followed by k_flush over the cells it could not take (s.ovf_list)
+enum FlushMode { FLUSH_STREAM = 0, FLUSH_TMA = 1, FLUSH_WARP = 2 };
+constexpr uint32_t OVF_PASS = 0xFFFFFFFFu;  // k_flush's `begin` for the overflow pass
 void launch_flush(const DevGraph& g, const DevState& s, const Arena& out,
                   unsigned long long* out_top, uint32_t begin, uint32_t objects_per_cell,
                   int full_vobj, int sm_count, uint32_t* spill, uint32_t spill_cap, uint32_t t_cut,
-                  uint32_t max_ctas, int tma, cudaStream_t st);
+                  uint32_t max_ctas, int mode, cudaStream_t st);
 
 // v_obj[v] = (start, n) is valid only if start lies inside the cell's current cleaned list
 // (lists only move up the arena between garbage collections, which rewrite every entry).

@@ -1,10 +1,11 @@
-"""The two ingest paths (opts.ingest_kernels) against the oracle (-m gpu).
+"""The ingest paths (opts.ingest_kernels) against the oracle (-m gpu).
 
 Alg. 1 (P@18177-19248) caches each message in the log of cell(src(e)); the index state it
-leaves must be the same whichever launch structure builds it: the single cooperative launch
-(classify / extent allocation / scatter separated by grid barriers; default for a batch that
-fits one resident wave) or the three-launch path (ingest_kernels=3; also the default's
-fallback for larger batches).  Bit-exact: cleaned cells equal the oracle's latest-per-object
+leaves must be the same whichever launch structure builds it: a single cooperative launch
+(classify / extent allocation / scatter separated by grid barriers) in its cell-hash variant
+(ingest_kernels=1) or its direct variant (one rank atomic per update, ingest_kernels=2) --
+the default picks one for a batch that fits one resident wave -- or the three-launch path
+(ingest_kernels=3; also the default's fallback for larger batches).  Bit-exact: cleaned cells equal the oracle's latest-per-object
 snapshot, kNN rows equal the full-Dijkstra oracle's.
 """
 import numpy as np
@@ -44,7 +45,7 @@ def _same(got, ref, msg):
     assert np.array_equal(got[0], ref[0]) and np.array_equal(got[1], ref[1]), msg
 
 
-@pytest.mark.parametrize("mode", [0, 3])
+@pytest.mark.parametrize("mode", [0, 1, 2, 3])
 def test_ingest_paths_same_state(gg, mode):
     """Multi-CTA batches (300k updates over a 53k-vertex graph, 207 cells of 256 vertices);
     a batch with one bad record in its middle is rejected whole by both paths."""
@@ -61,7 +62,7 @@ def test_ingest_paths_same_state(gg, mode):
     grid.ingest(upd[half:])
     st = grid.stats()
     assert st["n_updates"] == len(upd)
-    if mode == 0:
+    if mode != 3:
         assert st["kernel_launches"]["ingest_alloc"] == 0  # one launch per batch
     else:
         assert st["kernel_launches"]["ingest_alloc"] == 3
@@ -93,11 +94,12 @@ def test_fused_fallback_beyond_one_wave(gg):
     grid.close()
 
 
-def test_fused_many_small_batches(gg):
+@pytest.mark.parametrize("mode", [0, 1, 2])
+def test_fused_many_small_batches(gg, mode):
     """Single-update and tiny batches (one CTA, grid barrier of one) interleaved with queries."""
     g = synth.lattice_graph(16, 16, 1, 4)
     walk = synth.RandomWalk(g, 50, inject=True)
-    grid = gg.GGrid(g, 16, max_objects=64)
+    grid = gg.GGrid(g, 16, max_objects=64, ingest_kernels=mode)
     hist = []
     for r in range(6):
         u = walk.ticks(1)
@@ -173,7 +175,7 @@ def test_async_ingest_input_reuse_after_signal(gg):
     grid.close()
 
 
-@pytest.mark.parametrize("mode", [0, 3])
+@pytest.mark.parametrize("mode", [0, 1, 2, 3])
 def test_rejected_batch_leaves_t_now(gg, mode):
     """A rejected batch changes no observable state (ggrid.h): its valid records' far-future
     t must not become t_now of the expiry rule (reading R21), which would expire every cached

@@ -79,13 +79,13 @@ def test_c0_interleaved_rounds_lazy_equals_eager(gg):
     eager.close()
 
 
-@pytest.mark.parametrize("kernel", ["auto", "ring", "streaming"])
+@pytest.mark.parametrize("kernel", ["auto", "ring", "streaming", "warp"])
 def test_flush_parity_and_cells(gg, kernel, monkeypatch):
     """After ggrid_flush_all the cells' object lists are exactly the oracle's latest-per-object
     snapshot, each object once, in the cell of its arc's source vertex; flushing twice is a
-    no-op (idempotent).  Both flush kernels (the bulk-copy ring and the streaming one; GGRID_FLUSH_KERNEL
-    forces one, `auto` picks by log length per cell)."""
-    monkeypatch.setenv("GGRID_FLUSH_KERNEL", {"auto": "0", "ring": "1", "streaming": "2"}[kernel])
+    no-op (idempotent).  Every flush kernel (the bulk-copy ring, the streaming one and the
+    warp-per-cell one; GGRID_FLUSH_KERNEL forces one, `auto` picks by log length per cell)."""
+    monkeypatch.setenv("GGRID_FLUSH_KERNEL", {"auto": "0", "ring": "1", "streaming": "2", "warp": "3"}[kernel])
     g = synth.table_ii_graph("NY", scale=0.05)
     upd = synth.RandomWalk(g, 2000, inject=True).ticks(12)
     grid = gg.GGrid(g, 256, max_objects=4096)
@@ -627,7 +627,7 @@ def test_moved_objects_leave_clean_cells_stale(gg):
     grid.close()
 
 
-@pytest.mark.parametrize("kernel", ["1", "2"])
+@pytest.mark.parametrize("kernel", ["1", "2", "3"])
 def test_flush_kernels_interleaved_rounds(gg, kernel, monkeypatch):
     """Interleaved ingest / query rounds with either flush kernel forced (long chains of small
     extents, STALE cells, cleaned lists re-read): every round the oracle's answer."""
@@ -643,4 +643,37 @@ def test_flush_kernels_interleaved_rounds(gg, kernel, monkeypatch):
             grid.ingest(u)
         q = synth.queries(g, 200, seed=900 + r)
         _assert_same(grid.knn(q, 8), _oracle(g, np.concatenate(hist), q, 8), f"kernel {kernel} round {r}")
+    grid.close()
+
+
+@pytest.mark.parametrize("case", ["many_winners", "long_chains"])
+def test_flush_warp_overflow_cells(gg, case, monkeypatch):
+    """The warp-per-cell flush leaves a cell with more winners than it stages (WW = 128: 4096-vertex
+    cells of ~500 objects) or more extents than it walks (XW = 32: 40 batches between queries) to
+    the CTA kernel's overflow pass; cells of both kinds and ordinary ones in one flush, every round
+    the oracle's answer, and the cleaned cells the oracle's snapshot."""
+    monkeypatch.setenv("GGRID_FLUSH_KERNEL", "3")
+    g = synth.table_ii_graph("NY", scale=0.05)
+    walk = synth.RandomWalk(g, 2000, inject=True)
+    cs = 4096 if case == "many_winners" else 128
+    grid = gg.GGrid(g, cs, max_objects=2000)
+    hist = []
+    for r in range(3):
+        for _ in range(40 if case == "long_chains" else 2):
+            u = walk.ticks(1)
+            if case == "long_chains":
+                u = u[:300]
+            hist.append(u)
+            grid.ingest(u)
+        q = synth.queries(g, 150, seed=1200 + r)
+        _assert_same(grid.knn(q, 9), _oracle(g, np.concatenate(hist), q, 9), f"{case} round {r}")
+    grid.flush_all()
+    vcell = grid.vertex_cell()
+    rows = []
+    for c in range(grid.stats()["n_cells"]):
+        o, e, d = grid.cell_objects(c)
+        assert np.all(vcell[g["src"][e]] == c)
+        rows += list(zip(o.tolist(), e.tolist(), d.tolist()))
+    ids, e, d = oracle.snapshot_objects(np.concatenate(hist))
+    assert sorted(rows) == sorted(zip(ids.tolist(), e.tolist(), d.tolist()))
     grid.close()
