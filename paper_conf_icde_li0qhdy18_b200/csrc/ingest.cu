@@ -15,6 +15,7 @@
 // No tombstones: a record is valid iff its key equals ot_key[obj] (reading R8/R9), which
 // also makes out-of-order arrivals harmless.
 #include <algorithm>
+#include <cstdio>
 
 #include "internal.cuh"
 
@@ -553,42 +554,63 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
 // registers across the two grid barriers (no shared memory, no tmp/perm round trip), and the
 // scatter re-reads its record from L2.  Same arithmetic and rejection rules as the paths above.
 constexpr int DT = 512;   // threads per CTA (2 CTAs per SM)
+// (experiment hook) GG_INGEST_TIMING=1: phase timestamps of the first and last CTA, printed
+#ifndef GG_INGEST_TIMING
+#define GG_INGEST_TIMING 0
+#endif
+#if GG_INGEST_TIMING
+#define DTIME(k) unsigned long long _t##k; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(_t##k))
+#define DTIME_PRINT()                                                                              \
+  if (threadIdx.x == 0 && (blockIdx.x == 0 || blockIdx.x == gridDim.x - 1))                        \
+    printf("ingest_direct cta %u: p1 %llu bar1 %llu alloc %llu bar2 %llu scatter %llu ns\n", blockIdx.x, \
+           _t1 - _t0, _t2 - _t1, _t3 - _t2, _t4 - _t3, _t5 - _t4)
+#else
+#define DTIME(k)
+#define DTIME_PRINT()
+#endif
 constexpr int DPT = 8;    // updates per thread at most
-constexpr uint32_t RK_NEW = 1u << 30, RK_ZERO = 1u << 31;  // rank flags: key newer / key read 0
-constexpr uint32_t RK_MASK = RK_NEW - 1;
+// rank flags: a cell another rank owns / key newer than the one read / key read was 0
+constexpr uint32_t RK_REMOTE = 1u << 29, RK_NEW = 1u << 30, RK_ZERO = 1u << 31;
+constexpr uint32_t RK_MASK = RK_REMOTE - 1;
 
 __global__ void __launch_bounds__(DT, 2) k_ingest_direct(const uint4* __restrict__ upd, uint64_t n,
                                                          uint32_t seq0, DevGraph g, DevState s) {
   pdl_wait();   // (a programmatic dependent of the batch's status reset)
   pdl_allow();  // the next kernel may launch; it waits for this grid
+  DTIME(0);
   const uint32_t T = gridDim.x * DT;
   const uint32_t tid = blockIdx.x * DT + threadIdx.x;
   const int lane = threadIdx.x & 31;
-  uint32_t cl[DPT], rk[DPT], vs[DPT];  // cell (NONE: no update, REMOTE_CELL), rank | flags, src
+  // per update: source vertex (NONE: no update; its cell is cellof), rank | flags, and the cell
+  // whose cleaned list the object leaves (R8's STALE mark; NONE: none)
+  uint32_t rk[DPT], vs[DPT], lv[DPT];
   uint32_t tl = 0;
-  constexpr int HP = 2;  // (quarters: registers)
+  constexpr int HP = 2;  // (parts of 2: registers)
 #pragma unroll
   for (int hf = 0; hf < DPT / HP; ++hf) {  // a part's loads and gathers in flight together
     uint4 mm[HP];
     uint2 ee[HP];
     unsigned long long ck[HP];
+    uint32_t lc[HP];
 #pragma unroll
     for (int q = 0; q < HP; ++q) {
       const uint64_t i = (uint64_t)(hf * HP + q) * T + tid;
       mm[q] = i < n ? __ldg(upd + i) : make_uint4(0, 0xFFFFFFFFu, 0, 0);  // (re-read from L2)
     }
 #pragma unroll
-    for (int q = 0; q < HP; ++q) {
+    for (int q = 0; q < HP; ++q) {  // one memory round: inverted index, object key, listed cell
+      const bool ok = mm[q].x < s.max_objects;
       ee[q] = mm[q].y < g.A ? __ldg(g.einfo + mm[q].y) : make_uint2(0, 1);
-      ck[q] = mm[q].x < s.max_objects ? __ldcg(s.ot_key + mm[q].x) : 0ull;
+      ck[q] = ok ? __ldcg(s.ot_key + mm[q].x) : 0ull;
+      lc[q] = ok ? s.listed_cell[mm[q].x] : NONE;
     }
 #pragma unroll
     for (int q = 0; q < HP; ++q) {
       const int j = hf * HP + q;
       const uint64_t i = (uint64_t)j * T + tid;
-      cl[j] = NONE;
       rk[j] = 0;
-      vs[j] = 0;
+      vs[j] = NONE;
+      lv[j] = NONE;
       if (i >= n) continue;
       const uint4 m = mm[q];
       const uint2 e = ee[q];
@@ -607,9 +629,9 @@ __global__ void __launch_bounds__(DT, 2) k_ingest_direct(const uint4* __restrict
       const unsigned long long key = ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
       const uint32_t c0 = cellof(g, e.x);
       const bool remote = s.n_ranks > 1 && owner_of(c0, g.n_cells, s.n_ranks) != s.rank;
-      cl[j] = remote ? REMOTE_CELL : c0;
       vs[j] = e.x;
-      rk[j] = (key > ck[q] ? RK_NEW : 0u) | (ck[q] == 0ull ? RK_ZERO : 0u);
+      lv[j] = (lc[q] != NONE && lc[q] != c0) ? lc[q] : NONE;
+      rk[j] = (key > ck[q] ? RK_NEW : 0u) | (ck[q] == 0ull ? RK_ZERO : 0u) | (remote ? RK_REMOTE : 0u);
       if (!remote) atomicMax(&s.bcount[c0 * BCOUNT_STRIDE + 1], m.w);  // the extent's zeta.t
       tl = max(tl, m.w);
     }
@@ -617,47 +639,78 @@ __global__ void __launch_bounds__(DT, 2) k_ingest_direct(const uint4* __restrict
   // ranks: one returning atomic per update, all of a thread's in flight together
 #pragma unroll
   for (int j = 0; j < DPT; ++j) {
-    if (cl[j] < REMOTE_CELL) rk[j] |= atomicAdd(&s.bcount[cl[j] * BCOUNT_STRIDE], 1u);
+    if (vs[j] != NONE && !(rk[j] & RK_REMOTE)) rk[j] |= atomicAdd(&s.bcount[cellof(g, vs[j]) * BCOUNT_STRIDE], 1u);
   }
   tl = __reduce_max_sync(0xffffffffu, tl);
   if (lane == 0 && tl) atomicMax(&s.st->batch_tmax, tl);  // (folded into t_max once accepted)
 
   // ---- alloc: every rank is taken; one extent per (batch, cell)
   const unsigned G = gridDim.x;
+  DTIME(1);
   grid_barrier(&s.st->ingest_bar, G);
+  DTIME(2);
   {
     const bool err = *((volatile unsigned*)&s.st->ingest_err) != 0;
     commit_batch_tmax(s, err);
+    // an accepted batch marks the cells its objects leave STALE (mark_moved; a cell that also gets
+    // an extent here is dirty either way, so the order against the allocation does not matter)
+    if (!err) {
+#pragma unroll
+      for (int j = 0; j < DPT; ++j)
+        if (lv[j] != NONE) atomicCAS(&s.cell_head[lv[j]], NONE, STALE);
+    }
     const uint32_t nw = G * (DT / 32);
     for (uint32_t c0 = (blockIdx.x * (DT / 32) + (threadIdx.x >> 5)) * 32; c0 < g.n_cells; c0 += nw * 32)
       alloc_cell_warp(g, s, c0 + lane, err);
   }
+  DTIME(3);
   grid_barrier(&s.st->ingest_bar, 2 * G);
+  DTIME(4);
   if (*((volatile unsigned*)&s.st->ingest_err)) return;  // the batch is rejected as a whole
 
-  // ---- scatter: record j of this thread to its cell's extent at bbase + rank
+  // ---- scatter: record j of this thread to its cell's extent at bbase + rank (parts of 4: every
+  //      load of a part in flight before its stores)
+  uint32_t* __restrict__ a_obj = s.ar.obj;
+  unsigned long long* __restrict__ a_key = s.ar.key;
+  uint32_t* __restrict__ a_vsrc = s.ar.vsrc;
+  uint32_t* __restrict__ a_off = s.ar.off;
+  uint32_t* __restrict__ a_edge = s.ar.edge;
+  constexpr int SP = 4;
 #pragma unroll
-  for (int j = 0; j < DPT; ++j) {
-    if (cl[j] == NONE) continue;
-    const uint64_t i = (uint64_t)j * T + tid;
-    const uint4 m = __ldg(upd + i);
-    const uint32_t pos = cl[j] < REMOTE_CELL ? s.bbase[cl[j]] + (rk[j] & RK_MASK) : NONE;
-    const unsigned long long key = ((unsigned long long)m.w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
-    mark_moved(s, m.x, cellof(g, vs[j]));
-    if (pos != NONE) {  // (NONE: a cell another rank owns)
-      s.ar.obj[pos] = m.x;
-      s.ar.key[pos] = key;
-      s.ar.vsrc[pos] = vs[j];
-      s.ar.off[pos] = m.z;
-      s.ar.edge[pos] = m.y;
+  for (int h = 0; h < DPT / SP; ++h) {
+    uint4 m[SP];
+    uint32_t pos[SP];
+#pragma unroll
+    for (int q = 0; q < SP; ++q) {
+      const int j = h * SP + q;
+      const uint64_t i = (uint64_t)j * T + tid;
+      const bool own = vs[j] != NONE && !(rk[j] & RK_REMOTE);
+      m[q] = vs[j] != NONE ? __ldg(upd + i) : make_uint4(0, 0, 0, 0);
+      pos[q] = own ? __ldcg(s.bbase + cellof(g, vs[j])) + (rk[j] & RK_MASK) : NONE;
     }
-    if (rk[j] & RK_ZERO) {
-      const unsigned long long old = atomicMax(&s.ot_key[m.x], key);
-      if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
-    } else if (rk[j] & RK_NEW) {
-      atomicMax(&s.ot_key[m.x], key);
+#pragma unroll
+    for (int q = 0; q < SP; ++q) {
+      const int j = h * SP + q;
+      if (vs[j] == NONE) continue;
+      const uint64_t i = (uint64_t)j * T + tid;
+      const unsigned long long key = ((unsigned long long)m[q].w << 32) | (unsigned long long)(seq0 + (uint32_t)i);
+      if (pos[q] != NONE) {  // (NONE: a cell another rank owns)
+        a_obj[pos[q]] = m[q].x;
+        a_key[pos[q]] = key;
+        a_vsrc[pos[q]] = vs[j];
+        a_off[pos[q]] = m[q].z;
+        a_edge[pos[q]] = m[q].y;
+      }
+      if (rk[j] & RK_ZERO) {
+        const unsigned long long old = atomicMax(&s.ot_key[m[q].x], key);
+        if (old == 0ull && key != 0ull) atomicAdd(&s.st->n_live, 1u);
+      } else if (rk[j] & RK_NEW) {
+        atomicMax(&s.ot_key[m[q].x], key);
+      }
     }
   }
+  DTIME(5);
+  DTIME_PRINT();
 }
 
 // a tile whose 2-slots-per-cell hash does not fit shared memory: fused with a hash of one slot

@@ -150,6 +150,10 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 #ifndef GG_WARP_ARCS
 #define GG_WARP_ARCS 1
 #endif
+// the chunk's arcs staged slot-major by ballots (1) or vertex-major by a warp prefix sum (0)
+#ifndef GG_SLOT_MAJOR
+#define GG_SLOT_MAJOR 1
+#endif
 __device__ __forceinline__ void prefetch_vertex(const DevGraph& g, const DevState& s, uint32_t v) {
   if (GG_PREFETCH) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(g.vadj + (size_t)v * 4));
@@ -617,6 +621,20 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       const uint32_t room = INF - du;
       auto real = [&](uint32_t w) { return (w - 1u < WMAX - 1u) & (w < room); };
       const uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
+#if GG_SLOT_MAJOR
+      // slot-major order (every lane's slot-0 arc, then slot 1, ...): one ballot per inline slot
+      // instead of a warp prefix sum over the lanes' arc counts
+      const unsigned b0 = __ballot_sync(FULL, r0), b1 = __ballot_sync(FULL, r1);
+      const unsigned b2 = __ballot_sync(FULL, r2), b3 = __ballot_sync(FULL, r3);
+      const uint32_t o1 = __popc(b0), o2 = o1 + __popc(b1), o3 = o2 + __popc(b2);
+      const uint32_t n_arc = o3 + __popc(b3);
+      if (n_arc > STAGE) OVF_RES(1);  // (the next level's table takes it)
+      if (r0) m.stage[__popc(b0 & lt)] = make_uint2(a01.x, du + a01.y);
+      if (r1) m.stage[o1 + __popc(b1 & lt)] = make_uint2(a01.z, du + a01.w);
+      if (r2) m.stage[o2 + __popc(b2 & lt)] = make_uint2(a23.x, du + a23.y);
+      if (r3) m.stage[o3 + __popc(b3 & lt)] = make_uint2(a23.z, du + a23.w);
+      if (lane == 0) c_arcs += n_arc;
+#else
       const uint32_t cnt = r0 + r1 + r2 + r3;
       uint32_t pre = cnt;
 #pragma unroll
@@ -632,6 +650,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       if (r2) m.stage[pre++] = make_uint2(a23.x, du + a23.y);
       if (r3) m.stage[pre++] = make_uint2(a23.z, du + a23.w);
       c_arcs += cnt;
+#endif
       const bool dirty = harv && hd != NONE;
       const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
       const uint32_t ev = __reduce_or_sync(FULL, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
