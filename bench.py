@@ -117,7 +117,7 @@ class ClockSampler:
         self.mark_rows = 0
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(gpu), f"--query-gpu={self.Q}",
-                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                       "--format=csv,noheader,nounits", "-lms", "20"],
                                       stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
@@ -144,7 +144,7 @@ class ClockSampler:
         timed = rows[self.mark_rows:]
         if timed:
             rows = timed
-        else:  # a timed region shorter than the 100 ms sampling interval: the warm-up's last samples
+        else:  # a timed region shorter than the 20 ms sampling interval: the warm-up's last samples
             rows = rows[-3:]
             window = "last warm-up samples (timed region shorter than the sampling interval)"
         sm, mx, reasons = [], [], set()
@@ -279,8 +279,9 @@ def run_ours(args, cfg_name):
     n_step_upd = n_obj * cfg["step_ticks"]
     preload = walk.ticks(cfg["preload_ticks"]) if cfg["preload_ticks"] else np.empty((0, 4), np.uint32)
     # the record arena: superseded extents are reclaimed by a garbage collection when it fills;
-    # 2^28 records (6.4 GB of 180) keep it to one per ~190 steps at C3 (amortised, reported)
-    log_cap = args.log_capacity or max(1 << 28, int(1.25 * (len(preload) + 8 * n_step_upd)) + (1 << 20))
+    # 2^29 records (12.9 GB of 180) keep the setup's three re-ingested 64M-record flushes and
+    # ~160 steps after them (2M records per C3 step) collection-free (amortised, reported)
+    log_cap = args.log_capacity or max(1 << 29, int(1.25 * (len(preload) + 8 * n_step_upd)) + (1 << 20))
     hist = [preload]  # every update the index has seen, in arrival order (for the parity check)
 
     n_break = max(3, min(args.steps, 10))  # breakdown steps (every launch timed), after the timed ones
@@ -650,7 +651,7 @@ def self_launch(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=["C0", "C1", "C2", "C3"])

@@ -150,6 +150,11 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 #ifndef GG_WARP_ARCS
 #define GG_WARP_ARCS 1
 #endif
+// the one-warp table cleared with 16-byte stores (1) or 4-byte ones (0)
+#ifndef GG_VEC_INIT
+#define GG_VEC_INIT 1
+#endif
+static_assert(INF == EMPTY32, "a cleared slot's key and distance are the same word");
 // the chunk's arcs staged slot-major by ballots (1) or vertex-major by a warp prefix sum (0)
 #ifndef GG_SLOT_MAJOR
 #define GG_SLOT_MAJOR 1
@@ -443,9 +448,17 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
   const uint32_t k = P.k;
   const unsigned lt = lanemask_lt();
 
-  for (uint32_t i = lane; i < cp.H; i += 32) {
-    m.key[i] = EMPTY32;
-    m.dist[i] = INF;
+  if (GG_VEC_INIT && (cp.H & 3u) == 0) {  // 16-byte stores (carve() keeps both arrays 16-aligned)
+    const uint4 e4 = make_uint4(EMPTY32, EMPTY32, EMPTY32, EMPTY32);
+    for (uint32_t i = lane; i < cp.H / 4; i += 32) {
+      reinterpret_cast<uint4*>(m.key)[i] = e4;
+      reinterpret_cast<uint4*>(m.dist)[i] = e4;  // (INF == EMPTY32)
+    }
+  } else {
+    for (uint32_t i = lane; i < cp.H; i += 32) {
+      m.key[i] = EMPTY32;
+      m.dist[i] = INF;
+    }
   }
   for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) m.fin[i] = 0;
   for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) m.listed[i] = 0;

@@ -81,7 +81,8 @@ for cap in caps:
         wr *= scale.get(units[hdr.index("dram__bytes_write.sum")], 1)
         kind, cfg = cap.rsplit("_", 1)
         kind = {"ingestscatter": "ingest_bulk_scatter", "ingestclassify": "ingest_bulk_classify",
-                "stepscatter": "ingest_step_scatter"}.get(kind, kind)
+                "stepscatter": "ingest_step_scatter", "stepingest": "ingest_step",
+                "stepflush": "flush_step"}.get(kind, kind)
         traffic.setdefault(cfg, collections.defaultdict(float))[kind] += rd + wr
         if "smsp__issue_active.avg.pct_of_peak_sustained_active" in hdr:  # (non-HBM limiters)
             issue.setdefault(cfg, {})[kind] = {
@@ -109,6 +110,24 @@ for ll in [os.path.join(src, f) for f in sorted(os.listdir(src)) if f.startswith
         share = f"{100 * sum(v) / tot:.1f}%" if "gg::" in k else "(torch L2 flush, untimed)"
         lines.append(f"| `{k}` | {len(v)} | {sum(v) / len(v) / 1e3:.1f} | {share} |")
     lines.append("")
+    # the bench steps alone (from the first step ingest on; the setup's bulk ingests and full
+    # flushes excluded): the share each kernel takes of a step, to compare with the bench's
+    # CUDA-event split
+    names = [r[h.index("Kernel Name")].split("(")[0] for r in rows[hi + 1:]]
+    vals = [float(r[h.index("Metric Value")].replace(",", "")) for r in rows[hi + 1:]]
+    first = next((i for i, n in enumerate(names) if "k_ingest_direct" in n or "k_ingest_fused" in n), None)
+    if first is not None:  # (up to the e2e section's fresh index: its bulk preload ingest)
+        end = next((i for i in range(first, len(names)) if "k_ingest_classify" in names[i]), len(names))
+        st = collections.defaultdict(list)
+        for n, v in zip(names[first:end], vals[first:end]):
+            if "gg::" in n:
+                st[n].append(v)
+        tot = sum(sum(v) for v in st.values())
+        lines += [f"## Launch list, bench steps only ({lcfg}): share of the step", "",
+                  "| kernel | launches | mean µs | share of the step's library time |", "|---|---|---|---|"]
+        for k, v in sorted(st.items(), key=lambda x: -sum(x[1])):
+            lines.append(f"| `{k}` | {len(v)} | {sum(v) / len(v) / 1e3:.1f} | {100 * sum(v) / tot:.1f}% |")
+        lines.append("")
 
 open(os.path.join(dst, f"{tag}_summary.md"), "w").write("\n".join(lines) + "\n")
 for cfg, d in traffic.items():
