@@ -650,7 +650,8 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
   const double ball = (double)k * h->V / (double)std::max<uint64_t>(1, h->n_live_hi());
   while (lvl0 < L - 2 && (k > expand_max_k(lvl0) || GG_BALL_FACTOR * ball > expand_table_slots(lvl0))) lvl0++;
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
-  const uint32_t ball_hint = (uint32_t)std::min(ball, 4.0e9);
+  uint32_t ball_hint = (uint32_t)std::min(ball, 4.0e9);
+  if (k > expand_warp_max_k()) ball_hint = std::max(ball_hint, expand_cta_ball());  // (its candidate list)
   std::vector<uint32_t> n_in(L, 0);
   n_in[lvl0] = n_q;
   // The level above the starting one runs in the same round BESIDE it (a programmatic

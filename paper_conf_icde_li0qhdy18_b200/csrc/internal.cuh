@@ -357,6 +357,10 @@ uint32_t expand_max_k(int level);
 size_t expand_warp_bytes(int level, uint32_t V);
 // bytes per resumable-promotion record if `level` runs n queries one warp per query, else 0
 size_t expand_resume_bytes(int level, uint32_t n, int sm_count, uint32_t ball_hint);
+// the largest k the one-warp level-0 kernel takes, and the expected ball (vertices) from which the
+// starting level runs one CTA per query: a larger k starts at the CTA kernel
+uint32_t expand_warp_max_k();
+uint32_t expand_cta_ball();
 void launch_dump_cell(const DevGraph& g, const DevState& s, uint32_t c, uint32_t* obj,
                       uint32_t* edge, uint32_t* off, uint32_t cap, uint32_t* n_out, cudaStream_t st);
 }  // namespace gg

@@ -92,6 +92,8 @@ struct WarpMemT {
   S* act;                    // F: the round's active slots (the bucket being expanded)
   uint32_t* listed;          // H/32 bits: vertex expanded at least once (objects harvested)
   uint2* stage;              // STAGE: the chunk's arcs (dst, D + w), compacted (one-warp variant)
+  S* par;                    // H: (GG_PARENT) slot of the vertex that gave the slot its D
+  S* ssrc;                   // STAGE: (GG_PARENT) the staged arc's source slot
 };
 using WarpMem = WarpMemT<uint32_t>;   // global-memory level
 using WarpMemS = WarpMemT<uint16_t>;  // shared-memory levels
@@ -101,10 +103,25 @@ using WarpMemS = WarpMemT<uint16_t>;  // shared-memory levels
 #define GG_STAGE 112
 #endif
 constexpr uint32_t STAGE = GG_STAGE;
+// (GG_SHFL_ARCS=1) no arc stage: the chunk's arcs stay in their lanes' registers and each relax
+// pass fetches its arc from the owning lane with shuffles; shared memory keeps only the arc ->
+// source-lane map (128 bytes instead of 8 x STAGE), so more queries are resident per SM
+// Measured at C3 (r2 A/B): the shuffles cost ~9% at equal residency (28 per SM) and 32 resident
+// queries win back only ~6% (expansion 1.148 vs 1.117 ms) -- off
+#ifndef GG_SHFL_ARCS
+#define GG_SHFL_ARCS 0
+#endif
+constexpr size_t STAGE_BYTES = GG_SHFL_ARCS ? 128 : 8ull * STAGE;
 
+// (experiment hook) GG_PARENT=1: the one-warp kernel keeps each slot's parent (the vertex whose
+// relaxation set its D) and does not stage a vertex's arc back to its parent -- such an arc can
+// never improve it: D[x] = D[p] + w(p,x) so D[x] + w(x,p) > D[p]
+#ifndef GG_PARENT
+#define GG_PARENT 0
+#endif
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c, size_t slot_bytes) {
-  const size_t fr = (3ull * c.F * slot_bytes + 15) & ~size_t(15);
-  return 8ull * c.C + 8ull * STAGE + 8ull * c.H + 4ull * c.C + 8ull * ((c.H + 31) / 32) + fr;
+  const size_t fr = (3ull * c.F * slot_bytes + (GG_PARENT ? (size_t)(c.H + STAGE) * slot_bytes : 0) + 15) & ~size_t(15);
+  return 8ull * c.C + STAGE_BYTES + 8ull * c.H + 4ull * c.C + 8ull * ((c.H + 31) / 32) + fr;
 }
 
 template <class S>
@@ -112,7 +129,7 @@ __device__ inline WarpMemT<S> carve(unsigned char* base, const Caps& c) {
   WarpMemT<S> m;
   m.cand = reinterpret_cast<unsigned long long*>(base);
   m.stage = reinterpret_cast<uint2*>(m.cand + c.C);
-  uint32_t* p = reinterpret_cast<uint32_t*>(m.stage + STAGE);
+  uint32_t* p = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(m.stage) + STAGE_BYTES);
   m.key = p; p += c.H;
   m.dist = p; p += c.H;
   m.cobj = p; p += c.C;
@@ -121,7 +138,9 @@ __device__ inline WarpMemT<S> carve(unsigned char* base, const Caps& c) {
   S* f = reinterpret_cast<S*>(p);
   m.front0 = f; f += c.F;
   m.front1 = f; f += c.F;
-  m.act = f;
+  m.act = f; f += c.F;
+  m.par = f; f += GG_PARENT ? c.H : 0;
+  m.ssrc = f;
   return m;
 }
 
@@ -491,6 +510,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
   if (lane == 0) {
     bool imp;
     const int sl = tab_relax(m, H, seed_v, seed_d, imp);
+    if (GG_PARENT) m.par[sl] = (std::remove_pointer_t<decltype(m.par)>)~0u;  // (the seed: no parent)
     front[0] = (uint32_t)sl;
     m.fin[sl >> 5] |= 1u << (sl & 31);
   }
@@ -578,7 +598,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
     //         real arcs are then compacted into shared memory (warp prefix sum over the lanes'
     //         arc counts) and relaxed 32 at a time, lane = arc -- no lane idles on an empty slot
     struct ChunkLd {
-      uint32_t vslot, u, du, hcell, hd;
+      uint32_t vslot, u, du, hcell, hd, pv;
       uint4 a01, a23;
       uint2 cc, v0;
       bool vv, harv;
@@ -590,6 +610,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       x.vslot = 0;
       x.u = 0;
       x.du = INF;
+      x.pv = NONE;
       x.hcell = 0;
       x.hd = NONE;
       x.a01 = make_uint4(0, 0, 0, 0);
@@ -601,6 +622,10 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
         x.vslot = m.act[vi];
         x.u = m.key[x.vslot];
         x.du = m.dist[x.vslot];  // (an improvement after this read re-queues the vertex: fin cleared)
+        if (GG_PARENT) {  // the parent of this D (written with it): its arc back is not staged
+          const uint32_t ps = m.par[x.vslot];
+          x.pv = ps != (uint32_t)(std::remove_pointer_t<decltype(m.par)>)~0u ? m.key[ps] : NONE;
+        }
         const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)x.u * 4);
         x.a01 = rec[0];
         x.a23 = rec[1];
@@ -624,7 +649,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
     }
     for (uint32_t c0 = 0; c0 < na; c0 += 32) {
       const ChunkLd x = (GG_EARLY_LOADS && c0 == 0) ? first : load_chunk(c0);
-      const uint32_t vslot = x.vslot, u = x.u, du = x.du, hcell = x.hcell, hd = x.hd;
+      const uint32_t vslot = x.vslot, u = x.u, du = x.du, hcell = x.hcell, hd = x.hd, pv = x.pv;
       const uint4 a01 = x.a01, a23 = x.a23;
       const uint2 cc = x.cc, v0 = x.v0;
       const bool harv = x.harv;
@@ -633,8 +658,28 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       // a real arc (1 <= w < WMAX) whose sum stays below INF (du < INF: a bucket vertex); 32-bit
       const uint32_t room = INF - du;
       auto real = [&](uint32_t w) { return (w - 1u < WMAX - 1u) & (w < room); };
-      const uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
-#if GG_SLOT_MAJOR
+      uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
+      if (GG_PARENT) {
+        r0 &= a01.x != pv;
+        r1 &= a01.z != pv;
+        r2 &= a23.x != pv;
+        r3 &= a23.z != pv;
+      }
+#if GG_SHFL_ARCS
+      // slot-major order (every lane's slot-0 arc, then slot 1, ...): arc i of the chunk lives in
+      // lane smap[i], inline slot (i >= o1) + (i >= o2) + (i >= o3)
+      const unsigned b0 = __ballot_sync(FULL, r0), b1 = __ballot_sync(FULL, r1);
+      const unsigned b2 = __ballot_sync(FULL, r2), b3 = __ballot_sync(FULL, r3);
+      const uint32_t o1 = __popc(b0), o2 = o1 + __popc(b1), o3 = o2 + __popc(b2);
+      const uint32_t n_arc = o3 + __popc(b3);
+      unsigned char* smap = reinterpret_cast<unsigned char*>(m.stage);
+      if (r0) smap[__popc(b0 & lt)] = (unsigned char)lane;
+      if (r1) smap[o1 + __popc(b1 & lt)] = (unsigned char)lane;
+      if (r2) smap[o2 + __popc(b2 & lt)] = (unsigned char)lane;
+      if (r3) smap[o3 + __popc(b3 & lt)] = (unsigned char)lane;
+      if (lane == 0) c_arcs += n_arc;
+      const uint32_t n0 = du + a01.y, n1 = du + a01.w, n2 = du + a23.y, n3 = du + a23.w;
+#elif GG_SLOT_MAJOR
       // slot-major order (every lane's slot-0 arc, then slot 1, ...): one ballot per inline slot
       // instead of a warp prefix sum over the lanes' arc counts
       const unsigned b0 = __ballot_sync(FULL, r0), b1 = __ballot_sync(FULL, r1);
@@ -646,6 +691,13 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       if (r1) m.stage[o1 + __popc(b1 & lt)] = make_uint2(a01.z, du + a01.w);
       if (r2) m.stage[o2 + __popc(b2 & lt)] = make_uint2(a23.x, du + a23.y);
       if (r3) m.stage[o3 + __popc(b3 & lt)] = make_uint2(a23.z, du + a23.w);
+      if (GG_PARENT) {
+        using SS = std::remove_pointer_t<decltype(m.ssrc)>;
+        if (r0) m.ssrc[__popc(b0 & lt)] = (SS)vslot;
+        if (r1) m.ssrc[o1 + __popc(b1 & lt)] = (SS)vslot;
+        if (r2) m.ssrc[o2 + __popc(b2 & lt)] = (SS)vslot;
+        if (r3) m.ssrc[o3 + __popc(b3 & lt)] = (SS)vslot;
+      }
       if (lane == 0) c_arcs += n_arc;
 #else
       const uint32_t cnt = r0 + r1 + r2 + r3;
@@ -672,13 +724,38 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       for (uint32_t j0 = 0; j0 < n_arc; j0 += 32) {
         bool has = false, ovf = false;
         uint32_t nslot = 0;
+#if GG_SHFL_ARCS
+        uint2 a = make_uint2(0, INF);
+        {  // the pass's arc from its lane: one shuffle pair per inline slot the pass spans
+          const uint32_t i = j0 + lane, last = min(j0 + 31, n_arc - 1);
+          const uint32_t src = i < n_arc ? smap[i] : lane;
+          const uint32_t sj = (i >= o1) + (i >= o2) + (i >= o3);
+          const uint32_t jlo = (j0 >= o1) + (j0 >= o2) + (j0 >= o3);
+          const uint32_t jhi = (last >= o1) + (last >= o2) + (last >= o3);
+#define GG_TAKE(J, D, N)                                          \
+          if (jlo <= J && J <= jhi) {                             \
+            const uint32_t xd = __shfl_sync(FULL, D, src);        \
+            const uint32_t xn = __shfl_sync(FULL, N, src);        \
+            if (sj == J) a = make_uint2(xd, xn);                  \
+          }
+          GG_TAKE(0u, a01.x, n0)
+          GG_TAKE(1u, a01.z, n1)
+          GG_TAKE(2u, a23.x, n2)
+          GG_TAKE(3u, a23.z, n3)
+#undef GG_TAKE
+        }
+#endif
         if (j0 + lane < n_arc) {
+#if !GG_SHFL_ARCS
           const uint2 a = m.stage[j0 + lane];
+#endif
           bool imp;
           const int rr = tab_relax(m, H, a.x, a.y, imp);
           if (rr < 0) {
             ovf = true;
           } else if (imp) {
+            // (the lanes of this relaxation are done: the slot's D is the minimum they set)
+            if (GG_PARENT && ((volatile uint32_t*)m.dist)[rr] == a.y) m.par[rr] = m.ssrc[j0 + lane];
             mn = min(mn, a.y);
             const uint32_t bit = 1u << (rr & 31);
             if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
@@ -694,7 +771,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
         if (has) nfront[nn + __popc(hm & lt)] = nslot;
         nn += __popc(hm);
       }
-      __syncwarp();  // (the stage is rewritten by the next chunk)
+      __syncwarp();  // (the stage / source map is rewritten by the next chunk)
       // vertices with more than 4 arcs: arcs 3.. from the CSR, one per lane per step (rare)
       if (ev & 2u) {
         uint32_t b0 = 0, b1 = 0;
@@ -716,6 +793,8 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
               if (rr < 0) {
                 ovf = true;
               } else if (imp) {
+                if (GG_PARENT && ((volatile uint32_t*)m.dist)[rr] == (uint32_t)nd)
+                  m.par[rr] = (std::remove_pointer_t<decltype(m.par)>)vslot;
                 mn = min(mn, (uint32_t)nd);
                 const uint32_t bit = 1u << (rr & 31);
                 if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
@@ -927,8 +1006,18 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
 // scratch (the last level).  Two instantiations, so that every table access of the shared one
 // compiles to LDS/STS/ATOMS with 32-bit addresses (one pointer that may be either space makes
 // them generic 64-bit LD/ST/ATOM, measured ~10% slower overall).
+// (GG_SHFL_ARCS: its ~7 KB per query fits 8 CTAs of 4 queries per SM, so registers are capped at
+// 64; with the stage, shared memory allows 7 and ptxas is left its own choice)
+#if GG_SHFL_ARCS
+#define GG_EXPAND_BOUNDS __launch_bounds__(32 * GG_WARP_WPC, 8)
+#else
+#define GG_EXPAND_BOUNDS
+#endif
+#ifndef GG_WARP_WPC
+#define GG_WARP_WPC 4
+#endif
 template <bool SMEM>
-__global__ void k_expand(QParams P) {
+__global__ void GG_EXPAND_BOUNDS k_expand(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
   const uint32_t warp = threadIdx.x >> 5;
@@ -972,6 +1061,7 @@ __global__ void k_expand(QParams P) {
 #ifndef GG_PAIR
 #define GG_PAIR 0
 #endif
+static_assert(!(GG_PAIR && GG_SHFL_ARCS), "the paired kernel stages its arcs (GG_SHFL_ARCS=0)");
 
 struct HalfWarp {
   uint32_t h, hl, base;
@@ -1328,7 +1418,7 @@ __global__ void k_expand_pair(QParams P) {
           nn += __popc(hm);
         }
       }
-      __syncwarp();  // (the stage is rewritten by the next chunk)
+      __syncwarp();  // (the stage / source map is rewritten by the next chunk)
       // vertices with more than 4 arcs: arcs 3.. from the CSR, one per lane per step (rare)
       if (both_max(ev & 2u)) {
         uint32_t b0 = 0, b1 = 0;
@@ -1909,6 +1999,15 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 // ... and of the one-warp-per-query kernel (small expected balls, C3): fewer slots = more queries
 // resident per SM (with 4 warps per CTA: 1,024 -> 896 -> 768 slots = 18 -> 20 -> 24 warps per SM;
 // C3 expansion 1.66 -> 1.46 -> 1.37 ms, 7 promotions per 65,536 queries at 768)
+// the one-warp level 0's frontier and candidate capacities (C3 replay of 1,000 queries: frontier
+// <= 57, harvested candidates <= 16 at k = 10); k above GG_C0W - 32 starts at the CTA kernel
+#ifndef GG_F0W
+#define GG_F0W (GG_SHFL_ARCS ? 64 : 96)
+#endif
+#ifndef GG_C0W
+#define GG_C0W (GG_SHFL_ARCS ? 32 : 64)
+#endif
+static_assert((GG_C0W & (GG_C0W - 1)) == 0, "the candidate list is bitonic-sorted: a power of two");
 #ifndef GG_H0W
 #define GG_H0W 704
 #endif
@@ -1953,7 +2052,11 @@ uint32_t expand_max_k(int level) { return caps_for(level, 1).C - 32; }
 // the caps a level runs with in a given mode (the one-warp kernel's level 0 has its own table)
 static Caps caps_mode(int level, uint32_t V, bool cta) {
   Caps c = caps_for(level, V);
-  if (level == 0 && !cta) c.H = GG_H0W;
+  if (level == 0 && !cta) {
+    c.H = GG_H0W;
+    c.F = GG_F0W;
+    c.C = GG_C0W;
+  }
   return c;
 }
 static size_t warp_bytes_mode(int level, uint32_t V, bool cta) {
@@ -1970,6 +2073,8 @@ size_t expand_warp_bytes(int level, uint32_t V) {
 // kCtaBall vertices: measured C2 k=10, ball ~110: one warp 0.179 ms vs 4 warps 0.194 ms; C3,
 // ~240: 36.9 vs 36.3M q/s; C1, ~260: 0.330 vs 0.273 ms; C2 k=30, ~320: 0.398 vs 0.345 ms)
 constexpr uint32_t kCtaBall = 256;
+uint32_t expand_warp_max_k() { return GG_C0W - 32; }
+uint32_t expand_cta_ball() { return kCtaBall; }
 static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level >= NLEVELS - 1) return false;
   if (n <= (uint32_t)sm_count) return true;
