@@ -92,8 +92,6 @@ struct WarpMemT {
   S* act;                    // F: the round's active slots (the bucket being expanded)
   uint32_t* listed;          // H/32 bits: vertex expanded at least once (objects harvested)
   uint2* stage;              // STAGE: the chunk's arcs (dst, D + w), compacted (one-warp variant)
-  S* par;                    // H: (GG_PARENT) slot of the vertex that gave the slot its D
-  S* ssrc;                   // STAGE: (GG_PARENT) the staged arc's source slot
 };
 using WarpMem = WarpMemT<uint32_t>;   // global-memory level
 using WarpMemS = WarpMemT<uint16_t>;  // shared-memory levels
@@ -103,24 +101,15 @@ using WarpMemS = WarpMemT<uint16_t>;  // shared-memory levels
 #define GG_STAGE 112
 #endif
 constexpr uint32_t STAGE = GG_STAGE;
-// (GG_SHFL_ARCS=1) no arc stage: the chunk's arcs stay in their lanes' registers and each relax
-// pass fetches its arc from the owning lane with shuffles; shared memory keeps only the arc ->
-// source-lane map (128 bytes instead of 8 x STAGE), so more queries are resident per SM
-// Measured at C3 (r2 A/B): the shuffles cost ~9% at equal residency (28 per SM) and 32 resident
-// queries win back only ~6% (expansion 1.148 vs 1.117 ms) -- off
-#ifndef GG_SHFL_ARCS
-#define GG_SHFL_ARCS 0
+constexpr size_t STAGE_BYTES = 8ull * STAGE;
+static_assert(STAGE >= 64, "a half chunk (16 vertices x 4 inline arcs) must fit the stage");
+// a chunk with more arcs than the stage: staged in two halves (1) or its query promoted (0)
+#ifndef GG_HALF_SPLIT
+#define GG_HALF_SPLIT 0
 #endif
-constexpr size_t STAGE_BYTES = GG_SHFL_ARCS ? 128 : 8ull * STAGE;
 
-// (experiment hook) GG_PARENT=1: the one-warp kernel keeps each slot's parent (the vertex whose
-// relaxation set its D) and does not stage a vertex's arc back to its parent -- such an arc can
-// never improve it: D[x] = D[p] + w(p,x) so D[x] + w(x,p) > D[p]
-#ifndef GG_PARENT
-#define GG_PARENT 0
-#endif
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c, size_t slot_bytes) {
-  const size_t fr = (3ull * c.F * slot_bytes + (GG_PARENT ? (size_t)(c.H + STAGE) * slot_bytes : 0) + 15) & ~size_t(15);
+  const size_t fr = (3ull * c.F * slot_bytes + 15) & ~size_t(15);
   return 8ull * c.C + STAGE_BYTES + 8ull * c.H + 4ull * c.C + 8ull * ((c.H + 31) / 32) + fr;
 }
 
@@ -138,9 +127,7 @@ __device__ inline WarpMemT<S> carve(unsigned char* base, const Caps& c) {
   S* f = reinterpret_cast<S*>(p);
   m.front0 = f; f += c.F;
   m.front1 = f; f += c.F;
-  m.act = f; f += c.F;
-  m.par = f; f += GG_PARENT ? c.H : 0;
-  m.ssrc = f;
+  m.act = f;
   return m;
 }
 
@@ -174,10 +161,6 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 #define GG_VEC_INIT 1
 #endif
 static_assert(INF == EMPTY32, "a cleared slot's key and distance are the same word");
-// the chunk's arcs staged slot-major by ballots (1) or vertex-major by a warp prefix sum (0)
-#ifndef GG_SLOT_MAJOR
-#define GG_SLOT_MAJOR 1
-#endif
 __device__ __forceinline__ void prefetch_vertex(const DevGraph& g, const DevState& s, uint32_t v) {
   if (GG_PREFETCH) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(g.vadj + (size_t)v * 4));
@@ -510,7 +493,6 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
   if (lane == 0) {
     bool imp;
     const int sl = tab_relax(m, H, seed_v, seed_d, imp);
-    if (GG_PARENT) m.par[sl] = (std::remove_pointer_t<decltype(m.par)>)~0u;  // (the seed: no parent)
     front[0] = (uint32_t)sl;
     m.fin[sl >> 5] |= 1u << (sl & 31);
   }
@@ -598,7 +580,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
     //         real arcs are then compacted into shared memory (warp prefix sum over the lanes'
     //         arc counts) and relaxed 32 at a time, lane = arc -- no lane idles on an empty slot
     struct ChunkLd {
-      uint32_t vslot, u, du, hcell, hd, pv;
+      uint32_t vslot, u, du, hcell, hd;
       uint4 a01, a23;
       uint2 cc, v0;
       bool vv, harv;
@@ -610,7 +592,6 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       x.vslot = 0;
       x.u = 0;
       x.du = INF;
-      x.pv = NONE;
       x.hcell = 0;
       x.hd = NONE;
       x.a01 = make_uint4(0, 0, 0, 0);
@@ -622,10 +603,6 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
         x.vslot = m.act[vi];
         x.u = m.key[x.vslot];
         x.du = m.dist[x.vslot];  // (an improvement after this read re-queues the vertex: fin cleared)
-        if (GG_PARENT) {  // the parent of this D (written with it): its arc back is not staged
-          const uint32_t ps = m.par[x.vslot];
-          x.pv = ps != (uint32_t)(std::remove_pointer_t<decltype(m.par)>)~0u ? m.key[ps] : NONE;
-        }
         const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)x.u * 4);
         x.a01 = rec[0];
         x.a23 = rec[1];
@@ -649,7 +626,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
     }
     for (uint32_t c0 = 0; c0 < na; c0 += 32) {
       const ChunkLd x = (GG_EARLY_LOADS && c0 == 0) ? first : load_chunk(c0);
-      const uint32_t vslot = x.vslot, u = x.u, du = x.du, hcell = x.hcell, hd = x.hd, pv = x.pv;
+      const uint32_t vslot = x.vslot, u = x.u, du = x.du, hcell = x.hcell, hd = x.hd;
       const uint4 a01 = x.a01, a23 = x.a23;
       const uint2 cc = x.cc, v0 = x.v0;
       const bool harv = x.harv;
@@ -658,120 +635,62 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       // a real arc (1 <= w < WMAX) whose sum stays below INF (du < INF: a bucket vertex); 32-bit
       const uint32_t room = INF - du;
       auto real = [&](uint32_t w) { return (w - 1u < WMAX - 1u) & (w < room); };
-      uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
-      if (GG_PARENT) {
-        r0 &= a01.x != pv;
-        r1 &= a01.z != pv;
-        r2 &= a23.x != pv;
-        r3 &= a23.z != pv;
-      }
-#if GG_SHFL_ARCS
-      // slot-major order (every lane's slot-0 arc, then slot 1, ...): arc i of the chunk lives in
-      // lane smap[i], inline slot (i >= o1) + (i >= o2) + (i >= o3)
-      const unsigned b0 = __ballot_sync(FULL, r0), b1 = __ballot_sync(FULL, r1);
-      const unsigned b2 = __ballot_sync(FULL, r2), b3 = __ballot_sync(FULL, r3);
-      const uint32_t o1 = __popc(b0), o2 = o1 + __popc(b1), o3 = o2 + __popc(b2);
-      const uint32_t n_arc = o3 + __popc(b3);
-      unsigned char* smap = reinterpret_cast<unsigned char*>(m.stage);
-      if (r0) smap[__popc(b0 & lt)] = (unsigned char)lane;
-      if (r1) smap[o1 + __popc(b1 & lt)] = (unsigned char)lane;
-      if (r2) smap[o2 + __popc(b2 & lt)] = (unsigned char)lane;
-      if (r3) smap[o3 + __popc(b3 & lt)] = (unsigned char)lane;
-      if (lane == 0) c_arcs += n_arc;
-      const uint32_t n0 = du + a01.y, n1 = du + a01.w, n2 = du + a23.y, n3 = du + a23.w;
-#elif GG_SLOT_MAJOR
-      // slot-major order (every lane's slot-0 arc, then slot 1, ...): one ballot per inline slot
-      // instead of a warp prefix sum over the lanes' arc counts
-      const unsigned b0 = __ballot_sync(FULL, r0), b1 = __ballot_sync(FULL, r1);
-      const unsigned b2 = __ballot_sync(FULL, r2), b3 = __ballot_sync(FULL, r3);
-      const uint32_t o1 = __popc(b0), o2 = o1 + __popc(b1), o3 = o2 + __popc(b2);
-      const uint32_t n_arc = o3 + __popc(b3);
-      if (n_arc > STAGE) OVF_RES(1);  // (the next level's table takes it)
-      if (r0) m.stage[__popc(b0 & lt)] = make_uint2(a01.x, du + a01.y);
-      if (r1) m.stage[o1 + __popc(b1 & lt)] = make_uint2(a01.z, du + a01.w);
-      if (r2) m.stage[o2 + __popc(b2 & lt)] = make_uint2(a23.x, du + a23.y);
-      if (r3) m.stage[o3 + __popc(b3 & lt)] = make_uint2(a23.z, du + a23.w);
-      if (GG_PARENT) {
-        using SS = std::remove_pointer_t<decltype(m.ssrc)>;
-        if (r0) m.ssrc[__popc(b0 & lt)] = (SS)vslot;
-        if (r1) m.ssrc[o1 + __popc(b1 & lt)] = (SS)vslot;
-        if (r2) m.ssrc[o2 + __popc(b2 & lt)] = (SS)vslot;
-        if (r3) m.ssrc[o3 + __popc(b3 & lt)] = (SS)vslot;
-      }
-      if (lane == 0) c_arcs += n_arc;
-#else
-      const uint32_t cnt = r0 + r1 + r2 + r3;
-      uint32_t pre = cnt;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, pre, o);
-        if (lane >= (uint32_t)o) pre += y;
-      }
-      const uint32_t n_arc = __shfl_sync(FULL, pre, 31);
-      if (n_arc > STAGE) OVF_RES(1);  // (the next level's table takes it)
-      pre -= cnt;
-      if (r0) m.stage[pre++] = make_uint2(a01.x, du + a01.y);
-      if (r1) m.stage[pre++] = make_uint2(a01.z, du + a01.w);
-      if (r2) m.stage[pre++] = make_uint2(a23.x, du + a23.y);
-      if (r3) m.stage[pre++] = make_uint2(a23.z, du + a23.w);
-      c_arcs += cnt;
-#endif
+      const uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
       const bool dirty = harv && hd != NONE;
       const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
       const uint32_t ev = __reduce_or_sync(FULL, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
-      __syncwarp();
-      // relax: lane = arc of the staged list
-      for (uint32_t j0 = 0; j0 < n_arc; j0 += 32) {
-        bool has = false, ovf = false;
-        uint32_t nslot = 0;
-#if GG_SHFL_ARCS
-        uint2 a = make_uint2(0, INF);
-        {  // the pass's arc from its lane: one shuffle pair per inline slot the pass spans
-          const uint32_t i = j0 + lane, last = min(j0 + 31, n_arc - 1);
-          const uint32_t src = i < n_arc ? smap[i] : lane;
-          const uint32_t sj = (i >= o1) + (i >= o2) + (i >= o3);
-          const uint32_t jlo = (j0 >= o1) + (j0 >= o2) + (j0 >= o3);
-          const uint32_t jhi = (last >= o1) + (last >= o2) + (last >= o3);
-#define GG_TAKE(J, D, N)                                          \
-          if (jlo <= J && J <= jhi) {                             \
-            const uint32_t xd = __shfl_sync(FULL, D, src);        \
-            const uint32_t xn = __shfl_sync(FULL, N, src);        \
-            if (sj == J) a = make_uint2(xd, xn);                  \
-          }
-          GG_TAKE(0u, a01.x, n0)
-          GG_TAKE(1u, a01.z, n1)
-          GG_TAKE(2u, a23.x, n2)
-          GG_TAKE(3u, a23.z, n3)
-#undef GG_TAKE
+      // the chunk's real arcs staged slot-major (every lane's slot-0 arc, then slot 1, ...: one
+      // ballot per inline slot) and relaxed 32 at a time (lane = arc); a chunk with more arcs than
+      // the stage holds goes in two halves (lanes 0-15, then 16-31: <= 64 arcs each)
+      const unsigned a0 = __ballot_sync(FULL, r0), a1 = __ballot_sync(FULL, r1);
+      const unsigned a2 = __ballot_sync(FULL, r2), a3 = __ballot_sync(FULL, r3);
+      const uint32_t n_all = __popc(a0) + __popc(a1) + __popc(a2) + __popc(a3);
+#if GG_HALF_SPLIT
+      const unsigned half = n_all > STAGE ? 0x0000FFFFu : FULL;
+#else
+      if (n_all > STAGE) OVF_RES(1);  // (rare: the chained level resumes it with its own stage)
+      const unsigned half = FULL;
+#endif
+      for (unsigned pm = half;; pm = ~half) {
+        const unsigned b0 = a0 & pm, b1 = a1 & pm, b2 = a2 & pm, b3 = a3 & pm;
+        const uint32_t o1 = __popc(b0), o2 = o1 + __popc(b1), o3 = o2 + __popc(b2);
+        const uint32_t n_arc = o3 + __popc(b3);
+        if ((pm >> lane) & 1u) {
+          if (r0) m.stage[__popc(b0 & lt)] = make_uint2(a01.x, du + a01.y);
+          if (r1) m.stage[o1 + __popc(b1 & lt)] = make_uint2(a01.z, du + a01.w);
+          if (r2) m.stage[o2 + __popc(b2 & lt)] = make_uint2(a23.x, du + a23.y);
+          if (r3) m.stage[o3 + __popc(b3 & lt)] = make_uint2(a23.z, du + a23.w);
         }
-#endif
-        if (j0 + lane < n_arc) {
-#if !GG_SHFL_ARCS
-          const uint2 a = m.stage[j0 + lane];
-#endif
-          bool imp;
-          const int rr = tab_relax(m, H, a.x, a.y, imp);
-          if (rr < 0) {
-            ovf = true;
-          } else if (imp) {
-            // (the lanes of this relaxation are done: the slot's D is the minimum they set)
-            if (GG_PARENT && ((volatile uint32_t*)m.dist)[rr] == a.y) m.par[rr] = m.ssrc[j0 + lane];
-            mn = min(mn, a.y);
-            const uint32_t bit = 1u << (rr & 31);
-            if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
-              has = true;
-              nslot = (uint32_t)rr;
-              prefetch_vertex(g, s, a.x);
+        if (lane == 0) c_arcs += n_arc;
+        __syncwarp();
+        for (uint32_t j0 = 0; j0 < n_arc; j0 += 32) {
+          bool has = false, ovf = false;
+          uint32_t nslot = 0;
+          if (j0 + lane < n_arc) {
+            const uint2 a = m.stage[j0 + lane];
+            bool imp;
+            const int rr = tab_relax(m, H, a.x, a.y, imp);
+            if (rr < 0) {
+              ovf = true;
+            } else if (imp) {
+              mn = min(mn, a.y);
+              const uint32_t bit = 1u << (rr & 31);
+              if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
+                has = true;
+                nslot = (uint32_t)rr;
+                prefetch_vertex(g, s, a.x);
+              }
             }
           }
+          if (__any_sync(FULL, ovf)) OVF_RES(2);
+          const unsigned hm = __ballot_sync(FULL, has);
+          if (nn + __popc(hm) > cp.F) OVF_RES(3);
+          if (has) nfront[nn + __popc(hm & lt)] = nslot;
+          nn += __popc(hm);
         }
-        if (__any_sync(FULL, ovf)) OVF_RES(2);
-        const unsigned hm = __ballot_sync(FULL, has);
-        if (nn + __popc(hm) > cp.F) OVF_RES(3);
-        if (has) nfront[nn + __popc(hm & lt)] = nslot;
-        nn += __popc(hm);
+        __syncwarp();  // (the stage is rewritten by the next half / chunk)
+        if (pm != 0x0000FFFFu) break;  // (one part, or the second half done)
       }
-      __syncwarp();  // (the stage / source map is rewritten by the next chunk)
       // vertices with more than 4 arcs: arcs 3.. from the CSR, one per lane per step (rare)
       if (ev & 2u) {
         uint32_t b0 = 0, b1 = 0;
@@ -793,8 +712,6 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
               if (rr < 0) {
                 ovf = true;
               } else if (imp) {
-                if (GG_PARENT && ((volatile uint32_t*)m.dist)[rr] == (uint32_t)nd)
-                  m.par[rr] = (std::remove_pointer_t<decltype(m.par)>)vslot;
                 mn = min(mn, (uint32_t)nd);
                 const uint32_t bit = 1u << (rr & 31);
                 if (!(atomicOr(&m.fin[rr >> 5], bit) & bit)) {
@@ -1006,18 +923,8 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
 // scratch (the last level).  Two instantiations, so that every table access of the shared one
 // compiles to LDS/STS/ATOMS with 32-bit addresses (one pointer that may be either space makes
 // them generic 64-bit LD/ST/ATOM, measured ~10% slower overall).
-// (GG_SHFL_ARCS: its ~7 KB per query fits 8 CTAs of 4 queries per SM, so registers are capped at
-// 64; with the stage, shared memory allows 7 and ptxas is left its own choice)
-#if GG_SHFL_ARCS
-#define GG_EXPAND_BOUNDS __launch_bounds__(32 * GG_WARP_WPC, 8)
-#else
-#define GG_EXPAND_BOUNDS
-#endif
-#ifndef GG_WARP_WPC
-#define GG_WARP_WPC 4
-#endif
 template <bool SMEM>
-__global__ void GG_EXPAND_BOUNDS k_expand(QParams P) {
+__global__ void k_expand(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
   const uint32_t warp = threadIdx.x >> 5;
@@ -1061,7 +968,6 @@ __global__ void GG_EXPAND_BOUNDS k_expand(QParams P) {
 #ifndef GG_PAIR
 #define GG_PAIR 0
 #endif
-static_assert(!(GG_PAIR && GG_SHFL_ARCS), "the paired kernel stages its arcs (GG_SHFL_ARCS=0)");
 
 struct HalfWarp {
   uint32_t h, hl, base;
@@ -2000,12 +1906,15 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 // resident per SM (with 4 warps per CTA: 1,024 -> 896 -> 768 slots = 18 -> 20 -> 24 warps per SM;
 // C3 expansion 1.66 -> 1.46 -> 1.37 ms, 7 promotions per 65,536 queries at 768)
 // the one-warp level 0's frontier and candidate capacities (C3 replay of 1,000 queries: frontier
-// <= 57, harvested candidates <= 16 at k = 10); k above GG_C0W - 32 starts at the CTA kernel
+// <= 57, harvested candidates <= 16 at k = 10); k above GG_C0W - 32 starts at the CTA kernel.
+// Measured at C3 (r2 A/B): 32 resident queries per SM (696 slots, 64-entry stage with the half
+// split, F 64, C 32: 7,024 B, 64 registers with spills) 1.146 ms vs 1.115 ms for this 28-resident
+// configuration; without the half split 71% of the queries promote (chunks of > 64 arcs)
 #ifndef GG_F0W
-#define GG_F0W (GG_SHFL_ARCS ? 64 : 96)
+#define GG_F0W 96
 #endif
 #ifndef GG_C0W
-#define GG_C0W (GG_SHFL_ARCS ? 32 : 64)
+#define GG_C0W 64
 #endif
 static_assert((GG_C0W & (GG_C0W - 1)) == 0, "the candidate list is bitonic-sorted: a power of two");
 #ifndef GG_H0W
