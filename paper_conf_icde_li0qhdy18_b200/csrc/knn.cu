@@ -178,10 +178,68 @@ __device__ __forceinline__ bool valid_rec(const DevState& s, uint32_t p, uint32_
   return !GG_HARVEST_VALIDATE || s.ar.key[p] == s.ot_key[ob];
 }
 
+// GG_BUCKET_HASH=1: the vertex table probes 4-slot buckets with one 16-byte load (a vertex is
+// searched for in all four slots of a bucket at once; a new one claims the bucket's first free
+// slot) instead of single slots -- fewer probe iterations, and so less lane divergence, at the
+// same load.  C3 A/B: expansion 1.114 -> 1.054 ms (704 slots); 640 slots 1.076 (promotions)
+#ifndef GG_BUCKET_HASH
+#define GG_BUCKET_HASH 1
+#endif
+template <class M>
+__device__ __forceinline__ uint4 ld_bucket(const M& m, uint32_t b) {
+  uint4 r;
+  if constexpr (sizeof(*m.front0) == 2) {  // (shared-memory levels)
+    const uint32_t a = (uint32_t)__cvta_generic_to_shared(m.key + 4 * b);
+    asm volatile("ld.volatile.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(a));
+  } else {
+    asm volatile("ld.volatile.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(m.key + 4 * b));
+  }
+  return r;
+}
+// the slot of v in bucket b's keys kk, or -1
+__device__ __forceinline__ int bucket_match(const uint4& kk, uint32_t b, uint32_t v) {
+  const uint32_t mm = (kk.x == v ? 1u : 0u) | (kk.y == v ? 2u : 0u) | (kk.z == v ? 4u : 0u) | (kk.w == v ? 8u : 0u);
+  return mm ? (int)(4 * b + __ffs(mm) - 1) : -1;
+}
+
 // insert-or-min of (v, d); returns the slot (or -1 if the table is full)
 template <class M>
 __device__ __forceinline__ int tab_relax(const M& m, uint32_t H, uint32_t v, uint32_t d,
                                          bool& improved) {
+#if GG_BUCKET_HASH
+  // buckets b, b+1, ... (linear probing over buckets): v is in the first bucket holding it or a
+  // free slot (slots are never freed, so a bucket with a free slot ends every search)
+  const uint32_t NB = H >> 2;
+  uint32_t b = vhash(v, NB);
+  int fs = -1;
+#pragma unroll 1
+  for (int p = 0; p < MAXP / 4 && fs < 0; ++p) {
+    uint4 kk = ld_bucket(m, b);
+#pragma unroll 1
+    for (;;) {
+      fs = bucket_match(kk, b, v);
+      if (fs >= 0) break;
+      const uint32_t e = (kk.x == EMPTY32 ? 1u : 0u) | (kk.y == EMPTY32 ? 2u : 0u) |
+                         (kk.z == EMPTY32 ? 4u : 0u) | (kk.w == EMPTY32 ? 8u : 0u);
+      if (!e) break;  // full: the next bucket
+      const uint32_t j = 4 * b + __ffs(e) - 1;
+      const uint32_t old = atomicCAS(&m.key[j], EMPTY32, v);
+      if (old == EMPTY32 || old == v) {
+        fs = (int)j;
+        break;
+      }
+      kk = ld_bucket(m, b);  // another lane took that slot: look again
+    }
+    b = b + 1 == NB ? 0 : b + 1;
+  }
+  if (fs < 0) {
+    improved = false;
+    return -1;
+  }
+  const uint32_t sl = (uint32_t)fs;
+#else
   uint32_t sl = vhash(v, H);
   volatile uint32_t* vk = m.key;
   // find or claim v's slot (one exit; the distance update below is out of the probe loop)
@@ -199,6 +257,7 @@ __device__ __forceinline__ int tab_relax(const M& m, uint32_t H, uint32_t v, uin
     }
     sl = sl + 1 == H ? 0 : sl + 1;
   }
+#endif
   if (((volatile uint32_t*)m.dist)[sl] <= d) {  // not an improvement (e.g. the twin arc back)
     improved = false;
   } else {
@@ -276,6 +335,17 @@ __device__ inline RecView rec_view(unsigned char* base, const Caps& c) {
 // slot of a vertex known to be in the table (-1: not found)
 template <class M>
 __device__ __forceinline__ int tab_find(const M& m, uint32_t H, uint32_t v) {
+#if GG_BUCKET_HASH
+  const uint32_t NB = H >> 2;
+  uint32_t b = vhash(v, NB);
+  for (int p = 0; p < MAXP / 4; ++p) {
+    const uint4 kk = ld_bucket(m, b);
+    const int sl = bucket_match(kk, b, v);
+    if (sl >= 0) return sl;
+    b = b + 1 == NB ? 0 : b + 1;
+  }
+  return -1;
+#endif
   uint32_t sl = vhash(v, H);
   for (int p = 0; p < MAXP; ++p) {
     if (m.key[sl] == v) return (int)sl;
