@@ -460,7 +460,10 @@ def run_ours(args, cfg_name):
     if dom == "expand":
         nq = Qr * K
         rounds_q = dx["iterations"] / max(1, nq)
-        resident = int(os.environ.get("BENCH_EXPAND_RESIDENT", str(148 * 16)))  # 4-warp CTAs x 16 per SM
+        # the C3 starting level: the one-warp kernel, 7 CTAs x 4 queries per SM (shared memory),
+        # ~1,028 of the 1,036 CTAs (the rest reserved for the chained level beside it)
+        sms = torch.cuda.get_device_properties(dev).multi_processor_count
+        resident = int(os.environ.get("BENCH_EXPAND_RESIDENT", str(sms * 28)))
         cyc = rounds_q * (ROUND_TRIPS * L2_HIT_CYCLES + ROUND_ONCHIP_CYCLES)
         t_model_ms = nq / resident * cyc / (sm_mhz_max * 1e3)
         roofline["latency_model"] = {
