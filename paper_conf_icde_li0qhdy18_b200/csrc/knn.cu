@@ -74,6 +74,33 @@ constexpr int MAXP = 128;                  // probe limit of the vertex table
 constexpr uint32_t SPECIAL = 0xFFFFFFFFu;  // candidate slot of a same-arc object
 constexpr uint32_t WMAX = 0xFFFFFFFFu;     // inline-adjacency overflow marker
 
+// GG_BUCKET_HASH=1: the vertex table probes 4-slot buckets with one 16-byte load (a vertex is
+// searched for in all four slots of a bucket at once; a new one claims the bucket's first free
+// slot) instead of single slots -- fewer probe iterations, and so less lane divergence, at the
+// same load.  C3 A/B: expansion 1.114 -> 1.054 ms (704 slots); 640 slots 1.076 (promotions)
+#ifndef GG_BUCKET_HASH
+#define GG_BUCKET_HASH 1
+#endif
+// GG_KD_INTERLEAVE=1: each 4-slot bucket keeps its 4 keys and then its 4 distances in one 32-byte
+// block (one 16-byte load each, issued together), so a probe that finds its vertex already holds
+// the vertex's distance; 0: separate key and distance arrays
+// (measured at C3: 1.119 ms vs 1.046 ms separate -- the second 16-byte load and the lane
+// selects cost more than the dependent distance load they save; off)
+#ifndef GG_KD_INTERLEAVE
+#define GG_KD_INTERLEAVE 0
+#endif
+static_assert(!GG_KD_INTERLEAVE || GG_BUCKET_HASH, "the interleaved table is a bucketed one");
+constexpr uint32_t KB_STRIDE = GG_KD_INTERLEAVE ? 8u : 4u;  // words from one bucket's keys to the next's
+#if GG_KD_INTERLEAVE
+#define KEYR(M, I) ((M).key[(I) + ((I) & ~3u)])
+#define DISTR(M, I) ((M).dist[(I) + ((I) & ~3u)])
+#else
+#define KEYR(M, I) ((M).key[(I)])
+#define DISTR(M, I) ((M).dist[(I)])
+#endif
+#ifndef GG_BUCKET_ROT
+#define GG_BUCKET_ROT 1  // (C3 A/B: 1.054 -> 1.046 ms)
+#endif
 struct Caps {
   uint32_t H, F, C;  // table slots, frontier, candidates
 };
@@ -119,8 +146,9 @@ __device__ inline WarpMemT<S> carve(unsigned char* base, const Caps& c) {
   m.cand = reinterpret_cast<unsigned long long*>(base);
   m.stage = reinterpret_cast<uint2*>(m.cand + c.C);
   uint32_t* p = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(m.stage) + STAGE_BYTES);
-  m.key = p; p += c.H;
-  m.dist = p; p += c.H;
+  m.key = p;
+  m.dist = GG_KD_INTERLEAVE ? p + 4 : p + c.H;  // (interleaved: 4 keys, 4 distances per bucket)
+  p += 2 * c.H;
   m.cobj = p; p += c.C;
   m.fin = p; p += (c.H + 31) / 32;
   m.listed = p; p += (c.H + 31) / 32;
@@ -178,29 +206,21 @@ __device__ __forceinline__ bool valid_rec(const DevState& s, uint32_t p, uint32_
   return !GG_HARVEST_VALIDATE || s.ar.key[p] == s.ot_key[ob];
 }
 
-// GG_BUCKET_HASH=1: the vertex table probes 4-slot buckets with one 16-byte load (a vertex is
-// searched for in all four slots of a bucket at once; a new one claims the bucket's first free
-// slot) instead of single slots -- fewer probe iterations, and so less lane divergence, at the
-// same load.  C3 A/B: expansion 1.114 -> 1.054 ms (704 slots); 640 slots 1.076 (promotions)
-#ifndef GG_BUCKET_HASH
-#define GG_BUCKET_HASH 1
-#endif
-#ifndef GG_BUCKET_ROT
-#define GG_BUCKET_ROT 1  // (C3 A/B: 1.054 -> 1.046 ms)
-#endif
 template <class M>
-__device__ __forceinline__ uint4 ld_bucket(const M& m, uint32_t b) {
+__device__ __forceinline__ uint4 ld_words4(const M& m, const uint32_t* p) {
   uint4 r;
   if constexpr (sizeof(*m.front0) == 2) {  // (shared-memory levels)
-    const uint32_t a = (uint32_t)__cvta_generic_to_shared(m.key + 4 * b);
+    const uint32_t a = (uint32_t)__cvta_generic_to_shared(p);
     asm volatile("ld.volatile.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
                  : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(a));
   } else {
     asm volatile("ld.volatile.v4.u32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(m.key + 4 * b));
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
   }
   return r;
 }
+template <class M>
+__device__ __forceinline__ uint4 ld_bucket(const M& m, uint32_t b) { return ld_words4(m, m.key + KB_STRIDE * b); }
 // the slot of v in bucket b's keys kk, or -1
 __device__ __forceinline__ int bucket_match(const uint4& kk, uint32_t b, uint32_t v) {
   const uint32_t mm = (kk.x == v ? 1u : 0u) | (kk.y == v ? 2u : 0u) | (kk.z == v ? 4u : 0u) | (kk.w == v ? 8u : 0u);
@@ -217,13 +237,20 @@ __device__ __forceinline__ int tab_relax(const M& m, uint32_t H, uint32_t v, uin
   const uint32_t NB = H >> 2;
   uint32_t b = vhash(v, NB);
   int fs = -1;
+  uint32_t dpre = INF;  // (interleaved table) the slot's distance as loaded with its bucket
 #pragma unroll 1
   for (int p = 0; p < MAXP / 4 && fs < 0; ++p) {
     uint4 kk = ld_bucket(m, b);
+    uint4 dd = make_uint4(INF, INF, INF, INF);
+    if (GG_KD_INTERLEAVE) dd = ld_words4(m, m.key + KB_STRIDE * b + 4);
 #pragma unroll 1
     for (;;) {
       fs = bucket_match(kk, b, v);
-      if (fs >= 0) break;
+      if (fs >= 0) {
+        const uint32_t jj = (uint32_t)fs & 3u;
+        dpre = jj == 0 ? dd.x : jj == 1 ? dd.y : jj == 2 ? dd.z : dd.w;
+        break;
+      }
       const uint32_t e = (kk.x == EMPTY32 ? 1u : 0u) | (kk.y == EMPTY32 ? 2u : 0u) |
                          (kk.z == EMPTY32 ? 4u : 0u) | (kk.w == EMPTY32 ? 8u : 0u);
       if (!e) break;  // full: the next bucket
@@ -235,9 +262,10 @@ __device__ __forceinline__ int tab_relax(const M& m, uint32_t H, uint32_t v, uin
 #else
       const uint32_t j = 4 * b + __ffs(e) - 1;
 #endif
-      const uint32_t old = atomicCAS(&m.key[j], EMPTY32, v);
+      const uint32_t old = atomicCAS(&KEYR(m, j), EMPTY32, v);
       if (old == EMPTY32 || old == v) {
         fs = (int)j;
+        dpre = INF;  // (just claimed: the atomicMin below decides)
         break;
       }
       kk = ld_bucket(m, b);  // another lane took that slot: look again
@@ -249,15 +277,16 @@ __device__ __forceinline__ int tab_relax(const M& m, uint32_t H, uint32_t v, uin
     return -1;
   }
   const uint32_t sl = (uint32_t)fs;
+  // (a stale preloaded distance is never below the current one: distances only decrease)
+  const uint32_t dnow = GG_KD_INTERLEAVE ? dpre : *(volatile uint32_t*)&DISTR(m, sl);
 #else
   uint32_t sl = vhash(v, H);
-  volatile uint32_t* vk = m.key;
   // find or claim v's slot (one exit; the distance update below is out of the probe loop)
 #pragma unroll 1
   for (int p = 0;; ++p) {
-    uint32_t cur = vk[sl];
+    uint32_t cur = *(volatile uint32_t*)&KEYR(m, sl);
     if (cur == EMPTY32) {
-      cur = atomicCAS(&m.key[sl], EMPTY32, v);
+      cur = atomicCAS(&KEYR(m, sl), EMPTY32, v);
       if (cur == EMPTY32) cur = v;  // claimed (its distance is still INF)
     }
     if (cur == v) break;
@@ -268,10 +297,13 @@ __device__ __forceinline__ int tab_relax(const M& m, uint32_t H, uint32_t v, uin
     sl = sl + 1 == H ? 0 : sl + 1;
   }
 #endif
-  if (((volatile uint32_t*)m.dist)[sl] <= d) {  // not an improvement (e.g. the twin arc back)
+#if !GG_BUCKET_HASH
+  const uint32_t dnow = *(volatile uint32_t*)&DISTR(m, sl);
+#endif
+  if (dnow <= d) {  // not an improvement (e.g. the twin arc back)
     improved = false;
   } else {
-    improved = atomicMin(&m.dist[sl], d) > d;
+    improved = atomicMin(&DISTR(m, sl), d) > d;
   }
   return (int)sl;
 }
@@ -358,7 +390,7 @@ __device__ __forceinline__ int tab_find(const M& m, uint32_t H, uint32_t v) {
 #endif
   uint32_t sl = vhash(v, H);
   for (int p = 0; p < MAXP; ++p) {
-    if (m.key[sl] == v) return (int)sl;
+    if (KEYR(m, sl) == v) return (int)sl;
     sl = sl + 1 == H ? 0 : sl + 1;
   }
   return -1;
@@ -424,7 +456,7 @@ __device__ __forceinline__ unsigned long long cand_dist(const M& m, uint32_t i) 
   const unsigned long long a = m.cand[i];
   const uint32_t slot = (uint32_t)(a >> 32), off = (uint32_t)a;
   if (slot == SPECIAL) return off;
-  return (unsigned long long)m.dist[slot] + off;
+  return (unsigned long long)DISTR(m, slot) + off;
 }
 
 // Append one ballot's worth of candidates (false: capacity exceeded)
@@ -448,7 +480,7 @@ __device__ __forceinline__ bool cand_push(const M& m, uint32_t& nc, uint32_t C, 
 template <class M, class S>
 __device__ void request_lookahead(const QParams& P, const M& m, const S* front, uint32_t nf, int lane) {
   for (uint32_t i = lane; i < nf; i += 32) {
-    const uint32_t v = m.key[front[i]];
+    const uint32_t v = KEYR(m, front[i]);
     request_flush(P.s, cellof(P.g, v), P.epoch);
   }
 }
@@ -488,8 +520,8 @@ __device__ void promote_export(const QParams& P, const M& m, uint32_t qi, int la
     const uint32_t n_act = rs.ok ? rs.na - rs.c0 : 0;
     if (rs.ok) {
       for (uint32_t i = lane; i < c.H; i += 32) {
-        r.key[i] = m.key[i];
-        r.dist[i] = m.dist[i];
+        r.key[i] = KEYR(m, i);
+        r.dist[i] = DISTR(m, i);
       }
       for (uint32_t i = lane; i < (c.H + 31) / 32; i += 32) {
         r.listed[i] = m.listed[i];
@@ -532,14 +564,18 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
 
   if (GG_VEC_INIT && (cp.H & 3u) == 0) {  // 16-byte stores (carve() keeps both arrays 16-aligned)
     const uint4 e4 = make_uint4(EMPTY32, EMPTY32, EMPTY32, EMPTY32);
-    for (uint32_t i = lane; i < cp.H / 4; i += 32) {
-      reinterpret_cast<uint4*>(m.key)[i] = e4;
-      reinterpret_cast<uint4*>(m.dist)[i] = e4;  // (INF == EMPTY32)
+    if (GG_KD_INTERLEAVE) {  // (keys and distances: one 2H-word block)
+      for (uint32_t i = lane; i < cp.H / 2; i += 32) reinterpret_cast<uint4*>(m.key)[i] = e4;
+    } else {
+      for (uint32_t i = lane; i < cp.H / 4; i += 32) {
+        reinterpret_cast<uint4*>(m.key)[i] = e4;
+        reinterpret_cast<uint4*>(m.dist)[i] = e4;  // (INF == EMPTY32)
+      }
     }
   } else {
     for (uint32_t i = lane; i < cp.H; i += 32) {
-      m.key[i] = EMPTY32;
-      m.dist[i] = INF;
+      KEYR(m, i) = EMPTY32;
+      DISTR(m, i) = INF;
     }
   }
   for (uint32_t i = lane; i < (cp.H + 31) / 32; i += 32) m.fin[i] = 0;
@@ -634,7 +670,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
     for (uint32_t b0 = 0; b0 < nf; b0 += 32) {
       const uint32_t i = b0 + lane;
       const uint32_t sl = i < nf ? front[i] : NONE;
-      const uint32_t ent = sl != NONE ? m.dist[sl] : INF;
+      const uint32_t ent = sl != NONE ? DISTR(m, sl) : INF;
       const bool a = sl != NONE && ent < bhi;
       const bool r = sl != NONE && !a;
       const unsigned rm = __ballot_sync(FULL, r);
@@ -681,8 +717,8 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       x.harv = false;
       if (x.vv) {
         x.vslot = m.act[vi];
-        x.u = m.key[x.vslot];
-        x.du = m.dist[x.vslot];  // (an improvement after this read re-queues the vertex: fin cleared)
+        x.u = KEYR(m, x.vslot);
+        x.du = DISTR(m, x.vslot);  // (an improvement after this read re-queues the vertex: fin cleared)
         const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)x.u * 4);
         x.a01 = rec[0];
         x.a23 = rec[1];
@@ -857,7 +893,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       w.v0 = make_uint2(0, 0);
       if (w.vv) {
         w.vslot = m.act[vi];
-        w.u = m.key[w.vslot];
+        w.u = KEYR(m, w.vslot);
         w.arc = g.vadj[(size_t)w.u * 4 + s4];
         if (s4 == 0) {
           w.hcell = cellof(g, w.u);
@@ -874,7 +910,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       const Win nxt = load_win(w0 + 8);  // (all lanes out of range past the last window)
       // D re-read now: an earlier window may have improved it (the frontier bit was cleared
       // at partition, so such an improvement also re-queued the vertex)
-      const uint32_t du = cur.vv ? m.dist[cur.vslot] : INF;
+      const uint32_t du = cur.vv ? DISTR(m, cur.vslot) : INF;
       bool has = false, ovf = false;
       uint32_t nslot = 0;
       auto relax = [&](uint32_t dst, uint32_t w) {
@@ -1211,8 +1247,8 @@ __global__ void k_expand_pair(QParams P) {
       need = false;
       outcome = -1;
       for (uint32_t i = W.hl; i < H; i += 16) {
-        m.key[i] = EMPTY32;
-        m.dist[i] = INF;
+        KEYR(m, i) = EMPTY32;
+        DISTR(m, i) = INF;
       }
       for (uint32_t i = W.hl; i < (H + 31) / 32; i += 16) {
         m.fin[i] = 0;
@@ -1309,7 +1345,7 @@ __global__ void k_expand_pair(QParams P) {
     for (uint32_t b0 = 0; b0 < nf_b; b0 += 16) {
       const uint32_t i = b0 + W.hl;
       const uint32_t sl = (act && i < nf) ? front[i] : NONE;
-      const uint32_t ent = sl != NONE ? m.dist[sl] : INF;
+      const uint32_t ent = sl != NONE ? DISTR(m, sl) : INF;
       const bool a = sl != NONE && ent < bhi;
       const bool r = sl != NONE && !a;
       const unsigned rm = __ballot_sync(0xffffffffu, r) & W.mask;
@@ -1340,8 +1376,8 @@ __global__ void k_expand_pair(QParams P) {
       bool harv = false;
       if (vv) {
         vslot = m.act[vi];
-        u = m.key[vslot];
-        du = m.dist[vslot];
+        u = KEYR(m, vslot);
+        du = DISTR(m, vslot);
         const uint4* rec = reinterpret_cast<const uint4*>(g.vadj + (size_t)u * 4);
         a01 = rec[0];
         a23 = rec[1];
@@ -1446,7 +1482,7 @@ __global__ void k_expand_pair(QParams P) {
       }
       if (oc < 0 && (ev & 4u)) {  // a cell with cached updates: lazy flush, then retry
         if (dirty) request_flush(s, hcell, P.epoch);
-        for (uint32_t i = W.hl; i < nf; i += 16) request_flush(s, cellof(g, m.key[front[i]]), P.epoch);
+        for (uint32_t i = W.hl; i < nf; i += 16) request_flush(s, cellof(g, KEYR(m, front[i])), P.epoch);
         oc = RETRY;
       }
       if (oc < 0) {
@@ -1575,8 +1611,8 @@ __device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& 
   const uint32_t k = P.k;
 
   for (uint32_t i = tid; i < H; i += T) {
-    m.key[i] = EMPTY32;
-    m.dist[i] = INF;
+    KEYR(m, i) = EMPTY32;
+    DISTR(m, i) = INF;
   }
   for (uint32_t i = tid; i < (H + 31) / 32; i += T) m.fin[i] = 0;
   for (uint32_t i = tid; i < (H + 31) / 32; i += T) m.listed[i] = 0;
@@ -1658,7 +1694,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& 
     nf = sh.nn[1];
     if (nf > cp.F || nc0 > cp.C || (sh.flags & FL_OVF)) return OVERFLOW;
     uint32_t mn = INF;
-    for (uint32_t i = tid; i < nf; i += T) mn = min(mn, m.dist[m.front0[i]]);
+    for (uint32_t i = tid; i < nf; i += T) mn = min(mn, DISTR(m, m.front0[i]));
     mn = __reduce_min_sync(FULL, mn);
     if (lane == 0) sh.red[1][wid] = mn;
     __syncthreads();
@@ -1724,7 +1760,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& 
     uint32_t mn = INF;
     for (uint32_t i = tid; i < nf; i += T) {
       const uint32_t sl = front[i];
-      const uint32_t ent = m.dist[sl];
+      const uint32_t ent = DISTR(m, sl);
       if (ent < bhi) {
         m.act[atomicAdd(&sh.na[par], 1u)] = sl;  // (act has F entries: na <= nf <= F)
         atomicAnd(&m.fin[sl >> 5], ~(1u << (sl & 31)));
@@ -1749,7 +1785,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& 
       const uint32_t vi = w0 + (tid >> 2), s4 = tid & 3;
       if (vi < na) {
         const uint32_t vslot = m.act[vi];
-        const uint32_t u = m.key[vslot], du = m.dist[vslot];  // D re-read after the frontier bit
+        const uint32_t u = KEYR(m, vslot), du = DISTR(m, vslot);  // D re-read after the frontier bit
         const uint2 arc = g.vadj[(size_t)u * 4 + s4];
         bool harv = false;
         uint32_t hcell = 0, hd = NONE;
@@ -1827,7 +1863,7 @@ __device__ int run_query_cta(const QParams& P, const WarpMemS& m, CtaShared<W>& 
     const uint32_t fl = sh.flags;
     if (fl & FL_OVF) return OVERFLOW;
     if (fl & FL_RETRY) {  // ask for every dirty cell the frontier will need, then retry
-      for (uint32_t i = tid; i < nf; i += T) request_flush(s, cellof(g, m.key[front[i]]), P.epoch);
+      for (uint32_t i = tid; i < nf; i += T) request_flush(s, cellof(g, KEYR(m, front[i])), P.epoch);
       return RETRY;
     }
     blo = sh.red[par][0];
