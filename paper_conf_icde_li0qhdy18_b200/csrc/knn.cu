@@ -2097,7 +2097,12 @@ size_t expand_warp_bytes(int level, uint32_t V) {
 // starting level runs one warp per query when the caller expects small balls (ball_hint below
 // kCtaBall vertices: measured C2 k=10, ball ~110: one warp 0.179 ms vs 4 warps 0.194 ms; C3,
 // ~240: 36.9 vs 36.3M q/s; C1, ~260: 0.330 vs 0.273 ms; C2 k=30, ~320: 0.398 vs 0.345 ms)
-constexpr uint32_t kCtaBall = 256;
+// (with the bucketed table, r2: C1 expansion 0.301 -> 0.262 ms and C2 k=30 0.370 -> 0.268 ms one
+// warp per query; thresholds 400 and 600 equal on both, so 512)
+#ifndef GG_CTA_BALL
+#define GG_CTA_BALL 512
+#endif
+constexpr uint32_t kCtaBall = GG_CTA_BALL;
 uint32_t expand_warp_max_k() { return GG_C0W - 32; }
 uint32_t expand_cta_ball() { return kCtaBall; }
 static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
