@@ -134,6 +134,10 @@ static_assert(STAGE >= 64, "a half chunk (16 vertices x 4 inline arcs) must fit 
 #ifndef GG_HALF_SPLIT
 #define GG_HALF_SPLIT 0
 #endif
+// the chunk's harvest / rare-event vote after its relax passes (1) or before them (0)
+#ifndef GG_LATE_EVENTS
+#define GG_LATE_EVENTS 0  // (measured: 1.059 vs 1.046 ms -- off)
+#endif
 
 __host__ __device__ inline size_t warpmem_bytes(const Caps& c, size_t slot_bytes) {
   const size_t fr = (3ull * c.F * slot_bytes + 15) & ~size_t(15);
@@ -752,9 +756,11 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
       const uint32_t room = INF - du;
       auto real = [&](uint32_t w) { return (w - 1u < WMAX - 1u) & (w < room); };
       const uint32_t r0 = real(a01.y), r1 = real(a01.w), r2 = real(a23.y), r3 = real(a23.w);
+#if !GG_LATE_EVENTS
       const bool dirty = harv && hd != NONE;
       const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
       const uint32_t ev = __reduce_or_sync(FULL, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
+#endif
       // the chunk's real arcs staged slot-major (every lane's slot-0 arc, then slot 1, ...: one
       // ballot per inline slot) and relaxed 32 at a time (lane = arc); a chunk with more arcs than
       // the stage holds goes in two halves (lanes 0-15, then 16-31: <= 64 arcs each)
@@ -807,6 +813,13 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
         __syncwarp();  // (the stage is rewritten by the next half / chunk)
         if (pm != 0x0000FFFFu) break;  // (one part, or the second half done)
       }
+#if GG_LATE_EVENTS
+      // the chunk's harvest state (cell head, cleaned list, object index) is first used only now:
+      // its loads' latency overlaps the relax passes above
+      const bool dirty = harv && hd != NONE;
+      const uint2 vo = harv ? vobj_valid(v0, cc) : make_uint2(0, 0);
+      const uint32_t ev = __reduce_or_sync(FULL, (overflow_arcs ? 2u : 0u) | (dirty ? 4u : 0u) | (vo.y ? 8u : 0u));
+#endif
       // vertices with more than 4 arcs: arcs 3.. from the CSR, one per lane per step (rare)
       if (ev & 2u) {
         uint32_t b0 = 0, b1 = 0;
