@@ -628,25 +628,69 @@ __global__ void __launch_bounds__(FW * 32, 5) k_flush_warp(DevGraph g, DevState 
       }
       __syncwarp();
     }
-    // R[c] sorted by (source vertex, winner index): warp bitonic sort of the packed pairs
+    // R[c] sorted by (source vertex, winner index): a warp bitonic sort of the packed pairs --
+    // in registers (element j * 32 + lane in v[j], shuffles for strides below 32) on 32-bit keys
+    // ((vertex - cell base) << 7 | index) when the cell size allows, else in shared memory
     uint32_t n2 = 1;
     while (n2 < n_win) n2 <<= 1;
-    for (uint32_t i = lane; i < n2; i += 32)
-      m.srt[i] = i < n_win ? ((unsigned long long)m.w_vs[i] << 32 | i) : EMPTY64;
-    __syncwarp();
-    for (uint32_t size = 2; size <= n2; size <<= 1) {
-      for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
-        for (uint32_t i = lane; i < n2 / 2; i += 32) {
-          const uint32_t lo = 2 * i - (i & (stride - 1));
-          const uint32_t hi = lo + stride;
-          const bool asc = (lo & size) == 0;
-          const unsigned long long x = m.srt[lo], y = m.srt[hi];
-          if ((x > y) == asc) {
-            m.srt[lo] = y;
-            m.srt[hi] = x;
+    if (g.cs <= (1u << 25)) {
+      uint32_t v[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t i = j * 32 + lane;
+        v[j] = i < n_win ? ((m.w_vs[i] - cbeg) << 7 | i) : 0xFFFFFFFFu;
+      }
+      const uint32_t E = n2 > 32 ? n2 / 32 : 1;  // registers in use (n2 <= WW = 128)
+      for (uint32_t size = 2; size <= n2; size <<= 1) {
+        for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+          if (stride >= 32) {  // partner in this lane: register j ^ (stride / 32)
+            const uint32_t jj = stride >> 5;
+#pragma unroll
+            for (uint32_t j = 0; j < 4; ++j) {
+              if (j >= E || (j & jj)) continue;
+              const bool asc = ((j * 32 + lane) & size) == 0;
+              const uint32_t a = v[j], b = v[j | jj];
+              if ((a > b) == asc) {
+                v[j] = b;
+                v[j | jj] = a;
+              }
+            }
+          } else {  // partner in lane ^ stride, same register
+#pragma unroll
+            for (uint32_t j = 0; j < 4; ++j) {
+              if (j >= E) continue;
+              const uint32_t o = __shfl_xor_sync(0xffffffffu, v[j], stride);
+              const bool asc = ((j * 32 + lane) & size) == 0;
+              const bool lower = (lane & stride) == 0;
+              v[j] = (lower == asc) ? min(v[j], o) : max(v[j], o);
+            }
           }
         }
-        __syncwarp();
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t i = j * 32 + lane;
+        if (i < n_win) m.srt[i] = ((unsigned long long)((v[j] >> 7) + cbeg) << 32) | (v[j] & 127u);
+      }
+      __syncwarp();
+    } else {
+      for (uint32_t i = lane; i < n2; i += 32)
+        m.srt[i] = i < n_win ? ((unsigned long long)m.w_vs[i] << 32 | i) : EMPTY64;
+      __syncwarp();
+      for (uint32_t size = 2; size <= n2; size <<= 1) {
+        for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+          for (uint32_t i = lane; i < n2 / 2; i += 32) {
+            const uint32_t lo = 2 * i - (i & (stride - 1));
+            const uint32_t hi = lo + stride;
+            const bool asc = (lo & size) == 0;
+            const unsigned long long x = m.srt[lo], y = m.srt[hi];
+            if ((x > y) == asc) {
+              m.srt[lo] = y;
+              m.srt[hi] = x;
+            }
+          }
+          __syncwarp();
+        }
       }
     }
     for (uint32_t r = lane; r < n_win; r += 32) {

@@ -70,6 +70,24 @@ def test_loopback_index_bit_exact(gg, n):
     grid.close()
 
 
+@pytest.mark.parametrize("mode", [1, 2, 3])
+def test_loopback_ingest_paths(gg, mode):
+    """Every ingest path in sharded mode (4 shards): updates of other shards' cells only raise the
+    replicated object table (and mark the cell an object leaves STALE on its owner) -- the cell-hash
+    launch (1), the direct launch (2) and the three launches (3) all give the oracle's answers."""
+    g = synth.table_ii_graph("NY", scale=0.2)
+    walk = synth.RandomWalk(g, 20_000, inject=True)
+    grid = gg.GGrid(g, 256, max_objects=20_000, n_gpus=4, devices=[0] * 4, ingest_kernels=mode)
+    hist = []
+    for it in range(3):
+        u = walk.ticks(2 + it)
+        hist.append(u)
+        grid.ingest(u)
+        q = synth.queries(g, 500, seed=70 + it)
+        _same(grid.knn(q, 9), oracle.knn_from_updates(g, np.concatenate(hist), q, 9), f"mode {mode} round {it}")
+    grid.close()
+
+
 def test_loopback_edge_cases(gg):
     """Fewer queries than shards (empty origin shares), k beyond the objects (padding), ties
     (lattice weights 1..4), device inputs and outputs, a flush_all and the per-cell dump routed
