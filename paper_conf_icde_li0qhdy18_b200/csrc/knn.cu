@@ -70,7 +70,10 @@ __device__ __forceinline__ unsigned long long gtime() {
     __syncwarp();                                                                 \
     OVF_AT(why);                                                                  \
   } while (0)
-constexpr int MAXP = 128;                  // probe limit of the vertex table
+#ifndef GG_MAXP
+#define GG_MAXP 128
+#endif
+constexpr int MAXP = GG_MAXP;  // probe limit of the vertex table (slots)
 constexpr uint32_t SPECIAL = 0xFFFFFFFFu;  // candidate slot of a same-arc object
 constexpr uint32_t WMAX = 0xFFFFFFFFu;     // inline-adjacency overflow marker
 
