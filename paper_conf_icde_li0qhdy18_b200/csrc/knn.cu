@@ -191,6 +191,10 @@ constexpr uint32_t EMPTY32 = 0xFFFFFFFFu;  // free key slot (vertex ids are < 2^
 #ifndef GG_WARP_ARCS
 #define GG_WARP_ARCS 1
 #endif
+// the final candidate sort in registers (shuffles) when at most 32 candidates and k <= 32 (1)
+#ifndef GG_REG_SORT
+#define GG_REG_SORT 1
+#endif
 // the one-warp table cleared with 16-byte stores (1) or 4-byte ones (0)
 #ifndef GG_VEC_INIT
 #define GG_VEC_INIT 1
@@ -1028,6 +1032,28 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
   c_objs = __reduce_add_sync(FULL, c_objs);
 
   // ---- 4. the k smallest (dist, obj) ------------------------------------------------------
+  if (GG_REG_SORT && nc <= 32 && k <= 32) {  // one candidate per lane: bitonic sort by shuffles
+    unsigned long long v = EMPTY64;
+    if (lane < nc) {
+      const unsigned long long d = cand_dist(m, lane);
+      if (d < INF) v = (d << 32) | m.cobj[lane];
+    }
+#pragma unroll
+    for (uint32_t size = 2; size <= 32; size <<= 1) {
+#pragma unroll
+      for (uint32_t stride = size >> 1; stride > 0; stride >>= 1) {
+        const unsigned long long o = __shfl_xor_sync(FULL, v, stride);
+        const bool keep_min = ((lane & stride) == 0) == ((lane & size) == 0);
+        v = keep_min ? min(v, o) : max(v, o);
+      }
+    }
+    if (lane < k) {
+      const bool ok = v != EMPTY64 && (uint32_t)(v >> 32) <= lim;
+      P.out_obj[(size_t)qi * k + lane] = ok ? (uint32_t)v : GGRID_PAD;
+      P.out_dist[(size_t)qi * k + lane] = ok ? (uint32_t)(v >> 32) : GGRID_PAD;
+    }
+    goto finish;
+  }
   for (uint32_t i = lane; i < nc; i += 32) {
     const unsigned long long d = cand_dist(m, i);
     m.cand[i] = d < INF ? ((d << 32) | m.cobj[i]) : EMPTY64;
@@ -1040,6 +1066,7 @@ __device__ __forceinline__ int run_query(const QParams& P, const M& m, uint32_t 
     P.out_obj[(size_t)qi * k + r] = ok ? (uint32_t)dk : GGRID_PAD;
     P.out_dist[(size_t)qi * k + r] = ok ? (uint32_t)(dk >> 32) : GGRID_PAD;
   }
+finish:
   if (lane == 0 && P.remote) P.remote[qi] = rmask;
   if (lane == 0) {
     atomicAdd(&s.st->ex_iters, (unsigned long long)c_iter);
