@@ -677,3 +677,26 @@ def test_flush_warp_overflow_cells(gg, case, monkeypatch):
     ids, e, d = oracle.snapshot_objects(np.concatenate(hist))
     assert sorted(rows) == sorted(zip(ids.tolist(), e.tolist(), d.tolist()))
     grid.close()
+
+
+@pytest.mark.parametrize("k", [1, 10, 31, 32])
+def test_one_warp_candidate_sort_both_paths(gg, k):
+    """The one-warp level's final candidate sort runs in registers (one candidate per lane) when a
+    query harvested at most 32 candidates and k <= 32, else in shared memory: objects stacked 24 at
+    a time on a few hundred arcs (plus a uniform background) give queries on both sides of 32
+    harvested candidates, with ties at equal offsets.  Every row the oracle's."""
+    g = synth.table_ii_graph("NY", scale=0.2)
+    rng = np.random.default_rng(21)
+    hot = rng.choice(len(g["src"]), 250, replace=False)
+    arc_c = np.repeat(hot, 24)
+    off_c = (rng.integers(0, 3, len(arc_c)) * (g["w"][arc_c] // 3)).astype(np.int64)  # ties
+    arc_b, off_b = synth.random_locations(g, 2000, rng)
+    arc = np.concatenate([arc_c, arc_b]).astype(np.int64)
+    off = np.minimum(np.concatenate([off_c, off_b]).astype(np.int64), g["w"][arc].astype(np.int64) - 1)
+    n = len(arc)
+    upd = np.stack([rng.permutation(n), arc, off, np.full(n, 5, np.int64)], 1).astype(np.uint32)
+    q = synth.queries(g, 1200, seed=91)
+    grid = gg.GGrid(g, 256, max_objects=n)
+    grid.ingest(upd)
+    _assert_same(grid.knn(q, k), _oracle(g, upd, q, k), f"k={k}")
+    grid.close()
