@@ -2145,6 +2145,9 @@ size_t expand_warp_bytes(int level, uint32_t V) {
 #ifndef GG_CTA_BALL
 #define GG_CTA_BALL 512
 #endif
+#ifndef GG_CTA_BALL1
+#define GG_CTA_BALL1 1024  // (C2 k=40 / 50: expansion 0.427 -> 0.401 / 0.489 -> 0.474 ms; 0: always a CTA)
+#endif
 constexpr uint32_t kCtaBall = GG_CTA_BALL;
 uint32_t expand_warp_max_k() { return GG_C0W - 32; }
 uint32_t expand_cta_ball() { return kCtaBall; }
@@ -2152,6 +2155,8 @@ static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level >= NLEVELS - 1) return false;
   if (n <= (uint32_t)sm_count) return true;
   if (level == 0) return GG_CTA_LEVEL == 0 && ball_hint >= kCtaBall;
+  // (a starting level 1 -- 32 < k <= 96 -- also runs one warp per query below GG_CTA_BALL1)
+  if (level == 1) return ball_hint >= GG_CTA_BALL1;
   return true;
 }
 
