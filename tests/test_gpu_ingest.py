@@ -243,3 +243,25 @@ def test_overflowing_batch_is_eoverflow(gg):
     assert e.value.rc == gg.GGRID_EOVERFLOW
     assert grid.stats()["n_updates"] == 0
     grid.close()
+
+
+@pytest.mark.parametrize("extra", [0, 1])
+def test_direct_launch_at_capacity(gg, extra):
+    """The direct launch holds at most 2 CTAs x 512 threads x 8 updates per SM (1,212,416 on a
+    148-SM B200): a batch of exactly that many updates takes it with every register slot in use,
+    one more falls back to the other paths; both exact.  Single-vertex cells (many distinct cells
+    per tile, the direct path's regime)."""
+    import torch
+
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    n = sms * 2 * 512 * 8 + extra
+    g = synth.table_ii_graph("NY", scale=0.05)
+    walk = synth.RandomWalk(g, 8000, inject=True)
+    upd = walk.ticks(-(-n // 8000))[:n]
+    grid = gg.GGrid(g, 1, max_objects=8000, ingest_kernels=2)
+    grid.ingest(upd)
+    st = grid.stats()
+    assert st["kernel_launches"]["ingest_alloc"] == (1 if extra else 0)
+    q = synth.queries(g, 300, seed=123)
+    _same(grid.knn(q, 8), oracle.knn_from_updates(g, upd, q, 8), f"n={n}")
+    grid.close()
