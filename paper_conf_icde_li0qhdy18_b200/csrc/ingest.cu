@@ -145,12 +145,22 @@ __global__ void __launch_bounds__(CT) k_ingest_classify(const uint4* __restrict_
     for (int q = 0; q < SPC; ++q) h_cnt[tid * SPC + q] |= (excl + loc[q]) << 16;  // counts <= CU
   }
   __syncthreads();  // (the claims below read other threads' slots)
-  for (int i = tid; i < CH; i += CT) {
-    const uint32_t c = h_cell[i];
-    if (c != NONE && c != REMOTE_CELL) {
-      atomicMax(&s.bcount[c * BCOUNT_STRIDE + 1], h_tmax[i]);
-      h_cell[i] = atomicAdd(&s.bcount[c * BCOUNT_STRIDE], h_cnt[i] & 0xFFFFu);
+  {  // one claim per distinct cell of the tile: all of a thread's SPC returning atomics in flight
+     // together (a loop storing each result before the next load serialises their latencies)
+    uint32_t cs[SPC], base[SPC];
+#pragma unroll
+    for (int q = 0; q < SPC; ++q) cs[q] = h_cell[q * CT + tid];
+#pragma unroll
+    for (int q = 0; q < SPC; ++q) {
+      const uint32_t c = cs[q], i = q * CT + tid;
+      base[q] = c;
+      if (c != NONE && c != REMOTE_CELL) {
+        atomicMax(&s.bcount[c * BCOUNT_STRIDE + 1], h_tmax[i]);
+        base[q] = atomicAdd(&s.bcount[c * BCOUNT_STRIDE], h_cnt[i] & 0xFFFFu);
+      }
     }
+#pragma unroll
+    for (int q = 0; q < SPC; ++q) h_cell[q * CT + tid] = base[q];
   }
   __syncthreads();
   uint32_t si[CPT], rk[CPT];
