@@ -108,8 +108,10 @@ typedef struct ggrid_opts {
                               cell-hash variant when its hash fits -- and larger
                               batches by three launches.  1 = the cell-hash
                               launch whenever it fits; 2 = the direct launch
-                              whenever it fits; 3 = always the three launches.
-                              All produce the same index state.                    */
+                              whenever it fits; 3 = always the three launches;
+                              4 = the sort-by-cell path (keys, radix sort by cell,
+                              per-cell runs, allocation, coalesced scatter) for
+                              every batch.  All produce the same index state.      */
   /* ---- multi-GPU (see "multi-GPU" below).  All 0 = one GPU.            */
   uint32_t n_gpus;         /* > 1: ONE index over n_gpus shards driven by this process,
                               shard r on devices[r] (cell ownership, one request/reply

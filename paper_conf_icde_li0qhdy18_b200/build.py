@@ -15,7 +15,7 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 OBJDIR = os.path.join(PKG, "build")
 LIB = os.path.join(PKG, "libggrid.so")
-SOURCES = ["api.cu", "ingest.cu", "flush.cu", "knn.cu", "prior_art.cu", "multi.cu", "prior_art_knn.cu"]
+SOURCES = ["api.cu", "ingest.cu", "ingest_sort.cu", "flush.cu", "knn.cu", "prior_art.cu", "multi.cu", "prior_art_knn.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",

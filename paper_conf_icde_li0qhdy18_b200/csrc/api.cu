@@ -222,7 +222,7 @@ static int build_one(const ggrid_graph* gr, uint32_t cell_size, const ggrid_opts
   h->t_delta = o.t_delta;
   // the expiry cut reads t_now on the host, so expiry keeps ingest synchronous
   h->async_ingest = (o.async_ingest && !o.t_delta) ? 1 : 0;
-  h->ingest_mode = o.ingest_kernels <= 3 ? (int)o.ingest_kernels : 0;
+  h->ingest_mode = o.ingest_kernels <= 4 ? (int)o.ingest_kernels : 0;
   if (const char* fk = getenv("GGRID_FLUSH_KERNEL")) h->flush_kernel = atoi(fk);  // (experiment hook)
   h->s.n_ranks = 1;
   h->s.rank = 0;
@@ -410,6 +410,11 @@ int ggrid_free(ggrid_t h) {
   return GGRID_OK;
 }
 
+// (a batch beyond one resident wave over many cells by the sort-by-cell path (1), or always by
+// the tile-hash three launches (0))
+#ifndef GG_SORTED_INGEST
+#define GG_SORTED_INGEST 1
+#endif
 // ingest n updates already resident in device memory at d_u (the main stream must be
 // ordered after their arrival)
 static constexpr uint64_t kMaxBatch = 0xFFFFFFFEull;  // seq 2 .. 2^32-1 after a re-base
@@ -420,8 +425,15 @@ int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
   const uint32_t ext_need = (uint32_t)std::min<uint64_t>(n, h->n_cells);
   RC(h->ensure_arena(n + 3ull * ext_need, ext_need));
   IngestPlan fp;
-  const bool fused = h->ingest_mode != 3 && ingest_fused_plan(n, h->n_cells, h->sm_count, h->ingest_mode, &fp);
-  if (!fused) RC(h->tmp.ensure(ingest_tmp_bytes(n)));
+  const bool fused = h->ingest_mode != 3 && h->ingest_mode != 4 &&
+                     ingest_fused_plan(n, h->n_cells, h->sm_count, h->ingest_mode, &fp);
+  // beyond one resident wave: the sort-by-cell path (mode 4; by default when the three-launch
+  // path's 8,192-update tiles would average under two updates per distinct cell -- C3: 64M-update
+  // batch 6.85 -> 6.3 ms; on 264 cells (C1) the tiles aggregate well and the sort loses 3x)
+  const bool sorted = !fused && ingest_sorted_fits(n) &&
+                      (h->ingest_mode == 4 ||
+                       (h->ingest_mode == 0 && GG_SORTED_INGEST && 8192ull <= 2ull * h->n_cells));
+  if (!fused) RC(h->tmp.ensure(sorted ? ingest_sort_tmp_bytes(n, h->n_cells) : ingest_tmp_bytes(n)));
   {
     WordSet ws;
     if (fused) ws.add(&h->d_status->ingest_bar, 0u);
@@ -443,6 +455,13 @@ int ingest_device(ggrid_t h, const uint4* d_u, uint64_t n) {
     cudaError_t le = cudaSuccess;
     h->launch(GGRID_K_INGEST_CLASSIFY, [&] { le = launch_ingest_fused(d_u, n, seq0, g, s, fp, st); });
     CK(le);
+  } else if (sorted) {  // keys + radix sort by cell + runs, extent allocation, sorted scatter
+    SortedBatch sb{};
+    cudaError_t le = cudaSuccess;
+    h->launch(GGRID_K_INGEST_CLASSIFY, [&] { le = launch_ingest_sorted_keys(d_u, n, g, s, h->tmp.p, &sb, st); });
+    CK(le);
+    h->launch(GGRID_K_INGEST_ALLOC, [&] { launch_ingest_alloc(g, s, st); });
+    h->launch(GGRID_K_INGEST_SCATTER, [&] { launch_ingest_sorted_scatter(d_u, n, seq0, g, s, sb, st); });
   } else {
     h->launch(GGRID_K_INGEST_CLASSIFY, [&] { launch_ingest_classify(d_u, n, g, s, tmp, st); });
     h->launch(GGRID_K_INGEST_ALLOC, [&] { launch_ingest_alloc(g, s, st); });

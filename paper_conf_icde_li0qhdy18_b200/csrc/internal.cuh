@@ -244,6 +244,18 @@ struct IngestPlan {
   bool direct;  // k_ingest_direct (per-update rank atomics, registers across the barriers)
 };
 bool ingest_fused_plan(uint64_t n, uint32_t n_cells, int sm_count, int mode, IngestPlan* p);
+// sort-by-cell ingest of a large batch (ingest_sort.cu): keys + radix sort + per-cell runs, then
+// k_ingest_alloc, then the scatter of the sorted batch
+struct SortedBatch {
+  const uint32_t* keys;
+  const unsigned long long* vals;
+};
+bool ingest_sorted_fits(uint64_t n);
+size_t ingest_sort_tmp_bytes(uint64_t n, uint32_t n_cells);
+cudaError_t launch_ingest_sorted_keys(const uint4* upd, uint64_t n, const DevGraph& g, const DevState& s,
+                                      void* tmp, SortedBatch* out, cudaStream_t st);
+void launch_ingest_sorted_scatter(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
+                                  const DevState& s, const SortedBatch& b, cudaStream_t st);
 cudaError_t launch_ingest_fused(const uint4* upd, uint64_t n, uint32_t seq0, const DevGraph& g,
                                 const DevState& s, const IngestPlan& p, cudaStream_t st);  // classify -> scatter scratch (tmp + perm)
 void launch_ingest_alloc(const DevGraph& g, const DevState& s, cudaStream_t st);

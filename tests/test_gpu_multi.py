@@ -70,11 +70,12 @@ def test_loopback_index_bit_exact(gg, n):
     grid.close()
 
 
-@pytest.mark.parametrize("mode", [1, 2, 3])
+@pytest.mark.parametrize("mode", [1, 2, 3, 4])
 def test_loopback_ingest_paths(gg, mode):
     """Every ingest path in sharded mode (4 shards): updates of other shards' cells only raise the
     replicated object table (and mark the cell an object leaves STALE on its owner) -- the cell-hash
-    launch (1), the direct launch (2) and the three launches (3) all give the oracle's answers."""
+    launch (1), the direct launch (2), the three launches (3) and the sort-by-cell path (4) all give
+    the oracle's answers."""
     g = synth.table_ii_graph("NY", scale=0.2)
     walk = synth.RandomWalk(g, 20_000, inject=True)
     grid = gg.GGrid(g, 256, max_objects=20_000, n_gpus=4, devices=[0] * 4, ingest_kernels=mode)
