@@ -564,6 +564,9 @@ __global__ void __launch_bounds__(FT, 1) k_ingest_fused(const uint4* __restrict_
 // registers across the two grid barriers (no shared memory, no tmp/perm round trip), and the
 // scatter re-reads its record from L2.  Same arithmetic and rejection rules as the paths above.
 constexpr int DT = 512;   // threads per CTA (2 CTAs per SM)
+#ifndef GG_DIRECT_HP
+#define GG_DIRECT_HP 2
+#endif
 // (experiment hook) GG_INGEST_TIMING=1: phase timestamps of the first and last CTA, printed
 #ifndef GG_INGEST_TIMING
 #define GG_INGEST_TIMING 0
@@ -595,7 +598,7 @@ __global__ void __launch_bounds__(DT, 2) k_ingest_direct(const uint4* __restrict
   // whose cleaned list the object leaves (R8's STALE mark; NONE: none)
   uint32_t rk[DPT], vs[DPT], lv[DPT];
   uint32_t tl = 0;
-  constexpr int HP = 2;  // (parts of 2: registers)
+  constexpr int HP = GG_DIRECT_HP;  // (parts: registers vs gathers in flight)
 #pragma unroll
   for (int hf = 0; hf < DPT / HP; ++hf) {  // a part's loads and gathers in flight together
     uint4 mm[HP];
