@@ -1082,8 +1082,14 @@ finish:
 // scratch (the last level).  Two instantiations, so that every table access of the shared one
 // compiles to LDS/STS/ATOMS with 32-bit addresses (one pointer that may be either space makes
 // them generic 64-bit LD/ST/ATOM, measured ~10% slower overall).
+// registers capped for GG_WARP_MINB resident CTAs of 4 queries per SM: the 600-slot table makes a
+// query 7,008 B of shared memory, so 8 CTAs (32 queries) fit and 64 registers must too
+#ifndef GG_WARP_MINB
+#define GG_WARP_MINB 8
+#endif
+#define GG_EXPAND_BOUNDS __launch_bounds__(128, GG_WARP_MINB)
 template <bool SMEM>
-__global__ void k_expand(QParams P) {
+__global__ void GG_EXPAND_BOUNDS k_expand(QParams P) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
   const uint32_t warp = threadIdx.x >> 5;
@@ -2070,14 +2076,14 @@ constexpr int NLEVELS = EXPAND_LEVELS;
 // split, F 64, C 32: 7,024 B, 64 registers with spills) 1.146 ms vs 1.115 ms for this 28-resident
 // configuration; without the half split 71% of the queries promote (chunks of > 64 arcs)
 #ifndef GG_F0W
-#define GG_F0W 96
+#define GG_F0W 64
 #endif
 #ifndef GG_C0W
 #define GG_C0W 64
 #endif
 static_assert((GG_C0W & (GG_C0W - 1)) == 0, "the candidate list is bitonic-sorted: a power of two");
 #ifndef GG_H0W
-#define GG_H0W 704
+#define GG_H0W 600
 #endif
 #ifndef GG_F0
 #define GG_F0 96
@@ -2117,18 +2123,32 @@ uint32_t expand_table_slots(int level) { return caps_for(level, 1).H; }
 
 uint32_t expand_max_k(int level) { return caps_for(level, 1).C - 32; }
 
-// the caps a level runs with in a given mode (the one-warp kernel's level 0 has its own table)
-static Caps caps_mode(int level, uint32_t V, bool cta) {
+// The one-warp level 0 has two tables: the narrow one (600 slots, frontier 64: 7,008 B per query,
+// 32 queries per SM) and, when the caller's hint says the expected ball touches more vertices
+// (WIDE_BIT of ball_hint: expected ball x arcs per vertex above ~650, e.g. C1's denser NY-shaped
+// graph), the wide one (704 slots, frontier 96: 28 per SM).  Measured: C3 expansion 1.030 ->
+// 0.986 ms narrow; C1 0.262 ms wide vs 0.360 narrow; C2 k=30 0.268 wide vs 0.286 narrow.
+#ifndef GG_H0W_WIDE
+#define GG_H0W_WIDE 704
+#endif
+#ifndef GG_F0W_WIDE
+#define GG_F0W_WIDE 96
+#endif
+constexpr uint32_t WIDE_BIT = 1u << 31;
+__host__ __device__ inline bool wide0(uint32_t bh) { return (bh & WIDE_BIT) != 0; }
+__host__ __device__ inline uint32_t ball_of(uint32_t bh) { return bh & ~WIDE_BIT; }
+// the caps a level runs with in a given mode (the one-warp kernel's level 0 has its own tables)
+static Caps caps_mode(int level, uint32_t V, bool cta, bool wide = false) {
   Caps c = caps_for(level, V);
   if (level == 0 && !cta) {
-    c.H = GG_H0W;
-    c.F = GG_F0W;
+    c.H = wide ? GG_H0W_WIDE : GG_H0W;
+    c.F = wide ? GG_F0W_WIDE : GG_F0W;
     c.C = GG_C0W;
   }
   return c;
 }
-static size_t warp_bytes_mode(int level, uint32_t V, bool cta) {
-  return (warpmem_bytes(caps_mode(level, V, cta), level == NLEVELS - 1 ? 4 : 2) + 15) & ~size_t(15);
+static size_t warp_bytes_mode(int level, uint32_t V, bool cta, bool wide = false) {
+  return (warpmem_bytes(caps_mode(level, V, cta, wide), level == NLEVELS - 1 ? 4 : 2) + 15) & ~size_t(15);
 }
 
 size_t expand_warp_bytes(int level, uint32_t V) {
@@ -2149,9 +2169,13 @@ size_t expand_warp_bytes(int level, uint32_t V) {
 #define GG_CTA_BALL1 1024  // (C2 k=40 / 50: expansion 0.427 -> 0.401 / 0.489 -> 0.474 ms; 0: always a CTA)
 #endif
 constexpr uint32_t kCtaBall = GG_CTA_BALL;
-uint32_t expand_warp_max_k() { return GG_C0W - 32; }
+#ifndef GG_WARP_MAXK
+#define GG_WARP_MAXK (GG_C0W - 32)
+#endif
+uint32_t expand_warp_max_k() { return GG_WARP_MAXK; }
 uint32_t expand_cta_ball() { return kCtaBall; }
 static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
+  ball_hint = ball_of(ball_hint);
   if (level >= NLEVELS - 1) return false;
   if (n <= (uint32_t)sm_count) return true;
   if (level == 0) return GG_CTA_LEVEL == 0 && ball_hint >= kCtaBall;
@@ -2164,7 +2188,7 @@ static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
 // one-warp kernel (which exports the state of the queries it promotes), else 0
 size_t expand_resume_bytes(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level >= NLEVELS - 2 || use_cta(level, n, sm_count, ball_hint) || (GG_PAIR && level == 0)) return 0;
-  return resume_bytes(caps_mode(level, 1, false));
+  return resume_bytes(caps_mode(level, 1, false, wide0(ball_hint)));
 }
 
 // one-warp-per-query kernel: warps (independent queries) per CTA.  Each CTA costs 1 KB of reserved
@@ -2175,15 +2199,15 @@ size_t expand_resume_bytes(int level, uint32_t n, int sm_count, uint32_t ball_hi
 constexpr uint32_t WPC = GG_WARP_WPC;
 
 // resident CTAs per SM of a shared-memory level's kernel (occupancy calculator, cached)
-static uint32_t blocks_per_sm(int level, bool cta) {
-  static int bps[2][NLEVELS] = {};  // (occupancy: the same on every B200)
+static uint32_t blocks_per_sm(int level, bool cta, bool wide = false) {
+  static int bps[2][2][NLEVELS] = {};  // (occupancy: the same on every B200)
   // the attribute is per device: set on every device this process launches on
   if (cta) func_attr_once(cta_kernel(level), cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
   else if (GG_PAIR && level == 0) func_attr_once(k_expand_pair, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   else func_attr_once(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-  int& b = bps[cta ? 1 : 0][level];
+  int& b = bps[wide ? 1 : 0][cta ? 1 : 0][level];
   if (!b) {
-    const int smem = (int)warp_bytes_mode(level, 1, cta);
+    const int smem = (int)warp_bytes_mode(level, 1, cta, wide);
     if (cta) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, cta_kernel(level), cta_warps(level) * 32, smem);
     } else {
@@ -2204,14 +2228,14 @@ uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level == NLEVELS - 1) return 0;  // (global scratch: sized by the caller's scratch warps)
   const bool cta = use_cta(level, n, sm_count, ball_hint);
   const uint32_t per = cta ? 1u : (GG_PAIR && level == 0 ? 2 * WPC : WPC);  // queries a CTA runs at once
-  return std::min<uint32_t>((n + per - 1) / per, (uint32_t)sm_count * blocks_per_sm(level, cta));
+  return std::min<uint32_t>((n + per - 1) / per, (uint32_t)sm_count * blocks_per_sm(level, cta, wide0(ball_hint)));
 }
 
 size_t expand_block_bytes(int level, uint32_t V, uint32_t n, int sm_count, uint32_t ball_hint, bool chained) {
   if (level == NLEVELS - 1) return 0;
   const bool cta = chained || use_cta(level, n, sm_count, ball_hint);
   const uint32_t per = cta ? 1u : (GG_PAIR && level == 0 ? 2 * WPC : WPC);
-  return warp_bytes_mode(level, V, cta) * per + 1024;  // (+ the per-CTA reservation)
+  return warp_bytes_mode(level, V, cta, wide0(ball_hint)) * per + 1024;  // (+ the per-CTA reservation)
 }
 
 void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st) {
@@ -2235,7 +2259,8 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.bound = L.bound;
   P.remote = L.remote;
   const bool cta_mode = level < NLEVELS - 1 && (L.chain_in != nullptr || use_cta(level, L.n, sm_count, L.ball_hint));
-  P.caps = caps_mode(level, g.V, cta_mode);
+  const bool wide = wide0(L.ball_hint);
+  P.caps = caps_mode(level, g.V, cta_mode, wide);
   P.warps_per_cta = 1;  // (the one-warp shared-memory kernel: WPC, set below)
   P.scratch = nullptr;
   P.exited = L.exited;
@@ -2250,12 +2275,12 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.resume_bytes = 0;
   P.rcaps = Caps{0, 0, 0};
   if (L.resume && L.resume_cap) {  // (the exporting level: this one, or the one below a chained level)
-    P.rcaps = caps_mode(L.chain_in ? level - 1 : level, g.V, false);
+    P.rcaps = caps_mode(L.chain_in ? level - 1 : level, g.V, false, wide);
     P.resume = static_cast<unsigned char*>(L.resume);
     P.resume_cap = L.resume_cap;
     P.resume_bytes = (uint32_t)resume_bytes(P.rcaps);
   }
-  const int smem = (int)warp_bytes_mode(level, g.V, cta_mode);
+  const int smem = (int)warp_bytes_mode(level, g.V, cta_mode, wide);
   if (level == NLEVELS - 1) {
     P.scratch = static_cast<unsigned char*>(L.scratch);
     k_expand<false><<<std::min<uint32_t>(L.n, std::max<uint32_t>(1, L.scratch_warps)), 32, 0, st>>>(P);
@@ -2263,7 +2288,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   }
   const bool cta = L.chain_in != nullptr || use_cta(level, L.n, sm_count, L.ball_hint);
   const uint32_t grid = L.grid ? L.grid : std::max<uint32_t>(1, expand_grid(level, L.n, sm_count, L.ball_hint));
-  blocks_per_sm(level, cta);  // (sets the shared-memory attribute)
+  blocks_per_sm(level, cta, wide);  // (sets the shared-memory attribute)
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   const bool pair = !cta && GG_PAIR && level == 0;
