@@ -460,10 +460,10 @@ def run_ours(args, cfg_name):
     if dom == "expand":
         nq = Qr * K
         rounds_q = dx["iterations"] / max(1, nq)
-        # the C3 starting level: the one-warp kernel, 7 CTAs x 4 queries per SM (shared memory),
-        # ~1,028 of the 1,036 CTAs (the rest reserved for the chained level beside it)
+        # the C3 starting level: the one-warp kernel with its narrow table, 8 CTAs x 4 queries per
+        # SM (shared memory and 64 registers), less the few CTAs reserved for the chained level
         sms = torch.cuda.get_device_properties(dev).multi_processor_count
-        resident = int(os.environ.get("BENCH_EXPAND_RESIDENT", str(sms * 28)))
+        resident = int(os.environ.get("BENCH_EXPAND_RESIDENT", str(sms * 32)))
         cyc = rounds_q * (ROUND_TRIPS * L2_HIT_CYCLES + ROUND_ONCHIP_CYCLES)
         t_model_ms = nq / resident * cyc / (sm_mhz_max * 1e3)
         roofline["latency_model"] = {
