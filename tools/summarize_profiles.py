@@ -117,7 +117,8 @@ for ll in [os.path.join(src, f) for f in sorted(os.listdir(src)) if f.startswith
     vals = [float(r[h.index("Metric Value")].replace(",", "")) for r in rows[hi + 1:]]
     first = next((i for i, n in enumerate(names) if "k_ingest_direct" in n or "k_ingest_fused" in n), None)
     if first is not None:  # (up to the e2e section's fresh index: its bulk preload ingest)
-        end = next((i for i in range(first, len(names)) if "k_ingest_classify" in names[i]), len(names))
+        end = next((i for i in range(first, len(names))
+                    if "k_ingest_classify" in names[i] or "k_bulk_keys" in names[i]), len(names))
         st = collections.defaultdict(list)
         for n, v in zip(names[first:end], vals[first:end]):
             if "gg::" in n:
