@@ -672,11 +672,12 @@ int knn_impl(ggrid_t h, const ggrid_query* q, uint32_t n_q, uint32_t k, uint32_t
   const double ball = (double)k * h->V / (double)std::max<uint64_t>(1, h->n_live_hi());
   while (lvl0 < L - 2 && (k > expand_max_k(lvl0) || GG_BALL_FACTOR * ball > expand_table_slots(lvl0))) lvl0++;
   while (lvl0 < L - 1 && k > expand_max_k(lvl0)) lvl0++;
-  uint32_t ball_hint = (uint32_t)std::min(ball, 2.0e9);
+  uint32_t ball_hint = (uint32_t)std::min(ball, 1.0e9);  // (bits 30-31: table variant flags)
   if (k > expand_warp_max_k()) ball_hint = std::max(ball_hint, expand_cta_ball());  // (its candidate list)
   // bit 31: the one-warp level 0 takes its wide table (the expected ball touches more vertices:
   // ball x arcs per vertex, C1 ~730 vs C3 ~580)
   if (ball * (double)h->A / std::max(1u, h->V) > GG_WIDE_TABLE_HINT) ball_hint |= 1u << 31;
+  else if (k <= 16) ball_hint |= 1u << 30;  // (bit 30: the narrow table's short-candidate-list variant)
   std::vector<uint32_t> n_in(L, 0);
   n_in[lvl0] = n_q;
   // The level above the starting one runs in the same round BESIDE it (a programmatic

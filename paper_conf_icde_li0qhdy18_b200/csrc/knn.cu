@@ -2134,21 +2134,28 @@ uint32_t expand_max_k(int level) { return caps_for(level, 1).C - 32; }
 #ifndef GG_F0W_WIDE
 #define GG_F0W_WIDE 96
 #endif
-constexpr uint32_t WIDE_BIT = 1u << 31;
+// SMALLK_BIT (k <= 16 with the narrow table): a 32-entry candidate list buys 48 more slots (648)
+// at the same 32 resident queries per SM (C3: 0.988 -> 0.979 ms)
+#ifndef GG_H0W_SMALLK
+#define GG_H0W_SMALLK 648
+#endif
+constexpr uint32_t WIDE_BIT = 1u << 31, SMALLK_BIT = 1u << 30;
 __host__ __device__ inline bool wide0(uint32_t bh) { return (bh & WIDE_BIT) != 0; }
-__host__ __device__ inline uint32_t ball_of(uint32_t bh) { return bh & ~WIDE_BIT; }
+// table variant of the one-warp level 0: 0 narrow, 1 wide, 2 narrow with the short candidate list
+__host__ __device__ inline int var0(uint32_t bh) { return (bh & WIDE_BIT) ? 1 : (bh & SMALLK_BIT) ? 2 : 0; }
+__host__ __device__ inline uint32_t ball_of(uint32_t bh) { return bh & ~(WIDE_BIT | SMALLK_BIT); }
 // the caps a level runs with in a given mode (the one-warp kernel's level 0 has its own tables)
-static Caps caps_mode(int level, uint32_t V, bool cta, bool wide = false) {
+static Caps caps_mode(int level, uint32_t V, bool cta, int var = 0) {
   Caps c = caps_for(level, V);
   if (level == 0 && !cta) {
-    c.H = wide ? GG_H0W_WIDE : GG_H0W;
-    c.F = wide ? GG_F0W_WIDE : GG_F0W;
-    c.C = GG_C0W;
+    c.H = var == 1 ? GG_H0W_WIDE : var == 2 ? GG_H0W_SMALLK : GG_H0W;
+    c.F = var == 1 ? GG_F0W_WIDE : GG_F0W;
+    c.C = var == 2 ? 32u : (uint32_t)GG_C0W;
   }
   return c;
 }
-static size_t warp_bytes_mode(int level, uint32_t V, bool cta, bool wide = false) {
-  return (warpmem_bytes(caps_mode(level, V, cta, wide), level == NLEVELS - 1 ? 4 : 2) + 15) & ~size_t(15);
+static size_t warp_bytes_mode(int level, uint32_t V, bool cta, int var = 0) {
+  return (warpmem_bytes(caps_mode(level, V, cta, var), level == NLEVELS - 1 ? 4 : 2) + 15) & ~size_t(15);
 }
 
 size_t expand_warp_bytes(int level, uint32_t V) {
@@ -2188,7 +2195,7 @@ static bool use_cta(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
 // one-warp kernel (which exports the state of the queries it promotes), else 0
 size_t expand_resume_bytes(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level >= NLEVELS - 2 || use_cta(level, n, sm_count, ball_hint) || (GG_PAIR && level == 0)) return 0;
-  return resume_bytes(caps_mode(level, 1, false, wide0(ball_hint)));
+  return resume_bytes(caps_mode(level, 1, false, var0(ball_hint)));
 }
 
 // one-warp-per-query kernel: warps (independent queries) per CTA.  Each CTA costs 1 KB of reserved
@@ -2199,15 +2206,15 @@ size_t expand_resume_bytes(int level, uint32_t n, int sm_count, uint32_t ball_hi
 constexpr uint32_t WPC = GG_WARP_WPC;
 
 // resident CTAs per SM of a shared-memory level's kernel (occupancy calculator, cached)
-static uint32_t blocks_per_sm(int level, bool cta, bool wide = false) {
-  static int bps[2][2][NLEVELS] = {};  // (occupancy: the same on every B200)
+static uint32_t blocks_per_sm(int level, bool cta, int var = 0) {
+  static int bps[3][2][NLEVELS] = {};  // (occupancy: the same on every B200)
   // the attribute is per device: set on every device this process launches on
   if (cta) func_attr_once(cta_kernel(level), cudaFuncAttributeMaxDynamicSharedMemorySize, 226 * 1024);
   else if (GG_PAIR && level == 0) func_attr_once(k_expand_pair, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
   else func_attr_once(k_expand<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-  int& b = bps[wide ? 1 : 0][cta ? 1 : 0][level];
+  int& b = bps[var][cta ? 1 : 0][level];
   if (!b) {
-    const int smem = (int)warp_bytes_mode(level, 1, cta, wide);
+    const int smem = (int)warp_bytes_mode(level, 1, cta, var);
     if (cta) {
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, cta_kernel(level), cta_warps(level) * 32, smem);
     } else {
@@ -2228,14 +2235,14 @@ uint32_t expand_grid(int level, uint32_t n, int sm_count, uint32_t ball_hint) {
   if (level == NLEVELS - 1) return 0;  // (global scratch: sized by the caller's scratch warps)
   const bool cta = use_cta(level, n, sm_count, ball_hint);
   const uint32_t per = cta ? 1u : (GG_PAIR && level == 0 ? 2 * WPC : WPC);  // queries a CTA runs at once
-  return std::min<uint32_t>((n + per - 1) / per, (uint32_t)sm_count * blocks_per_sm(level, cta, wide0(ball_hint)));
+  return std::min<uint32_t>((n + per - 1) / per, (uint32_t)sm_count * blocks_per_sm(level, cta, var0(ball_hint)));
 }
 
 size_t expand_block_bytes(int level, uint32_t V, uint32_t n, int sm_count, uint32_t ball_hint, bool chained) {
   if (level == NLEVELS - 1) return 0;
   const bool cta = chained || use_cta(level, n, sm_count, ball_hint);
   const uint32_t per = cta ? 1u : (GG_PAIR && level == 0 ? 2 * WPC : WPC);
-  return warp_bytes_mode(level, V, cta, wide0(ball_hint)) * per + 1024;  // (+ the per-CTA reservation)
+  return warp_bytes_mode(level, V, cta, var0(ball_hint)) * per + 1024;  // (+ the per-CTA reservation)
 }
 
 void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, int sm_count, cudaStream_t st) {
@@ -2259,8 +2266,8 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.bound = L.bound;
   P.remote = L.remote;
   const bool cta_mode = level < NLEVELS - 1 && (L.chain_in != nullptr || use_cta(level, L.n, sm_count, L.ball_hint));
-  const bool wide = wide0(L.ball_hint);
-  P.caps = caps_mode(level, g.V, cta_mode, wide);
+  const int var = var0(L.ball_hint);
+  P.caps = caps_mode(level, g.V, cta_mode, var);
   P.warps_per_cta = 1;  // (the one-warp shared-memory kernel: WPC, set below)
   P.scratch = nullptr;
   P.exited = L.exited;
@@ -2275,12 +2282,12 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   P.resume_bytes = 0;
   P.rcaps = Caps{0, 0, 0};
   if (L.resume && L.resume_cap) {  // (the exporting level: this one, or the one below a chained level)
-    P.rcaps = caps_mode(L.chain_in ? level - 1 : level, g.V, false, wide);
+    P.rcaps = caps_mode(L.chain_in ? level - 1 : level, g.V, false, var);
     P.resume = static_cast<unsigned char*>(L.resume);
     P.resume_cap = L.resume_cap;
     P.resume_bytes = (uint32_t)resume_bytes(P.rcaps);
   }
-  const int smem = (int)warp_bytes_mode(level, g.V, cta_mode, wide);
+  const int smem = (int)warp_bytes_mode(level, g.V, cta_mode, var);
   if (level == NLEVELS - 1) {
     P.scratch = static_cast<unsigned char*>(L.scratch);
     k_expand<false><<<std::min<uint32_t>(L.n, std::max<uint32_t>(1, L.scratch_warps)), 32, 0, st>>>(P);
@@ -2288,7 +2295,7 @@ void launch_expand(const ExpandLaunch& L, const DevGraph& g, const DevState& s, 
   }
   const bool cta = L.chain_in != nullptr || use_cta(level, L.n, sm_count, L.ball_hint);
   const uint32_t grid = L.grid ? L.grid : std::max<uint32_t>(1, expand_grid(level, L.n, sm_count, L.ball_hint));
-  blocks_per_sm(level, cta, wide);  // (sets the shared-memory attribute)
+  blocks_per_sm(level, cta, var);  // (sets the shared-memory attribute)
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   const bool pair = !cta && GG_PAIR && level == 0;
